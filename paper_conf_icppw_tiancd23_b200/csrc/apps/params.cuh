@@ -1,0 +1,279 @@
+// csrc/apps/params.cuh — S5 (instance CLI parse) and the arena / shared-
+// memory layout of every app, compiled for BOTH host and device: the host
+// sizes the slot arenas and the dynamic shared memory from exactly the code
+// the instance runs, so a valid line can never run out of arena.
+//
+// Flag grammars follow SURVEY.md §8(c) XS-1 / RS-1 / AMG-1; an unknown flag,
+// a missing value or a bad value makes the instance print the usage text and
+// exit 1 (the paper's loader passes each line to the app's own main,
+// Fig. 4).
+#pragma once
+#include "../rt/device_rt.cuh"
+
+namespace ens {
+
+enum AppId : uint32_t { APP_BY_ARGV0 = 0, APP_ECHO = 1, APP_XSBENCH = 2, APP_RSBENCH = 3, APP_AMGMK = 4,
+                        APP_NOTFOUND = 5 /* internal: argv[0] names no app */ };
+
+// ============================ XSBench-style ================================
+enum { XS_UNIONIZED = 0, XS_NUCLIDE = 1, XS_HASH = 2 };
+constexpr int kXsMaxGp = 16384;  // per-nuclide sort fits one SM's shared memory
+
+struct XsParams {
+  int n_iso = 355;
+  int n_gp = 11303;
+  long long lookups = 17000000;
+  int grid = XS_UNIONIZED;
+  int bins = 10000;
+  unsigned long long seed = 1070, gseed = 42;
+};
+
+// returns the offending argv index, or -1
+ENS_HD int xs_parse(int argc, const char *const *argv, XsParams &p) {
+  for (int i = 1; i < argc; i++) {
+    const char *f = argv[i];
+    if (i + 1 >= argc) return i;
+    const char *v = argv[i + 1];
+    long long x;
+    if (str_eq(f, "-s")) {
+      if (str_eq(v, "small")) p.n_iso = 68;
+      else if (str_eq(v, "large")) p.n_iso = 355;
+      else return i + 1;
+    } else if (str_eq(f, "-g")) {
+      if (!parse_i64(v, &x) || x < 2 || x > kXsMaxGp) return i + 1;
+      p.n_gp = (int)x;
+    } else if (str_eq(f, "-l")) {
+      if (!parse_i64(v, &x) || x < 0 || x > (1LL << 40)) return i + 1;
+      p.lookups = x;
+    } else if (str_eq(f, "-G")) {
+      if (str_eq(v, "unionized")) p.grid = XS_UNIONIZED;
+      else if (str_eq(v, "nuclide")) p.grid = XS_NUCLIDE;
+      else if (str_eq(v, "hash")) p.grid = XS_HASH;
+      else return i + 1;
+    } else if (str_eq(f, "-h")) {
+      if (!parse_i64(v, &x) || x < 1 || x > 10000000) return i + 1;
+      p.bins = (int)x;
+    } else if (str_eq(f, "-m")) {
+      if (!str_eq(v, "event")) return i + 1;
+    } else if (str_eq(f, "-r")) {
+      if (!parse_i64(v, &x) || x < 0) return i + 1;
+      p.seed = (unsigned long long)x;
+    } else if (str_eq(f, "-R")) {
+      if (!parse_i64(v, &x) || x < 0) return i + 1;
+      p.gseed = (unsigned long long)x;
+    } else {
+      return i;
+    }
+    i++;
+  }
+  return -1;
+}
+
+ENS_HD int xs_max_nucs(int n_iso) { return n_iso == 68 ? 34 : 321; }
+ENS_HD int pow2_ceil(int n) {
+  int p = 1;
+  while (p < n) p <<= 1;
+  return p;
+}
+
+// arena layout (byte offsets, 256-B aligned)
+struct XsLayout {
+  uint64_t recs;      // [n_iso][n_gp] x 48 B records, sorted per nuclide
+  uint64_t scratch;   // [n_gp] x 48 B unsorted records of one nuclide
+  uint64_t uenergy;   // unionized: [n_u] sorted union energies (u64 bits)
+  uint64_t utmp;      // unionized: [n_u] merge ping-pong
+  uint64_t uown;      // unionized: [n_u] u16 owner nuclide
+  uint64_t uowntmp;   // unionized: [n_u] u16 ping-pong
+  uint64_t index;     // unionized [n_u][n_iso] / hash [n_iso][bins+1] int32
+  uint64_t total;
+};
+ENS_HD XsLayout xs_layout(const XsParams &p) {
+  XsLayout L{};
+  const uint64_t n_u = (uint64_t)p.n_iso * p.n_gp;
+  uint64_t o = 0;
+  L.recs = o; o = align_up(o + n_u * 48, 256);
+  L.scratch = o; o = align_up(o + (uint64_t)p.n_gp * 48, 256);
+  if (p.grid == XS_UNIONIZED) {
+    L.uenergy = o; o = align_up(o + n_u * 8, 256);
+    L.utmp = o; o = align_up(o + n_u * 8, 256);
+    L.uown = o; o = align_up(o + n_u * 2, 256);
+    L.uowntmp = o; o = align_up(o + n_u * 2, 256);
+    L.index = o; o = align_up(o + n_u * (uint64_t)p.n_iso * 4, 256);
+  } else if (p.grid == XS_HASH) {
+    L.index = o; o = align_up(o + (uint64_t)p.n_iso * (p.bins + 1) * 4, 256);
+  }
+  L.total = o;
+  return L;
+}
+
+// dynamic shared memory layout
+struct XsSmem {
+  uint32_t thr, nn, mats, concs, keys, perm, total;
+};
+ENS_HD XsSmem xs_smem(const XsParams &p) {
+  XsSmem S{};
+  const uint32_t mx = (uint32_t)xs_max_nucs(p.n_iso);
+  const uint32_t P2 = (uint32_t)pow2_ceil(p.n_gp);
+  uint32_t o = 0;
+  S.thr = o; o += 12 * 8;                 // pick_mat thresholds
+  S.nn = o; o += 16 * 4;                  // num_nucs
+  S.concs = o; o += 12 * mx * 8;          // concentrations
+  S.mats = o; o += (uint32_t)align_up(12 * mx * 2, 16);  // nuclide ids (u16)
+  S.keys = o; o += P2 * 8;                // sort keys (energy bits)
+  S.perm = o; o += (uint32_t)align_up(P2 * 2, 16);       // sort payload (u16)
+  S.total = o;
+  return S;
+}
+
+// ============================ RSBench-style ================================
+struct RsParams {
+  int n_nuc = 355;
+  long long lookups = 10000000;
+  int avg_poles = 1000;
+  int avg_windows = 100;
+  int doppler = 1;
+  unsigned long long seed = 1070, iseed = 42;
+};
+
+ENS_HD int rs_parse(int argc, const char *const *argv, RsParams &p) {
+  for (int i = 1; i < argc; i++) {
+    const char *f = argv[i];
+    if (str_eq(f, "-d")) {
+      p.doppler = 0;
+      continue;
+    }
+    if (i + 1 >= argc) return i;
+    const char *v = argv[i + 1];
+    long long x;
+    if (str_eq(f, "-s")) {
+      if (str_eq(v, "small")) p.n_nuc = 68;
+      else if (str_eq(v, "large")) p.n_nuc = 355;
+      else return i + 1;
+    } else if (str_eq(f, "-l")) {
+      if (!parse_i64(v, &x) || x < 0 || x > (1LL << 40)) return i + 1;
+      p.lookups = x;
+    } else if (str_eq(f, "-p")) {
+      if (!parse_i64(v, &x) || x < 1 || x > 100000) return i + 1;
+      p.avg_poles = (int)x;
+    } else if (str_eq(f, "-w")) {
+      if (!parse_i64(v, &x) || x < 1 || x > 100000) return i + 1;
+      p.avg_windows = (int)x;
+    } else if (str_eq(f, "-r")) {
+      if (!parse_i64(v, &x) || x < 0) return i + 1;
+      p.seed = (unsigned long long)x;
+    } else if (str_eq(f, "-R")) {
+      if (!parse_i64(v, &x) || x < 0) return i + 1;
+      p.iseed = (unsigned long long)x;
+    } else {
+      return i;
+    }
+    i++;
+  }
+  return -1;
+}
+
+struct RsLayout {
+  uint64_t pole_off;   // [n_nuc+1] int32 prefix of n_poles
+  uint64_t win_off;    // [n_nuc+1] int32 prefix of n_windows
+  uint64_t poles;      // [total_poles] x 64 B {EA, RT, RA, RF} complex
+  uint64_t pole_l;     // [total_poles] u8 l_value
+  uint64_t windows;    // [total_windows] x 32 B {T, A, F, (start,end)}
+  uint64_t k0rs;       // [n_nuc][4] double
+  uint64_t total;
+};
+ENS_HD RsLayout rs_layout(const RsParams &p) {
+  RsLayout L{};
+  const uint64_t tp = (uint64_t)p.avg_poles * p.n_nuc, tw = (uint64_t)p.avg_windows * p.n_nuc;
+  uint64_t o = 0;
+  L.pole_off = o; o = align_up(o + (p.n_nuc + 1) * 4ULL, 256);
+  L.win_off = o; o = align_up(o + (p.n_nuc + 1) * 4ULL, 256);
+  L.poles = o; o = align_up(o + tp * 64, 256);
+  L.pole_l = o; o = align_up(o + tp, 256);
+  L.windows = o; o = align_up(o + tw * 32, 256);
+  L.k0rs = o; o = align_up(o + p.n_nuc * 32ULL, 256);
+  L.total = o;
+  return L;
+}
+struct RsSmem {
+  uint32_t thr, nn, concs, mats, npol, nwin, total;
+};
+ENS_HD RsSmem rs_smem(const RsParams &p) {
+  RsSmem S{};
+  const uint32_t mx = (uint32_t)xs_max_nucs(p.n_nuc);
+  uint32_t o = 0;
+  S.thr = o; o += 12 * 8;
+  S.nn = o; o += 16 * 4;
+  S.concs = o; o += 12 * mx * 8;
+  S.mats = o; o += (uint32_t)align_up(12 * mx * 2, 16);
+  S.npol = o; o += (uint32_t)align_up((p.n_nuc + 1) * 4, 16);   // pole counts -> offsets
+  S.nwin = o; o += (uint32_t)align_up((p.n_nuc + 1) * 4, 16);   // window counts -> offsets
+  S.total = o;
+  return S;
+}
+
+// ============================ AMGmk-style ==================================
+struct AmgParams {
+  int nx = 50, ny = 50, nz = 50;
+  int iters = 100;
+  int kind = 0;  // 0 relax, 1 matvec, 2 both
+  unsigned long long seed = 0;
+};
+ENS_HD int amg_parse(int argc, const char *const *argv, AmgParams &p) {
+  for (int i = 1; i < argc; i++) {
+    const char *f = argv[i];
+    if (i + 1 >= argc) return i;
+    const char *v = argv[i + 1];
+    long long x;
+    if (str_eq(f, "-x") || str_eq(f, "-y") || str_eq(f, "-z")) {
+      if (!parse_i64(v, &x) || x < 1 || x > 1024) return i + 1;
+      (str_eq(f, "-x") ? p.nx : str_eq(f, "-y") ? p.ny : p.nz) = (int)x;
+    } else if (str_eq(f, "-i")) {
+      if (!parse_i64(v, &x) || x < 0 || x > 1000000) return i + 1;
+      p.iters = (int)x;
+    } else if (str_eq(f, "-k")) {
+      if (str_eq(v, "relax")) p.kind = 0;
+      else if (str_eq(v, "matvec")) p.kind = 1;
+      else if (str_eq(v, "both")) p.kind = 2;
+      else return i + 1;
+    } else if (str_eq(f, "-r")) {
+      if (!parse_i64(v, &x) || x < 0) return i + 1;
+      p.seed = (unsigned long long)x;
+    } else {
+      return i;
+    }
+    i++;
+  }
+  if ((long long)p.nx * p.ny * p.nz > (1LL << 24)) return 0;  // reading R-amg-range
+  return -1;
+}
+
+// SELL-32 layout: rows in slices of 32; within a slice entries are stored
+// column-major by entry position (entry e of the slice's 32 rows are
+// contiguous), padded to 7 entries per row; padding entries have col = -1.
+struct AmgLayout {
+  long long n, nnz, n_slices;
+  uint64_t col;    // [n_slices][7][32] int32
+  uint64_t val;    // [n_slices][7][32] double
+  uint64_t rlen;   // [n] u8 entries per row
+  uint64_t f, u, u2, y;  // [n] double
+  uint64_t total;
+};
+ENS_HD AmgLayout amg_layout(const AmgParams &p) {
+  AmgLayout L{};
+  L.n = (long long)p.nx * p.ny * p.nz;
+  L.nnz = 7 * L.n - 2 * ((long long)p.nx * p.ny + (long long)p.ny * p.nz + (long long)p.nx * p.nz);
+  L.n_slices = (L.n + 31) / 32;
+  const uint64_t ent = (uint64_t)L.n_slices * 7 * 32;
+  uint64_t o = 0;
+  L.col = o; o = align_up(o + ent * 4, 256);
+  L.val = o; o = align_up(o + ent * 8, 256);
+  L.rlen = o; o = align_up(o + (uint64_t)L.n, 256);
+  L.f = o; o = align_up(o + (uint64_t)L.n * 8, 256);
+  L.u = o; o = align_up(o + (uint64_t)L.n * 8, 256);
+  L.u2 = o; o = align_up(o + (uint64_t)L.n * 8, 256);
+  L.y = o; o = align_up(o + (uint64_t)L.n * 8, 256);
+  L.total = o;
+  return L;
+}
+
+}  // namespace ens

@@ -1,0 +1,544 @@
+// csrc/host/api.cpp — N3, the C ABI of libens.so (declared in include/ens.h).
+//
+// S1  ens_load_args / ens_parse_args: the enhanced loader of §3.2
+//      / Fig. 4 — one instance per line, argv[0]
+//     first.  The paper's StringCache keeps c_str() pointers into a growing
+//     vector<string> (dangling after reallocation for short strings); here
+//     every token lives once in an immutable packed blob with offsets.
+// S2  ens_launch: one pinned host->device copy of blob + offsets + instance
+//     map, then one persistent launch per app present (kernels.cu).
+// S10 ens_collect: records, tallies and the compacted stdout back to the
+//     host (P:380 `map(from: Ret[:NI])`), stdout formatted here.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../../include/ens.h"
+#include "../apps/params.cuh"
+#include "../kparams.h"
+
+namespace ens {
+long format_raw(const void *raw, size_t raw_len, std::string &out);
+}
+
+using namespace ens;
+
+// ---------------------------------------------------------------------------
+// errors
+// ---------------------------------------------------------------------------
+static thread_local std::string g_err;
+static int fail(int code, const std::string &msg) {
+  g_err = msg;
+  return code;
+}
+static int cuda_fail(cudaError_t e, const char *what) {
+  g_err = std::string(what) + ": " + cudaGetErrorString(e);
+  return ENS_ECUDA;
+}
+#define CU(call)                                   \
+  do {                                             \
+    cudaError_t e_ = (call);                       \
+    if (e_ != cudaSuccess) return cuda_fail(e_, #call); \
+  } while (0)
+
+// ---------------------------------------------------------------------------
+// S1: args
+// ---------------------------------------------------------------------------
+struct ens_args {
+  bool has_argv0 = false;
+  std::vector<char> blob;            // NUL-terminated tokens
+  std::vector<uint32_t> tok_off;     // argv entries of all lines, in order
+  std::vector<uint32_t> line_tok;    // [n+1]
+  std::vector<const char *> hptr;    // host argv arrays, NULL after each line
+  std::vector<uint32_t> hfirst;      // [n] start of line i in hptr
+};
+
+static uint32_t blob_add(ens_args *a, const char *s, size_t n) {
+  const uint32_t off = (uint32_t)a->blob.size();
+  a->blob.insert(a->blob.end(), s, s + n);
+  a->blob.push_back('\0');
+  return off;
+}
+
+extern "C" int ens_parse_args(const char *text, size_t len, const char *argv0, ens_args **out) {
+  if (!out || (!text && len)) return fail(ENS_EINVAL, "ens_parse_args: NULL argument");
+  *out = nullptr;
+  if (len && std::memchr(text, '\0', len)) return fail(ENS_EPARSE, "ens_parse_args: embedded NUL byte");
+  ens_args *a = new ens_args();
+  uint32_t a0 = 0;
+  if (argv0) {
+    a->has_argv0 = true;
+    a0 = blob_add(a, argv0, std::strlen(argv0));
+  }
+  a->line_tok.push_back(0);
+  size_t pos = 0;
+  while (pos < len) {
+    const char *nl = (const char *)std::memchr(text + pos, '\n', len - pos);
+    size_t end = nl ? (size_t)(nl - text) : len;
+    size_t e = end;
+    if (e > pos && text[e - 1] == '\r') e--;  // reading Q1
+    if (end - pos > ENS_MAX_LINE) {
+      delete a;
+      return fail(ENS_EINVAL, "ens_parse_args: line longer than ENS_MAX_LINE");
+    }
+    int argc = 0;
+    if (argv0) {
+      a->tok_off.push_back(a0);
+      argc++;
+    }
+    size_t i = pos;
+    while (i < e) {
+      while (i < e && (text[i] == ' ' || text[i] == '\t')) i++;
+      const size_t s = i;
+      while (i < e && text[i] != ' ' && text[i] != '\t') i++;
+      if (i > s) {
+        a->tok_off.push_back(blob_add(a, text + s, i - s));
+        argc++;
+      }
+    }
+    if (argc > ENS_MAX_ARGC) {
+      delete a;
+      return fail(ENS_EINVAL, "ens_parse_args: more than ENS_MAX_ARGC argv entries on a line");
+    }
+    a->line_tok.push_back((uint32_t)a->tok_off.size());
+    if (!nl) break;
+    pos = end + 1;
+  }
+  if (a->blob.size() > 0xFFFFFFF0u) {
+    delete a;
+    return fail(ENS_EINVAL, "ens_parse_args: args larger than 4 GiB");
+  }
+  const size_t n = a->line_tok.size() - 1;
+  for (size_t l = 0; l < n; l++) {
+    a->hfirst.push_back((uint32_t)a->hptr.size());
+    for (uint32_t t = a->line_tok[l]; t < a->line_tok[l + 1]; t++) a->hptr.push_back(a->blob.data() + a->tok_off[t]);
+    a->hptr.push_back(nullptr);
+  }
+  *out = a;
+  return ENS_OK;
+}
+
+extern "C" int ens_load_args(const char *path, const char *argv0, ens_args **out) {
+  if (!path || !out) return fail(ENS_EINVAL, "ens_load_args: NULL argument");
+  FILE *f = std::fopen(path, "rb");
+  if (!f) return fail(ENS_ENOENT, std::string("ens_load_args: cannot open ") + path);
+  std::string s;
+  char buf[1 << 16];
+  size_t k;
+  while ((k = std::fread(buf, 1, sizeof buf, f)) > 0) s.append(buf, k);
+  std::fclose(f);
+  return ens_parse_args(s.data(), s.size(), argv0, out);
+}
+
+extern "C" int ens_args_count(const ens_args *a) {
+  if (!a) return fail(ENS_EINVAL, "ens_args_count: NULL");
+  return (int)(a->line_tok.size() - 1);
+}
+
+extern "C" int ens_args_get(const ens_args *a, int i, int *argc, const char *const **argv) {
+  if (!a || !argc || !argv) return fail(ENS_EINVAL, "ens_args_get: NULL");
+  if (i < 0 || i >= ens_args_count(a)) return fail(ENS_ERANGE, "ens_args_get: index out of range");
+  *argc = (int)(a->line_tok[i + 1] - a->line_tok[i]);
+  *argv = a->hptr.data() + a->hfirst[i];
+  return ENS_OK;
+}
+
+extern "C" void ens_args_free(ens_args *a) { delete a; }
+
+// ---------------------------------------------------------------------------
+// S2..S9: launch
+// ---------------------------------------------------------------------------
+struct Group {
+  uint32_t app = 0;
+  int T = 0, grid = 0;
+  uint32_t smem = 0;
+  uint64_t arena = 0;
+  std::vector<uint32_t> kmap;
+  size_t kmap_off = 0;
+};
+
+struct Plan {  // workspace layout (byte offsets) and groups
+  int n = 0;
+  uint32_t stdout_cap = 4096;
+  uint64_t arena_bytes = 0;
+  int slots = 0;
+  std::vector<Group> groups;
+  std::vector<uint32_t> line_of_k;
+  // staged (H2D) part
+  size_t o_blob = 0, o_tok = 0, o_line = 0, o_lok = 0, o_kmap = 0, staged = 0;
+  // zeroed part: counters (n_groups + 1 u64 stdout total), recs, pos
+  size_t o_ctr = 0, o_recs = 0, o_pos = 0, zeroed_end = 0;
+  size_t o_tal = 0, o_out = 0, o_cmp = 0, o_arena = 0, total = 0;
+};
+
+struct ens_run {
+  Plan P;
+  const ens_args *args_copy_src = nullptr;
+  char *ws = nullptr;
+  size_t ws_bytes = 0;
+  bool owns_ws = false;
+  cudaStream_t stream = nullptr;
+  char *h_stage = nullptr;
+  cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  uint32_t flags = 0;
+  bool launched = false;
+};
+
+static size_t al(size_t x) { return (x + 255) / 256 * 256; }
+
+static uint32_t app_of_argv0(const char *a0) {
+  const char *b = std::strrchr(a0, '/');
+  b = b ? b + 1 : a0;
+  if (!std::strcmp(b, "echo")) return APP_ECHO;
+  if (!std::strcmp(b, "xsbench")) return APP_XSBENCH;
+  if (!std::strcmp(b, "rsbench")) return APP_RSBENCH;
+  if (!std::strcmp(b, "amgmk")) return APP_AMGMK;
+  return APP_NOTFOUND;
+}
+
+static int threads_for(int32_t t) {
+  if (t <= 0) t = 256;
+  int T = 32;
+  while (T * 2 <= t && T < 1024) T *= 2;
+  return T;
+}
+
+// Build the plan: groups, geometry, layout.  mem_cap: bytes available for
+// the whole workspace (0 = unlimited).
+static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, size_t mem_cap, Plan &P) {
+  if (!a || !c) return fail(ENS_EINVAL, "ens_launch: NULL args or cfg");
+  if ((uint32_t)app > ENS_APP_AMGMK) return fail(ENS_EINVAL, "ens_launch: unknown app");
+  const int count = ens_args_count(a);
+  const int64_t n = c->n_instances, first = c->first, stride = c->stride <= 0 ? 1 : c->stride;
+  if (n < 0 || first < 0) return fail(ENS_EINVAL, "ens_launch: negative first / n_instances");
+  if (n > 0 && first + (n - 1) * stride >= count)
+    return fail(ENS_ERANGE, "ens_launch: instance id beyond the args file (reading Q4)");
+  if (c->grid_blocks < 0) return fail(ENS_EINVAL, "ens_launch: negative grid_blocks");
+  P.n = (int)n;
+  P.stdout_cap = c->stdout_bytes ? (c->stdout_bytes + 7u) / 8u * 8u : 4096u;
+  const int T = threads_for(c->block_threads);
+  int dev = 0, sms = 148;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceGetAttribute");
+
+  Group g_by_app[6];
+  uint64_t need_arena = 0;
+  P.line_of_k.resize((size_t)n);
+  for (int64_t k = 0; k < n; k++) {
+    const uint32_t line = (uint32_t)(first + k * stride);
+    P.line_of_k[(size_t)k] = line;
+    int argc;
+    const char *const *argv;
+    ens_args_get(a, (int)line, &argc, &argv);
+    uint32_t ap = (uint32_t)app;
+    if (app == ENS_APP_BY_ARGV0) ap = argc > 0 ? app_of_argv0(argv[0]) : (uint32_t)APP_NOTFOUND;
+    uint64_t ar = 0;
+    uint32_t sm = 0;
+    app_size(ap, argc, argv, &ar, &sm);
+    Group &g = g_by_app[ap];
+    g.app = ap;
+    g.arena = std::max(g.arena, ar);
+    g.smem = std::max(g.smem, sm);
+    g.kmap.push_back((uint32_t)k);
+    need_arena = std::max(need_arena, ar);
+  }
+  P.arena_bytes = c->arena_bytes ? al(c->arena_bytes) : al(need_arena);
+  for (uint32_t ap : {(uint32_t)APP_XSBENCH, (uint32_t)APP_RSBENCH, (uint32_t)APP_AMGMK, (uint32_t)APP_ECHO,
+                      (uint32_t)APP_NOTFOUND}) {
+    Group &g = g_by_app[ap];
+    if (g.kmap.empty()) continue;
+    g.T = T;
+    int occ = 0;
+    e = group_occupancy(ap, T, g.smem, &occ);
+    if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor");
+    if (occ <= 0) return fail(ENS_EINVAL, "ens_launch: an instance needs more shared memory than one SM has");
+    int grid = c->grid_blocks ? c->grid_blocks : occ * sms;
+    grid = std::min<int64_t>(grid, (int64_t)g.kmap.size());
+    g.grid = std::max(grid, 1);
+    P.groups.push_back(g);
+  }
+  // layout: staged part
+  size_t o = 0;
+  P.o_blob = o; o = al(o + a->blob.size());
+  P.o_tok = o; o = al(o + a->tok_off.size() * 4);
+  P.o_line = o; o = al(o + a->line_tok.size() * 4);
+  P.o_lok = o; o = al(o + (size_t)n * 4);
+  P.o_kmap = o;
+  for (Group &g : P.groups) {
+    g.kmap_off = o;
+    o += g.kmap.size() * 4;
+  }
+  o = al(o);
+  P.staged = o;
+  // zeroed part
+  P.o_ctr = o; o = al(o + (P.groups.size() + 1) * 8);
+  P.o_recs = o; o = al(o + (size_t)n * sizeof(ens_record));
+  P.o_pos = o; o = al(o + (size_t)n * 8);
+  P.zeroed_end = o;
+  P.o_tal = o; o = al(o + (size_t)n * ENS_TALLIES * 4);
+  P.o_out = o; o = al(o + (size_t)n * P.stdout_cap);
+  P.o_cmp = o; o = al(o + (size_t)n * P.stdout_cap);
+  P.o_arena = o;
+  int want = 0;
+  for (const Group &g : P.groups) want = std::max(want, g.grid);
+  if (P.arena_bytes && mem_cap) {
+    if (mem_cap <= o + P.arena_bytes) return fail(ENS_ENOMEM, "ens_launch: workspace cannot hold one arena slot");
+    const uint64_t fit = (mem_cap - o) / P.arena_bytes;
+    if ((uint64_t)want > fit) {
+      if (c->grid_blocks) return fail(ENS_ENOMEM, "ens_launch: grid_blocks x arena does not fit the workspace");
+      want = (int)fit;
+      for (Group &g : P.groups) g.grid = std::min(g.grid, want);
+    }
+  }
+  P.slots = want;
+  P.total = o + (size_t)want * P.arena_bytes;
+  return ENS_OK;
+}
+
+static size_t free_device_bytes() {
+  size_t fr = 0, tot = 0;
+  if (cudaMemGetInfo(&fr, &tot) != cudaSuccess) return 0;
+  return fr > (512u << 20) ? fr - (512u << 20) : fr / 2;  // leave headroom
+}
+
+extern "C" int ens_workspace_bytes(ens_app app, const ens_args *a, const ens_launch_cfg *c, size_t *bytes) {
+  if (!bytes) return fail(ENS_EINVAL, "ens_workspace_bytes: NULL");
+  Plan P;
+  int rc = make_plan(app, a, c, c && c->grid_blocks ? 0 : free_device_bytes(), P);
+  if (rc) return rc;
+  *bytes = P.total;
+  return ENS_OK;
+}
+
+static int enqueue(ens_run *r) {
+  const Plan &P = r->P;
+  CU(cudaMemsetAsync(r->ws + P.o_ctr, 0, P.zeroed_end - P.o_ctr, r->stream));
+  CU(cudaEventRecord(r->ev0, r->stream));
+  for (size_t gi = 0; gi < P.groups.size(); gi++) {
+    const Group &g = P.groups[gi];
+    KParams k{};
+    k.blob = r->ws + P.o_blob;
+    k.tok_off = (const uint32_t *)(r->ws + P.o_tok);
+    k.line_tok = (const uint32_t *)(r->ws + P.o_line);
+    k.kmap = (const uint32_t *)(r->ws + g.kmap_off);
+    k.line_of_k = (const uint32_t *)(r->ws + P.o_lok);
+    k.n = (uint32_t)g.kmap.size();
+    k.flags = r->flags;
+    k.counter = (uint32_t *)(r->ws + P.o_ctr + 8 * gi);
+    k.stdout_total = (unsigned long long *)(r->ws + P.o_ctr + 8 * P.groups.size());
+    k.recs = (ens_record *)(r->ws + P.o_recs);
+    k.stdout_pos = (unsigned long long *)(r->ws + P.o_pos);
+    k.tallies = (uint32_t *)(r->ws + P.o_tal);
+    k.stdout_base = r->ws + P.o_out;
+    k.stdout_cmp = r->ws + P.o_cmp;
+    k.stdout_cap = P.stdout_cap;
+    k.arena_base = r->ws + P.o_arena;
+    k.arena_bytes = P.arena_bytes;
+    cudaError_t e = launch_group(g.app, g.T, g.grid, g.smem, k, r->stream);
+    if (e != cudaSuccess) return cuda_fail(e, "ens_kernel launch");
+  }
+  CU(cudaEventRecord(r->ev1, r->stream));
+  r->launched = true;
+  return ENS_OK;
+}
+
+extern "C" int ens_launch(ens_app app, const ens_args *a, const ens_launch_cfg *c, void *d_workspace, size_t ws_bytes,
+                          void *cuda_stream, ens_run **out) {
+  if (!out) return fail(ENS_EINVAL, "ens_launch: NULL out");
+  *out = nullptr;
+  ens_run *r = new ens_run();
+  r->stream = (cudaStream_t)cuda_stream;
+  r->flags = c ? c->flags : 0;
+  const size_t cap = d_workspace ? ws_bytes : (c && c->grid_blocks ? 0 : free_device_bytes());
+  int rc = make_plan(app, a, c, cap, r->P);
+  if (rc) {
+    delete r;
+    return rc;
+  }
+  Plan &P = r->P;
+  if (d_workspace) {
+    if (ws_bytes < P.total) {
+      delete r;
+      return fail(ENS_ENOMEM, "ens_launch: ws_bytes < ens_workspace_bytes");
+    }
+    r->ws = (char *)d_workspace;
+    r->ws_bytes = ws_bytes;
+  } else if (P.n > 0) {
+    cudaError_t e = cudaMalloc(&r->ws, P.total);
+    if (e != cudaSuccess) {
+      delete r;
+      return fail(ENS_ENOMEM, std::string("ens_launch: cudaMalloc: ") + cudaGetErrorString(e));
+    }
+    r->owns_ws = true;
+    r->ws_bytes = P.total;
+  }
+  cudaError_t e = cudaEventCreate(&r->ev0);
+  if (e == cudaSuccess) e = cudaEventCreate(&r->ev1);
+  if (e != cudaSuccess) {
+    ens_run_free(r);
+    return cuda_fail(e, "cudaEventCreate");
+  }
+  *out = r;
+  if (P.n == 0) return ENS_OK;
+  // one pinned staging buffer, one H2D copy
+  e = cudaHostAlloc((void **)&r->h_stage, P.staged, cudaHostAllocDefault);
+  if (e != cudaSuccess) {
+    *out = nullptr;
+    ens_run_free(r);
+    return cuda_fail(e, "cudaHostAlloc");
+  }
+  std::memset(r->h_stage, 0, P.staged);
+  std::memcpy(r->h_stage + P.o_blob, a->blob.data(), a->blob.size());
+  std::memcpy(r->h_stage + P.o_tok, a->tok_off.data(), a->tok_off.size() * 4);
+  std::memcpy(r->h_stage + P.o_line, a->line_tok.data(), a->line_tok.size() * 4);
+  std::memcpy(r->h_stage + P.o_lok, P.line_of_k.data(), P.line_of_k.size() * 4);
+  for (const Group &g : P.groups) std::memcpy(r->h_stage + g.kmap_off, g.kmap.data(), g.kmap.size() * 4);
+  e = cudaMemcpyAsync(r->ws, r->h_stage, P.staged, cudaMemcpyHostToDevice, r->stream);
+  if (e != cudaSuccess) {
+    *out = nullptr;
+    ens_run_free(r);
+    return cuda_fail(e, "cudaMemcpyAsync H2D");
+  }
+  rc = enqueue(r);
+  if (rc) {
+    *out = nullptr;
+    ens_run_free(r);
+  }
+  return rc;
+}
+
+extern "C" int ens_run_relaunch(ens_run *r, void *cuda_stream) {
+  if (!r) return fail(ENS_EINVAL, "ens_run_relaunch: NULL");
+  if (cuda_stream) r->stream = (cudaStream_t)cuda_stream;
+  if (r->P.n == 0) return ENS_OK;
+  return enqueue(r);
+}
+
+// ---------------------------------------------------------------------------
+// S10: collect
+// ---------------------------------------------------------------------------
+extern "C" int ens_collect(ens_run *r, ens_record *recs, uint32_t *tallies, char *stdout_buf, size_t cap,
+                           uint64_t *stdout_off) {
+  if (!r) return fail(ENS_EINVAL, "ens_collect: NULL run");
+  const Plan &P = r->P;
+  const int n = P.n;
+  if (n == 0) {
+    if (stdout_off) stdout_off[0] = 0;
+    return ENS_OK;
+  }
+  CU(cudaStreamSynchronize(r->stream));
+  CU(cudaGetLastError());
+  // counters | records | stdout positions: one copy
+  std::vector<char> zb(P.zeroed_end - P.o_ctr);
+  CU(cudaMemcpy(zb.data(), r->ws + P.o_ctr, zb.size(), cudaMemcpyDeviceToHost));
+  const uint64_t total = *(const uint64_t *)(zb.data() + 8 * P.groups.size());
+  std::vector<ens_record> R((size_t)n);
+  std::memcpy(R.data(), zb.data() + (P.o_recs - P.o_ctr), (size_t)n * sizeof(ens_record));
+  const uint64_t *pos = (const uint64_t *)(zb.data() + (P.o_pos - P.o_ctr));
+  if (tallies) CU(cudaMemcpy(tallies, r->ws + P.o_tal, (size_t)n * ENS_TALLIES * 4, cudaMemcpyDeviceToHost));
+  std::vector<uint64_t> cmp((size_t)(total + 7) / 8 + 1);
+  if (total) CU(cudaMemcpy(cmp.data(), r->ws + P.o_cmp, (size_t)total, cudaMemcpyDeviceToHost));
+  std::string text;
+  std::vector<uint64_t> off((size_t)n + 1, 0);
+  int bad = 0;
+  for (int k = 0; k < n; k++) {
+    ens_record &x = R[(size_t)k];
+    if (!(x.flags & ENS_RF_DONE)) {  // never completed
+      std::memset(&x, 0, sizeof x);
+      x.instance = P.line_of_k[(size_t)k];
+      x.flags = ENS_RF_NOT_RUN;
+    } else if (x.stdout_len) {
+      const size_t before = text.size();
+      if (pos[k] + x.stdout_len > total || format_raw((const char *)cmp.data() + pos[k], x.stdout_len, text) < 0) {
+        bad++;
+        text.resize(before);
+      }
+      x.stdout_len = (uint32_t)(text.size() - before);
+    }
+    off[(size_t)k + 1] = text.size();
+  }
+  if (recs) std::memcpy(recs, R.data(), R.size() * sizeof(ens_record));
+  if (stdout_off) std::memcpy(stdout_off, off.data(), off.size() * 8);
+  if (bad) return fail(ENS_ECUDA, "ens_collect: malformed device stdout records");
+  if (stdout_buf) {
+    if (cap < text.size()) return fail(ENS_ERANGE, "ens_collect: stdout buffer too small");
+    std::memcpy(stdout_buf, text.data(), text.size());
+  }
+  return ENS_OK;
+}
+
+extern "C" int ens_run_elapsed_ms(ens_run *r, float *ms) {
+  if (!r || !ms) return fail(ENS_EINVAL, "ens_run_elapsed_ms: NULL");
+  if (!r->launched) {
+    *ms = 0.f;
+    return ENS_OK;
+  }
+  cudaError_t e = cudaEventQuery(r->ev1);
+  if (e == cudaErrorNotReady) return fail(ENS_EBUSY, "ens_run_elapsed_ms: not finished");
+  CU(cudaEventElapsedTime(ms, r->ev0, r->ev1));
+  return ENS_OK;
+}
+
+extern "C" int ens_run_get_info(const ens_run *r, ens_run_info *info) {
+  if (!r || !info) return fail(ENS_EINVAL, "ens_run_get_info: NULL");
+  std::memset(info, 0, sizeof *info);
+  const Plan &P = r->P;
+  info->n_instances = P.n;
+  info->n_groups = (int32_t)P.groups.size();
+  for (const Group &g : P.groups) {
+    const uint32_t ap = g.app == APP_NOTFOUND ? 0u : g.app;
+    info->grid_blocks[ap] = g.grid;
+    info->block_threads[ap] = g.T;
+  }
+  info->kernel_launches = (int32_t)P.groups.size();
+  info->arena_bytes = P.arena_bytes;
+  info->ws_bytes = r->ws_bytes;
+  info->records_offset = P.o_recs;
+  info->tallies_offset = P.o_tal;
+  info->stdout_offset = P.o_out;
+  info->stdout_bytes = P.stdout_cap;
+  info->h2d_bytes = P.n ? P.staged : 0;
+  return ENS_OK;
+}
+
+extern "C" long ens_format_stdout(uint32_t app, const void *raw, size_t raw_len, char *out, size_t cap) {
+  (void)app;
+  std::string s;
+  long k = format_raw(raw, raw_len, s);
+  if (k < 0) return fail(ENS_EINVAL, "ens_format_stdout: malformed records");
+  if (out) std::memcpy(out, s.data(), std::min(cap, s.size()));
+  return (long)s.size();
+}
+
+extern "C" void ens_run_free(ens_run *r) {
+  if (!r) return;
+  if (r->launched) cudaStreamSynchronize(r->stream);
+  if (r->owns_ws && r->ws) cudaFree(r->ws);
+  if (r->h_stage) cudaFreeHost(r->h_stage);
+  if (r->ev0) cudaEventDestroy(r->ev0);
+  if (r->ev1) cudaEventDestroy(r->ev1);
+  delete r;
+}
+
+extern "C" const char *ens_strerror(int err) {
+  switch (err) {
+    case ENS_OK: return "ok";
+    case ENS_EINVAL: return "invalid argument";
+    case ENS_ENOENT: return "args file not found";
+    case ENS_ENOMEM: return "out of memory";
+    case ENS_ECUDA: return "CUDA error";
+    case ENS_ERANGE: return "out of range";
+    case ENS_EBUSY: return "busy";
+    case ENS_EPARSE: return "parse error";
+  }
+  return "unknown error";
+}
+
+extern "C" const char *ens_last_error(void) { return g_err.c_str(); }
+extern "C" const char *ens_version(void) { return "ens 0.1.0 (sm_100a)"; }

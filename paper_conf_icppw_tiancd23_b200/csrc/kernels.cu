@@ -1,0 +1,161 @@
+// csrc/kernels.cu — N2, the ensemble scheduler kernel, and its instances.
+//
+// The paper maps NI instances onto N teams with `target teams distribute
+// num_teams(N) thread_limit(T)` (Fig. 4), one team = one CUDA
+// thread block (§2.3), with N = NI in its evaluation.
+// Here the grid is persistent: min(NI, occupancy x 148) blocks pull instance
+// slots from an atomic counter (reading Q5), so NI may exceed the blocks that
+// fit at once, and each block's heap arena is a fixed slot of the workspace
+// (memory = resident blocks x arena, not NI x arena).
+#include <cuda_runtime.h>
+
+#include "apps/amgmk.cuh"
+#include "apps/echo.cuh"
+#include "apps/rsbench.cuh"
+#include "apps/xsbench.cuh"
+#include "kparams.h"
+
+namespace ens {
+
+__device__ __forceinline__ uint64_t globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+__device__ __forceinline__ uint32_t smid() {
+  uint32_t s;
+  asm volatile("mov.u32 %0, %%smid;" : "=r"(s));
+  return s;
+}
+
+template <class App, int T>
+__global__ void __launch_bounds__(T, (1024 / T) > 0 ? (1024 / T) : 1) ens_kernel(const KParams p) {
+  extern __shared__ __align__(16) char dsmem[];
+  __shared__ char *s_argv[ENS_MAX_ARGC + 1];
+  __shared__ uint32_t s_j;
+  __shared__ unsigned long long s_pos;
+  __shared__ Shared sh;
+  const int tid = threadIdx.x;
+  char *const arena = p.arena_base + (size_t)blockIdx.x * p.arena_bytes;
+  for (;;) {
+    if (tid == 0) s_j = atomicAdd(p.counter, 1u);
+    __syncthreads();
+    const uint32_t j = s_j;
+    if (j >= p.n) break;  // block-uniform
+    const uint32_t k = p.kmap[j];
+    const uint32_t line = p.line_of_k[k];
+    const uint32_t t0 = p.line_tok[line];
+    const int argc = (int)(p.line_tok[line + 1] - t0);
+    for (int i = tid; i < argc; i += T) s_argv[i] = const_cast<char *>(p.blob) + p.tok_off[t0 + i];
+    if (tid == 0) s_argv[argc] = nullptr;
+    if (tid < 32) sh.tallies[tid] = 0;
+    if (tid == 0) {
+      sh.out_len = 0;
+      sh.flags = 0;
+    }
+    uint64_t t_start = 0;
+    if ((p.flags & ENS_F_TIMESTAMPS) && tid == 0) t_start = globaltimer();
+    __syncthreads();
+
+    Ctx c;
+    c.k = k;
+    c.id = line;
+    c.arena = arena;
+    c.arena_cap = p.arena_bytes;
+    c.out = p.stdout_base + (size_t)k * p.stdout_cap;
+    c.out_cap = p.stdout_cap;
+    c.sh = &sh;
+    c.smem = dsmem;
+    const Result r = App::run(c, argc, s_argv);
+    __syncthreads();
+
+    if (tid < ENS_TALLIES) p.tallies[(size_t)k * ENS_TALLIES + tid] = sh.tallies[tid];
+    if (tid == 0) {
+      ens_record rec;
+      rec.instance = line;
+      rec.exit_code = r.exit_code;
+      rec.app = App::kId == APP_NOTFOUND ? 0u : App::kId;
+      rec.flags = sh.flags | ENS_RF_DONE;
+      rec.vhash = r.vhash;
+      rec.bitsum = r.bitsum;
+      rec.fsum = r.fsum;
+      rec.fabs = r.fabs;
+      rec.work = r.work;
+      rec.stdout_len = sh.out_len;
+      rec.smid = (p.flags & ENS_F_TIMESTAMPS) ? smid() : 0u;
+      rec.t_start_ns = t_start;
+      rec.t_end_ns = (p.flags & ENS_F_TIMESTAMPS) ? globaltimer() : 0ull;
+      p.recs[k] = rec;
+      s_pos = atomicAdd(p.stdout_total, (unsigned long long)sh.out_len);
+      p.stdout_pos[k] = s_pos;
+    }
+    __syncthreads();
+    {  // compact this instance's stdout (whole 8-B words)
+      const unsigned long long *src = reinterpret_cast<const unsigned long long *>(c.out);
+      unsigned long long *dst = reinterpret_cast<unsigned long long *>(p.stdout_cmp + s_pos);
+      for (uint32_t w = tid; w < sh.out_len / 8; w += T) dst[w] = src[w];
+    }
+    __syncthreads();  // s_j, s_pos, s_argv, sh reused by the next instance
+  }
+}
+
+template <class App>
+static const void *kernel_for(int T) {
+  switch (T) {
+    case 32: return (const void *)ens_kernel<App, 32>;
+    case 64: return (const void *)ens_kernel<App, 64>;
+    case 128: return (const void *)ens_kernel<App, 128>;
+    case 256: return (const void *)ens_kernel<App, 256>;
+    case 512: return (const void *)ens_kernel<App, 512>;
+    case 1024: return (const void *)ens_kernel<App, 1024>;
+  }
+  return nullptr;
+}
+
+const void *kernel_ptr(uint32_t app, int T) {
+  switch (app) {
+    case APP_ECHO: return kernel_for<EchoApp>(T);
+    case APP_XSBENCH: return kernel_for<XsApp>(T);
+    case APP_RSBENCH: return kernel_for<RsApp>(T);
+    case APP_AMGMK: return kernel_for<AmgApp>(T);
+    case APP_NOTFOUND: return kernel_for<NotFoundApp>(T);
+  }
+  return nullptr;
+}
+
+// host-side sizing from the same parse/layout code the instance runs
+bool app_size(uint32_t app, int argc, const char *const *argv, uint64_t *arena, uint32_t *smem) {
+  switch (app) {
+    case APP_ECHO: return EchoApp::size(argc, argv, arena, smem);
+    case APP_XSBENCH: return XsApp::size(argc, argv, arena, smem);
+    case APP_RSBENCH: return RsApp::size(argc, argv, arena, smem);
+    case APP_AMGMK: return AmgApp::size(argc, argv, arena, smem);
+    case APP_NOTFOUND: return NotFoundApp::size(argc, argv, arena, smem);
+  }
+  *arena = 0;
+  *smem = 0;
+  return false;
+}
+
+cudaError_t launch_group(uint32_t app, int T, int grid, size_t smem, const KParams &p, cudaStream_t st) {
+  const void *fn = kernel_ptr(app, T);
+  if (!fn) return cudaErrorInvalidValue;
+  if (smem > 48 * 1024) {
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+  }
+  void *args[] = {const_cast<KParams *>(&p)};
+  return cudaLaunchKernel(fn, dim3(grid), dim3(T), args, smem, st);
+}
+
+cudaError_t group_occupancy(uint32_t app, int T, size_t smem, int *blocks_per_sm) {
+  const void *fn = kernel_ptr(app, T);
+  if (!fn) return cudaErrorInvalidValue;
+  if (smem > 48 * 1024) {
+    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+  }
+  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, fn, T, smem);
+}
+
+}  // namespace ens

@@ -1,0 +1,36 @@
+// csrc/kparams.h — kernel parameters of one app group launch and the
+// host <-> kernel-file interface (internal to libens).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+#include "../../include/ens.h"
+
+namespace ens {
+
+struct KParams {
+  const char *blob;           // NUL-terminated tokens (argv0 once + all lines)
+  const uint32_t *tok_off;    // byte offset of each argv entry in blob
+  const uint32_t *line_tok;   // [n_lines+1] first argv entry of each line
+  const uint32_t *kmap;       // [n] group-local index -> record slot k
+  const uint32_t *line_of_k;  // [n_instances] record slot -> line
+  uint32_t n;                 // instances in this group
+  uint32_t flags;             // ENS_F_*
+  uint32_t *counter;          // scheduler counter (zeroed before launch)
+  unsigned long long *stdout_total;  // compacted stdout bytes (zeroed)
+  ens_record *recs;           // [n_instances]
+  unsigned long long *stdout_pos;    // [n_instances] offset in stdout_cmp
+  uint32_t *tallies;          // [n_instances][ENS_TALLIES]
+  char *stdout_base;          // [n_instances][stdout_cap] raw, per instance
+  char *stdout_cmp;           // compacted raw stdout (for a small D2H)
+  uint32_t stdout_cap;
+  char *arena_base;           // [grid][arena_bytes]
+  uint64_t arena_bytes;
+};
+
+const void *kernel_ptr(uint32_t app, int T);
+bool app_size(uint32_t app, int argc, const char *const *argv, uint64_t *arena, uint32_t *smem);
+cudaError_t launch_group(uint32_t app, int T, int grid, size_t smem, const KParams &p, cudaStream_t st);
+cudaError_t group_occupancy(uint32_t app, int T, size_t smem, int *blocks_per_sm);
+
+}  // namespace ens

@@ -1,0 +1,226 @@
+// csrc/rt/device_rt.cuh — N0, the per-instance device runtime.
+//
+// Everything an instance owns (§3.3: instances must not share
+// mutable globals) lives in its Ctx: its argv (shared memory), its heap
+// arena (a slot of the workspace, bump-allocated through a host-computed
+// layout), its stdout buffer, its tallies and its exit code.  No mutable
+// __device__ globals exist anywhere in the instance bodies.
+#pragma once
+#include <cstdint>
+
+#include "fmt_ids.h"
+#include "../../../include/ens.h"
+
+namespace ens {
+
+#define ENS_HD __host__ __device__ __forceinline__
+
+// ---------------------------------------------------------------------------
+// LCG (SURVEY.md §8(c) "Shared primitives"): s <- (a*s + 1) mod 2^63, held
+// as an affine map so that n steps are one multiply-add (jump constants).
+// ---------------------------------------------------------------------------
+constexpr uint64_t kLcgA = 2806196910506780709ULL;
+constexpr uint64_t kMask63 = 0x7FFFFFFFFFFFFFFFULL;
+
+struct Affine {
+  uint64_t a, c;  // s -> a*s + c  (mod 2^64; reduced mod 2^63 on apply)
+  ENS_HD uint64_t operator()(uint64_t s) const { return (a * s + c) & kMask63; }
+  // this ∘ then: apply `first` then this
+  ENS_HD Affine after(const Affine &first) const { return {a * first.a, a * first.c + c}; }
+};
+
+// the map of n LCG steps, by repeated squaring
+ENS_HD Affine lcg_pow(uint64_t n) {
+  Affine r{1ULL, 0ULL};
+  Affine b{kLcgA, 1ULL};
+  n &= kMask63;
+  while (n) {
+    if (n & 1ULL) r = b.after(r);
+    b = b.after(b);
+    n >>= 1;
+  }
+  return r;
+}
+
+ENS_HD uint64_t lcg_next(uint64_t s) { return (kLcgA * s + 1ULL) & kMask63; }
+
+// advance, then scale by 2^-63 (exact: the conversion rounds, the scale is a
+// power of two)
+__device__ __forceinline__ double lcg_double(uint64_t &s) {
+  s = lcg_next(s);
+  return __ull2double_rn(s) * 0x1p-63;
+}
+__device__ __forceinline__ uint64_t lcg_int(uint64_t &s) {
+  s = lcg_next(s);
+  return s;
+}
+
+// ---------------------------------------------------------------------------
+// strings / integer flags (reading R-int: optional sign, 1..18 digits)
+// ---------------------------------------------------------------------------
+ENS_HD bool str_eq(const char *a, const char *b) {
+  while (*a && *a == *b) {
+    a++;
+    b++;
+  }
+  return *a == *b;
+}
+ENS_HD uint32_t str_len(const char *a) {
+  uint32_t n = 0;
+  while (a[n]) n++;
+  return n;
+}
+ENS_HD bool parse_i64(const char *s, long long *v) {
+  bool neg = false;
+  if (*s == '+' || *s == '-') {
+    neg = *s == '-';
+    s++;
+  }
+  long long x = 0;
+  int nd = 0;
+  for (; *s; s++, nd++) {
+    if (*s < '0' || *s > '9' || nd >= 18) return false;
+    x = x * 10 + (*s - '0');
+  }
+  if (nd == 0) return false;
+  *v = neg ? -x : x;
+  return true;
+}
+
+ENS_HD uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
+
+// ---------------------------------------------------------------------------
+// per-instance context (identical copy in every thread of the block)
+// ---------------------------------------------------------------------------
+struct Shared {             // static shared memory of the scheduler
+  uint32_t tallies[32];     // per-instance tallies (smem atomics)
+  uint32_t out_len;         // stdout bytes used (thread 0 only)
+  uint32_t flags;           // record flags (thread 0 only)
+  unsigned long long red_u[32];  // block reduction scratch
+  double red_d[32];
+};
+
+struct Result {  // meaningful in thread 0 after the body returns
+  int exit_code;
+  uint64_t vhash, bitsum;
+  double fsum, fabs;
+  uint64_t work;
+};
+
+struct Ctx {
+  uint32_t k, id;      // record slot, instance id (line)
+  char *arena;         // this block's slot
+  uint64_t arena_cap;
+  char *out;           // this instance's raw stdout buffer
+  uint32_t out_cap;
+  Shared *sh;
+  char *smem;          // dynamic shared memory of the app
+};
+
+// ---- stdout: {u32 fmt, u32 payload bytes, 8-B slots}; strings = len slot +
+// bytes padded to 8.  Called by thread 0 only.
+struct OutArg {
+  int kind;  // 0 int64, 1 uint64, 2 double, 3 string
+  union {
+    long long i;
+    unsigned long long u;
+    double d;
+    const char *s;
+  };
+};
+__device__ __forceinline__ OutArg oa(int v) { OutArg a; a.kind = 0; a.i = v; return a; }
+__device__ __forceinline__ OutArg oa(long long v) { OutArg a; a.kind = 0; a.i = v; return a; }
+__device__ __forceinline__ OutArg oa(unsigned long long v) { OutArg a; a.kind = 1; a.u = v; return a; }
+__device__ __forceinline__ OutArg oa(double v) { OutArg a; a.kind = 2; a.d = v; return a; }
+__device__ __forceinline__ OutArg oa(const char *v) { OutArg a; a.kind = 3; a.s = v; return a; }
+
+__device__ inline void out_write(Ctx &c, unsigned fmt, const OutArg *args, int n) {
+  uint32_t payload = 0;
+  for (int i = 0; i < n; i++) payload += args[i].kind == 3 ? 8u + (uint32_t)align_up(str_len(args[i].s), 8) : 8u;
+  uint32_t need = 8u + payload;
+  uint32_t len = c.sh->out_len;
+  if (len + need > c.out_cap) {
+    c.sh->flags |= 1u;  // ENS_RF_STDOUT_TRUNC
+    return;
+  }
+  unsigned long long *w = reinterpret_cast<unsigned long long *>(c.out + len);
+  *w++ = (unsigned long long)fmt | ((unsigned long long)payload << 32);
+  for (int i = 0; i < n; i++) {
+    if (args[i].kind == 3) {
+      uint32_t L = str_len(args[i].s);
+      *w++ = L;
+      for (uint32_t b = 0; b < L; b += 8) {
+        unsigned long long v = 0;
+        for (uint32_t q = 0; q < 8 && b + q < L; q++) v |= (unsigned long long)(unsigned char)args[i].s[b + q] << (8 * q);
+        *w++ = v;
+      }
+    } else {
+      *w++ = args[i].u;
+    }
+  }
+  c.sh->out_len = len + need;
+}
+
+template <class... A>
+__device__ __forceinline__ void ens_printf(Ctx &c, unsigned fmt, A... a) {
+  if (threadIdx.x != 0) return;
+  OutArg args[sizeof...(A) > 0 ? sizeof...(A) : 1] = {oa(a)...};
+  out_write(c, fmt, args, (int)sizeof...(A));
+}
+
+// ---------------------------------------------------------------------------
+// block reductions (result valid in every thread)
+// ---------------------------------------------------------------------------
+__device__ __forceinline__ unsigned long long warp_sum_u64(unsigned long long v) {
+  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+__device__ __forceinline__ double warp_sum_f64(double v) {
+  for (int o = 16; o; o >>= 1) v += __shfl_xor_sync(0xffffffffu, v, o);
+  return v;
+}
+__device__ __forceinline__ double warp_max_f64(double v) {  // NaN never wins
+  for (int o = 16; o; o >>= 1) {
+    double w = __shfl_xor_sync(0xffffffffu, v, o);
+    v = (w > v) ? w : v;
+  }
+  return v;
+}
+
+__device__ inline unsigned long long block_sum_u64(Shared *sh, unsigned long long v) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  v = warp_sum_u64(v);
+  __syncthreads();
+  if (lane == 0) sh->red_u[w] = v;
+  __syncthreads();
+  v = lane < nw ? sh->red_u[lane] : 0ULL;
+  return warp_sum_u64(v);
+}
+__device__ inline double block_sum_f64(Shared *sh, double v) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  v = warp_sum_f64(v);
+  __syncthreads();
+  if (lane == 0) sh->red_d[w] = v;
+  __syncthreads();
+  v = lane < nw ? sh->red_d[lane] : 0.0;
+  return warp_sum_f64(v);
+}
+__device__ inline double block_max_f64(Shared *sh, double v) {
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+  v = warp_max_f64(v);
+  __syncthreads();
+  if (lane == 0) sh->red_d[w] = v;
+  __syncthreads();
+  v = lane < nw ? sh->red_d[lane] : v;
+  return warp_max_f64(v);
+}
+
+// Arena data is written and re-read inside the same persistent launch (and a
+// slot is reused by the block's next instance), so it must NOT go through the
+// non-coherent read-only path (ld.global.nc / __ldg): plain coherent loads.
+template <class T>
+__device__ __forceinline__ T ld_(const T *p) { return *p; }
+
+__device__ __forceinline__ uint64_t dbits(double d) { return (uint64_t)__double_as_longlong(d); }
+
+}  // namespace ens

@@ -1,0 +1,109 @@
+"""GPU ensemble semantics and fault paths (Fig. 4; §3.2).
+
+Invariants: instance i inside an ensemble == a solo launch of line i; N
+copies of one line give N identical records; permuting the lines permutes
+the records; sharded launches (first, stride) reproduce the full launch.
+Faults: bad flags -> exit 1 + usage text; arena too small -> exit 12 +
+NOMEM; stdout buffer too small -> STDOUT_TRUNC; n = 0; ids beyond the file.
+"""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+from parity import assert_parity  # noqa: E402
+
+LINES = [
+    "xsbench -s small -g 64 -l 900 -r 1",
+    "rsbench -s small -l 300 -p 30 -w 6 -r 2",
+    "amgmk -x 6 -y 5 -z 4 -i 3 -r 9",
+    "echo hello world",
+    "xsbench -s small -g 40 -l 300 -G hash -h 30 -r 3",
+    "xsbench -g 1",
+    "nosuchapp -x",
+]
+FIELDS = ["instance", "exit_code", "app", "flags", "vhash", "bitsum", "fsum", "fabs", "work", "stdout_len"]
+
+
+def ens():
+    from paper_conf_icppw_tiancd23_b200 import ensemble
+    return ensemble
+
+
+def text(lines):
+    return "".join(l + "\n" for l in lines)
+
+
+def test_fig5_loader_on_device(oracle):
+    """Fig. 5: 4 lines, -n 4 -t 128, argv[0] of the loader first."""
+    import os
+    t = open(os.path.join(os.path.dirname(__file__), "golden", "fig5_arguments.txt")).read()
+    g = ens().run_text(t, app="echo", argv0="./user_app_gpu", threads=128)
+    o = oracle.run_text(t, app=oracle.APP_ECHO, argv0="./user_app_gpu")
+    assert_parity(g, o)
+    assert list(g.records["exit_code"]) == [6, 6, 6, 6]
+
+
+def test_solo_equals_ensemble():
+    full = ens().run_text(text(LINES))
+    for i, l in enumerate(LINES):
+        solo = ens().run_text(text([l]))
+        for f in FIELDS[1:]:
+            assert solo.records[0][f] == full.records[i][f], (i, f)
+        assert solo.stdout[0] == full.stdout[i]
+        assert np.array_equal(solo.tallies[0], full.tallies[i])
+
+
+def test_copies_and_permutation():
+    r = ens().run_text(text([LINES[0]] * 37))
+    for f in FIELDS[1:]:
+        assert np.all(r.records[f] == r.records[f][0])
+    perm = [3, 0, 6, 2, 5, 1, 4]
+    a = ens().run_text(text(LINES))
+    b = ens().run_text(text([LINES[p] for p in perm]))
+    for j, p in enumerate(perm):
+        for f in FIELDS[1:]:
+            assert a.records[p][f] == b.records[j][f]
+
+
+def test_sharded_launches_match_full():
+    from paper_conf_icppw_tiancd23_b200 import Args
+    full = ens().run_text(text(LINES))
+    G = 3
+    for rank in range(G):
+        e = ens().Ensemble(Args.parse(text(LINES)), app="auto", first=rank, stride=G).launch()
+        r = e.collect()
+        for k in range(e.n):
+            i = rank + k * G
+            for f in FIELDS:
+                assert r.records[k][f] == full.records[i][f]
+            assert r.stdout[k] == full.stdout[i]
+        e.close()
+
+
+def test_arena_too_small_is_nomem():
+    r = ens().run_text(text(["xsbench -s small -g 100 -l 10", "echo x"]), arena_bytes=4096)
+    assert r.records[0]["exit_code"] == 12 and r.records[0]["flags"] & 2
+    assert r.records[1]["exit_code"] == 2
+
+
+def test_stdout_truncation_flag():
+    r = ens().run_text(text(["echo " + " ".join(["abcdefgh"] * 20)]), stdout_bytes=64)
+    assert r.records[0]["flags"] & 1
+    assert r.records[0]["exit_code"] == 21
+    assert r.stdout[0].startswith(b"argc=21\n")
+
+
+def test_empty_and_range():
+    from paper_conf_icppw_tiancd23_b200 import Args, EnsError
+    r = ens().run_text("", app="echo")
+    assert len(r.records) == 0
+    with pytest.raises(EnsError):
+        ens().Ensemble(Args.parse("a\nb\n"), app="echo", n=3).launch()
+
+
+def test_timestamps_and_smid():
+    r = ens().run_text(text([LINES[0]] * 300), timestamps=True)
+    assert np.all(r.records["t_end_ns"] >= r.records["t_start_ns"])
+    assert np.all(r.records["t_start_ns"] > 0)
+    assert len(set(r.records["smid"].tolist())) > 16

@@ -1,0 +1,104 @@
+"""GPU parity: the CUDA path (libens.so through its C ABI) vs the oracle.
+
+Small and ragged cases compare every instance element by element; the
+full-size configurations compare a sample of instances the oracle can run in
+seconds (tests/test_gpu_fullsize.py).
+"""
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+from parity import assert_parity  # noqa: E402
+
+XS_CASES = [
+    # n_gp ragged vs the pow2 sort (37 -> 64), several tiles, one below T
+    "xsbench -s small -g 37 -l 1000 -G unionized -r 3",
+    "xsbench -s small -g 37 -l 1000 -G nuclide -r 3",
+    "xsbench -s small -g 37 -l 1000 -G hash -h 7 -r 3",
+    "xsbench -s small -g 1000 -l 10000 -m event -G unionized -r 1070",
+    "xsbench -s small -g 1500 -l 3000 -G hash -h 1000 -r 11 -R 5",
+    "xsbench -s small -g 2 -l 500 -G unionized -r 2",
+    "xsbench -s small -g 2 -l 500 -G hash -h 1 -r 2",
+    "xsbench -s small -g 300 -l 0 -r 2",
+    "xsbench -s small -g 300 -l 5 -G hash -h 3 -r 9",
+    "xsbench -s large -g 40 -l 2000 -G unionized -r 5",
+    "xsbench -s large -g 200 -l 2000 -G hash -h 500 -r 6",
+    "xsbench -s small -g 16384 -l 2000 -G hash -h 100 -r 4",
+]
+
+RS_CASES = [
+    "rsbench -s small -l 2000 -p 100 -w 10 -r 1",
+    "rsbench -s small -l 2000 -p 100 -w 10 -d -r 2",
+    "rsbench -s small -l 500 -p 5 -w 9 -r 3",
+    "rsbench -s large -l 300 -p 50 -w 7 -r 4 -R 8",
+    "rsbench -s small -l 0 -p 20 -w 3",
+]
+
+AMG_CASES = [
+    "amgmk -x 1 -y 1 -z 1 -i 3 -r 1",
+    "amgmk -x 5 -y 3 -z 7 -i 4 -r 2",
+    "amgmk -x 33 -y 2 -z 3 -i 6 -k matvec -r 3",
+    "amgmk -x 9 -y 9 -z 9 -i 5 -k both -r 4",
+    "amgmk -x 16 -y 16 -z 16 -i 20 -k relax -r 0",
+    "amgmk -x 32 -y 32 -z 32 -i 3 -k relax -r 7",
+]
+
+MISC_CASES = [
+    "echo",
+    "echo a b  c",
+    "nosuchapp -x 1",
+    "xsbench -g 1",
+    "xsbench -s tiny",
+    "xsbench -l",
+    "rsbench -q",
+    "amgmk -k jacobi",
+    "amgmk -x 2000",
+]
+
+
+def run_both(oracle, lines, threads=256, grid=0, **kw):
+    from paper_conf_icppw_tiancd23_b200.ensemble import run_text
+    text = "".join(l + "\n" for l in lines)
+    g = run_text(text, app="auto", threads=threads, grid=grid, **kw)
+    o = oracle.run_text(text)
+    return g, o
+
+
+@pytest.mark.parametrize("line", XS_CASES)
+def test_xs_parity(oracle, line):
+    g, o = run_both(oracle, [line])
+    assert_parity(g, o)
+
+
+@pytest.mark.parametrize("line", RS_CASES)
+def test_rs_parity(oracle, line):
+    g, o = run_both(oracle, [line])
+    assert_parity(g, o)
+
+
+@pytest.mark.parametrize("line", AMG_CASES)
+def test_amg_parity(oracle, line):
+    g, o = run_both(oracle, [line])
+    assert_parity(g, o)
+
+
+def test_misc_parity(oracle):
+    g, o = run_both(oracle, MISC_CASES)
+    assert_parity(g, o)
+
+
+@pytest.mark.parametrize("threads", [32, 64, 128, 512, 1024, 100, 5000])
+def test_thread_limit_independence(oracle, threads):
+    """-t is an upper bound and results never depend on it (reading Q6)."""
+    lines = [XS_CASES[0], XS_CASES[2], RS_CASES[0], AMG_CASES[1], AMG_CASES[2], "echo t"]
+    g, o = run_both(oracle, lines, threads=threads)
+    assert_parity(g, o)
+
+
+@pytest.mark.parametrize("grid", [1, 2, 3])
+def test_more_instances_than_blocks(oracle, grid):
+    """Persistent blocks pull ids from the counter; a slot arena is reused (reading Q5)."""
+    lines = [f"xsbench -s small -g {50 + 7 * i} -l 700 -G {['unionized', 'nuclide', 'hash'][i % 3]} -h 13 -r {i}"
+             for i in range(9)]
+    g, o = run_both(oracle, lines, grid=grid)
+    assert_parity(g, o)
