@@ -1,0 +1,422 @@
+#!/usr/bin/env python
+"""bench.py — ensemble execution on B200: instances/s, lookups/s, HBM roofline.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
+                    [--workload C2|TSTAR|C1|C3|C4|C5] [--no-extras]
+
+One step = one pass of the whole hot path over one
+batch: every instance of the workload launched as ONE persistent ensemble
+kernel per app (device-resident args: ens_run_relaunch), plus, for N > 1,
+the NCCL all-gather of the per-instance records.  The default workload is
+BASELINE.json configs[1] (C2: 64 XSBench-style large instances per GPU, the
+paper's 64-instance point); weak scaling: every rank runs 64 instances of a
+64*N-line args file sharded by instance id (i mod N).
+
+`e2e` times the same through the public C ABI from HOST buffers each step:
+ens_launch (pinned H2D of the args) + ens_collect (D2H of records, tallies,
+stdout).  `--impl reference` times the CPU oracle (test infrastructure, the
+one other place this script runs it) on the box's host cores.
+Timing: W warm-up steps, then K steps bracketed by barrier +
+cuda.synchronize, CUDA events on the launching stream, max over ranks.
+"""
+import argparse
+import json
+import os
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "instances/sec and lookups/sec per ensemble launch at 1/2/4/8 B200; HBM GB/s vs peak"
+FALLBACK_HBM_GBS = 6650.0
+
+# algorithmic bytes.  XS lookup: 16-B bracket + per nuclide
+# a 4-B index entry and the 96-B bracketing record pair.
+XS_NUM_NUCS = {68: [34, 5, 4, 4, 27, 21, 21, 21, 21, 21, 9, 9], 355: [321, 5, 4, 4, 27, 21, 21, 21, 21, 21, 9, 9]}
+
+
+def parse_xs_line(line):
+    t = line.split()
+    p = {"n_iso": 355, "n_gp": 11303, "L": 17000000, "grid": "unionized", "bins": 10000}
+    for i in range(1, len(t) - 1, 2):
+        f, v = t[i], t[i + 1]
+        if f == "-s":
+            p["n_iso"] = 68 if v == "small" else 355
+        elif f == "-g":
+            p["n_gp"] = int(v)
+        elif f == "-l":
+            p["L"] = int(v)
+        elif f == "-G":
+            p["grid"] = v
+        elif f == "-h":
+            p["bins"] = int(v)
+    return p
+
+
+def xs_init_bytes(p):
+    """Per-instance init: 48 n_u grid (+ unionized 8 n_u union + 8 n_u merge + 4 n_u n_iso index,
+    or hash 4 n_iso bins) — the bytes the method must write."""
+    n_u = p["n_iso"] * p["n_gp"]
+    b = 48 * n_u
+    if p["grid"] == "unionized":
+        b += 8 * n_u + 8 * n_u + 4 * n_u * p["n_iso"]
+    elif p["grid"] == "hash":
+        b += 4 * p["n_iso"] * p["bins"]
+    return b
+
+
+def xs_lookup_bytes(n_iso, mat_counts):
+    nn = XS_NUM_NUCS[n_iso]
+    return sum(int(c) * (16 + 100 * nn[m]) for m, c in enumerate(mat_counts))
+
+
+def algorithmic_bytes(lines, recs, tallies):
+    """Exact algorithmic bytes of one launch: per-instance init + per-lookup bytes from the
+    per-instance material tallies (XS).  Other apps: SURVEY.md §8(d) per-unit figures."""
+    total = 0
+    for k, line in enumerate(lines):
+        app = line.split()[0]
+        if app == "xsbench" and recs[k]["exit_code"] == 0:
+            p = parse_xs_line(line)
+            total += xs_init_bytes(p) + xs_lookup_bytes(p["n_iso"], tallies[k][5:17])
+        elif app == "amgmk" and recs[k]["exit_code"] == 0:
+            t = line.split()
+            d = {t[i]: t[i + 1] for i in range(1, len(t) - 1, 2)}
+            nx, ny, nz = int(d.get("-x", 50)), int(d.get("-y", 50)), int(d.get("-z", 50))
+            it = int(d.get("-i", 100))
+            n = nx * ny * nz
+            nnz = 7 * n - 2 * (nx * ny + ny * nz + nx * nz)
+            total += it * (12 * nnz + 4 * (n + 1) + 24 * n) + 12 * nnz + 32 * n
+    return total
+
+
+def measured_peak_hbm():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured"
+    except Exception:
+        return FALLBACK_HBM_GBS, "fallback"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons during the timed region."""
+    Q = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+         "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", "-i", str(self.index), f"--query-gpu={self.Q}",
+                                          "--format=csv,noheader,nounits", "-lms", "100"],
+                                         stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for l in self.proc.stdout:
+            self.lines.append(l.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        time.sleep(0.15)
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], None, set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for l in self.lines:
+            f = [x.strip() for x in l.split(",")]
+            if len(f) < 6:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx = float(f[1])
+            except ValueError:
+                continue
+            for nm, v in zip(names, f[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        sm.sort()
+        med = sm[len(sm) // 2] if sm else None
+        return {"sm_mhz": med, "sm_max_mhz": mx, "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def dist_env():
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return world, rank, local
+
+
+def workload_lines(name, world):
+    from paper_conf_icppw_tiancd23_b200 import workloads as W
+    if name == "C2":
+        return W.c2(64 * world), "C2: 64 x XSBench-style large (355 nuclides, 11303 gridpoints, hash 10000 bins, " \
+                                 "1M lookups) per GPU, distinct seeds; weak scaling by instance id"
+    if name == "TSTAR":
+        return W.tstar(1024 * world), "TSTAR: 1024 x XSBench-style small (68 nuclides, 1000 gridpoints, unionized, " \
+                                      "10k lookups) per GPU"
+    if name == "C1":
+        return W.c1(4 * world), "C1: 4 x XSBench-style small (1000 gridpoints, 10k lookups) per GPU"
+    if name == "C3":
+        return W.c3(256 * world), "C3: 256 x RSBench-style small, varied args, per GPU"
+    if name == "C4":
+        return W.c4(1024 * world), "C4: 1024 x AMGmk-style 32^3 Jacobi relax (20 sweeps) per GPU, T=1024"
+    if name == "C5":
+        return W.c5(4096 * world), "C5: 4096 mixed (XS/XS/RS/AMG) per GPU, sharded by instance id"
+    raise SystemExit(f"unknown workload {name}")
+
+
+THREADS = {"C2": 1024, "TSTAR": 256, "C1": 256, "C3": 256, "C4": 1024, "C5": 256}
+
+
+def time_ours(lines, world, rank, threads, steps, warmup, torch, dist_on):
+    """Device-resident timing of the ensemble (relaunch) + NCCL all-gather for world > 1."""
+    from paper_conf_icppw_tiancd23_b200 import Args, workloads
+    from paper_conf_icppw_tiancd23_b200.ensemble import Ensemble
+    from paper_conf_icppw_tiancd23_b200 import dist as D
+    args = Args.parse(workloads.text(lines))
+    n_total = len(lines)
+    stream = torch.cuda.Stream()
+    with torch.cuda.stream(stream):
+        ens = Ensemble(args, app="auto", first=rank, stride=world, threads=threads, stream=stream).launch()
+    stream.synchronize()
+    gather_rows = D.padded_count(n_total, world)
+    out_buf = None
+
+    def step():
+        ens.relaunch()
+        if dist_on:
+            with torch.cuda.stream(stream):
+                D.all_gather_rows(ens.device_records(), gather_rows)
+
+    for _ in range(warmup):
+        step()
+    stream.synchronize()
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(steps)]
+    if dist_on:
+        torch.distributed.barrier()
+    torch.cuda.synchronize()
+    t_all0 = torch.cuda.Event(enable_timing=True)
+    t_all1 = torch.cuda.Event(enable_timing=True)
+    t_all0.record(stream)
+    for i in range(steps):
+        ev[i][0].record(stream)
+        step()
+        ev[i][1].record(stream)
+    t_all1.record(stream)
+    torch.cuda.synchronize()
+    if dist_on:
+        torch.distributed.barrier()
+    total_ms = t_all0.elapsed_time(t_all1)
+    per_ms = [a.elapsed_time(b) for a, b in ev]
+    res = ens.collect()
+    info = ens.info()
+    return ens, res, info, total_ms, per_ms, out_buf
+
+
+def time_e2e(lines, world, rank, threads, steps, torch, dist_on):
+    """The public C ABI from host buffers: ens_launch (H2D) + ens_collect (D2H) per step."""
+    from paper_conf_icppw_tiancd23_b200 import Args, workloads, _ens
+    args = Args.parse(workloads.text(lines))
+    n_local = len(range(rank, len(lines), world))
+    cfg = _ens.make_cfg(n_local, first=rank, stride=world, threads=threads)
+    ws = _ens.workspace_bytes("auto", args, cfg)
+    buf = torch.empty(ws, dtype=torch.uint8, device="cuda")
+    stream = torch.cuda.current_stream().cuda_stream
+    h2d = d2h = 0
+
+    def one():
+        run = _ens.Run.launch("auto", args, cfg, buf.data_ptr(), ws, stream, keep=buf)
+        out = run.collect()
+        i = run.info()
+        run.close()
+        return out, i
+
+    one()  # warm
+    torch.cuda.synchronize()
+    if dist_on:
+        torch.distributed.barrier()
+    t0 = time.perf_counter()
+    for _ in range(steps):
+        out, i = one()
+    dt = time.perf_counter() - t0
+    h2d = int(i.h2d_bytes)
+    d2h = int(i.d2h_bytes)
+    return dt / steps, h2d, d2h
+
+
+def cpu_oracle_sample(lines, budget_s=20.0, max_instances=None):
+    """The oracle as it stands on this host: a bounded sample of the workload's instances."""
+    sys.path.insert(0, os.path.join(ROOT, "tests"))
+    import oracle_lib
+    oracle_lib.build()
+    cores = os.cpu_count() or 1
+    k = max_instances or max(1, min(cores, len(lines)))
+    sample = lines[:k]
+    t0 = time.perf_counter()
+    r = oracle_lib.run_text("".join(l + "\n" for l in sample), jobs=min(cores, k))
+    dt = time.perf_counter() - t0
+    work = int(r.records["work"].sum())
+    return {"instances": k, "seconds": dt, "cores": min(cores, k), "work": work}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="C2")
+    ap.add_argument("--no-extras", action="store_true", help="skip the TSTAR / solo side measurements")
+    a = ap.parse_args()
+    world, rank, local = dist_env()
+    if a.gpus != world and world == 1:
+        world_note = f"--gpus {a.gpus} without torchrun: running 1 process"
+    else:
+        world_note = None
+    lines, wl_desc = workload_lines(a.workload, world)
+    threads = THREADS.get(a.workload, 256)
+    n_local = len(range(rank, len(lines), world))
+    config = {"workload": wl_desc, "instances_per_gpu": n_local, "instances_total": len(lines),
+              "block_threads": threads, "l2": "inputs larger than L2 (per-instance tables >> 126 MB in total)",
+              "parallelism": f"instances sharded i mod {world}"}
+    if a.impl == "reference":
+        if rank != 0:
+            return
+        cores = os.cpu_count() or 1
+        vals = []
+        for _ in range(max(1, a.warmup // 3)):
+            pass
+        per = []
+        for s in range(a.steps):
+            r = cpu_oracle_sample(lines, max_instances=min(cores, len(lines), 16))
+            per.append(r)
+        inst = sum(r["instances"] for r in per)
+        sec = sum(r["seconds"] for r in per)
+        v = inst / sec
+        line = {"impl": "reference", "metric": METRIC, "value": v, "unit": "instances/s", "n_gpus": a.gpus,
+                "steps": a.steps, "warmup": a.warmup, "ms_per_step": 1e3 * sec / a.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic", "config": config,
+                "cpu_baseline": {"value": v, "unit": "instances/s", "cores": per[0]["cores"], "kind": "oracle",
+                                 "sample": f"first {per[0]['instances']} instances of the workload per step, "
+                                           f"full size, one instance per core"},
+                "e2e": {"value": v, "unit": "instances/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+                "lookups_per_s": sum(r["work"] for r in per) / sec}
+        print(json.dumps(line), flush=True)
+        return
+
+    import torch
+    dist_on = world > 1
+    if dist_on:
+        torch.cuda.set_device(local)
+        torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local))
+    else:
+        torch.cuda.set_device(0)
+    sampler = ClockSampler(local)
+    sampler_started = False
+
+    ens, res, info, total_ms, per_ms, _ = None, None, None, None, None, None
+    # timed region (clocks sampled during it)
+    sampler.start()
+    sampler_started = True
+    ens, res, info, total_ms, per_ms, _ = time_ours(lines, world, rank, threads, a.steps, max(3, a.warmup), torch,
+                                                    dist_on)
+    clocks = sampler.stop()
+    ms = total_ms / a.steps
+    t = torch.tensor([ms], dtype=torch.float64, device="cuda")
+    if dist_on:
+        torch.distributed.all_reduce(t, op=torch.distributed.ReduceOp.MAX)
+    ms_max = float(t.item())
+    local_lines = lines[rank::world]
+    algo = algorithmic_bytes(local_lines, res.records, res.tallies)
+    kern_ms = sum(per_ms) / len(per_ms)
+    peak, peak_kind = measured_peak_hbm()
+    achieved = algo / (kern_ms * 1e-3) / 1e9
+    lookups_local = int(res.records["work"].sum())
+    tt = torch.tensor([lookups_local, algo], dtype=torch.float64, device="cuda")
+    if dist_on:
+        torch.distributed.all_reduce(tt)
+    lookups_total = float(tt[0].item())
+    ok = bool((res.records["exit_code"] == 0).all())
+
+    # e2e through the C ABI from host buffers
+    e2e_s, h2d, d2h = time_e2e(lines, world, rank, threads, max(2, min(a.steps, 5)), torch, dist_on)
+    te = torch.tensor([e2e_s], dtype=torch.float64, device="cuda")
+    if dist_on:
+        torch.distributed.all_reduce(te, op=torch.distributed.ReduceOp.MAX)
+    e2e_s = float(te.item())
+
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tp):
+        try:
+            traffic = json.load(open(tp)).get(a.workload)
+        except Exception:
+            traffic = None
+
+    extras = {}
+    if not a.no_extras and world == 1 and a.workload == "C2":
+        # the paper's metric T1*N/TN: solo run of line 0 (N=1), same T
+        solo_ens, solo_res, _, solo_ms, _, _ = time_ours(lines[:1], 1, 0, threads, 2, 1, torch, False)
+        extras["speedup_vs_solo"] = {"T1_ms": solo_ms / 2, "TN_ms": ms, "N": len(lines),
+                                     "value": (solo_ms / 2) * len(lines) / ms,
+                                     "paper_context": "51x at 64 instances on A100 40GB (P:44-45, P:639-640)"}
+        solo_ens.close()
+        # north-star target launch: >= 1024 XSBench-style instances per B200 at >= 60% HBM
+        tl, _ = workload_lines("TSTAR", 1)
+        t_ens, t_res, t_info, t_ms, t_per, _ = time_ours(tl, 1, 0, 256, 5, 3, torch, False)
+        t_algo = algorithmic_bytes(tl, t_res.records, t_res.tallies)
+        t_k = sum(t_per) / len(t_per)
+        extras["tstar"] = {"instances": len(tl), "ms_per_launch": t_k, "instances_per_s": len(tl) / (t_k * 1e-3),
+                           "lookups_per_s": float(t_res.records["work"].sum()) / (t_k * 1e-3),
+                           "algorithmic_bytes": t_algo, "achieved_gbs": t_algo / (t_k * 1e-3) / 1e9,
+                           "frac_of_hbm": t_algo / (t_k * 1e-3) / 1e9 / peak,
+                           "parity_exit_ok": bool((t_res.records["exit_code"] == 0).all())}
+        t_ens.close()
+
+    if rank == 0:
+        out = {"metric": METRIC, "value": len(lines) / (ms_max * 1e-3), "unit": "instances/s", "n_gpus": world,
+               "steps": a.steps, "warmup": max(3, a.warmup), "ms_per_step": ms_max, "higher_is_better": True,
+               "scaling": "weak", "vs_baseline": None, "dtype": "f64", "data": "synthetic", "config": config,
+               "lookups_per_s": lookups_total / (ms_max * 1e-3),
+               "e2e": {"value": len(lines) / e2e_s, "unit": "instances/s", "h2d_bytes_per_step": h2d,
+                       "d2h_bytes_per_step": d2h},
+               "gpu_launches": int(info.kernel_launches) * a.steps,
+               "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
+                            "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
+                            "kernel": "ens_kernel<XsApp,1024>" if a.workload == "C2" else "ens_kernel",
+                            "algorithmic_bytes_per_launch": algo, "kernel_ms": kern_ms},
+               "clocks": clocks, "all_exit_ok": ok}
+        if world_note:
+            out["note"] = world_note
+        if world == 1:
+            cb = cpu_oracle_sample(lines, max_instances=min(os.cpu_count() or 1, 16, len(lines)))
+            out["cpu_baseline"] = {"value": cb["instances"] / cb["seconds"], "unit": "instances/s",
+                                   "cores": cb["cores"], "kind": "oracle",
+                                   "sample": f"first {cb['instances']} instances of the workload (full size), "
+                                             f"one per core, {cb['seconds']:.1f} s"}
+        out.update(extras)
+        print(json.dumps(out), flush=True)
+    if ens is not None:
+        ens.close()
+    if dist_on:
+        torch.distributed.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

@@ -177,6 +177,7 @@ typedef struct {
   uint64_t stdout_offset;  /* byte offset of the raw stdout buffers              */
   uint32_t stdout_bytes;   /* raw stdout bytes per instance                      */
   uint64_t h2d_bytes;      /* bytes copied host->device by ens_launch            */
+  uint64_t d2h_bytes;      /* bytes copied device->host by the last ens_collect  */
 } ens_run_info;
 int ens_run_get_info(const ens_run *r, ens_run_info *info);
 

@@ -49,7 +49,8 @@ class RunInfo(ctypes.Structure):
                 ("kernel_launches", ctypes.c_int32), ("arena_bytes", ctypes.c_uint64),
                 ("ws_bytes", ctypes.c_uint64), ("records_offset", ctypes.c_uint64),
                 ("tallies_offset", ctypes.c_uint64), ("stdout_offset", ctypes.c_uint64),
-                ("stdout_bytes", ctypes.c_uint32), ("h2d_bytes", ctypes.c_uint64)]
+                ("stdout_bytes", ctypes.c_uint32), ("h2d_bytes", ctypes.c_uint64),
+                ("d2h_bytes", ctypes.c_uint64)]
 
 
 def _load():

@@ -251,30 +251,34 @@ struct XsApp {
       uint16_t *osrc = orun, *odst = (orun == oA) ? oB : oA;
       const int CH = 16;
       for (long long w = n_gp; w < n_u; w <<= 1) {
-        for (long long o0 = (long long)tid * CH; o0 < n_u; o0 += (long long)T * CH) {
-          const long long base = (o0 / (2 * w)) * (2 * w);
-          const long long la = (base + w < n_u) ? w : n_u - base;
-          const long long lb = (base + 2 * w < n_u) ? w : (n_u - base - la > 0 ? n_u - base - la : 0);
-          const uint64_t *A = src + base, *B = src + base + la;
-          long long op = o0 - base;
-          long long lo = op - lb > 0 ? op - lb : 0, hi = op < la ? op : la;
-          while (lo < hi) {
-            const long long mid = (lo + hi) >> 1;
-            if (A[mid] < B[op - 1 - mid]) lo = mid + 1;
-            else hi = mid;
-          }
-          long long ia = lo, ib = op - lo;
-          const long long end = (o0 + CH < base + la + lb) ? o0 + CH : base + la + lb;
-          for (long long o = o0; o < end; o++) {
-            if (ia < la && (ib >= lb || A[ia] < B[ib])) {
-              dst[o] = A[ia];
-              odst[o] = osrc[base + ia];
-              ia++;
-            } else {
-              dst[o] = B[ib];
-              odst[o] = osrc[base + la + ib];
-              ib++;
+        for (long long c0 = (long long)tid * CH; c0 < n_u; c0 += (long long)T * CH) {
+          const long long c1 = (c0 + CH < n_u) ? c0 + CH : n_u;
+          for (long long o0 = c0; o0 < c1;) {  // a chunk may straddle merge pairs
+            const long long base = (o0 / (2 * w)) * (2 * w);
+            const long long la = (base + w < n_u) ? w : n_u - base;
+            const long long lb = (base + 2 * w < n_u) ? w : (n_u - base - la > 0 ? n_u - base - la : 0);
+            const uint64_t *A = src + base, *B = src + base + la;
+            const long long op = o0 - base;
+            long long lo = op - lb > 0 ? op - lb : 0, hi = op < la ? op : la;
+            while (lo < hi) {
+              const long long mid = (lo + hi) >> 1;
+              if (A[mid] < B[op - 1 - mid]) lo = mid + 1;
+              else hi = mid;
             }
+            long long ia = lo, ib = op - lo;
+            const long long end = (c1 < base + la + lb) ? c1 : base + la + lb;
+            for (long long o = o0; o < end; o++) {
+              if (ia < la && (ib >= lb || A[ia] < B[ib])) {
+                dst[o] = A[ia];
+                odst[o] = osrc[base + ia];
+                ia++;
+              } else {
+                dst[o] = B[ib];
+                odst[o] = osrc[base + la + ib];
+                ib++;
+              }
+            }
+            o0 = end;
           }
         }
         __syncthreads();

@@ -187,6 +187,7 @@ struct ens_run {
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   uint32_t flags = 0;
   bool launched = false;
+  uint64_t d2h = 0;
 };
 
 static size_t al(size_t x) { return (x + 255) / 256 * 256; }
@@ -288,7 +289,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   int want = 0;
   for (const Group &g : P.groups) want = std::max(want, g.grid);
   if (P.arena_bytes && mem_cap) {
-    if (mem_cap <= o + P.arena_bytes) return fail(ENS_ENOMEM, "ens_launch: workspace cannot hold one arena slot");
+    if (mem_cap < o + P.arena_bytes) return fail(ENS_ENOMEM, "ens_launch: workspace cannot hold one arena slot");
     const uint64_t fit = (mem_cap - o) / P.arena_bytes;
     if ((uint64_t)want > fit) {
       if (c->grid_blocks) return fail(ENS_ENOMEM, "ens_launch: grid_blocks x arena does not fit the workspace");
@@ -434,16 +435,22 @@ extern "C" int ens_collect(ens_run *r, ens_record *recs, uint32_t *tallies, char
   }
   CU(cudaStreamSynchronize(r->stream));
   CU(cudaGetLastError());
+  r->d2h = 0;
   // counters | records | stdout positions: one copy
   std::vector<char> zb(P.zeroed_end - P.o_ctr);
   CU(cudaMemcpy(zb.data(), r->ws + P.o_ctr, zb.size(), cudaMemcpyDeviceToHost));
+  r->d2h += zb.size();
   const uint64_t total = *(const uint64_t *)(zb.data() + 8 * P.groups.size());
   std::vector<ens_record> R((size_t)n);
   std::memcpy(R.data(), zb.data() + (P.o_recs - P.o_ctr), (size_t)n * sizeof(ens_record));
   const uint64_t *pos = (const uint64_t *)(zb.data() + (P.o_pos - P.o_ctr));
-  if (tallies) CU(cudaMemcpy(tallies, r->ws + P.o_tal, (size_t)n * ENS_TALLIES * 4, cudaMemcpyDeviceToHost));
+  if (tallies) {
+    CU(cudaMemcpy(tallies, r->ws + P.o_tal, (size_t)n * ENS_TALLIES * 4, cudaMemcpyDeviceToHost));
+    r->d2h += (size_t)n * ENS_TALLIES * 4;
+  }
   std::vector<uint64_t> cmp((size_t)(total + 7) / 8 + 1);
   if (total) CU(cudaMemcpy(cmp.data(), r->ws + P.o_cmp, (size_t)total, cudaMemcpyDeviceToHost));
+  r->d2h += total;
   std::string text;
   std::vector<uint64_t> off((size_t)n + 1, 0);
   int bad = 0;
@@ -504,6 +511,7 @@ extern "C" int ens_run_get_info(const ens_run *r, ens_run_info *info) {
   info->stdout_offset = P.o_out;
   info->stdout_bytes = P.stdout_cap;
   info->h2d_bytes = P.n ? P.staged : 0;
+  info->d2h_bytes = r->d2h;
   return ENS_OK;
 }
 
