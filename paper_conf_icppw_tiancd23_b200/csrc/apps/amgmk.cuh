@@ -17,6 +17,7 @@ namespace ens {
 
 struct AmgApp {
   static constexpr uint32_t kId = APP_AMGMK;
+  static constexpr int kMaxT = 1024;  // 64 registers suffice
 
   __device__ static Result run(Ctx &c, int argc, char **argv) {
     Result R{};
@@ -136,7 +137,7 @@ struct AmgApp {
     return R;
   }
 
-  __host__ static bool size(int argc, const char *const *argv, uint64_t *arena, uint32_t *smem) {
+  __host__ static bool size(int argc, const char *const *argv, int, uint64_t *arena, uint32_t *smem) {
     AmgParams p;
     *smem = 0;
     if (amg_parse(argc, argv, p) >= 0) {

@@ -76,10 +76,17 @@ ENS_HD int pow2_ceil(int n) {
   return p;
 }
 
+// per-nuclide bucket count of the init sort (power of two)
+ENS_HD int xs_nb(int n_gp) {
+  int nb = pow2_ceil(n_gp) / 2;
+  return nb < 32 ? 32 : (nb > 8192 ? 8192 : nb);
+}
+
 // arena layout (byte offsets, 256-B aligned)
 struct XsLayout {
   uint64_t recs;      // [n_iso][n_gp] x 48 B records, sorted per nuclide
   uint64_t scratch;   // [n_gp] x 48 B unsorted records of one nuclide
+  uint64_t keys;      // [n_gp] x 16 B {energy bits, index} being sorted
   uint64_t uenergy;   // unionized: [n_u] sorted union energies (u64 bits)
   uint64_t utmp;      // unionized: [n_u] merge ping-pong
   uint64_t uown;      // unionized: [n_u] u16 owner nuclide
@@ -93,6 +100,7 @@ ENS_HD XsLayout xs_layout(const XsParams &p) {
   uint64_t o = 0;
   L.recs = o; o = align_up(o + n_u * 48, 256);
   L.scratch = o; o = align_up(o + (uint64_t)p.n_gp * 48, 256);
+  L.keys = o; o = align_up(o + (uint64_t)p.n_gp * 16, 256);
   if (p.grid == XS_UNIONIZED) {
     L.uenergy = o; o = align_up(o + n_u * 8, 256);
     L.utmp = o; o = align_up(o + n_u * 8, 256);
@@ -106,21 +114,28 @@ ENS_HD XsLayout xs_layout(const XsParams &p) {
   return L;
 }
 
-// dynamic shared memory layout
+// dynamic shared memory layout: material tables + the sort's bucket counters
+constexpr int kXsU = 2;       // nuclide gathers in flight per lane
+constexpr int kXsMaxT = 512;  // XsApp::kMaxT
+// lookups per thread per material-sorted batch: enough that every thread
+// gets several fuel lookups (321 nuclides large / 34 small)
+ENS_HD int xs_batch_k(int n_iso) { return n_iso == 68 ? 8 : 24; }
 struct XsSmem {
-  uint32_t thr, nn, mats, concs, keys, perm, total;
+  uint32_t thr, nn, mats, concs, bkt, mcnt, slot, total;
 };
-ENS_HD XsSmem xs_smem(const XsParams &p) {
+// T = the block size the instance runs with
+ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   XsSmem S{};
   const uint32_t mx = (uint32_t)xs_max_nucs(p.n_iso);
-  const uint32_t P2 = (uint32_t)pow2_ceil(p.n_gp);
   uint32_t o = 0;
   S.thr = o; o += 12 * 8;                 // pick_mat thresholds
   S.nn = o; o += 16 * 4;                  // num_nucs
   S.concs = o; o += 12 * mx * 8;          // concentrations
   S.mats = o; o += (uint32_t)align_up(12 * mx * 2, 16);  // nuclide ids (u16)
-  S.keys = o; o += P2 * 8;                // sort keys (energy bits)
-  S.perm = o; o += (uint32_t)align_up(P2 * 2, 16);       // sort payload (u16)
+  S.bkt = o; o += (uint32_t)align_up((uint64_t)xs_nb(p.n_gp) * 4, 16);  // bucket counters / offsets
+  S.mcnt = o; o += 32 * 4;                // batch material counts / offsets
+  S.slot = o;                             // batch slots: energy (+ union index)
+  o += (uint32_t)xs_batch_k(p.n_iso) * (uint32_t)T * (p.grid == XS_UNIONIZED ? 12u : 8u);
   S.total = o;
   return S;
 }

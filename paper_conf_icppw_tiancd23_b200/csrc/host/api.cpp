@@ -241,7 +241,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     if (app == ENS_APP_BY_ARGV0) ap = argc > 0 ? app_of_argv0(argv[0]) : (uint32_t)APP_NOTFOUND;
     uint64_t ar = 0;
     uint32_t sm = 0;
-    app_size(ap, argc, argv, &ar, &sm);
+    app_size(ap, argc, argv, std::min(T, app_max_threads(ap)), &ar, &sm);
     Group &g = g_by_app[ap];
     g.app = ap;
     g.arena = std::max(g.arena, ar);
@@ -254,9 +254,9 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
                       (uint32_t)APP_NOTFOUND}) {
     Group &g = g_by_app[ap];
     if (g.kmap.empty()) continue;
-    g.T = T;
+    g.T = std::min(T, app_max_threads(ap));
     int occ = 0;
-    e = group_occupancy(ap, T, g.smem, &occ);
+    e = group_occupancy(ap, g.T, g.smem, &occ);
     if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor");
     if (occ <= 0) return fail(ENS_EINVAL, "ens_launch: an instance needs more shared memory than one SM has");
     int grid = c->grid_blocks ? c->grid_blocks : occ * sms;

@@ -29,7 +29,7 @@ __device__ __forceinline__ uint32_t smid() {
 }
 
 template <class App, int T>
-__global__ void __launch_bounds__(T, (1024 / T) > 0 ? (1024 / T) : 1) ens_kernel(const KParams p) {
+__global__ void __launch_bounds__(T, (512 / T) > 0 ? (512 / T) : 1) ens_kernel(const KParams p) {
   extern __shared__ __align__(16) char dsmem[];
   __shared__ char *s_argv[ENS_MAX_ARGC + 1];
   __shared__ uint32_t s_j;
@@ -99,17 +99,35 @@ __global__ void __launch_bounds__(T, (1024 / T) > 0 ? (1024 / T) : 1) ens_kernel
   }
 }
 
+template <class App, int T>
+static const void *kernel_if() {
+  if constexpr (T <= App::kMaxT) return (const void *)ens_kernel<App, T>;
+  return nullptr;
+}
 template <class App>
 static const void *kernel_for(int T) {
   switch (T) {
-    case 32: return (const void *)ens_kernel<App, 32>;
-    case 64: return (const void *)ens_kernel<App, 64>;
-    case 128: return (const void *)ens_kernel<App, 128>;
-    case 256: return (const void *)ens_kernel<App, 256>;
-    case 512: return (const void *)ens_kernel<App, 512>;
-    case 1024: return (const void *)ens_kernel<App, 1024>;
+    case 32: return kernel_if<App, 32>();
+    case 64: return kernel_if<App, 64>();
+    case 128: return kernel_if<App, 128>();
+    case 256: return kernel_if<App, 256>();
+    case 512: return kernel_if<App, 512>();
+    case 1024: return kernel_if<App, 1024>();
   }
   return nullptr;
+}
+
+// the largest block size an app's kernel is built for (the thread limit is an
+// upper bound)
+int app_max_threads(uint32_t app) {
+  switch (app) {
+    case APP_ECHO: return EchoApp::kMaxT;
+    case APP_XSBENCH: return XsApp::kMaxT;
+    case APP_RSBENCH: return RsApp::kMaxT;
+    case APP_AMGMK: return AmgApp::kMaxT;
+    case APP_NOTFOUND: return NotFoundApp::kMaxT;
+  }
+  return 32;
 }
 
 const void *kernel_ptr(uint32_t app, int T) {
@@ -124,13 +142,13 @@ const void *kernel_ptr(uint32_t app, int T) {
 }
 
 // host-side sizing from the same parse/layout code the instance runs
-bool app_size(uint32_t app, int argc, const char *const *argv, uint64_t *arena, uint32_t *smem) {
+bool app_size(uint32_t app, int argc, const char *const *argv, int T, uint64_t *arena, uint32_t *smem) {
   switch (app) {
-    case APP_ECHO: return EchoApp::size(argc, argv, arena, smem);
-    case APP_XSBENCH: return XsApp::size(argc, argv, arena, smem);
-    case APP_RSBENCH: return RsApp::size(argc, argv, arena, smem);
-    case APP_AMGMK: return AmgApp::size(argc, argv, arena, smem);
-    case APP_NOTFOUND: return NotFoundApp::size(argc, argv, arena, smem);
+    case APP_ECHO: return EchoApp::size(argc, argv, T, arena, smem);
+    case APP_XSBENCH: return XsApp::size(argc, argv, T, arena, smem);
+    case APP_RSBENCH: return RsApp::size(argc, argv, T, arena, smem);
+    case APP_AMGMK: return AmgApp::size(argc, argv, T, arena, smem);
+    case APP_NOTFOUND: return NotFoundApp::size(argc, argv, T, arena, smem);
   }
   *arena = 0;
   *smem = 0;
@@ -140,7 +158,7 @@ bool app_size(uint32_t app, int argc, const char *const *argv, uint64_t *arena, 
 cudaError_t launch_group(uint32_t app, int T, int grid, size_t smem, const KParams &p, cudaStream_t st) {
   const void *fn = kernel_ptr(app, T);
   if (!fn) return cudaErrorInvalidValue;
-  if (smem > 48 * 1024) {
+  if (smem > 0) {
     cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
   }
@@ -151,7 +169,7 @@ cudaError_t launch_group(uint32_t app, int T, int grid, size_t smem, const KPara
 cudaError_t group_occupancy(uint32_t app, int T, size_t smem, int *blocks_per_sm) {
   const void *fn = kernel_ptr(app, T);
   if (!fn) return cudaErrorInvalidValue;
-  if (smem > 48 * 1024) {
+  if (smem > 0) {
     cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
   }

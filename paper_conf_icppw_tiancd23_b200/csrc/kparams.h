@@ -29,7 +29,8 @@ struct KParams {
 };
 
 const void *kernel_ptr(uint32_t app, int T);
-bool app_size(uint32_t app, int argc, const char *const *argv, uint64_t *arena, uint32_t *smem);
+int app_max_threads(uint32_t app);
+bool app_size(uint32_t app, int argc, const char *const *argv, int T, uint64_t *arena, uint32_t *smem);
 cudaError_t launch_group(uint32_t app, int T, int grid, size_t smem, const KParams &p, cudaStream_t st);
 cudaError_t group_occupancy(uint32_t app, int T, size_t smem, int *blocks_per_sm);
 
