@@ -76,21 +76,27 @@ ENS_HD int pow2_ceil(int n) {
   return p;
 }
 
-// per-nuclide bucket count of the init sort (power of two)
-ENS_HD int xs_nb(int n_gp) {
-  int nb = pow2_ceil(n_gp) / 2;
-  return nb < 32 ? 32 : (nb > 8192 ? 8192 : nb);
+// Init sort = one bucket sort of all n_u records (energies are uniform in
+// [0,1)): unionized by energy alone (the union order; each nuclide's order
+// is its subsequence), otherwise by (nuclide, energy).  Power-of-two bucket
+// counts keep floor(E * nb) exact.
+ENS_HD long long xs_buckets(const XsParams &p) {
+  const long long n_u = (long long)p.n_iso * p.n_gp;
+  if (p.grid == XS_UNIONIZED) return pow2_ceil((int)((n_u + 1) / 2));
+  return (long long)p.n_iso * (pow2_ceil(p.n_gp) / 2 > 0 ? pow2_ceil(p.n_gp) / 2 : 1);
 }
+ENS_HD int xs_nbn(int n_gp) { return pow2_ceil(n_gp) / 2 > 0 ? pow2_ceil(n_gp) / 2 : 1; }
+// union-sweep chunks (rows per chunk) for the index grid
+constexpr int kXsSweepRows = 512;
 
 // arena layout (byte offsets, 256-B aligned)
 struct XsLayout {
   uint64_t recs;      // [n_iso][n_gp] x 48 B records, sorted per nuclide
-  uint64_t scratch;   // [n_gp] x 48 B unsorted records of one nuclide
-  uint64_t keys;      // [n_gp] x 16 B {energy bits, index} being sorted
+  uint64_t scratch;   // [n_u] x 48 B records in generation order
+  uint64_t keys;      // [n_u] x 16 B {energy bits, record id}, bucket-sorted
+  uint64_t bkt;       // [xs_buckets] u32 bucket counts -> offsets
   uint64_t uenergy;   // unionized: [n_u] sorted union energies (u64 bits)
-  uint64_t utmp;      // unionized: [n_u] merge ping-pong
-  uint64_t uown;      // unionized: [n_u] u16 owner nuclide
-  uint64_t uowntmp;   // unionized: [n_u] u16 ping-pong
+  uint64_t chist;     // unionized: [n_chunks][n_iso] u32 owner counts per sweep chunk
   uint64_t index;     // unionized [n_u][n_iso] / hash [n_iso][bins+1] int32
   uint64_t total;
 };
@@ -98,14 +104,17 @@ ENS_HD XsLayout xs_layout(const XsParams &p) {
   XsLayout L{};
   const uint64_t n_u = (uint64_t)p.n_iso * p.n_gp;
   uint64_t o = 0;
+  // unionized: one sort of all n_u records; otherwise one nuclide at a time
+  const uint64_t n_s = p.grid == XS_UNIONIZED ? n_u : (uint64_t)p.n_gp;
   L.recs = o; o = align_up(o + n_u * 48, 256);
-  L.scratch = o; o = align_up(o + (uint64_t)p.n_gp * 48, 256);
-  L.keys = o; o = align_up(o + (uint64_t)p.n_gp * 16, 256);
+  L.scratch = o; o = align_up(o + n_s * 48, 256);
+  L.keys = o; o = align_up(o + n_s * 16, 256);
+  L.bkt = o;
+  if (p.grid == XS_UNIONIZED) o = align_up(o + (uint64_t)xs_buckets(p) * 4, 256);
   if (p.grid == XS_UNIONIZED) {
+    const uint64_t nch = (n_u + kXsSweepRows - 1) / kXsSweepRows;
     L.uenergy = o; o = align_up(o + n_u * 8, 256);
-    L.utmp = o; o = align_up(o + n_u * 8, 256);
-    L.uown = o; o = align_up(o + n_u * 2, 256);
-    L.uowntmp = o; o = align_up(o + n_u * 2, 256);
+    L.chist = o; o = align_up(o + nch * (uint64_t)p.n_iso * 4, 256);
     L.index = o; o = align_up(o + n_u * (uint64_t)p.n_iso * 4, 256);
   } else if (p.grid == XS_HASH) {
     L.index = o; o = align_up(o + (uint64_t)p.n_iso * (p.bins + 1) * 4, 256);
@@ -121,7 +130,7 @@ constexpr int kXsMaxT = 512;  // XsApp::kMaxT
 // gets several fuel lookups (321 nuclides large / 34 small)
 ENS_HD int xs_batch_k(int n_iso) { return n_iso == 68 ? 8 : 24; }
 struct XsSmem {
-  uint32_t thr, nn, mats, concs, bkt, mcnt, slot, total;
+  uint32_t thr, nn, mats, concs, mcnt, nbkt, slot, total;
 };
 // T = the block size the instance runs with
 ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
@@ -132,8 +141,9 @@ ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   S.nn = o; o += 16 * 4;                  // num_nucs
   S.concs = o; o += 12 * mx * 8;          // concentrations
   S.mats = o; o += (uint32_t)align_up(12 * mx * 2, 16);  // nuclide ids (u16)
-  S.bkt = o; o += (uint32_t)align_up((uint64_t)xs_nb(p.n_gp) * 4, 16);  // bucket counters / offsets
   S.mcnt = o; o += 32 * 4;                // batch material counts / offsets
+  S.nbkt = o;                             // per-nuclide sort buckets (hash / nuclide grids)
+  if (p.grid != XS_UNIONIZED) o += (uint32_t)align_up((uint64_t)xs_nbn(p.n_gp) * 4, 16);
   S.slot = o;                             // batch slots: energy (+ union index)
   o += (uint32_t)xs_batch_k(p.n_iso) * (uint32_t)T * (p.grid == XS_UNIONIZED ? 12u : 8u);
   S.total = o;

@@ -124,43 +124,89 @@ __device__ __forceinline__ long long gs_u64(const uint64_t *A, double q, long lo
   return lo;
 }
 
-// exclusive prefix sum of a[0..n) in shared memory, block-wide (n >= 1)
-__device__ inline void block_exclusive_scan(uint32_t *a, int n, Shared *sh) {
+// exclusive (or inclusive) prefix sum of a[0..n) (global or shared memory,
+// 16-B aligned), block-wide, in coalesced tiles of 8 consecutive elements per
+// thread (two 16-B loads)
+template <bool INCL = false>
+__device__ inline void global_exclusive_scan(uint32_t *a, long long n, Shared *sh) {
   const int tid = threadIdx.x, T = blockDim.x, lane = tid & 31, w = tid >> 5, nw = T >> 5;
-  const int per = (n + T - 1) / T;
-  const int b0 = tid * per < n ? tid * per : n, b1 = b0 + per < n ? b0 + per : n;
-  uint32_t sum = 0;
-  for (int i = b0; i < b1; i++) sum += a[i];
-  uint32_t inc = sum;
-  for (int o = 1; o < 32; o <<= 1) {
-    const uint32_t v = __shfl_up_sync(0xffffffffu, inc, o);
-    if (lane >= o) inc += v;
-  }
-  if (lane == 31) sh->red_u[w] = inc;
-  __syncthreads();
-  if (w == 0) {
-    unsigned long long t = lane < nw ? sh->red_u[lane] : 0ULL;
-    unsigned long long ti = t;
-    for (int o = 1; o < 32; o <<= 1) {
-      const unsigned long long v = __shfl_up_sync(0xffffffffu, ti, o);
-      if (lane >= o) ti += v;
+  constexpr int V = 8;
+  const bool vec = (reinterpret_cast<uintptr_t>(a) & 15) == 0;
+  uint32_t carry = 0;
+  for (long long base = 0; base < n; base += (long long)T * V) {
+    const long long i0 = base + (long long)tid * V;
+    uint32_t v[V];
+    if (vec && i0 + V <= n) {
+      const uint4 x = *reinterpret_cast<const uint4 *>(a + i0), y = *reinterpret_cast<const uint4 *>(a + i0 + 4);
+      v[0] = x.x; v[1] = x.y; v[2] = x.z; v[3] = x.w; v[4] = y.x; v[5] = y.y; v[6] = y.z; v[7] = y.w;
+    } else {
+#pragma unroll
+      for (int k = 0; k < V; k++) v[k] = i0 + k < n ? a[i0 + k] : 0u;
     }
-    if (lane < nw) sh->red_u[lane] = ti - t;  // exclusive warp offsets
+    uint32_t sum = 0;
+#pragma unroll
+    for (int k = 0; k < V; k++) sum += v[k];
+    uint32_t inc = sum;
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t t = __shfl_up_sync(0xffffffffu, inc, o);
+      if (lane >= o) inc += t;
+    }
+    if (lane == 31) sh->red_u[w] = inc;
+    __syncthreads();
+    if (w == 0) {
+      const unsigned long long t = lane < nw ? sh->red_u[lane] : 0ULL;
+      unsigned long long ti = t;
+      for (int o = 1; o < 32; o <<= 1) {
+        const unsigned long long u = __shfl_up_sync(0xffffffffu, ti, o);
+        if (lane >= o) ti += u;
+      }
+      if (lane < nw) sh->red_u[lane] = ti - t;                         // exclusive warp offsets
+      if (lane == 31) sh->red_d[0] = __longlong_as_double((long long)ti);  // tile total
+    }
+    __syncthreads();
+    uint32_t run = carry + (uint32_t)sh->red_u[w] + inc - sum;
+    const uint32_t total = (uint32_t)__double_as_longlong(sh->red_d[0]);
+#pragma unroll
+    for (int k = 0; k < V; k++) {
+      const uint32_t t = v[k];
+      v[k] = INCL ? run + t : run;
+      run += t;
+    }
+    if (vec && i0 + V <= n) {
+      *reinterpret_cast<uint4 *>(a + i0) = make_uint4(v[0], v[1], v[2], v[3]);
+      *reinterpret_cast<uint4 *>(a + i0 + 4) = make_uint4(v[4], v[5], v[6], v[7]);
+    } else {
+#pragma unroll
+      for (int k = 0; k < V; k++)
+        if (i0 + k < n) a[i0 + k] = v[k];
+    }
+    carry += total;
+    __syncthreads();
   }
-  __syncthreads();
-  uint32_t run = (uint32_t)sh->red_u[w] + inc - sum;
-  for (int i = b0; i < b1; i++) {
-    const uint32_t v = a[i];
-    a[i] = run;
-    run += v;
-  }
-  __syncthreads();
 }
+
+#ifdef ENS_XS_STOP  // profiling builds only: stop init after phase k
+#define XS_STOP(k) do { if (ENS_XS_STOP == (k)) { __syncthreads(); return; } } while (0)
+#else
+#define XS_STOP(k) do { } while (0)
+#endif
 
 struct XsKey {
   unsigned long long key;  // energy bit pattern (positive doubles order as integers)
   unsigned int idx, pad;
 };
+
+// init-sort bucket of record r with energy e in [0, 1]: by energy alone
+// (unionized) or by (nuclide, energy); nb / nbn are powers of two, so
+// e * nb is exact and floor() is monotone in e.
+__device__ __forceinline__ long long bucket_of(double e, long long r, int n_gp, bool uni, long long nb, int nbn) {
+  if (uni) {
+    const long long b = (long long)(e * (double)nb);
+    return b < nb - 1 ? b : nb - 1;
+  }
+  const long long b = (long long)(e * (double)nbn);
+  return (r / n_gp) * nbn + (b < nbn - 1 ? b : nbn - 1);
+}
 
 struct XsApp {
   static constexpr uint32_t kId = APP_XSBENCH;
@@ -195,7 +241,8 @@ struct XsApp {
     hm_tables(n_iso, mx, thr, nn, concs, mats);
     __syncthreads();
     hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
-    init(c, p, L, S);
+    if (p.grid == XS_UNIONIZED) init(c, p, L, S);
+    else init_nuc(c, p, L, S);
     if (p.grid == XS_HASH) lookups<XS_HASH>(c, p, L, thr, nn, concs, mats, R);
     else if (p.grid == XS_UNIONIZED) lookups<XS_UNIONIZED>(c, p, L, thr, nn, concs, mats, R);
     else lookups<XS_NUCLIDE>(c, p, L, thr, nn, concs, mats, R);
@@ -207,201 +254,437 @@ struct XsApp {
     return R;
   }
 
-  // ---- XS-3/4/5: nuclide grid, per-nuclide sort, acceleration structure --
-  __device__ static __noinline__ void init(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
+  // sort keys[lo, hi) by (energy, record id): <= 8 in registers, else in place
+  __device__ static __forceinline__ void sort_bucket(XsKey *keys, long long lo, long long hi) {
+    const int cnt = (int)(hi - lo);
+    if (cnt <= 1) return;
+    if (cnt <= 8) {
+      unsigned long long kk[8];
+      unsigned ii[8];
+#pragma unroll
+      for (int q = 0; q < 8; q++)
+        if (q < cnt) {
+          const XsKey v = keys[lo + q];
+          kk[q] = v.key;
+          ii[q] = v.idx;
+        }
+#pragma unroll
+      for (int x = 1; x < 8; x++) {
+#pragma unroll
+        for (int y = x; y > 0; y--) {
+          if (x < cnt && (kk[y - 1] > kk[y] || (kk[y - 1] == kk[y] && ii[y - 1] > ii[y]))) {
+            const unsigned long long tk = kk[y - 1];
+            kk[y - 1] = kk[y];
+            kk[y] = tk;
+            const unsigned ti = ii[y - 1];
+            ii[y - 1] = ii[y];
+            ii[y] = ti;
+          }
+        }
+      }
+#pragma unroll
+      for (int q = 0; q < 8; q++)
+        if (q < cnt) {
+          XsKey v;
+          v.key = kk[q];
+          v.idx = ii[q];
+          v.pad = 0;
+          keys[lo + q] = v;
+        }
+      return;
+    }
+    for (long long x = lo + 1; x < hi; x++) {
+      const XsKey v = keys[x];
+      long long y = x - 1;
+      while (y >= lo && (keys[y].key > v.key || (keys[y].key == v.key && keys[y].idx > v.idx))) {
+        keys[y + 1] = keys[y];
+        y--;
+      }
+      keys[y + 1] = v;
+    }
+  }
+
+  // ---- XS-3/4/5, hash and nuclide grids: one nuclide at a time -------------
+  // Nuclide i's n_gp records (draws 6r+1..6r+6, r = i*n_gp + j; XS-3) are
+  // generated into an L2-resident scratch, bucket-sorted by energy (XS-4:
+  // shared-memory counts -> scan -> scatter -> per-bucket sort), written to
+  // their sorted position, and (hash) the nuclide's index column is built as
+  // a histogram of each energy's first bin followed by an inclusive scan
+  // (XS-5: ig[i][b] = grid_search(E_i, b*du) = min(#{k>=1: E_k <= b*du}, n_gp-2)).
+  __device__ static __noinline__ void init_nuc(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
     const int tid = threadIdx.x, T = blockDim.x;
     const int n_iso = p.n_iso, n_gp = p.n_gp;
-    const long long n_u = (long long)n_iso * n_gp;
-    const int NB = xs_nb(n_gp);
-    uint32_t *bkt = (uint32_t *)(c.smem + S.bkt);
+    const int nbn = xs_nbn(n_gp);
+    uint32_t *nb = (uint32_t *)(c.smem + S.nbkt);
     double *recs = (double *)(c.arena + L.recs);
     double *scr = (double *)(c.arena + L.scratch);
     XsKey *keys = (XsKey *)(c.arena + L.keys);
     int *ig = (int *)(c.arena + L.index);
-    uint64_t *uA = (uint64_t *)(c.arena + L.uenergy), *uB = (uint64_t *)(c.arena + L.utmp);
-    uint16_t *oA = (uint16_t *)(c.arena + L.uown), *oB = (uint16_t *)(c.arena + L.uowntmp);
-    int rounds = 0;
-    while ((1 << rounds) < n_iso) rounds++;
-    uint64_t *urun = (rounds & 1) ? uB : uA;  // merge rounds alternate; end in uA
-    uint16_t *orun = (rounds & 1) ? oB : oA;
+    const bool hash = p.grid == XS_HASH;
     const double du = 1.0 / p.bins;
     const Affine J6T = lcg_pow(6ULL * T);
     const Affine Jnuc = lcg_pow(6ULL * n_gp);
     uint64_t s_nuc = lcg_pow(6ULL * tid)(p.gseed);  // before record (i*n_gp + tid)
-
     for (int i = 0; i < n_iso; i++) {
-      for (int b = tid; b < NB; b += T) bkt[b] = 0;
+      int *col = ig + (size_t)i * (p.bins + 1);
+      for (int b = tid; b < nbn; b += T) nb[b] = 0;
+      if (hash)
+        for (int b = tid; b <= p.bins; b += T) col[b] = 0;
       __syncthreads();
-      // (a) generate: record r = i*n_gp + j takes draws 6r+1 .. 6r+6 (XS-3)
-      uint64_t s = s_nuc;
-      for (int j = tid; j < n_gp; j += T, s = J6T(s)) {
+      {  // generate + count
+        uint64_t s = s_nuc;
+        for (int j = tid; j < n_gp; j += T, s = J6T(s)) {
+          uint64_t t = s;
+          double v[6];
+#pragma unroll
+          for (int f = 0; f < 6; f++) v[f] = lcg_double(t);
+          double2 *d = reinterpret_cast<double2 *>(scr + 6 * (size_t)j);
+          d[0] = make_double2(v[0], v[1]);
+          d[1] = make_double2(v[2], v[3]);
+          d[2] = make_double2(v[4], v[5]);
+          atomicAdd(&nb[bucket_of(v[0], j, n_gp, false, 0, nbn)], 1u);
+        }
+        s_nuc = Jnuc(s_nuc);
+      }
+      __syncthreads();
+      global_exclusive_scan(nb, nbn, c.sh);
+      for (int j0 = tid; j0 < n_gp; j0 += 4 * T) {  // scatter {energy, j}
+        double e[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++) e[q] = j0 + q * T < n_gp ? ld_(scr + 6 * (size_t)(j0 + q * T)) : 0.0;
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+          const int j = j0 + q * T;
+          if (j < n_gp) {
+            const uint32_t pos = atomicAdd(&nb[bucket_of(e[q], j, n_gp, false, 0, nbn)], 1u);
+            XsKey k;
+            k.key = dbits(e[q]);
+            k.idx = (unsigned)j;
+            k.pad = 0;
+            keys[pos] = k;
+          }
+        }
+      }
+      __syncthreads();
+      for (int b = tid; b < nbn; b += T) sort_bucket(keys, b ? nb[b - 1] : 0, nb[b]);
+      __syncthreads();
+      double *rec_i = recs + (size_t)i * n_gp * 6;
+      for (int k0 = tid; k0 < n_gp; k0 += 4 * T) {  // records to sorted position; bin histogram
+        unsigned jj[4];
+        unsigned long long kb[4];
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+          const int k = k0 + q * T;
+          if (k < n_gp) {
+            const XsKey v = keys[k];
+            jj[q] = v.idx;
+            kb[q] = v.key;
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < 4; q++) {
+          const int k = k0 + q * T;
+          if (k < n_gp) {
+            const double2 *src = reinterpret_cast<const double2 *>(scr + 6 * (size_t)jj[q]);
+            double2 *dst = reinterpret_cast<double2 *>(rec_i + 6 * (size_t)k);
+            const double2 a = src[0], b = src[1], x = src[2];
+            dst[0] = a;
+            dst[1] = b;
+            dst[2] = x;
+            if (hash && k >= 1) {  // first bin b with E_k <= b*du
+              const double e = __longlong_as_double((long long)kb[q]);
+              long long bb = (long long)(e * p.bins);
+              while (bb > 0 && (double)(bb - 1) * du >= e) bb--;
+              while (bb < p.bins && (double)bb * du < e) bb++;
+              if (bb < p.bins) atomicAdd((unsigned *)&col[bb], 1u);
+            }
+          }
+        }
+      }
+      __syncthreads();
+      if (hash) {
+        global_exclusive_scan<true>((uint32_t *)col, p.bins, c.sh);
+        for (int b = tid; b < p.bins; b += T) {
+          const int v = col[b];
+          if (v > n_gp - 2) col[b] = n_gp - 2;
+        }
+        if (tid == 0) col[p.bins] = n_gp - 2;
+        __syncthreads();
+      }
+    }
+  }
+
+  // ---- XS-3/4/5: nuclide grid, sort, acceleration structure --------------
+  // One block-wide bucket sort of all n_u records replaces n_iso per-nuclide
+  // sorts: (G) generate every record (draws 6r+1..6r+6, XS-3) into scratch
+  // and count its bucket; (S) scan; (P) scatter {energy, record id}; (B)
+  // insertion-sort each ~2-element bucket.  Unionized buckets are by energy
+  // alone, so the sorted keys ARE the union (XS-5) and a nuclide's records in
+  // union order are its sorted records (XS-4); otherwise buckets are
+  // (nuclide, energy).  Ties are measure-zero (reading Q13) and broken by
+  // record id, deterministically.
+  __device__ static __noinline__ void init(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
+    const int tid = threadIdx.x, T = blockDim.x;
+    const int n_iso = p.n_iso, n_gp = p.n_gp;
+    const long long n_u = (long long)n_iso * n_gp;
+    const long long NB = xs_buckets(p);
+    const int nbn = xs_nbn(n_gp);
+    double *recs = (double *)(c.arena + L.recs);
+    double *scr = (double *)(c.arena + L.scratch);
+    XsKey *keys = (XsKey *)(c.arena + L.keys);
+    uint32_t *bkt = (uint32_t *)(c.arena + L.bkt);
+    int *ig = (int *)(c.arena + L.index);
+    const bool uni = p.grid == XS_UNIONIZED;
+
+    for (long long b = tid; b < NB; b += T) bkt[b] = 0;
+    if (p.grid == XS_HASH)
+      for (long long x = tid; x < (long long)n_iso * (p.bins + 1); x += T) ig[x] = 0;
+    __syncthreads();
+    // (G) generate + count
+    {
+      const Affine J6T = lcg_pow(6ULL * T);
+      uint64_t s = lcg_pow(6ULL * tid)(p.gseed);
+      for (long long r = tid; r < n_u; r += T, s = J6T(s)) {
         uint64_t t = s;
         double v[6];
 #pragma unroll
         for (int f = 0; f < 6; f++) v[f] = lcg_double(t);
-        double2 *d = reinterpret_cast<double2 *>(scr + 6 * (size_t)j);
+        double2 *d = reinterpret_cast<double2 *>(scr + 6 * r);
         d[0] = make_double2(v[0], v[1]);
         d[1] = make_double2(v[2], v[3]);
         d[2] = make_double2(v[4], v[5]);
-        const int b = min((int)(v[0] * NB), NB - 1);
-        atomicAdd(&bkt[b], 1u);
+        atomicAdd(&bkt[bucket_of(v[0], r, n_gp, uni, NB, nbn)], 1u);
       }
-      s_nuc = Jnuc(s_nuc);
-      __syncthreads();
-      // (b) XS-4 sort: bucket offsets, scatter, per-bucket insertion sort
-      block_exclusive_scan(bkt, NB, c.sh);
-      for (int j = tid; j < n_gp; j += T) {
-        const double e = ld_(scr + 6 * (size_t)j);
-        const int b = min((int)(e * NB), NB - 1);
-        const uint32_t pos = atomicAdd(&bkt[b], 1u);
-        XsKey k;
-        k.key = dbits(e);
-        k.idx = (unsigned)j;
-        k.pad = 0;
-        keys[pos] = k;
+    }
+    __syncthreads();
+    XS_STOP(1);
+    // (S) bucket offsets
+    global_exclusive_scan(bkt, NB, c.sh);
+    XS_STOP(2);
+    // (P) scatter
+    for (long long r0 = tid; r0 < n_u; r0 += 4LL * T) {  // 4 independent atomics in flight
+      double e[4];
+      uint32_t pos[4];
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        const long long r = r0 + (long long)q * T;
+        e[q] = r < n_u ? ld_(scr + 6 * r) : 0.0;
       }
-      __syncthreads();
-      for (int b = tid; b < NB; b += T) {  // bkt[b] is now the end of bucket b
-        const int lo = b ? (int)bkt[b - 1] : 0, hi = (int)bkt[b];
-        for (int x = lo + 1; x < hi; x++) {
-          XsKey v = keys[x];
-          int y = x - 1;
-          while (y >= lo && keys[y].key > v.key) {
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        const long long r = r0 + (long long)q * T;
+        if (r < n_u) pos[q] = atomicAdd(&bkt[bucket_of(e[q], r, n_gp, uni, NB, nbn)], 1u);
+      }
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        const long long r = r0 + (long long)q * T;
+        if (r < n_u) {
+          XsKey k;
+          k.key = dbits(e[q]);
+          k.idx = (unsigned)r;
+          k.pad = 0;
+          keys[pos[q]] = k;
+        }
+      }
+    }
+    __syncthreads();
+    XS_STOP(3);
+    // (B) sort each bucket by (energy, record id); bkt[b] = end of bucket b.
+    // Buckets hold ~2 keys: up to 8 are sorted in registers, more in memory.
+    for (long long b = tid; b < NB; b += T) {
+      const long long lo = b ? (long long)bkt[b - 1] : 0, hi = (long long)bkt[b];
+      const int cnt = (int)(hi - lo);
+      if (cnt <= 1) continue;
+      if (cnt <= 8) {
+        unsigned long long kk[8];
+        unsigned ii[8];
+#pragma unroll
+        for (int q = 0; q < 8; q++)
+          if (q < cnt) {
+            const XsKey v = keys[lo + q];
+            kk[q] = v.key;
+            ii[q] = v.idx;
+          }
+#pragma unroll
+        for (int x = 1; x < 8; x++) {  // insertion sort, fully unrolled
+#pragma unroll
+          for (int y = x; y > 0; y--) {
+            if (x < cnt) {
+              const bool sw = kk[y - 1] > kk[y] || (kk[y - 1] == kk[y] && ii[y - 1] > ii[y]);
+              if (sw) {
+                const unsigned long long tk = kk[y - 1];
+                kk[y - 1] = kk[y];
+                kk[y] = tk;
+                const unsigned ti = ii[y - 1];
+                ii[y - 1] = ii[y];
+                ii[y] = ti;
+              }
+            }
+          }
+        }
+#pragma unroll
+        for (int q = 0; q < 8; q++)
+          if (q < cnt) {
+            XsKey v;
+            v.key = kk[q];
+            v.idx = ii[q];
+            v.pad = 0;
+            keys[lo + q] = v;
+          }
+      } else {
+        for (long long x = lo + 1; x < hi; x++) {
+          const XsKey v = keys[x];
+          long long y = x - 1;
+          while (y >= lo && (keys[y].key > v.key || (keys[y].key == v.key && keys[y].idx > v.idx))) {
             keys[y + 1] = keys[y];
             y--;
           }
           keys[y + 1] = v;
         }
       }
-      __syncthreads();
-      // (c) scatter the records to their sorted position
-      double *rec_i = recs + (size_t)i * n_gp * 6;
-      for (int k = tid; k < n_gp; k += T) {
-        const unsigned j = keys[k].idx;
-        const double2 *src = reinterpret_cast<const double2 *>(scr + 6 * (size_t)j);
-        double2 *dst = reinterpret_cast<double2 *>(rec_i + 6 * (size_t)k);
+    }
+    __syncthreads();
+
+    XS_STOP(4);
+    if (!uni) {
+      // (R) records to their sorted position: bucket order is nuclide-major
+      for (long long k = tid; k < n_u; k += T) {
+        const unsigned r = keys[k].idx;
+        const double2 *src = reinterpret_cast<const double2 *>(scr + 6 * (size_t)r);
+        double2 *dst = reinterpret_cast<double2 *>(recs + 6 * k);
         const double2 a = src[0], b = src[1], e = src[2];
         dst[0] = a;
         dst[1] = b;
         dst[2] = e;
       }
-      // (d) XS-5
-      if (p.grid == XS_HASH) {
-        // ig[i][b] = grid_search(E_i, b*du, 0, n_gp-1) = min(#{k>=1: E_k <= b*du}, n_gp-2),
-        // a merge walk over the sorted keys per contiguous chunk of bins
-        int *col = ig + (size_t)i * (p.bins + 1);
-        const int C = (p.bins + T - 1) / T;
-        const int b0 = tid * C, b1 = min(b0 + C, p.bins);
-        if (b0 < b1) {
-          const double q0 = (double)b0 * du;
-          int lo = 1, hi = n_gp;  // first k >= 1 with E_k > q0
-          while (lo < hi) {
-            const int mid = (lo + hi) >> 1;
-            if (__longlong_as_double((long long)keys[mid].key) <= q0) lo = mid + 1;
-            else hi = mid;
+      if (p.grid != XS_HASH) {
+        __syncthreads();
+        return;
+      }
+    XS_STOP(5);
+      // (H) hash grid ig[i][b] = grid_search(E_i, b*du, 0, n_gp-1)
+      //      = min(#{k >= 1 : E_i[k] <= b*du}, n_gp-2): histogram of each
+      //      energy's first bin b_k (smallest b with E_k <= b*du), then a
+      //      per-nuclide prefix sum over the bins.
+      const double du = 1.0 / p.bins;
+      for (long long k = tid; k < n_u; k += T) {
+        const int i = (int)(k / n_gp), kk = (int)(k % n_gp);
+        if (kk == 0) continue;
+        const double e = __longlong_as_double((long long)keys[k].key);
+        long long b = (long long)(e * p.bins);
+        while (b > 0 && (double)(b - 1) * du >= e) b--;
+        while (b < p.bins && (double)b * du < e) b++;
+        if (b < p.bins) atomicAdd((unsigned *)&ig[(size_t)i * (p.bins + 1) + b], 1u);
+      }
+      __syncthreads();
+      {
+        const int lane = tid & 31, warp = tid >> 5, nw = T >> 5;
+        constexpr int R = 16;  // rows of 32 bins loaded per step (coalesced)
+        for (int i = warp; i < n_iso; i += nw) {
+          int *col = ig + (size_t)i * (p.bins + 1);
+          int carry = 0;  // inclusive prefix of all earlier bins
+          for (int b0 = 0; b0 < p.bins; b0 += 32 * R) {
+            int v[R];
+#pragma unroll
+            for (int q = 0; q < R; q++) {
+              const int b = b0 + 32 * q + lane;
+              v[q] = b < p.bins ? col[b] : 0;
+            }
+#pragma unroll
+            for (int q = 0; q < R; q++) {
+              int inc = v[q];
+              for (int o = 1; o < 32; o <<= 1) {
+                const int t = __shfl_up_sync(0xffffffffu, inc, o);
+                if (lane >= o) inc += t;
+              }
+              const int run = carry + inc;
+              const int b = b0 + 32 * q + lane;
+              if (b < p.bins) col[b] = run < n_gp - 2 ? run : n_gp - 2;
+              carry = __shfl_sync(0xffffffffu, run, 31);
+            }
           }
-          int cnt = lo - 1;  // #{k >= 1 : E_k <= q0}
-          for (int b = b0; b < b1; b++) {
-            const double q = (double)b * du;
-            while (cnt < n_gp - 1 && __longlong_as_double((long long)keys[cnt + 1].key) <= q) cnt++;
-            col[b] = cnt < n_gp - 2 ? cnt : n_gp - 2;
-          }
-        }
-        if (tid == 0) col[p.bins] = n_gp - 2;
-      } else if (p.grid == XS_UNIONIZED) {
-        for (int k = tid; k < n_gp; k += T) {
-          urun[(size_t)i * n_gp + k] = keys[k].key;
-          orun[(size_t)i * n_gp + k] = (uint16_t)i;
+          if (lane == 0) col[p.bins] = n_gp - 2;
         }
       }
       __syncthreads();
+      return;
     }
 
-    if (p.grid != XS_UNIONIZED) return;
-    // ---- union: bottom-up merge of the n_iso sorted runs (merge path) ------
-    {
-      uint64_t *src = urun, *dst = (urun == uA) ? uB : uA;
-      uint16_t *osrc = orun, *odst = (orun == oA) ? oB : oA;
-      const int CH = 16;
-      for (long long w = n_gp; w < n_u; w <<= 1) {
-        for (long long c0 = (long long)tid * CH; c0 < n_u; c0 += (long long)T * CH) {
-          const long long c1 = (c0 + CH < n_u) ? c0 + CH : n_u;
-          for (long long o0 = c0; o0 < c1;) {  // a chunk may straddle merge pairs
-            const long long base = (o0 / (2 * w)) * (2 * w);
-            const long long la = (base + w < n_u) ? w : n_u - base;
-            const long long lb = (base + 2 * w < n_u) ? w : (n_u - base - la > 0 ? n_u - base - la : 0);
-            const uint64_t *A = src + base, *B = src + base + la;
-            const long long op = o0 - base;
-            long long lo = op - lb > 0 ? op - lb : 0, hi = op < la ? op : la;
-            while (lo < hi) {
-              const long long mid = (lo + hi) >> 1;
-              if (A[mid] < B[op - 1 - mid]) lo = mid + 1;
-              else hi = mid;
-            }
-            long long ia = lo, ib = op - lo;
-            const long long end = (c1 < base + la + lb) ? c1 : base + la + lb;
-            for (long long o = o0; o < end; o++) {
-              if (ia < la && (ib >= lb || A[ia] < B[ib])) {
-                dst[o] = A[ia];
-                odst[o] = osrc[base + ia];
-                ia++;
-              } else {
-                dst[o] = B[ib];
-                odst[o] = osrc[base + la + ib];
-                ib++;
-              }
-            }
-            o0 = end;
-          }
-        }
-        __syncthreads();
-        uint64_t *t = src; src = dst; dst = t;
-        uint16_t *to = osrc; osrc = odst; odst = to;
+    // ---- unionized: keys[] is the union (XS-5); owner = record id / n_gp ----
+    uint64_t *uA = (uint64_t *)(c.arena + L.uenergy);
+    uint32_t *chist = (uint32_t *)(c.arena + L.chist);
+    const long long nch = (n_u + kXsSweepRows - 1) / kXsSweepRows;
+    for (long long x = tid; x < nch * n_iso; x += T) chist[x] = 0;
+    __syncthreads();
+    XS_STOP(5);
+    for (long long e = tid; e < n_u; e += T) {  // union energies + chunk owner counts
+      const XsKey k = keys[e];
+      uA[e] = k.key;
+      atomicAdd(&chist[(e / kXsSweepRows) * n_iso + k.idx / n_gp], 1u);
+    }
+    __syncthreads();
+    for (int i = tid; i < n_iso; i += T) {  // exclusive scan over chunks per owner
+      uint32_t run = 0;
+      for (long long ch = 0; ch < nch; ch++) {
+        const uint32_t v = chist[ch * n_iso + i];
+        chist[ch * n_iso + i] = run;
+        run += v;
       }
     }
-    // ---- index grid: ig[e][i] = clip(#{k>=1: E_i[k] <= u_e}, 0, n_gp-2), a
-    // warp sweeps a chunk of rows, lanes own nuclides (coalesced row stores)
+    __syncthreads();
+    XS_STOP(6);
+    // sweep: a warp per chunk, lanes own nuclides; row e of the index grid is
+    // clip(#{k>=1: E_i[k] <= u_e}, 0, n_gp-2) = clip(cnt_i(e) - 1, ...), and
+    // the owner's new count is the sorted position of that record (XS-4).
     {
       const int lane = tid & 31, warp = tid >> 5, nw = T >> 5;
-      const long long per = (n_u + nw * 4 - 1) / (nw * 4);
-      const long long C = per > 512 ? per : 512;
-      const long long ntask = (n_u + C - 1) / C;
-      for (long long task = warp; task < ntask; task += nw) {
-        const long long e0 = task * C, e1 = (e0 + C < n_u) ? e0 + C : n_u;
+      for (long long ch = warp; ch < nch; ch += nw) {
+        const long long e0 = ch * kXsSweepRows, e1 = (e0 + kXsSweepRows < n_u) ? e0 + kXsSweepRows : n_u;
         int cnt[12];
-        const double ue0 = __longlong_as_double((long long)uA[e0]);
 #pragma unroll
         for (int m = 0; m < 12; m++) {
           const int i = lane + 32 * m;
-          cnt[m] = 0;
-          if (i < n_iso) {  // #{k : E_i[k] < u[e0]}
-            const double *E = recs + (size_t)i * n_gp * 6;
-            int lo = 0, hi = n_gp;
-            while (lo < hi) {
-              const int mid = (lo + hi) >> 1;
-              if (ld_(E + 6 * (size_t)mid) < ue0) lo = mid + 1;
-              else hi = mid;
-            }
-            cnt[m] = lo;
-          }
+          cnt[m] = i < n_iso ? (int)chist[ch * n_iso + i] : 0;
         }
-        for (long long e = e0; e < e1; e++) {
-          const int own = oA[e];
-          int *row = ig + (size_t)e * n_iso;
+        // owners of the next 32 rows are prefetched while this group is swept
+        int own_next = e0 + lane < e1 ? (int)(keys[e0 + lane].idx / (unsigned)n_gp) : -1;
+        for (long long g = e0; g < e1; g += 32) {
+          const int own_cur = own_next;
+          own_next = g + 32 + lane < e1 ? (int)(keys[g + 32 + lane].idx / (unsigned)n_gp) : -1;
+          const int ng = (int)(e1 - g < 32 ? e1 - g : 32);
+          for (int sl = 0; sl < ng; sl++) {
+            const long long e = g + sl;
+            const int own = __shfl_sync(0xffffffffu, own_cur, sl);
+            int *row = ig + (size_t)e * n_iso;
 #pragma unroll
-          for (int m = 0; m < 12; m++) {
-            const int i = lane + 32 * m;
-            if (i < n_iso) {
-              if (own == i) cnt[m]++;
-              int v = cnt[m] - 1;
-              v = v < 0 ? 0 : (v > n_gp - 2 ? n_gp - 2 : v);
-              row[i] = v;
+            for (int m = 0; m < 12; m++) {
+              const int i = lane + 32 * m;
+              if (i < n_iso) {
+                if (own == i) {  // sorted position of this record (XS-4)
+                  keys[e].pad = (unsigned)((size_t)i * n_gp + cnt[m]);
+                  cnt[m]++;
+                }
+                int v = cnt[m] - 1;
+                v = v < 0 ? 0 : (v > n_gp - 2 ? n_gp - 2 : v);
+                row[i] = v;
+              }
             }
           }
         }
       }
-      __syncthreads();
     }
+    __syncthreads();
+    // records to their sorted positions (coalesced over the union order)
+    for (long long e = tid; e < n_u; e += T) {
+      const XsKey k = keys[e];
+      const double2 *src = reinterpret_cast<const double2 *>(scr + 6 * (size_t)k.idx);
+      double2 *dst = reinterpret_cast<double2 *>(recs + 6 * (size_t)k.pad);
+      const double2 a = src[0], b = src[1], x = src[2];
+      dst[0] = a;
+      dst[1] = b;
+      dst[2] = x;
+    }
+    __syncthreads();
   }
 
   // ---- XS-6..XS-10: lookups ----------------------------------------------
