@@ -304,6 +304,48 @@ struct XsApp {
     }
   }
 
+  // Unionized index grid sweep: a warp per chunk of union rows, lane l owns
+  // nuclides l, l+32, ... (NM = ceil(n_iso/32) of them, counts in registers);
+  // row e is ig[e][i] = clip(cnt_i(e) - 1, 0, n_gp-2) with cnt_i(e) =
+  // #{k: E_i[k] <= u_e}, and the owner's count before its increment is the
+  // sorted position of that record (stored in keys[e].pad).  Branch-free.
+  template <int NM>
+  __device__ static __forceinline__ void sweep(XsKey *keys, const uint32_t *chist, int *ig, long long n_u, int n_iso,
+                                               int n_gp, long long nch) {
+    const int tid = threadIdx.x, T = blockDim.x, lane = tid & 31, warp = tid >> 5, nw = T >> 5;
+    for (long long ch = warp; ch < nch; ch += nw) {
+      const long long e0 = ch * kXsSweepRows, e1 = (e0 + kXsSweepRows < n_u) ? e0 + kXsSweepRows : n_u;
+      int cnt[NM];
+#pragma unroll
+      for (int m = 0; m < NM; m++) {
+        const int i = lane + 32 * m;
+        cnt[m] = i < n_iso ? (int)chist[ch * n_iso + i] : 0;
+      }
+      // owners of the next 32 rows are prefetched while this group is swept
+      int own_next = e0 + lane < e1 ? (int)(keys[e0 + lane].idx / (unsigned)n_gp) : -1;
+      for (long long g = e0; g < e1; g += 32) {
+        const int own_cur = own_next;
+        own_next = g + 32 + lane < e1 ? (int)(keys[g + 32 + lane].idx / (unsigned)n_gp) : -1;
+        const int ng = (int)(e1 - g < 32 ? e1 - g : 32);
+        int *row = ig + (size_t)g * n_iso;
+        for (int sl = 0; sl < ng; sl++, row += n_iso) {
+          const int own = __shfl_sync(0xffffffffu, own_cur, sl);
+          int pos = -1;
+#pragma unroll
+          for (int m = 0; m < NM; m++) {
+            const int i = lane + 32 * m;
+            const int hit = own == i;
+            pos = hit ? i * n_gp + cnt[m] : pos;
+            cnt[m] += hit;
+            const int v = cnt[m] - 1;
+            if (i < n_iso) row[i] = v < 0 ? 0 : (v > n_gp - 2 ? n_gp - 2 : v);
+          }
+          if (pos >= 0) keys[g + sl].pad = (unsigned)pos;
+        }
+      }
+    }
+  }
+
   // ---- XS-3/4/5, hash and nuclide grids: one nuclide at a time -------------
   // Nuclide i's n_gp records (draws 6r+1..6r+6, r = i*n_gp + j; XS-3) are
   // generated into an L2-resident scratch, bucket-sorted by energy (XS-4:
@@ -636,44 +678,10 @@ struct XsApp {
     // sweep: a warp per chunk, lanes own nuclides; row e of the index grid is
     // clip(#{k>=1: E_i[k] <= u_e}, 0, n_gp-2) = clip(cnt_i(e) - 1, ...), and
     // the owner's new count is the sorted position of that record (XS-4).
-    {
-      const int lane = tid & 31, warp = tid >> 5, nw = T >> 5;
-      for (long long ch = warp; ch < nch; ch += nw) {
-        const long long e0 = ch * kXsSweepRows, e1 = (e0 + kXsSweepRows < n_u) ? e0 + kXsSweepRows : n_u;
-        int cnt[12];
-#pragma unroll
-        for (int m = 0; m < 12; m++) {
-          const int i = lane + 32 * m;
-          cnt[m] = i < n_iso ? (int)chist[ch * n_iso + i] : 0;
-        }
-        // owners of the next 32 rows are prefetched while this group is swept
-        int own_next = e0 + lane < e1 ? (int)(keys[e0 + lane].idx / (unsigned)n_gp) : -1;
-        for (long long g = e0; g < e1; g += 32) {
-          const int own_cur = own_next;
-          own_next = g + 32 + lane < e1 ? (int)(keys[g + 32 + lane].idx / (unsigned)n_gp) : -1;
-          const int ng = (int)(e1 - g < 32 ? e1 - g : 32);
-          for (int sl = 0; sl < ng; sl++) {
-            const long long e = g + sl;
-            const int own = __shfl_sync(0xffffffffu, own_cur, sl);
-            int *row = ig + (size_t)e * n_iso;
-#pragma unroll
-            for (int m = 0; m < 12; m++) {
-              const int i = lane + 32 * m;
-              if (i < n_iso) {
-                if (own == i) {  // sorted position of this record (XS-4)
-                  keys[e].pad = (unsigned)((size_t)i * n_gp + cnt[m]);
-                  cnt[m]++;
-                }
-                int v = cnt[m] - 1;
-                v = v < 0 ? 0 : (v > n_gp - 2 ? n_gp - 2 : v);
-                row[i] = v;
-              }
-            }
-          }
-        }
-      }
-    }
+    if (n_iso <= 96) sweep<3>(keys, chist, ig, n_u, n_iso, n_gp, nch);
+    else sweep<12>(keys, chist, ig, n_u, n_iso, n_gp, nch);
     __syncthreads();
+    XS_STOP(7);
     // records to their sorted positions (coalesced over the union order)
     for (long long e = tid; e < n_u; e += T) {
       const XsKey k = keys[e];
