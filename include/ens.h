@@ -110,6 +110,10 @@ typedef struct {
   uint64_t arena_bytes;
   uint32_t stdout_bytes;
   uint32_t flags;
+  int32_t team_ctas;  /* CTAs per team for team-aware bodies (XSBench): 1, 2,
+                         4 or 8 (a thread-block cluster with distributed shared
+                         memory); 0 = auto (largest power of two <= 8 with
+                         n x team_ctas <= resident CTAs), ignored by other apps */
 } ens_launch_cfg;
 
 /* Device bytes ens_launch needs for (app, a, c).  With c->grid_blocks == 0
@@ -167,7 +171,7 @@ int ens_run_elapsed_ms(ens_run *r, float *ms);
 typedef struct {
   int32_t n_instances;
   int32_t n_groups;        /* kernel launches (one per app present)            */
-  int32_t grid_blocks[5];  /* per ens_app, 0 if absent                           */
+  int32_t grid_blocks[5];  /* CTAs launched, per ens_app, 0 if absent            */
   int32_t block_threads[5];
   int32_t kernel_launches; /* kernels per (re)launch                             */
   uint64_t arena_bytes;    /* per slot (max over groups)                         */
@@ -178,6 +182,7 @@ typedef struct {
   uint32_t stdout_bytes;   /* raw stdout bytes per instance                      */
   uint64_t h2d_bytes;      /* bytes copied host->device by ens_launch            */
   uint64_t d2h_bytes;      /* bytes copied device->host by the last ens_collect  */
+  int32_t team_ctas[5];    /* CTAs per team (cluster size), per ens_app           */
 } ens_run_info;
 int ens_run_get_info(const ens_run *r, ens_run_info *info);
 

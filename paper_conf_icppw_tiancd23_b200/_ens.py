@@ -40,7 +40,8 @@ class EnsError(RuntimeError):
 class LaunchCfg(ctypes.Structure):
     _fields_ = [("first", ctypes.c_int32), ("n_instances", ctypes.c_int32), ("stride", ctypes.c_int32),
                 ("grid_blocks", ctypes.c_int32), ("block_threads", ctypes.c_int32),
-                ("arena_bytes", ctypes.c_uint64), ("stdout_bytes", ctypes.c_uint32), ("flags", ctypes.c_uint32)]
+                ("arena_bytes", ctypes.c_uint64), ("stdout_bytes", ctypes.c_uint32), ("flags", ctypes.c_uint32),
+                ("team_ctas", ctypes.c_int32)]
 
 
 class RunInfo(ctypes.Structure):
@@ -50,7 +51,7 @@ class RunInfo(ctypes.Structure):
                 ("ws_bytes", ctypes.c_uint64), ("records_offset", ctypes.c_uint64),
                 ("tallies_offset", ctypes.c_uint64), ("stdout_offset", ctypes.c_uint64),
                 ("stdout_bytes", ctypes.c_uint32), ("h2d_bytes", ctypes.c_uint64),
-                ("d2h_bytes", ctypes.c_uint64)]
+                ("d2h_bytes", ctypes.c_uint64), ("team_ctas", ctypes.c_int32 * 5)]
 
 
 def _load():
@@ -149,8 +150,8 @@ class Args:
             pass
 
 
-def make_cfg(n, first=0, stride=1, grid=0, threads=0, arena_bytes=0, stdout_bytes=0, flags=0):
-    return LaunchCfg(first, n, stride, grid, threads, arena_bytes, stdout_bytes, flags)
+def make_cfg(n, first=0, stride=1, grid=0, threads=0, arena_bytes=0, stdout_bytes=0, flags=0, team_ctas=0):
+    return LaunchCfg(first, n, stride, grid, threads, arena_bytes, stdout_bytes, flags, team_ctas)
 
 
 def workspace_bytes(app, args, cfg):

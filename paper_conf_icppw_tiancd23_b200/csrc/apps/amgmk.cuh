@@ -18,6 +18,7 @@ namespace ens {
 struct AmgApp {
   static constexpr uint32_t kId = APP_AMGMK;
   static constexpr int kMaxT = 1024;  // 64 registers suffice
+  static constexpr bool kTeam = false;
 
   __device__ static Result run(Ctx &c, int argc, char **argv) {
     Result R{};
@@ -137,7 +138,7 @@ struct AmgApp {
     return R;
   }
 
-  __host__ static bool size(int argc, const char *const *argv, int, uint64_t *arena, uint32_t *smem) {
+  __host__ static bool size(int argc, const char *const *argv, int, int, uint64_t *arena, uint32_t *smem) {
     AmgParams p;
     *smem = 0;
     if (amg_parse(argc, argv, p) >= 0) {

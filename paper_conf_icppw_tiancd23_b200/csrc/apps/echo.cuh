@@ -11,6 +11,7 @@ namespace ens {
 struct EchoApp {
   static constexpr uint32_t kId = APP_ECHO;
   static constexpr int kMaxT = 1024;
+  static constexpr bool kTeam = false;
   __device__ static Result run(Ctx &c, int argc, char **argv) {
     Result R{};
     ens_printf(c, FMT_ECHO_ARGC, argc);
@@ -19,7 +20,7 @@ struct EchoApp {
     R.work = (uint64_t)argc;
     return R;
   }
-  __host__ static bool size(int, const char *const *, int, uint64_t *arena, uint32_t *smem) {
+  __host__ static bool size(int, const char *const *, int, int, uint64_t *arena, uint32_t *smem) {
     *arena = 0;
     *smem = 0;
     return true;
@@ -29,13 +30,14 @@ struct EchoApp {
 struct NotFoundApp {
   static constexpr uint32_t kId = APP_NOTFOUND;
   static constexpr int kMaxT = 1024;
+  static constexpr bool kTeam = false;
   __device__ static Result run(Ctx &c, int argc, char **argv) {
     Result R{};
     ens_printf(c, FMT_NOTFOUND, argc > 0 ? (const char *)argv[0] : "");
     R.exit_code = ENS_EXIT_NOTFOUND;
     return R;
   }
-  __host__ static bool size(int, const char *const *, int, uint64_t *arena, uint32_t *smem) {
+  __host__ static bool size(int, const char *const *, int, int, uint64_t *arena, uint32_t *smem) {
     *arena = 0;
     *smem = 0;
     return true;

@@ -100,12 +100,14 @@ struct XsLayout {
   uint64_t index;     // unionized [n_u][n_iso] / hash [n_iso][bins+1] int32
   uint64_t total;
 };
-ENS_HD XsLayout xs_layout(const XsParams &p) {
+// cs = CTAs in the team: hash / nuclide grids give each CTA its own
+// per-nuclide scratch
+ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
   XsLayout L{};
   const uint64_t n_u = (uint64_t)p.n_iso * p.n_gp;
   uint64_t o = 0;
   // unionized: one sort of all n_u records; otherwise one nuclide at a time
-  const uint64_t n_s = p.grid == XS_UNIONIZED ? n_u : (uint64_t)p.n_gp;
+  const uint64_t n_s = p.grid == XS_UNIONIZED ? n_u : (uint64_t)p.n_gp * (uint64_t)cs;
   L.recs = o; o = align_up(o + n_u * 48, 256);
   L.scratch = o; o = align_up(o + n_s * 48, 256);
   L.keys = o; o = align_up(o + n_s * 16, 256);

@@ -213,6 +213,7 @@ struct XsApp {
   // thread limit is an upper bound: 512 keeps 128 registers
   static constexpr int kMaxT = 512;
   static constexpr int kU = kXsU;
+  static constexpr bool kTeam = true;  // splits nuclides and lookup batches over a cluster
 
   __device__ static Result run(Ctx &c, int argc, char **argv) {
     Result R{};
@@ -224,7 +225,7 @@ struct XsApp {
       R.exit_code = ENS_EXIT_USAGE;
       return R;
     }
-    const XsLayout L = xs_layout(p);
+    const XsLayout L = xs_layout(p, c.csize);
     if (L.total > c.arena_cap) {
       if (threadIdx.x == 0) c.sh->flags |= 2u;  // ENS_RF_NOMEM
       R.exit_code = ENS_EXIT_NOMEM;
@@ -241,8 +242,12 @@ struct XsApp {
     hm_tables(n_iso, mx, thr, nn, concs, mats);
     __syncthreads();
     hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
-    if (p.grid == XS_UNIONIZED) init(c, p, L, S);
-    else init_nuc(c, p, L, S);
+    if (p.grid == XS_UNIONIZED) {
+      if (c.crank == 0) init(c, p, L, S);  // one CTA builds the union
+    } else {
+      init_nuc(c, p, L, S);  // nuclides striped over the team's CTAs
+    }
+    team_sync(c);
     if (p.grid == XS_HASH) lookups<XS_HASH>(c, p, L, thr, nn, concs, mats, R);
     else if (p.grid == XS_UNIONIZED) lookups<XS_UNIONIZED>(c, p, L, thr, nn, concs, mats, R);
     else lookups<XS_NUCLIDE>(c, p, L, thr, nn, concs, mats, R);
@@ -365,9 +370,12 @@ struct XsApp {
     const bool hash = p.grid == XS_HASH;
     const double du = 1.0 / p.bins;
     const Affine J6T = lcg_pow(6ULL * T);
-    const Affine Jnuc = lcg_pow(6ULL * n_gp);
-    uint64_t s_nuc = lcg_pow(6ULL * tid)(p.gseed);  // before record (i*n_gp + tid)
-    for (int i = 0; i < n_iso; i++) {
+    // this CTA takes nuclides crank, crank + csize, ... with its own scratch
+    scr += (size_t)c.crank * n_gp * 6;
+    keys += (size_t)c.crank * n_gp;
+    const Affine Jnuc = lcg_pow(6ULL * n_gp * c.csize);
+    uint64_t s_nuc = lcg_pow(6ULL * ((uint64_t)c.crank * n_gp + tid))(p.gseed);  // record (i*n_gp + tid)
+    for (int i = (int)c.crank; i < n_iso; i += (int)c.csize) {
       int *col = ig + (size_t)i * (p.bins + 1);
       for (int b = tid; b < nbn; b += T) nb[b] = 0;
       if (hash)
@@ -722,7 +730,7 @@ struct XsApp {
     double fsum = 0.0, fabs_ = 0.0;
     const long long NBt = (long long)K * T;
     const Affine JT = lcg_pow(2ULL * T);
-    for (long long b0 = 0; b0 < nL; b0 += NBt) {
+    for (long long b0 = (long long)c.crank * NBt; b0 < nL; b0 += NBt * c.csize) {  // batches striped over the team
       const int nb = (int)((nL - b0 < NBt) ? nL - b0 : NBt);
       if (tid < 12) mcnt[tid] = 0;
       __syncthreads();
@@ -859,10 +867,10 @@ struct XsApp {
       }
       __syncthreads();  // slots reused by the next batch
     }
-    ver = block_sum_u64(c.sh, ver);
-    bsum = block_sum_u64(c.sh, bsum);
-    fsum = block_sum_f64(c.sh, fsum);
-    fabs_ = block_sum_f64(c.sh, fabs_);
+    ver = team_sum_u64(c, ver);
+    bsum = team_sum_u64(c, bsum);
+    fsum = team_sum_f64(c, fsum);
+    fabs_ = team_sum_f64(c, fabs_);
     R.vhash = ver % 999983ULL;
     R.bitsum = bsum;
     R.fsum = fsum;
@@ -870,14 +878,14 @@ struct XsApp {
     R.work = (uint64_t)p.lookups;
   }
 
-  __host__ static bool size(int argc, const char *const *argv, int T, uint64_t *arena, uint32_t *smem) {
+  __host__ static bool size(int argc, const char *const *argv, int T, int cs, uint64_t *arena, uint32_t *smem) {
     XsParams p;
     if (xs_parse(argc, argv, p) >= 0) {
       *arena = 0;
       *smem = 0;
       return false;
     }
-    *arena = xs_layout(p).total;
+    *arena = xs_layout(p, cs).total;
     *smem = xs_smem(p, T).total;
     return true;
   }

@@ -155,7 +155,8 @@ extern "C" void ens_args_free(ens_args *a) { delete a; }
 // ---------------------------------------------------------------------------
 struct Group {
   uint32_t app = 0;
-  int T = 0, grid = 0;
+  int T = 0, grid = 0;  // grid = teams (arena slots); CTAs launched = grid * cs
+  int cs = 1;           // CTAs per team (cluster size)
   uint32_t smem = 0;
   uint64_t arena = 0;
   std::vector<uint32_t> kmap;
@@ -228,8 +229,8 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceGetAttribute");
 
+  // group instances by app; shared memory per group (independent of team size)
   Group g_by_app[6];
-  uint64_t need_arena = 0;
   P.line_of_k.resize((size_t)n);
   for (int64_t k = 0; k < n; k++) {
     const uint32_t line = (uint32_t)(first + k * stride);
@@ -241,29 +242,56 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     if (app == ENS_APP_BY_ARGV0) ap = argc > 0 ? app_of_argv0(argv[0]) : (uint32_t)APP_NOTFOUND;
     uint64_t ar = 0;
     uint32_t sm = 0;
-    app_size(ap, argc, argv, std::min(T, app_max_threads(ap)), &ar, &sm);
+    app_size(ap, argc, argv, std::min(T, app_max_threads(ap)), 1, &ar, &sm);
     Group &g = g_by_app[ap];
     g.app = ap;
-    g.arena = std::max(g.arena, ar);
     g.smem = std::max(g.smem, sm);
     g.kmap.push_back((uint32_t)k);
-    need_arena = std::max(need_arena, ar);
   }
-  P.arena_bytes = c->arena_bytes ? al(c->arena_bytes) : al(need_arena);
+  // team size: team-aware bodies get a cluster of cs CTAs when the group has
+  // fewer instances than resident CTAs (the largest power of two <= 8 with
+  // n_group * cs <= resident CTAs), or the cfg's team_ctas
+  uint64_t need_arena = 0;
   for (uint32_t ap : {(uint32_t)APP_XSBENCH, (uint32_t)APP_RSBENCH, (uint32_t)APP_AMGMK, (uint32_t)APP_ECHO,
                       (uint32_t)APP_NOTFOUND}) {
     Group &g = g_by_app[ap];
     if (g.kmap.empty()) continue;
     g.T = std::min(T, app_max_threads(ap));
-    int occ = 0;
-    e = group_occupancy(ap, g.T, g.smem, &occ);
+    int ctas = 0;
+    e = group_occupancy(ap, g.T, 1, g.smem, &ctas);
     if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor");
-    if (occ <= 0) return fail(ENS_EINVAL, "ens_launch: an instance needs more shared memory than one SM has");
-    int grid = c->grid_blocks ? c->grid_blocks : occ * sms;
-    grid = std::min<int64_t>(grid, (int64_t)g.kmap.size());
+    if (ctas <= 0) return fail(ENS_EINVAL, "ens_launch: an instance needs more shared memory than one SM has");
+    int cs = 1;
+    if (app_team_aware(ap)) {
+      if (c->team_ctas > 0) {
+        while (cs * 2 <= c->team_ctas && cs < kMaxTeamCtas) cs *= 2;
+      } else if (!c->grid_blocks) {
+        while (cs < kMaxTeamCtas && (int64_t)g.kmap.size() * cs * 2 <= ctas) cs *= 2;
+      }
+    }
+    int teams = ctas;
+    if (cs > 1) {
+      e = group_occupancy(ap, g.T, cs, g.smem, &teams);
+      if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters");
+      if (teams <= 0) cs = 1, teams = ctas;
+    }
+    g.cs = cs;
+    int grid = c->grid_blocks ? std::max(1, c->grid_blocks / cs) : teams;
+    grid = (int)std::min<int64_t>(grid, (int64_t)g.kmap.size());
     g.grid = std::max(grid, 1);
+    for (uint32_t k : g.kmap) {  // arena of this team size
+      int argc;
+      const char *const *argv;
+      ens_args_get(a, (int)P.line_of_k[k], &argc, &argv);
+      uint64_t ar = 0;
+      uint32_t sm = 0;
+      app_size(ap, argc, argv, g.T, cs, &ar, &sm);
+      g.arena = std::max(g.arena, ar);
+    }
+    need_arena = std::max(need_arena, g.arena);
     P.groups.push_back(g);
   }
+  P.arena_bytes = c->arena_bytes ? al(c->arena_bytes) : al(need_arena);
   // layout: staged part
   size_t o = 0;
   P.o_blob = o; o = al(o + a->blob.size());
@@ -341,7 +369,8 @@ static int enqueue(ens_run *r) {
     k.stdout_cap = P.stdout_cap;
     k.arena_base = r->ws + P.o_arena;
     k.arena_bytes = P.arena_bytes;
-    cudaError_t e = launch_group(g.app, g.T, g.grid, g.smem, k, r->stream);
+    k.team_ctas = (uint32_t)g.cs;
+    cudaError_t e = launch_group(g.app, g.T, g.grid * g.cs, g.cs, g.smem, k, r->stream);
     if (e != cudaSuccess) return cuda_fail(e, "ens_kernel launch");
   }
   CU(cudaEventRecord(r->ev1, r->stream));
@@ -500,7 +529,8 @@ extern "C" int ens_run_get_info(const ens_run *r, ens_run_info *info) {
   info->n_groups = (int32_t)P.groups.size();
   for (const Group &g : P.groups) {
     const uint32_t ap = g.app == APP_NOTFOUND ? 0u : g.app;
-    info->grid_blocks[ap] = g.grid;
+    info->grid_blocks[ap] = g.grid * g.cs;
+    info->team_ctas[ap] = g.cs;
     info->block_threads[ap] = g.T;
   }
   info->kernel_launches = (int32_t)P.groups.size();

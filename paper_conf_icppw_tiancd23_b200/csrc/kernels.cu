@@ -3,10 +3,12 @@
 // The paper maps NI instances onto N teams with `target teams distribute
 // num_teams(N) thread_limit(T)` (Fig. 4), one team = one CUDA
 // thread block (§2.3), with N = NI in its evaluation.
-// Here the grid is persistent: min(NI, occupancy x 148) blocks pull instance
-// slots from an atomic counter (reading Q5), so NI may exceed the blocks that
-// fit at once, and each block's heap arena is a fixed slot of the workspace
-// (memory = resident blocks x arena, not NI x arena).
+// Here the grid is persistent: min(NI, occupancy x 148) teams pull instance
+// slots from an atomic counter (reading Q5), so NI may exceed the teams that
+// fit at once, and each team's heap arena is a fixed slot of the workspace
+// (memory = resident teams x arena, not NI x arena).
+// A team is one CTA, or (team-aware bodies, ensembles with fewer instances
+// than SMs) a thread-block cluster of up to 8 CTAs (see rt/device_rt.cuh).
 #include <cuda_runtime.h>
 
 #include "apps/amgmk.cuh"
@@ -36,12 +38,23 @@ __global__ void __launch_bounds__(T, (512 / T) > 0 ? (512 / T) : 1) ens_kernel(c
   __shared__ unsigned long long s_pos;
   __shared__ Shared sh;
   const int tid = threadIdx.x;
-  char *const arena = p.arena_base + (size_t)blockIdx.x * p.arena_bytes;
+  const uint32_t cs = p.team_ctas;  // cluster dims (cs, 1, 1)
+  const uint32_t cr = cs > 1 ? cooperative_groups::this_cluster().block_rank() : 0u;
+  char *const arena = p.arena_base + (size_t)(blockIdx.x / cs) * p.arena_bytes;
+  Ctx c;
+  c.arena = arena;
+  c.arena_cap = p.arena_bytes;
+  c.out_cap = p.stdout_cap;
+  c.sh = &sh;
+  c.smem = dsmem;
+  c.crank = cr;
+  c.csize = cs;
   for (;;) {
-    if (tid == 0) s_j = atomicAdd(p.counter, 1u);
-    __syncthreads();
-    const uint32_t j = s_j;
-    if (j >= p.n) break;  // block-uniform
+    if (tid == 0 && cr == 0) s_j = atomicAdd(p.counter, 1u);
+    team_sync(c);
+    const uint32_t j = cr == 0 ? s_j : *cta_shared(&s_j, 0);
+    if (cs > 1) team_sync(c);  // every rank has read s_j before rank 0 may exit
+    if (j >= p.n) break;       // team-uniform
     const uint32_t k = p.kmap[j];
     const uint32_t line = p.line_of_k[k];
     const uint32_t t0 = p.line_tok[line];
@@ -57,45 +70,45 @@ __global__ void __launch_bounds__(T, (512 / T) > 0 ? (512 / T) : 1) ens_kernel(c
     if ((p.flags & ENS_F_TIMESTAMPS) && tid == 0) t_start = globaltimer();
     __syncthreads();
 
-    Ctx c;
     c.k = k;
     c.id = line;
-    c.arena = arena;
-    c.arena_cap = p.arena_bytes;
     c.out = p.stdout_base + (size_t)k * p.stdout_cap;
-    c.out_cap = p.stdout_cap;
-    c.sh = &sh;
-    c.smem = dsmem;
-    const Result r = App::run(c, argc, s_argv);
-    __syncthreads();
+    Result r{};
+    if (App::kTeam || cr == 0) r = App::run(c, argc, s_argv);
+    team_sync(c);
+    if (cs > 1 && cr != 0 && tid < ENS_TALLIES && sh.tallies[tid])  // combine tallies into rank 0
+      atomicAdd(cta_shared(&sh.tallies[tid], 0), sh.tallies[tid]);
+    team_sync(c);
 
-    if (tid < ENS_TALLIES) p.tallies[(size_t)k * ENS_TALLIES + tid] = sh.tallies[tid];
-    if (tid == 0) {
-      ens_record rec;
-      rec.instance = line;
-      rec.exit_code = r.exit_code;
-      rec.app = App::kId == APP_NOTFOUND ? 0u : App::kId;
-      rec.flags = sh.flags | ENS_RF_DONE;
-      rec.vhash = r.vhash;
-      rec.bitsum = r.bitsum;
-      rec.fsum = r.fsum;
-      rec.fabs = r.fabs;
-      rec.work = r.work;
-      rec.stdout_len = sh.out_len;
-      rec.smid = (p.flags & ENS_F_TIMESTAMPS) ? smid() : 0u;
-      rec.t_start_ns = t_start;
-      rec.t_end_ns = (p.flags & ENS_F_TIMESTAMPS) ? globaltimer() : 0ull;
-      p.recs[k] = rec;
-      s_pos = atomicAdd(p.stdout_total, (unsigned long long)sh.out_len);
-      p.stdout_pos[k] = s_pos;
+    if (cr == 0) {
+      if (tid < ENS_TALLIES) p.tallies[(size_t)k * ENS_TALLIES + tid] = sh.tallies[tid];
+      if (tid == 0) {
+        ens_record rec;
+        rec.instance = line;
+        rec.exit_code = r.exit_code;
+        rec.app = App::kId == APP_NOTFOUND ? 0u : App::kId;
+        rec.flags = sh.flags | ENS_RF_DONE;
+        rec.vhash = r.vhash;
+        rec.bitsum = r.bitsum;
+        rec.fsum = r.fsum;
+        rec.fabs = r.fabs;
+        rec.work = r.work;
+        rec.stdout_len = sh.out_len;
+        rec.smid = (p.flags & ENS_F_TIMESTAMPS) ? smid() : 0u;
+        rec.t_start_ns = t_start;
+        rec.t_end_ns = (p.flags & ENS_F_TIMESTAMPS) ? globaltimer() : 0ull;
+        p.recs[k] = rec;
+        s_pos = atomicAdd(p.stdout_total, (unsigned long long)sh.out_len);
+        p.stdout_pos[k] = s_pos;
+      }
+      __syncthreads();
+      {  // compact this instance's stdout (whole 8-B words)
+        const unsigned long long *src = reinterpret_cast<const unsigned long long *>(c.out);
+        unsigned long long *dst = reinterpret_cast<unsigned long long *>(p.stdout_cmp + s_pos);
+        for (uint32_t w = tid; w < sh.out_len / 8; w += T) dst[w] = src[w];
+      }
     }
-    __syncthreads();
-    {  // compact this instance's stdout (whole 8-B words)
-      const unsigned long long *src = reinterpret_cast<const unsigned long long *>(c.out);
-      unsigned long long *dst = reinterpret_cast<unsigned long long *>(p.stdout_cmp + s_pos);
-      for (uint32_t w = tid; w < sh.out_len / 8; w += T) dst[w] = src[w];
-    }
-    __syncthreads();  // s_j, s_pos, s_argv, sh reused by the next instance
+    team_sync(c);  // s_j, s_pos, s_argv, sh reused by the next instance
   }
 }
 
@@ -129,6 +142,8 @@ int app_max_threads(uint32_t app) {
   }
   return 32;
 }
+// whether the body splits its work over a multi-CTA team
+bool app_team_aware(uint32_t app) { return app == APP_XSBENCH ? XsApp::kTeam : false; }
 
 const void *kernel_ptr(uint32_t app, int T) {
   switch (app) {
@@ -142,38 +157,71 @@ const void *kernel_ptr(uint32_t app, int T) {
 }
 
 // host-side sizing from the same parse/layout code the instance runs
-bool app_size(uint32_t app, int argc, const char *const *argv, int T, uint64_t *arena, uint32_t *smem) {
+bool app_size(uint32_t app, int argc, const char *const *argv, int T, int cs, uint64_t *arena, uint32_t *smem) {
   switch (app) {
-    case APP_ECHO: return EchoApp::size(argc, argv, T, arena, smem);
-    case APP_XSBENCH: return XsApp::size(argc, argv, T, arena, smem);
-    case APP_RSBENCH: return RsApp::size(argc, argv, T, arena, smem);
-    case APP_AMGMK: return AmgApp::size(argc, argv, T, arena, smem);
-    case APP_NOTFOUND: return NotFoundApp::size(argc, argv, T, arena, smem);
+    case APP_ECHO: return EchoApp::size(argc, argv, T, cs, arena, smem);
+    case APP_XSBENCH: return XsApp::size(argc, argv, T, cs, arena, smem);
+    case APP_RSBENCH: return RsApp::size(argc, argv, T, cs, arena, smem);
+    case APP_AMGMK: return AmgApp::size(argc, argv, T, cs, arena, smem);
+    case APP_NOTFOUND: return NotFoundApp::size(argc, argv, T, cs, arena, smem);
   }
   *arena = 0;
   *smem = 0;
   return false;
 }
 
-cudaError_t launch_group(uint32_t app, int T, int grid, size_t smem, const KParams &p, cudaStream_t st) {
-  const void *fn = kernel_ptr(app, T);
-  if (!fn) return cudaErrorInvalidValue;
-  if (smem > 0) {
-    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
-  }
-  void *args[] = {const_cast<KParams *>(&p)};
-  return cudaLaunchKernel(fn, dim3(grid), dim3(T), args, smem, st);
+static cudaError_t set_smem(const void *fn, size_t smem) {
+  if (smem == 0) return cudaSuccess;
+  return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
 }
 
-cudaError_t group_occupancy(uint32_t app, int T, size_t smem, int *blocks_per_sm) {
+cudaError_t launch_group(uint32_t app, int T, int grid, int cs, size_t smem, const KParams &p, cudaStream_t st) {
   const void *fn = kernel_ptr(app, T);
   if (!fn) return cudaErrorInvalidValue;
-  if (smem > 0) {
-    cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
+  cudaError_t e = set_smem(fn, smem);
+  if (e != cudaSuccess) return e;
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3((unsigned)grid);
+  cfg.blockDim = dim3((unsigned)T);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = st;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = (unsigned)cs;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  void *args[] = {const_cast<KParams *>(&p)};
+  return cudaLaunchKernelExC(&cfg, fn, args);
+}
+
+// resident teams (clusters of cs CTAs) on the whole device
+cudaError_t group_occupancy(uint32_t app, int T, int cs, size_t smem, int *teams) {
+  const void *fn = kernel_ptr(app, T);
+  if (!fn) return cudaErrorInvalidValue;
+  cudaError_t e = set_smem(fn, smem);
+  if (e != cudaSuccess) return e;
+  if (cs <= 1) {
+    int per_sm = 0, dev = 0, sms = 0;
+    e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, T, smem);
+    if (e == cudaSuccess) e = cudaGetDevice(&dev);
+    if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    *teams = per_sm * sms;
+    return e;
   }
-  return cudaOccupancyMaxActiveBlocksPerMultiprocessor(blocks_per_sm, fn, T, smem);
+  cudaLaunchConfig_t cfg{};
+  cfg.gridDim = dim3((unsigned)(cs * 64));
+  cfg.blockDim = dim3((unsigned)T);
+  cfg.dynamicSmemBytes = smem;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = (unsigned)cs;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  return cudaOccupancyMaxActiveClusters(teams, fn, &cfg);
 }
 
 }  // namespace ens

@@ -24,14 +24,16 @@ struct KParams {
   char *stdout_base;          // [n_instances][stdout_cap] raw, per instance
   char *stdout_cmp;           // compacted raw stdout (for a small D2H)
   uint32_t stdout_cap;
-  char *arena_base;           // [grid][arena_bytes]
+  char *arena_base;           // [teams][arena_bytes]
   uint64_t arena_bytes;
+  uint32_t team_ctas;         // CTAs per team (thread-block cluster size)
 };
 
 const void *kernel_ptr(uint32_t app, int T);
 int app_max_threads(uint32_t app);
-bool app_size(uint32_t app, int argc, const char *const *argv, int T, uint64_t *arena, uint32_t *smem);
-cudaError_t launch_group(uint32_t app, int T, int grid, size_t smem, const KParams &p, cudaStream_t st);
-cudaError_t group_occupancy(uint32_t app, int T, size_t smem, int *blocks_per_sm);
+bool app_team_aware(uint32_t app);
+bool app_size(uint32_t app, int argc, const char *const *argv, int T, int cs, uint64_t *arena, uint32_t *smem);
+cudaError_t launch_group(uint32_t app, int T, int grid, int cs, size_t smem, const KParams &p, cudaStream_t st);
+cudaError_t group_occupancy(uint32_t app, int T, int cs, size_t smem, int *teams);
 
 }  // namespace ens

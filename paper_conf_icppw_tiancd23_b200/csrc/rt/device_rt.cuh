@@ -6,6 +6,8 @@
 // layout), its stdout buffer, its tallies and its exit code.  No mutable
 // __device__ globals exist anywhere in the instance bodies.
 #pragma once
+#include <cooperative_groups.h>
+
 #include <cstdint>
 
 #include "fmt_ids.h"
@@ -92,12 +94,16 @@ ENS_HD uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 // ---------------------------------------------------------------------------
 // per-instance context (identical copy in every thread of the block)
 // ---------------------------------------------------------------------------
+constexpr int kMaxTeamCtas = 8;  // portable thread-block-cluster size
+
 struct Shared {             // static shared memory of the scheduler
   uint32_t tallies[32];     // per-instance tallies (smem atomics)
   uint32_t out_len;         // stdout bytes used (thread 0 only)
   uint32_t flags;           // record flags (thread 0 only)
   unsigned long long red_u[32];  // block reduction scratch
   double red_d[32];
+  unsigned long long team_u[kMaxTeamCtas];  // cross-CTA partials (rank 0's copy)
+  double team_d[kMaxTeamCtas];
 };
 
 struct Result {  // meaningful in thread 0 after the body returns
@@ -107,15 +113,32 @@ struct Result {  // meaningful in thread 0 after the body returns
   uint64_t work;
 };
 
+// The team running one instance: one CTA (the paper's team = thread block,
+// P:313-318), or on B200 a thread-block cluster of csize CTAs with a hardware
+// barrier and distributed shared memory — for ensembles with fewer instances
+// than SMs (team-aware bodies only; others run on rank 0 alone).
 struct Ctx {
   uint32_t k, id;      // record slot, instance id (line)
-  char *arena;         // this block's slot
+  char *arena;         // this team's slot
   uint64_t arena_cap;
   char *out;           // this instance's raw stdout buffer
   uint32_t out_cap;
   Shared *sh;
   char *smem;          // dynamic shared memory of the app
+  uint32_t crank, csize;  // CTA rank in the team, team CTAs
 };
+
+// barrier of the whole team (cluster barrier: release/acquire at cluster
+// scope, so global and shared writes before it are visible after it)
+__device__ __forceinline__ void team_sync(const Ctx &c) {
+  if (c.csize > 1) cooperative_groups::this_cluster().sync();
+  else __syncthreads();
+}
+// `p` (a shared variable of this CTA) in the shared memory of team CTA `rank`
+template <class X>
+__device__ __forceinline__ X *cta_shared(X *p, uint32_t rank) {
+  return cooperative_groups::this_cluster().map_shared_rank(p, rank);
+}
 
 // ---- stdout: {u32 fmt, u32 payload bytes, 8-B slots}; strings = len slot +
 // bytes padded to 8.  Called by thread 0 only.
@@ -163,7 +186,7 @@ __device__ inline void out_write(Ctx &c, unsigned fmt, const OutArg *args, int n
 
 template <class... A>
 __device__ __forceinline__ void ens_printf(Ctx &c, unsigned fmt, A... a) {
-  if (threadIdx.x != 0) return;
+  if (threadIdx.x != 0 || c.crank != 0) return;
   OutArg args[sizeof...(A) > 0 ? sizeof...(A) : 1] = {oa(a)...};
   out_write(c, fmt, args, (int)sizeof...(A));
 }
@@ -222,5 +245,31 @@ template <class T>
 __device__ __forceinline__ T ld_(const T *p) { return *p; }
 
 __device__ __forceinline__ uint64_t dbits(double d) { return (uint64_t)__double_as_longlong(d); }
+
+// team reductions: block reduction, then CTA partials gathered in rank 0's
+// shared memory and summed in rank order (deterministic); result valid in
+// rank 0 (in every thread of it).
+__device__ inline unsigned long long team_sum_u64(Ctx &c, unsigned long long v) {
+  v = block_sum_u64(c.sh, v);
+  if (c.csize == 1) return v;
+  if (threadIdx.x == 0) *cta_shared(&c.sh->team_u[c.crank], 0) = v;
+  team_sync(c);
+  unsigned long long t = 0;
+  if (c.crank == 0)
+    for (uint32_t r = 0; r < c.csize; r++) t += c.sh->team_u[r];
+  team_sync(c);
+  return t;
+}
+__device__ inline double team_sum_f64(Ctx &c, double v) {
+  v = block_sum_f64(c.sh, v);
+  if (c.csize == 1) return v;
+  if (threadIdx.x == 0) *cta_shared(&c.sh->team_d[c.crank], 0) = v;
+  team_sync(c);
+  double t = 0.0;
+  if (c.crank == 0)
+    for (uint32_t r = 0; r < c.csize; r++) t += c.sh->team_d[r];
+  team_sync(c);
+  return t;
+}
 
 }  // namespace ens

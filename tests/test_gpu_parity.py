@@ -102,3 +102,12 @@ def test_more_instances_than_blocks(oracle, grid):
              for i in range(9)]
     g, o = run_both(oracle, lines, grid=grid)
     assert_parity(g, o)
+
+
+@pytest.mark.parametrize("team", [2, 4, 8])
+def test_cluster_team_parity(oracle, team):
+    """A team = a thread-block cluster of `team` CTAs (XS is team-aware): same results."""
+    lines = [XS_CASES[0], XS_CASES[1], XS_CASES[2], XS_CASES[4], XS_CASES[10], "xsbench -s small -g 77 -l 999 -G hash -h 5 -r 2",
+             RS_CASES[0], AMG_CASES[1], "echo team"]
+    g, o = run_both(oracle, lines, threads=128, team_ctas=team)
+    assert_parity(g, o)
