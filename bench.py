@@ -181,7 +181,7 @@ def workload_lines(name, world):
     raise SystemExit(f"unknown workload {name}")
 
 
-THREADS = {"C2": 1024, "TSTAR": 256, "C1": 256, "C3": 256, "C4": 1024, "C5": 256}
+THREADS = {"C2": 1024, "TSTAR": 512, "C1": 256, "C3": 256, "C4": 1024, "C5": 512}
 
 
 def time_ours(lines, world, rank, threads, steps, warmup, torch, dist_on, team_ctas=0):
@@ -386,7 +386,7 @@ def main():
                                      "paper_context": "51x at 64 instances on A100 40GB (P:44-45, P:639-640)"}
         # north-star target launch: >= 1024 XSBench-style instances per B200 at >= 60% HBM
         tl, _ = workload_lines("TSTAR", 1)
-        t_ens, t_res, t_info, t_ms, t_per, _ = time_ours(tl, 1, 0, 256, 5, 3, torch, False)
+        t_ens, t_res, t_info, t_ms, t_per, _ = time_ours(tl, 1, 0, THREADS["TSTAR"], 5, 3, torch, False)
         t_algo = algorithmic_bytes(tl, t_res.records, t_res.tallies)
         t_k = sum(t_per) / len(t_per)
         extras["tstar"] = {"instances": len(tl), "ms_per_launch": t_k, "instances_per_s": len(tl) / (t_k * 1e-3),

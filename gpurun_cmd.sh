@@ -1,3 +1,13 @@
-timeout 600 python bench.py > gpurun_out/bench3.json 2> gpurun_out/bench3.err; echo bench=$?
-timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none --csv --log-file gpurun_out/launches_r1b.csv python bench.py --steps 2 --warmup 3 --no-extras > /dev/null 2>&1; echo list=$?
-timeout 900 ncu --set full --clock-control none --import-source on -k regex:ens_kernel -s 1 -c 1 -o gpurun_out/c2_r1b python bench.py --steps 1 --warmup 3 --no-extras > /dev/null 2>&1; echo full=$?
+P="python tools/probe.py"
+C=paper_conf_icppw_tiancd23_b200/csrc
+for cfg in "512 2" "1024 1" "1024 2" "512 1" "512 4"; do
+  set -- $cfg
+  rm -f $C/kernels.o
+  make -s -C $C NVFLAGS="-gencode arch=compute_100a,code=sm_100a -O3 --fmad=false -std=c++17 -Xcompiler -fPIC -DENS_MINB_NUM=$1 -DENS_XS_U=$2" > /dev/null 2>&1
+  echo "== MINB_NUM=$1 U=$2"
+  $P "xsbench -s small -g 1000 -G unionized -l 10000 -r {i}" 1024 256 2
+  $P "xsbench -s small -g 1000 -G unionized -l 10000 -r {i}" 1024 512 2
+  $P "xsbench -s small -g 1000 -G unionized -l 10000 -r {i}" 1024 128 2
+  $P "xsbench -s large -g 11303 -G hash -h 10000 -l 1000000 -r {i}" 64 512 2
+  $P "xsbench -s large -g 11303 -G hash -h 10000 -l 1000000 -r {i}" 64 256 2
+done

@@ -86,6 +86,11 @@ ENS_HD long long xs_buckets(const XsParams &p) {
   return (long long)p.n_iso * (pow2_ceil(p.n_gp) / 2 > 0 ? pow2_ceil(p.n_gp) / 2 : 1);
 }
 ENS_HD int xs_nbn(int n_gp) { return pow2_ceil(n_gp) / 2 > 0 ? pow2_ceil(n_gp) / 2 : 1; }
+// bins of the union search table: ufind[b] = #{k >= 1 : u_k <= b / ubins}
+// (power of two, ~1 union energy per bin), so the union position of energy
+// p is ufind[floor(p * ubins)] plus a short forward scan — the same index as
+// XS-7's binary search, in two dependent loads instead of ~17
+ENS_HD long long xs_ubins(const XsParams &p) { return pow2_ceil((int)(((long long)p.n_iso * p.n_gp + 1) / 2)); }
 // union-sweep chunks (rows per chunk) for the index grid
 constexpr int kXsSweepRows = 512;
 
@@ -96,6 +101,7 @@ struct XsLayout {
   uint64_t keys;      // [n_u] x 16 B {energy bits, record id}, bucket-sorted
   uint64_t bkt;       // [xs_buckets] u32 bucket counts -> offsets
   uint64_t uenergy;   // unionized: [n_u] sorted union energies (u64 bits)
+  uint64_t ufind;     // unionized: [xs_ubins] u32 union search table (private accelerator)
   uint64_t chist;     // unionized: [n_chunks][n_iso] u32 owner counts per sweep chunk
   uint64_t index;     // unionized [n_u][n_iso] / hash [n_iso][bins+1] int32
   uint64_t total;
@@ -116,6 +122,7 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
   if (p.grid == XS_UNIONIZED) {
     const uint64_t nch = (n_u + kXsSweepRows - 1) / kXsSweepRows;
     L.uenergy = o; o = align_up(o + n_u * 8, 256);
+    L.ufind = o; o = align_up(o + (uint64_t)xs_ubins(p) * 4, 256);
     L.chist = o; o = align_up(o + nch * (uint64_t)p.n_iso * 4, 256);
     L.index = o; o = align_up(o + n_u * (uint64_t)p.n_iso * 4, 256);
   } else if (p.grid == XS_HASH) {
@@ -126,7 +133,10 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
 }
 
 // dynamic shared memory layout: material tables + the sort's bucket counters
-constexpr int kXsU = 2;       // nuclide gathers in flight per lane
+#ifndef ENS_XS_U
+#define ENS_XS_U 1  // measured on B200: 1 beats 2 and 4 (register pressure)
+#endif
+constexpr int kXsU = ENS_XS_U;  // nuclide gathers in flight per lane
 constexpr int kXsMaxT = 512;  // XsApp::kMaxT
 // lookups per thread per material-sorted batch: enough that every thread
 // gets several fuel lookups (321 nuclides large / 34 small)

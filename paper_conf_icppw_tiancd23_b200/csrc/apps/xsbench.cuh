@@ -664,15 +664,25 @@ struct XsApp {
     uint64_t *uA = (uint64_t *)(c.arena + L.uenergy);
     uint32_t *chist = (uint32_t *)(c.arena + L.chist);
     const long long nch = (n_u + kXsSweepRows - 1) / kXsSweepRows;
+    uint32_t *uf = (uint32_t *)(c.arena + L.ufind);
+    const long long UB = xs_ubins(p);
     for (long long x = tid; x < nch * n_iso; x += T) chist[x] = 0;
+    for (long long b = tid; b < UB; b += T) uf[b] = 0;
     __syncthreads();
     XS_STOP(5);
-    for (long long e = tid; e < n_u; e += T) {  // union energies + chunk owner counts
-      const XsKey k = keys[e];
+    for (long long e = tid; e < n_u; e += T) {  // union energies, chunk owner counts,
+      const XsKey k = keys[e];                   // search-table histogram
       uA[e] = k.key;
       atomicAdd(&chist[(e / kXsSweepRows) * n_iso + k.idx / n_gp], 1u);
+      if (e >= 1) {  // first bin b with u_e <= b / UB (UB a power of two: exact)
+        const double x = __longlong_as_double((long long)k.key) * (double)UB;
+        long long bk = (long long)x;
+        if ((double)bk < x) bk++;
+        if (bk < UB) atomicAdd(&uf[bk], 1u);
+      }
     }
     __syncthreads();
+    global_exclusive_scan<true>(uf, UB, c.sh);  // ufind[b] = #{k >= 1 : u_k <= b / UB}
     for (int i = tid; i < n_iso; i += T) {  // exclusive scan over chunks per owner
       uint32_t run = 0;
       for (long long ch = 0; ch < nch; ch++) {
@@ -720,6 +730,8 @@ struct XsApp {
     const double *recs = (const double *)(c.arena + L.recs);
     const int *ig = (const int *)(c.arena + L.index);
     const uint64_t *uA = (const uint64_t *)(c.arena + L.uenergy);
+    const uint32_t *uf = (const uint32_t *)(c.arena + L.ufind);
+    const long long UB = xs_ubins(p);
     const XsSmem S = xs_smem(p, T);
     const int K = xs_batch_k(n_iso);
     double *slot_pe = (double *)(c.smem + S.slot);
@@ -768,7 +780,13 @@ struct XsApp {
           const int mat = pick_mat_thr(thr, lcg_double(t));
           const uint32_t pos = atomicAdd(&mcnt[mat], 1u);
           slot_pe[pos] = pe;
-          if (GRID == XS_UNIONIZED) slot_idx[pos] = (int)gs_u64(uA, pe, 0, n_u - 1);
+          if (GRID == XS_UNIONIZED) {  // == grid_search(u, pe, 0, n_u-1) (XS-7)
+            long long b = (long long)(pe * (double)UB);
+            if (b > UB - 1) b = UB - 1;
+            long long cc = ld_(uf + b);
+            while (cc < n_u - 1 && __longlong_as_double((long long)ld_(uA + cc + 1)) <= pe) cc++;
+            slot_idx[pos] = (int)(cc < n_u - 2 ? cc : n_u - 2);
+          }
         }
       }
       __syncthreads();

@@ -30,8 +30,13 @@ __device__ __forceinline__ uint32_t smid() {
   return s;
 }
 
+// register budget: min blocks per SM = ENS_MINB_NUM / T (512: 128 registers)
+#ifndef ENS_MINB_NUM
+#define ENS_MINB_NUM 512
+#endif
+
 template <class App, int T>
-__global__ void __launch_bounds__(T, (512 / T) > 0 ? (512 / T) : 1) ens_kernel(const KParams p) {
+__global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T) : 1) ens_kernel(const KParams p) {
   extern __shared__ __align__(16) char dsmem[];
   __shared__ char *s_argv[ENS_MAX_ARGC + 1];
   __shared__ uint32_t s_j;
