@@ -55,8 +55,10 @@ enum {
 
 /* ens_launch_cfg.flags */
 enum {
-  ENS_F_TIMESTAMPS = 1u << 0 /* fill smid / t_start_ns / t_end_ns in records   */
+  ENS_F_TIMESTAMPS = 1u << 0, /* fill smid / t_start_ns / t_end_ns in records  */
+  ENS_F_PHASES = 1u << 1      /* accumulate per-phase device time (tracing)    */
 };
+#define ENS_PHASES 16
 
 typedef enum {
   ENS_APP_BY_ARGV0 = 0, /* basename of argv[0] selects the app per instance */
@@ -165,6 +167,14 @@ int ens_collect(ens_run *r, ens_record *recs, uint32_t *tallies, char *stdout_bu
 
 /* CUDA-event time of the last (re)launch's kernels, in ms.                   */
 int ens_run_elapsed_ms(ens_run *r, float *ms);
+
+/* Tracing (launched with ENS_F_PHASES): ns[p] = sum over instances of the
+ * %globaltimer time team thread 0 spent in phase p of the last (re)launch
+ * (XS: 0 materials, 1 generate, 2 bucket scan, 3 scatter, 4 bucket sort,
+ * 5 clear tables, 6 union tables, 7 index sweep, 8 record permute, 9 hash
+ * column, 10 lookup sampling + sort, 11 lookup gathers).  Blocks on the
+ * stream.                                                                    */
+int ens_run_phases(ens_run *r, uint64_t ns[ENS_PHASES]);
 
 /* Launch geometry actually used, and where the device-side results live
  * inside the workspace (for an in-place NCCL all-gather of the records).     */

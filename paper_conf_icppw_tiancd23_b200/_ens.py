@@ -16,7 +16,8 @@ LIB_PATH = os.path.join(PKG_DIR, "libens.so")
 ENS_OK, ENS_EINVAL, ENS_ENOENT, ENS_ENOMEM, ENS_ECUDA, ENS_ERANGE, ENS_EBUSY, ENS_EPARSE = 0, -1, -2, -3, -4, -5, -6, -7
 ENS_EXIT_USAGE, ENS_EXIT_NOMEM, ENS_EXIT_NOTFOUND = 1, 12, 127
 ENS_RF_STDOUT_TRUNC, ENS_RF_NOMEM, ENS_RF_NOT_RUN, ENS_RF_DONE = 1, 2, 4, 8
-ENS_F_TIMESTAMPS = 1
+ENS_F_TIMESTAMPS, ENS_F_PHASES = 1, 2
+ENS_PHASES = 16
 ENS_APP_BY_ARGV0, ENS_APP_ECHO, ENS_APP_XSBENCH, ENS_APP_RSBENCH, ENS_APP_AMGMK = 0, 1, 2, 3, 4
 APP_IDS = {"auto": 0, "echo": 1, "xsbench": 2, "rsbench": 3, "amgmk": 4}
 ENS_TALLIES = 32
@@ -72,6 +73,7 @@ def _load():
         "ens_run_relaunch": (i, [p, p]),
         "ens_collect": (i, [p, p, p, p, sz, p]),
         "ens_run_elapsed_ms": (i, [p, ctypes.POINTER(ctypes.c_float)]),
+        "ens_run_phases": (i, [p, ctypes.POINTER(ctypes.c_uint64)]),
         "ens_run_get_info": (i, [p, ctypes.POINTER(RunInfo)]),
         "ens_format_stdout": (ctypes.c_long, [u32, p, sz, p, sz]),
         "ens_run_free": (None, [p]),
@@ -89,6 +91,7 @@ def _load():
 lib = _load()
 EXPORTED = ["ens_load_args", "ens_parse_args", "ens_args_count", "ens_args_get", "ens_args_free",
             "ens_workspace_bytes", "ens_launch", "ens_run_relaunch", "ens_collect", "ens_run_elapsed_ms",
+            "ens_run_phases",
             "ens_run_get_info", "ens_format_stdout", "ens_run_free", "ens_strerror", "ens_last_error",
             "ens_version"]
 
@@ -207,6 +210,12 @@ class Run:
         ms = ctypes.c_float()
         _check("ens_run_elapsed_ms", lib.ens_run_elapsed_ms(self._h, ctypes.byref(ms)))
         return ms.value
+
+    def phases_ns(self):
+        """Per-phase device time summed over instances (launched with ENS_F_PHASES)."""
+        a = (ctypes.c_uint64 * ENS_PHASES)()
+        _check("ens_run_phases", lib.ens_run_phases(self._h, a))
+        return list(a)
 
     def info(self):
         i = RunInfo()

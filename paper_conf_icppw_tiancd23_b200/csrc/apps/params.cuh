@@ -103,8 +103,16 @@ struct XsLayout {
   uint64_t uenergy;   // unionized: [n_u] sorted union energies (u64 bits)
   uint64_t ufind;     // unionized: [xs_ubins] u32 union search table (private accelerator)
   uint64_t chist;     // unionized: [n_chunks][n_iso] u32 owner counts per sweep chunk
-  uint64_t index;     // unionized [n_u][n_iso] / hash [n_iso][bins+1] int32
+  uint64_t index;     // unionized [n_u][n_iso] int32 / hash [n_iso][bins+1] XsHashEnt
+  uint64_t hcol;      // hash: [cs][bins+1] int32 column being built
   uint64_t total;
+};
+// hash index entry: the upstream index u_low = ig[b][i] plus E_i[u_low+1], so
+// a lookup knows from one 16-B load whether its energy lies in the first
+// record pair of the bin (a private accelerator; results are unchanged)
+struct XsHashEnt {
+  int u_low, pad;
+  double e_next;
 };
 // cs = CTAs in the team: hash / nuclide grids give each CTA its own
 // per-nuclide scratch
@@ -126,7 +134,8 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
     L.chist = o; o = align_up(o + nch * (uint64_t)p.n_iso * 4, 256);
     L.index = o; o = align_up(o + n_u * (uint64_t)p.n_iso * 4, 256);
   } else if (p.grid == XS_HASH) {
-    L.index = o; o = align_up(o + (uint64_t)p.n_iso * (p.bins + 1) * 4, 256);
+    L.index = o; o = align_up(o + (uint64_t)p.n_iso * (p.bins + 1) * 16, 256);
+    L.hcol = o; o = align_up(o + (uint64_t)cs * (p.bins + 1) * 4, 256);
   }
   L.total = o;
   return L;

@@ -188,7 +188,7 @@ __device__ inline void global_exclusive_scan(uint32_t *a, long long n, Shared *s
 #ifdef ENS_XS_STOP  // profiling builds only: stop init after phase k
 #define XS_STOP(k) do { if (ENS_XS_STOP == (k)) { __syncthreads(); return; } } while (0)
 #else
-#define XS_STOP(k) do { } while (0)
+#define XS_STOP(k) phase_mark(c, (k))  // tracing (ENS_F_PHASES): end of init phase k
 #endif
 
 struct XsKey {
@@ -242,6 +242,7 @@ struct XsApp {
     hm_tables(n_iso, mx, thr, nn, concs, mats);
     __syncthreads();
     hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
+    phase_mark(c, 0);
     if (p.grid == XS_UNIONIZED) {
       if (c.crank == 0) init(c, p, L, S);  // one CTA builds the union
     } else {
@@ -376,7 +377,8 @@ struct XsApp {
     const Affine Jnuc = lcg_pow(6ULL * n_gp * c.csize);
     uint64_t s_nuc = lcg_pow(6ULL * ((uint64_t)c.crank * n_gp + tid))(p.gseed);  // record (i*n_gp + tid)
     for (int i = (int)c.crank; i < n_iso; i += (int)c.csize) {
-      int *col = ig + (size_t)i * (p.bins + 1);
+      int *col = (int *)(c.arena + L.hcol) + (size_t)c.crank * (p.bins + 1);  // this CTA's column
+      XsHashEnt *ent = (XsHashEnt *)ig + (size_t)i * (p.bins + 1);
       for (int b = tid; b < nbn; b += T) nb[b] = 0;
       if (hash)
         for (int b = tid; b <= p.bins; b += T) col[b] = 0;
@@ -397,7 +399,9 @@ struct XsApp {
         s_nuc = Jnuc(s_nuc);
       }
       __syncthreads();
+      phase_mark(c, 1);
       global_exclusive_scan(nb, nbn, c.sh);
+      phase_mark(c, 2);
       for (int j0 = tid; j0 < n_gp; j0 += 4 * T) {  // scatter {energy, j}
         double e[4];
 #pragma unroll
@@ -416,8 +420,10 @@ struct XsApp {
         }
       }
       __syncthreads();
+      phase_mark(c, 3);
       for (int b = tid; b < nbn; b += T) sort_bucket(keys, b ? nb[b - 1] : 0, nb[b]);
       __syncthreads();
+      phase_mark(c, 4);
       double *rec_i = recs + (size_t)i * n_gp * 6;
       for (int k0 = tid; k0 < n_gp; k0 += 4 * T) {  // records to sorted position; bin histogram
         unsigned jj[4];
@@ -452,6 +458,7 @@ struct XsApp {
         }
       }
       __syncthreads();
+      phase_mark(c, 8);
       if (hash) {
         global_exclusive_scan<true>((uint32_t *)col, p.bins, c.sh);
         for (int b = tid; b < p.bins; b += T) {
@@ -460,6 +467,16 @@ struct XsApp {
         }
         if (tid == 0) col[p.bins] = n_gp - 2;
         __syncthreads();
+        for (int b = tid; b <= p.bins; b += T) {  // entries {u_low, E[u_low+1]}
+          const int ul = col[b];
+          XsHashEnt h;
+          h.u_low = ul;
+          h.pad = 0;
+          h.e_next = ld_(rec_i + 6 * (size_t)(ul + 1));
+          ent[b] = h;
+        }
+        __syncthreads();
+        phase_mark(c, 9);
       }
     }
   }
@@ -700,17 +717,26 @@ struct XsApp {
     else sweep<12>(keys, chist, ig, n_u, n_iso, n_gp, nch);
     __syncthreads();
     XS_STOP(7);
-    // records to their sorted positions (coalesced over the union order)
-    for (long long e = tid; e < n_u; e += T) {
-      const XsKey k = keys[e];
-      const double2 *src = reinterpret_cast<const double2 *>(scr + 6 * (size_t)k.idx);
-      double2 *dst = reinterpret_cast<double2 *>(recs + 6 * (size_t)k.pad);
-      const double2 a = src[0], b = src[1], x = src[2];
-      dst[0] = a;
-      dst[1] = b;
-      dst[2] = x;
+    // records to their sorted positions (coalesced over the union order),
+    // four in flight per thread
+    for (long long e0 = tid; e0 < n_u; e0 += 4LL * T) {
+      XsKey k[4];
+#pragma unroll
+      for (int q = 0; q < 4; q++)
+        if (e0 + q * T < n_u) k[q] = keys[e0 + q * T];
+#pragma unroll
+      for (int q = 0; q < 4; q++)
+        if (e0 + q * T < n_u) {
+          const double2 *src = reinterpret_cast<const double2 *>(scr + 6 * (size_t)k[q].idx);
+          double2 *dst = reinterpret_cast<double2 *>(recs + 6 * (size_t)k[q].pad);
+          const double2 a = src[0], b = src[1], x = src[2];
+          dst[0] = a;
+          dst[1] = b;
+          dst[2] = x;
+        }
     }
     __syncthreads();
+    phase_mark(c, 8);
   }
 
   // ---- XS-6..XS-10: lookups ----------------------------------------------
@@ -790,6 +816,7 @@ struct XsApp {
         }
       }
       __syncthreads();
+      phase_mark(c, 10);
       // (B) thread-per-lookup over sorted slots
       for (int sl = tid; sl < nb; sl += T) {
         int mat = 0;
@@ -807,7 +834,7 @@ struct XsApp {
         const double *crow = concs + mat * mx;
         double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
         for (int j0 = 0; j0 < nm; j0 += kU) {
-          int nuc[kU], lo[kU];
+          int nuc[kU], lo[kU], uh[kU];
           bool on[kU];
           double2 a0[kU], a1[kU], a2[kU], b0v[kU], b1[kU], b2[kU];
 #pragma unroll
@@ -815,9 +842,18 @@ struct XsApp {
             on[u] = j0 + u < nm;
             nuc[u] = on[u] ? mrow[j0 + u] : 0;
             lo[u] = 0;
+            uh[u] = 0;
             if (on[u]) {
-              if (GRID == XS_HASH) lo[u] = ld_(ig + (size_t)nuc[u] * (p.bins + 1) + idx);
-              else if (GRID == XS_UNIONIZED) {
+              if (GRID == XS_HASH) {
+                // {u_low, E[u_low+1]} and the next bin's u_low: the bracket is
+                // u_low if pe < E[u_low+1], else (usually) u_low+1 — verified
+                // against the loaded pair below
+                const XsHashEnt *he = (const XsHashEnt *)ig + (size_t)nuc[u] * (p.bins + 1) + idx;
+                const int4 h = ld_(reinterpret_cast<const int4 *>(he));
+                const double e_next = __hiloint2double(h.w, h.z);
+                uh[u] = ld_(&he[1].u_low) + 1;
+                lo[u] = pe < e_next ? h.x : h.x + 1;
+              } else if (GRID == XS_UNIONIZED) {
                 const int k = ld_(ig + (size_t)idx * n_iso + nuc[u]);
                 lo[u] = (k == n_gp - 1) ? k - 1 : k;
               } else {
@@ -837,15 +873,26 @@ struct XsApp {
           if (GRID == XS_HASH) {
 #pragma unroll
             for (int u = 0; u < kU; u++) {
-              // E[u_low] < pe < E[u_low+1] is exactly grid_search's answer
-              // u_low on [u_low, u_high]; otherwise the full upstream logic
-              if (on[u] && !(a0[u].x < pe && pe < b0v[u].x)) {
+              // the guess lo is exactly upstream's bracket (grid_search on
+              // [u_low, u_high], its edge cases excluded) iff E[lo] < pe <
+              // E[lo+1] and lo+1 <= u_high; otherwise the full upstream logic
+              // walk forward while pe is past the pair (one gather per step;
+              // the guess is short by more than one record for ~1 in 8)
+              while (on[u] && pe >= b0v[u].x && a0[u].x < pe && lo[u] + 2 <= uh[u]) {
+                lo[u]++;
+                const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)nuc[u] * n_gp + lo[u]) * 6);
+                a0[u] = b0v[u]; a1[u] = b1[u]; a2[u] = b2[u];
+                b0v[u] = ld_(r2 + 3); b1[u] = ld_(r2 + 4); b2[u] = ld_(r2 + 5);
+              }
+              if (on[u] && !(a0[u].x < pe && pe < b0v[u].x && lo[u] + 1 <= uh[u])) {  // edges: upstream logic
                 const double *E = recs + (size_t)nuc[u] * n_gp * 6;
-                const int u_low = lo[u];
-                const int u_high = ld_(ig + (size_t)nuc[u] * (p.bins + 1) + idx + 1) + 1;
+                const XsHashEnt *he = (const XsHashEnt *)ig + (size_t)nuc[u] * (p.bins + 1) + idx;
+                const int u_low = ld_(&he->u_low);
+                const int u_high = uh[u];
+                const double e_low = ld_(E + 6 * (size_t)u_low);
                 const double e_high = ld_(E + 6 * (size_t)u_high);
                 int lower;
-                if (pe <= a0[u].x) lower = 0;
+                if (pe <= e_low) lower = 0;
                 else if (pe >= e_high) lower = n_gp - 1;
                 else lower = gs_recs(E, pe, u_low, u_high);
                 const int l2 = lower == n_gp - 1 ? lower - 1 : lower;
@@ -884,6 +931,7 @@ struct XsApp {
         fabs_ += fabs(m0); fabs_ += fabs(m1); fabs_ += fabs(m2); fabs_ += fabs(m3); fabs_ += fabs(m4);
       }
       __syncthreads();  // slots reused by the next batch
+      phase_mark(c, 11);
     }
     ver = team_sum_u64(c, ver);
     bsum = team_sum_u64(c, bsum);

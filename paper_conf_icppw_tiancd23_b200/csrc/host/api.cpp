@@ -173,7 +173,7 @@ struct Plan {  // workspace layout (byte offsets) and groups
   // staged (H2D) part
   size_t o_blob = 0, o_tok = 0, o_line = 0, o_lok = 0, o_kmap = 0, staged = 0;
   // zeroed part: counters (n_groups + 1 u64 stdout total), recs, pos
-  size_t o_ctr = 0, o_recs = 0, o_pos = 0, zeroed_end = 0;
+  size_t o_ctr = 0, o_recs = 0, o_pos = 0, o_phase = 0, zeroed_end = 0;
   size_t o_tal = 0, o_out = 0, o_cmp = 0, o_arena = 0, total = 0;
 };
 
@@ -309,6 +309,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   P.o_ctr = o; o = al(o + (P.groups.size() + 1) * 8);
   P.o_recs = o; o = al(o + (size_t)n * sizeof(ens_record));
   P.o_pos = o; o = al(o + (size_t)n * 8);
+  P.o_phase = o; o = al(o + ENS_PHASES * 8);
   P.zeroed_end = o;
   P.o_tal = o; o = al(o + (size_t)n * ENS_TALLIES * 4);
   P.o_out = o; o = al(o + (size_t)n * P.stdout_cap);
@@ -370,6 +371,7 @@ static int enqueue(ens_run *r) {
     k.arena_base = r->ws + P.o_arena;
     k.arena_bytes = P.arena_bytes;
     k.team_ctas = (uint32_t)g.cs;
+    k.phases = (r->flags & ENS_F_PHASES) ? (unsigned long long *)(r->ws + P.o_phase) : nullptr;
     cudaError_t e = launch_group(g.app, g.T, g.grid * g.cs, g.cs, g.smem, k, r->stream);
     if (e != cudaSuccess) return cuda_fail(e, "ens_kernel launch");
   }
@@ -506,6 +508,16 @@ extern "C" int ens_collect(ens_run *r, ens_record *recs, uint32_t *tallies, char
     if (cap < text.size()) return fail(ENS_ERANGE, "ens_collect: stdout buffer too small");
     std::memcpy(stdout_buf, text.data(), text.size());
   }
+  return ENS_OK;
+}
+
+extern "C" int ens_run_phases(ens_run *r, uint64_t ns[ENS_PHASES]) {
+  if (!r || !ns) return fail(ENS_EINVAL, "ens_run_phases: NULL");
+  std::memset(ns, 0, sizeof(uint64_t) * ENS_PHASES);
+  if (r->P.n == 0 || !r->launched) return ENS_OK;
+  if (!(r->flags & ENS_F_PHASES)) return fail(ENS_EINVAL, "ens_run_phases: launched without ENS_F_PHASES");
+  CU(cudaStreamSynchronize(r->stream));
+  CU(cudaMemcpy(ns, r->ws + r->P.o_phase, sizeof(uint64_t) * ENS_PHASES, cudaMemcpyDeviceToHost));
   return ENS_OK;
 }
 

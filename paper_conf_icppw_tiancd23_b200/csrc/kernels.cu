@@ -78,6 +78,8 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
     c.k = k;
     c.id = line;
     c.out = p.stdout_base + (size_t)k * p.stdout_cap;
+    c.phases = p.phases;
+    phase_mark(c, -1);
     Result r{};
     if (App::kTeam || cr == 0) r = App::run(c, argc, s_argv);
     team_sync(c);

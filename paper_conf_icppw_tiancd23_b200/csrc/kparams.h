@@ -27,6 +27,7 @@ struct KParams {
   char *arena_base;           // [teams][arena_bytes]
   uint64_t arena_bytes;
   uint32_t team_ctas;         // CTAs per team (thread-block cluster size)
+  unsigned long long *phases; // [ENS_PHASES] ns per phase (ENS_F_PHASES) or null
 };
 
 const void *kernel_ptr(uint32_t app, int T);

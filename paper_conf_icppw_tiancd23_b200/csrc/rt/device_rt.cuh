@@ -126,7 +126,23 @@ struct Ctx {
   Shared *sh;
   char *smem;          // dynamic shared memory of the app
   uint32_t crank, csize;  // CTA rank in the team, team CTAs
+  unsigned long long *phases;  // tracing: ns per phase, or null
+  unsigned long long t_mark;   // tracing: last mark (team thread 0)
 };
+
+__device__ __forceinline__ unsigned long long gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+// tracing: charge the time since the last mark to phase k (team thread 0)
+__device__ __forceinline__ void phase_mark(Ctx &c, int k) {
+  if (c.phases && threadIdx.x == 0 && c.crank == 0) {
+    const unsigned long long now = gtimer();
+    if (k >= 0) atomicAdd(&c.phases[k], now - c.t_mark);
+    c.t_mark = now;
+  }
+}
 
 // barrier of the whole team (cluster barrier: release/acquire at cluster
 // scope, so global and shared writes before it are visible after it)

@@ -1,20 +1,30 @@
 """Time ensembles of arbitrary lines on the GPU (phase probes, not the bench).
 
-    python tools/probe.py "xsbench -s large -g 11303 -G hash -l 0 -r {i}" 64 [threads] [reps]
+    python tools/probe.py "<line template with {i}>" N [threads] [reps] [--phases] [--team K]
+
+Prints the best-of-reps CUDA-event time of the ensemble launch; with
+--phases also the per-phase device time (ENS_F_PHASES tracing), summed over
+instances and divided by the number of concurrently running teams (so the
+numbers are comparable to the wall time).
 """
-import sys
 import os
+import sys
+
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 import torch  # noqa: E402
 from paper_conf_icppw_tiancd23_b200 import Args  # noqa: E402
 from paper_conf_icppw_tiancd23_b200.ensemble import Ensemble  # noqa: E402
 
+XS_PHASES = ["materials", "generate", "bucket scan", "scatter", "bucket sort", "clear tables", "union tables",
+             "index sweep", "record permute", "hash column", "lookup sample+sort", "lookup gathers"]
 
-def probe(template, n, threads=512, reps=3):
+
+def probe(template, n, threads=512, reps=3, phases=False, team=0):
     text = "".join(template.format(i=i) + "\n" for i in range(n))
-    e = Ensemble(Args.parse(text), app="auto", threads=threads).launch()
+    e = Ensemble(Args.parse(text), app="auto", threads=threads, phases=phases, team_ctas=team).launch()
     torch.cuda.synchronize()
     ts = []
+    ph = None
     for _ in range(reps):
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         a.record()
@@ -22,29 +32,27 @@ def probe(template, n, threads=512, reps=3):
         b.record()
         torch.cuda.synchronize()
         ts.append(a.elapsed_time(b))
+        if phases:
+            ph = e.run.phases_ns()
     r = e.collect(stdout=False)
     ok = bool((r.records["exit_code"] == 0).all())
     info = e.info()
     e.close()
-    return min(ts), ok, list(info.grid_blocks), list(info.block_threads)
+    return min(ts), ok, list(info.grid_blocks), list(info.block_threads), list(info.team_ctas), ph
 
 
 if __name__ == "__main__":
-    if len(sys.argv) > 2:
-        t, ok, g, T = probe(sys.argv[1], int(sys.argv[2]), *(int(x) for x in sys.argv[3:]))
-        print(f"{t:9.3f} ms ok={ok} grid={g} T={T} :: {sys.argv[1]} x{sys.argv[2]}")
-    else:
-        cases = [
-            ("xsbench -s large -g 11303 -G hash -h 10000 -l 0 -r {i}", 64, 512),
-            ("xsbench -s large -g 11303 -G hash -h 10000 -l 1000000 -r {i}", 64, 512),
-            ("xsbench -s large -g 11303 -G hash -h 10000 -l 1000000 -r {i}", 1, 512),
-            ("xsbench -s small -g 1000 -G unionized -l 0 -r {i}", 1024, 256),
-            ("xsbench -s small -g 1000 -G unionized -l 10000 -r {i}", 1024, 256),
-            ("xsbench -s small -g 1000 -G unionized -l 10000 -r {i}", 1024, 128),
-            ("xsbench -s small -g 1000 -G unionized -l 10000 -r {i}", 1024, 512),
-            ("rsbench -s small -l 10000 -p 1000 -w 100 -r {i}", 256, 256),
-            ("amgmk -x 32 -y 32 -z 32 -i 20 -k relax -r {i}", 1024, 1024),
-        ]
-        for tpl, n, T in cases:
-            t, ok, g, TT = probe(tpl, n, T)
-            print(f"{t:9.3f} ms ok={ok} grid={g} T={TT} :: {tpl} x{n}", flush=True)
+    args = [x for x in sys.argv[1:] if not x.startswith("--")]
+    phases = "--phases" in sys.argv
+    team = 0
+    if "--team" in sys.argv:
+        team = int(sys.argv[sys.argv.index("--team") + 1])
+        args.remove(str(team))
+    t, ok, g, T, cs, ph = probe(args[0], int(args[1]), *(int(x) for x in args[2:]), phases=phases, team=team)
+    print(f"{t:9.3f} ms ok={ok} grid={g} T={T} team={cs} :: {args[0]} x{args[1]}", flush=True)
+    if ph:
+        teams = max(max(g) // max(1, max(cs)), 1)
+        for k, v in enumerate(ph):
+            if v:
+                name = XS_PHASES[k] if k < len(XS_PHASES) else str(k)
+                print(f"    phase {k:2d} {name:20s} {v / 1e6 / teams:9.3f} ms per team", flush=True)
