@@ -86,6 +86,14 @@ typedef struct ens_run ens_run;
 #define ENS_MAX_LINE 65536
 int ens_load_args(const char *path, const char *argv0, ens_args **out);
 int ens_parse_args(const char *text, size_t len, const char *argv0, ens_args **out);
+/* Args-file script language (the paper's planned extension, §3.2):
+ * a line "@repeat N <template>" stands for N lines, i = 0..N-1, where
+ * "{expr}" is an integer expression in i (+ - * / % parentheses literals)
+ * and "{a|b|c}" the (i mod 3)-th alternative; other lines are unchanged.
+ * ens_load_args / ens_parse_args expand such lines (ENS_EPARSE if malformed).
+ * ens_expand_args writes the expanded text (at most cap bytes) and returns
+ * its full length, or <0.                                                      */
+long ens_expand_args(const char *text, size_t len, char *out, size_t cap);
 int ens_args_count(const ens_args *a); /* number of instances (lines), or <0 */
 /* host view of instance i: *argv borrowed from a, valid until ens_args_free */
 int ens_args_get(const ens_args *a, int i, int *argc, const char *const **argv);

@@ -66,6 +66,7 @@ def _load():
         "ens_load_args": (i, [ctypes.c_char_p, ctypes.c_char_p, pp]),
         "ens_parse_args": (i, [ctypes.c_char_p, sz, ctypes.c_char_p, pp]),
         "ens_args_count": (i, [p]),
+        "ens_expand_args": (ctypes.c_long, [ctypes.c_char_p, sz, p, sz]),
         "ens_args_get": (i, [p, i, ctypes.POINTER(ctypes.c_int), ctypes.POINTER(ctypes.POINTER(ctypes.c_char_p))]),
         "ens_args_free": (None, [p]),
         "ens_workspace_bytes": (i, [i, p, ctypes.POINTER(LaunchCfg), ctypes.POINTER(sz)]),
@@ -89,7 +90,7 @@ def _load():
 
 
 lib = _load()
-EXPORTED = ["ens_load_args", "ens_parse_args", "ens_args_count", "ens_args_get", "ens_args_free",
+EXPORTED = ["ens_load_args", "ens_parse_args", "ens_expand_args", "ens_args_count", "ens_args_get", "ens_args_free",
             "ens_workspace_bytes", "ens_launch", "ens_run_relaunch", "ens_collect", "ens_run_elapsed_ms",
             "ens_run_phases",
             "ens_run_get_info", "ens_format_stdout", "ens_run_free", "ens_strerror", "ens_last_error",
@@ -246,3 +247,15 @@ def format_stdout(app, raw):
 
 def version():
     return lib.ens_version().decode()
+
+
+def expand_args(text):
+    """Expand "@repeat N <template>" lines (the args-file script language)."""
+    if isinstance(text, str):
+        text = text.encode()
+    n = lib.ens_expand_args(text, len(text), None, 0)
+    if n < 0:
+        raise EnsError("ens_expand_args", n, "malformed @repeat template")
+    buf = ctypes.create_string_buffer(n + 1)
+    lib.ens_expand_args(text, len(text), buf, n + 1)
+    return buf.raw[:n].decode()

@@ -24,6 +24,7 @@
 
 namespace ens {
 long format_raw(const void *raw, size_t raw_len, std::string &out);
+int expand_args(const char *text, size_t len, std::string &out, long *bad_line);
 }
 
 using namespace ens;
@@ -69,6 +70,15 @@ extern "C" int ens_parse_args(const char *text, size_t len, const char *argv0, e
   if (!out || (!text && len)) return fail(ENS_EINVAL, "ens_parse_args: NULL argument");
   *out = nullptr;
   if (len && std::memchr(text, '\0', len)) return fail(ENS_EPARSE, "ens_parse_args: embedded NUL byte");
+  // "@repeat N <template>" lines (the args-file script language)
+  std::string expanded;
+  if ((len && text[0] == '@') || (len && std::strstr(std::string(text, len).c_str(), "\n@"))) {
+    long bad = -1;
+    if (expand_args(text, len, expanded, &bad))
+      return fail(ENS_EPARSE, "ens_parse_args: malformed @repeat template on line " + std::to_string(bad + 1));
+    text = expanded.data();
+    len = expanded.size();
+  }
   ens_args *a = new ens_args();
   uint32_t a0 = 0;
   if (argv0) {

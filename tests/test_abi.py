@@ -111,3 +111,49 @@ def test_stdout_formatter_rejects_garbage():
         format_stdout(1, struct.pack("<II", 99, 0))
     with pytest.raises(EnsError):
         format_stdout(1, struct.pack("<II", 5, 64))
+
+
+def py_expand(n, tpl):
+    """Independent reference for @repeat: Python eval of {expr} with C integer semantics."""
+    import re as _re
+
+    def cdiv(a, b):
+        q = abs(a) // abs(b)
+        return q if (a >= 0) == (b >= 0) else -q
+
+    out = []
+    for i in range(n):
+        def sub(mo):
+            body = mo.group(1)
+            if "|" in body:
+                alts = body.split("|")
+                return alts[i % len(alts)]
+            expr = body.replace("i", str(i))
+            expr = _re.sub(r"(\d+)\s*/\s*(\d+)", lambda m: str(cdiv(int(m.group(1)), int(m.group(2)))), expr)
+            return str(eval(expr))
+        out.append(_re.sub(r"\{([^}]*)\}", sub, tpl))
+    return "".join(l + "\n" for l in out)
+
+
+@pytest.mark.parametrize("n,tpl", [
+    (4, "xsbench -s small -r {1070+i}"),
+    (5, "rsbench -l {10000*(1+i%3)} -p {500|1000|2000} -w {50|100|200}{ -d|||}"),
+    (3, "amgmk -x {32} -y {i*8+24} -z {(i+1)*(i+2)}"),
+    (0, "echo {i}"),
+])
+def test_repeat_templates(n, tpl):
+    from paper_conf_icppw_tiancd23_b200 import Args, _ens
+    text = f"echo first\n@repeat {n} {tpl}\necho last\n"
+    exp = "echo first\n" + py_expand(n, tpl) + "echo last\n"
+    assert _ens.expand_args(text) == exp
+    a = Args.parse(text)
+    assert len(a) == n + 2
+    ref = Args.parse(exp)
+    assert [a.argv(k) for k in range(len(a))] == [ref.argv(k) for k in range(len(ref))]
+
+
+@pytest.mark.parametrize("bad", ["@repeat x echo", "@repeat 3 echo {i", "@repeat 2 echo {i/0}", "@repeat 2 echo {j}"])
+def test_repeat_errors(bad):
+    from paper_conf_icppw_tiancd23_b200 import Args, EnsError
+    with pytest.raises(EnsError):
+        Args.parse(bad + "\n")
