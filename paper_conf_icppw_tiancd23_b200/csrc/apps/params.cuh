@@ -22,10 +22,13 @@ constexpr int kXsMaxGp = 16384;  // per-nuclide sort fits one SM's shared memory
 struct XsParams {
   int n_iso = 355;
   int n_gp = 11303;
-  long long lookups = 17000000;
+  long long lookups = 17000000;  // event: total; history: per particle (default 34)
   int grid = XS_UNIONIZED;
   int bins = 10000;
   unsigned long long seed = 1070, gseed = 42;
+  bool history = false;          // -m history
+  long long particles = 500000;  // -p
+  bool lookups_set = false;
 };
 
 // returns the offending argv index, or -1
@@ -45,6 +48,7 @@ ENS_HD int xs_parse(int argc, const char *const *argv, XsParams &p) {
     } else if (str_eq(f, "-l")) {
       if (!parse_i64(v, &x) || x < 0 || x > (1LL << 40)) return i + 1;
       p.lookups = x;
+      p.lookups_set = true;
     } else if (str_eq(f, "-G")) {
       if (str_eq(v, "unionized")) p.grid = XS_UNIONIZED;
       else if (str_eq(v, "nuclide")) p.grid = XS_NUCLIDE;
@@ -54,7 +58,12 @@ ENS_HD int xs_parse(int argc, const char *const *argv, XsParams &p) {
       if (!parse_i64(v, &x) || x < 1 || x > 10000000) return i + 1;
       p.bins = (int)x;
     } else if (str_eq(f, "-m")) {
-      if (!str_eq(v, "event")) return i + 1;
+      if (str_eq(v, "event")) p.history = false;
+      else if (str_eq(v, "history")) p.history = true;
+      else return i + 1;
+    } else if (str_eq(f, "-p")) {
+      if (!parse_i64(v, &x) || x < 0 || x > (1LL << 32)) return i + 1;
+      p.particles = x;
     } else if (str_eq(f, "-r")) {
       if (!parse_i64(v, &x) || x < 0) return i + 1;
       p.seed = (unsigned long long)x;
@@ -66,6 +75,7 @@ ENS_HD int xs_parse(int argc, const char *const *argv, XsParams &p) {
     }
     i++;
   }
+  if (p.history && !p.lookups_set) p.lookups = 34;
   return -1;
 }
 

@@ -249,12 +249,22 @@ struct XsApp {
       init_nuc(c, p, L, S);  // nuclides striped over the team's CTAs
     }
     team_sync(c);
-    if (p.grid == XS_HASH) lookups<XS_HASH>(c, p, L, thr, nn, concs, mats, R);
-    else if (p.grid == XS_UNIONIZED) lookups<XS_UNIONIZED>(c, p, L, thr, nn, concs, mats, R);
-    else lookups<XS_NUCLIDE>(c, p, L, thr, nn, concs, mats, R);
+    if (p.history) {
+      if (p.grid == XS_HASH) lookups_history<XS_HASH>(c, p, L, thr, nn, concs, mats, R);
+      else if (p.grid == XS_UNIONIZED) lookups_history<XS_UNIONIZED>(c, p, L, thr, nn, concs, mats, R);
+      else lookups_history<XS_NUCLIDE>(c, p, L, thr, nn, concs, mats, R);
+    } else {
+      if (p.grid == XS_HASH) lookups<XS_HASH>(c, p, L, thr, nn, concs, mats, R);
+      else if (p.grid == XS_UNIONIZED) lookups<XS_UNIONIZED>(c, p, L, thr, nn, concs, mats, R);
+      else lookups<XS_NUCLIDE>(c, p, L, thr, nn, concs, mats, R);
+    }
     const char *grid = p.grid == XS_UNIONIZED ? "unionized" : p.grid == XS_NUCLIDE ? "nuclide" : "hash";
-    ens_printf(c, FMT_XS_HDR, n_iso == 68 ? "small" : "large", n_iso, (long long)p.n_gp, grid, p.lookups,
-               (unsigned long long)p.seed);
+    if (p.history)
+      ens_printf(c, FMT_XS_HIST, n_iso == 68 ? "small" : "large", n_iso, (long long)p.n_gp, grid, p.particles,
+                 p.lookups, (unsigned long long)p.seed);
+    else
+      ens_printf(c, FMT_XS_HDR, n_iso == 68 ? "small" : "large", n_iso, (long long)p.n_gp, grid, p.lookups,
+                 (unsigned long long)p.seed);
     ens_printf(c, FMT_VERIFY, (unsigned long long)R.vhash);
     R.exit_code = 0;
     return R;
@@ -739,6 +749,188 @@ struct XsApp {
     phase_mark(c, 8);
   }
 
+  // XS-7..XS-9 for one lookup (energy pe, material mat, union / hash index
+  // idx): the macroscopic XS m[0..4], nuclides summed in list order.
+  template <int GRID>
+  __device__ static __forceinline__ void macro_lookup(const XsParams &p, const double *recs, const int *ig,
+                                                      const int *nn, const double *concs, const uint16_t *mats,
+                                                      double pe, int mat, int idx, double *m) {
+    const int n_iso = p.n_iso, n_gp = p.n_gp, mx = xs_max_nucs(n_iso);
+    const int nm = nn[mat];
+    const uint16_t *mrow = mats + mat * mx;
+    const double *crow = concs + mat * mx;
+    double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
+    for (int j0 = 0; j0 < nm; j0 += kU) {
+      int nuc[kU], lo[kU], uh[kU];
+      bool on[kU];
+      double2 a0[kU], a1[kU], a2[kU], b0v[kU], b1[kU], b2[kU];
+#pragma unroll
+      for (int u = 0; u < kU; u++) {  // XS-7 step 1: index entries
+        on[u] = j0 + u < nm;
+        nuc[u] = on[u] ? mrow[j0 + u] : 0;
+        lo[u] = 0;
+        uh[u] = 0;
+        if (on[u]) {
+          if (GRID == XS_HASH) {
+            // {u_low, E[u_low+1]} and the next bin's u_low: the bracket is
+            // u_low if pe < E[u_low+1], else (usually) u_low+1 — verified
+            // against the loaded pair below
+            const XsHashEnt *he = (const XsHashEnt *)ig + (size_t)nuc[u] * (p.bins + 1) + idx;
+            const int4 h = ld_(reinterpret_cast<const int4 *>(he));
+            const double e_next = __hiloint2double(h.w, h.z);
+            uh[u] = ld_(&he[1].u_low) + 1;
+            lo[u] = pe < e_next ? h.x : h.x + 1;
+          } else if (GRID == XS_UNIONIZED) {
+            const int k = ld_(ig + (size_t)idx * n_iso + nuc[u]);
+            lo[u] = (k == n_gp - 1) ? k - 1 : k;
+          } else {
+            const int k = gs_recs(recs + (size_t)nuc[u] * n_gp * 6, pe, 0, n_gp - 1);
+            lo[u] = (k == n_gp - 1) ? k - 1 : k;
+          }
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < kU; u++) {  // step 2: record pair at lo (hash: at u_low)
+        if (on[u]) {
+          const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)nuc[u] * n_gp + lo[u]) * 6);
+          a0[u] = ld_(r2 + 0); a1[u] = ld_(r2 + 1); a2[u] = ld_(r2 + 2);
+          b0v[u] = ld_(r2 + 3); b1[u] = ld_(r2 + 4); b2[u] = ld_(r2 + 5);
+        }
+      }
+      if (GRID == XS_HASH) {
+#pragma unroll
+        for (int u = 0; u < kU; u++) {
+          // the guess lo is exactly upstream's bracket (grid_search on
+          // [u_low, u_high], its edge cases excluded) iff E[lo] < pe <
+          // E[lo+1] and lo+1 <= u_high; otherwise the full upstream logic
+          // walk forward while pe is past the pair (one gather per step;
+          // the guess is short by more than one record for ~1 in 8)
+          while (on[u] && pe >= b0v[u].x && a0[u].x < pe && lo[u] + 2 <= uh[u]) {
+            lo[u]++;
+            const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)nuc[u] * n_gp + lo[u]) * 6);
+            a0[u] = b0v[u]; a1[u] = b1[u]; a2[u] = b2[u];
+            b0v[u] = ld_(r2 + 3); b1[u] = ld_(r2 + 4); b2[u] = ld_(r2 + 5);
+          }
+          if (on[u] && !(a0[u].x < pe && pe < b0v[u].x && lo[u] + 1 <= uh[u])) {  // edges: upstream logic
+            const double *E = recs + (size_t)nuc[u] * n_gp * 6;
+            const XsHashEnt *he = (const XsHashEnt *)ig + (size_t)nuc[u] * (p.bins + 1) + idx;
+            const int u_low = ld_(&he->u_low);
+            const int u_high = uh[u];
+            const double e_low = ld_(E + 6 * (size_t)u_low);
+            const double e_high = ld_(E + 6 * (size_t)u_high);
+            int lower;
+            if (pe <= e_low) lower = 0;
+            else if (pe >= e_high) lower = n_gp - 1;
+            else lower = gs_recs(E, pe, u_low, u_high);
+            const int l2 = lower == n_gp - 1 ? lower - 1 : lower;
+            const double2 *r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)l2);
+            a0[u] = ld_(r2 + 0); a1[u] = ld_(r2 + 1); a2[u] = ld_(r2 + 2);
+            b0v[u] = ld_(r2 + 3); b1[u] = ld_(r2 + 4); b2[u] = ld_(r2 + 5);
+          }
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < kU; u++) {  // XS-8, XS-9 in nuclide order
+        if (on[u]) {
+          const double conc = crow[j0 + u];
+          // low = {E, total, elastic, absorption, fission, nu_fission}
+          const double f = (b0v[u].x - pe) / (b0v[u].x - a0[u].x);
+          m0 += (b0v[u].y - f * (b0v[u].y - a0[u].y)) * conc;
+          m1 += (b1[u].x - f * (b1[u].x - a1[u].x)) * conc;
+          m2 += (b1[u].y - f * (b1[u].y - a1[u].y)) * conc;
+          m3 += (b2[u].x - f * (b2[u].x - a2[u].x)) * conc;
+          m4 += (b2[u].y - f * (b2[u].y - a2[u].y)) * conc;
+        }
+      }
+    }
+    m[0] = m0;
+    m[1] = m1;
+    m[2] = m2;
+    m[3] = m3;
+    m[4] = m4;
+  }
+
+  // union position of energy pe == grid_search(u, pe, 0, n_u-1) (XS-7), via
+  // the search table: ufind[floor(pe*UB)] then a short forward scan
+  __device__ static __forceinline__ int union_idx(const uint32_t *uf, const uint64_t *uA, long long UB, long long n_u,
+                                                  double pe) {
+    long long b = (long long)(pe * (double)UB);
+    if (b > UB - 1) b = UB - 1;
+    long long cc = ld_(uf + b);
+    while (cc < n_u - 1 && __longlong_as_double((long long)ld_(uA + cc + 1)) <= pe) cc++;
+    return (int)(cc < n_u - 2 ? cc : n_u - 2);
+  }
+
+  // ---- history mode: thread per particle --------
+  // Particle q's stream starts at ff(seed, q * L * 10); its L lookups are a
+  // dependent chain (after each, skip one draw per macro channel > 1.0, then
+  // sample the next energy and material), so particles run in parallel.
+  template <int GRID>
+  __device__ static __noinline__ void lookups_history(Ctx &c, const XsParams &p, const XsLayout &L,
+                                                      const double *thr, const int *nn, const double *concs,
+                                                      const uint16_t *mats, Result &R) {
+    const int tid = threadIdx.x, T = blockDim.x;
+    const long long n_u = (long long)p.n_iso * p.n_gp, nL = p.lookups;
+    const double *recs = (const double *)(c.arena + L.recs);
+    const int *ig = (const int *)(c.arena + L.index);
+    const uint64_t *uA = (const uint64_t *)(c.arena + L.uenergy);
+    const uint32_t *uf = (const uint32_t *)(c.arena + L.ufind);
+    const long long UB = xs_ubins(p);
+    const double du = 1.0 / p.bins;
+    const long long g0 = (long long)c.crank * T + tid, gs = (long long)c.csize * T;
+    Affine fwd[6];  // skip 0..5 draws
+#pragma unroll
+    for (int k = 0; k < 6; k++) fwd[k] = lcg_pow((uint64_t)k);
+    const Affine J = lcg_pow((uint64_t)gs * (uint64_t)nL * 10ULL);
+    uint64_t s0 = lcg_pow((uint64_t)g0 * (uint64_t)nL * 10ULL)(p.seed);
+    unsigned long long ver = 0, bsum = 0;
+    double fsum = 0.0, fabs_ = 0.0;
+    for (long long q = g0; q < p.particles; q += gs, s0 = J(s0)) {
+      uint64_t s = s0;
+      double pe = lcg_double(s);
+      int mat = pick_mat_thr(thr, lcg_double(s));
+      for (long long i = 0; i < nL; i++) {
+        int idx = 0;
+        if (GRID == XS_UNIONIZED) idx = union_idx(uf, uA, UB, n_u, pe);
+        else if (GRID == XS_HASH) {
+          const long long bb = (long long)(pe / du);
+          idx = bb > p.bins - 1 ? p.bins - 1 : (int)bb;  // reading Q14
+        }
+        double m[5];
+        macro_lookup<GRID>(p, recs, ig, nn, concs, mats, pe, mat, idx, m);
+        double mxv = -1.0;
+        int am = 0;
+        int n_forward = 0;
+#pragma unroll
+        for (int x = 0; x < 5; x++) {
+          if (m[x] > mxv) {
+            mxv = m[x];
+            am = x;
+          }
+          n_forward += m[x] > 1.0 ? 1 : 0;
+          bsum += dbits(m[x]);
+          fsum += m[x];
+          fabs_ += fabs(m[x]);
+        }
+        ver += (unsigned long long)(am + 1);
+        atomicAdd(&c.sh->tallies[am], 1u);
+        atomicAdd(&c.sh->tallies[5 + mat], 1u);
+        s = fwd[n_forward](s);
+        pe = lcg_double(s);
+        mat = pick_mat_thr(thr, lcg_double(s));
+      }
+    }
+    ver = team_sum_u64(c, ver);
+    bsum = team_sum_u64(c, bsum);
+    fsum = team_sum_f64(c, fsum);
+    fabs_ = team_sum_f64(c, fabs_);
+    R.vhash = ver % 999983ULL;
+    R.bitsum = bsum;
+    R.fsum = fsum;
+    R.fabs = fabs_;
+    R.work = (uint64_t)p.particles * (uint64_t)nL;
+  }
+
   // ---- XS-6..XS-10: lookups ----------------------------------------------
   // Batches of K*T lookups: (A) every thread samples its K lookups (XS-6),
   // the batch is counting-sorted by material into shared memory; (B) thread
@@ -829,93 +1021,9 @@ struct XsApp {
           const long long bb = (long long)(pe / du);
           idx = bb > p.bins - 1 ? p.bins - 1 : (int)bb;  // reading Q14
         }
-        const int nm = nn[mat];
-        const uint16_t *mrow = mats + mat * mx;
-        const double *crow = concs + mat * mx;
-        double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
-        for (int j0 = 0; j0 < nm; j0 += kU) {
-          int nuc[kU], lo[kU], uh[kU];
-          bool on[kU];
-          double2 a0[kU], a1[kU], a2[kU], b0v[kU], b1[kU], b2[kU];
-#pragma unroll
-          for (int u = 0; u < kU; u++) {  // XS-7 step 1: index entries
-            on[u] = j0 + u < nm;
-            nuc[u] = on[u] ? mrow[j0 + u] : 0;
-            lo[u] = 0;
-            uh[u] = 0;
-            if (on[u]) {
-              if (GRID == XS_HASH) {
-                // {u_low, E[u_low+1]} and the next bin's u_low: the bracket is
-                // u_low if pe < E[u_low+1], else (usually) u_low+1 — verified
-                // against the loaded pair below
-                const XsHashEnt *he = (const XsHashEnt *)ig + (size_t)nuc[u] * (p.bins + 1) + idx;
-                const int4 h = ld_(reinterpret_cast<const int4 *>(he));
-                const double e_next = __hiloint2double(h.w, h.z);
-                uh[u] = ld_(&he[1].u_low) + 1;
-                lo[u] = pe < e_next ? h.x : h.x + 1;
-              } else if (GRID == XS_UNIONIZED) {
-                const int k = ld_(ig + (size_t)idx * n_iso + nuc[u]);
-                lo[u] = (k == n_gp - 1) ? k - 1 : k;
-              } else {
-                const int k = gs_recs(recs + (size_t)nuc[u] * n_gp * 6, pe, 0, n_gp - 1);
-                lo[u] = (k == n_gp - 1) ? k - 1 : k;
-              }
-            }
-          }
-#pragma unroll
-          for (int u = 0; u < kU; u++) {  // step 2: record pair at lo (hash: at u_low)
-            if (on[u]) {
-              const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)nuc[u] * n_gp + lo[u]) * 6);
-              a0[u] = ld_(r2 + 0); a1[u] = ld_(r2 + 1); a2[u] = ld_(r2 + 2);
-              b0v[u] = ld_(r2 + 3); b1[u] = ld_(r2 + 4); b2[u] = ld_(r2 + 5);
-            }
-          }
-          if (GRID == XS_HASH) {
-#pragma unroll
-            for (int u = 0; u < kU; u++) {
-              // the guess lo is exactly upstream's bracket (grid_search on
-              // [u_low, u_high], its edge cases excluded) iff E[lo] < pe <
-              // E[lo+1] and lo+1 <= u_high; otherwise the full upstream logic
-              // walk forward while pe is past the pair (one gather per step;
-              // the guess is short by more than one record for ~1 in 8)
-              while (on[u] && pe >= b0v[u].x && a0[u].x < pe && lo[u] + 2 <= uh[u]) {
-                lo[u]++;
-                const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)nuc[u] * n_gp + lo[u]) * 6);
-                a0[u] = b0v[u]; a1[u] = b1[u]; a2[u] = b2[u];
-                b0v[u] = ld_(r2 + 3); b1[u] = ld_(r2 + 4); b2[u] = ld_(r2 + 5);
-              }
-              if (on[u] && !(a0[u].x < pe && pe < b0v[u].x && lo[u] + 1 <= uh[u])) {  // edges: upstream logic
-                const double *E = recs + (size_t)nuc[u] * n_gp * 6;
-                const XsHashEnt *he = (const XsHashEnt *)ig + (size_t)nuc[u] * (p.bins + 1) + idx;
-                const int u_low = ld_(&he->u_low);
-                const int u_high = uh[u];
-                const double e_low = ld_(E + 6 * (size_t)u_low);
-                const double e_high = ld_(E + 6 * (size_t)u_high);
-                int lower;
-                if (pe <= e_low) lower = 0;
-                else if (pe >= e_high) lower = n_gp - 1;
-                else lower = gs_recs(E, pe, u_low, u_high);
-                const int l2 = lower == n_gp - 1 ? lower - 1 : lower;
-                const double2 *r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)l2);
-                a0[u] = ld_(r2 + 0); a1[u] = ld_(r2 + 1); a2[u] = ld_(r2 + 2);
-                b0v[u] = ld_(r2 + 3); b1[u] = ld_(r2 + 4); b2[u] = ld_(r2 + 5);
-              }
-            }
-          }
-#pragma unroll
-          for (int u = 0; u < kU; u++) {  // XS-8, XS-9 in nuclide order
-            if (on[u]) {
-              const double conc = crow[j0 + u];
-              // low = {E, total, elastic, absorption, fission, nu_fission}
-              const double f = (b0v[u].x - pe) / (b0v[u].x - a0[u].x);
-              m0 += (b0v[u].y - f * (b0v[u].y - a0[u].y)) * conc;
-              m1 += (b1[u].x - f * (b1[u].x - a1[u].x)) * conc;
-              m2 += (b1[u].y - f * (b1[u].y - a1[u].y)) * conc;
-              m3 += (b2[u].x - f * (b2[u].x - a2[u].x)) * conc;
-              m4 += (b2[u].y - f * (b2[u].y - a2[u].y)) * conc;
-            }
-          }
-        }
+        double mv[5];
+        macro_lookup<GRID>(p, recs, ig, nn, concs, mats, pe, mat, idx, mv);
+        const double m0 = mv[0], m1 = mv[1], m2 = mv[2], m3 = mv[3], m4 = mv[4];
         // XS-10
         double mxv = -1.0;
         int am = 0;

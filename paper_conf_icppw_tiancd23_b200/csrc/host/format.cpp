@@ -18,7 +18,7 @@ static const char *const kFmt[FMT_COUNT] = {
     /* FMT_BADARG    */ "%s: invalid argument '%s'\n",
     /* FMT_USAGE_XS  */
     "usage: %s [-s small|large] [-g gridpoints] [-l lookups] [-G unionized|nuclide|hash] [-h hash_bins] "
-    "[-m event] [-r seed] [-R grid_seed]\n",
+    "[-m event|history] [-p particles] [-r seed] [-R grid_seed]\n",
     /* FMT_USAGE_RS  */ "usage: %s [-s small|large] [-l lookups] [-p poles] [-w windows] [-d] [-r seed] [-R init_seed]\n",
     /* FMT_USAGE_AMG */ "usage: %s [-x nx] [-y ny] [-z nz] [-i iters] [-k relax|matvec|both] [-r seed]\n",
     /* FMT_NOTFOUND  */ "%s: command not found\n",
@@ -28,6 +28,7 @@ static const char *const kFmt[FMT_COUNT] = {
     /* FMT_VERIFY    */ "Verification checksum: %lu\n",
     /* FMT_RS_HDR    */ "RSBench-style HM=%s n_nuc=%d poles=%d windows=%d doppler=%d L=%ld seed=%lu\n",
     /* FMT_AMG       */ "AMGmk-style n=%d nnz=%d iters=%d maxerr=%.17g\n",
+    /* FMT_XS_HIST   */ "XSBench-style history HM=%s n_iso=%d n_gp=%ld grid=%s particles=%ld L=%ld seed=%lu\n",
 };
 
 // Expand one format with its slots; returns false on malformed input.

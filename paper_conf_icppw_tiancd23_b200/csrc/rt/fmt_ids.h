@@ -19,6 +19,7 @@ enum FmtId : unsigned {
   FMT_VERIFY = 8,     // "Verification checksum: %lu\n"
   FMT_RS_HDR = 9,     // RSBench-style header line
   FMT_AMG = 10,       // AMGmk-style result line
-  FMT_COUNT = 11
+  FMT_XS_HIST = 11,   // XSBench-style history-mode header line
+  FMT_COUNT = 12
 };
 }  // namespace ens

@@ -44,12 +44,20 @@ def test_fig5_loader_on_device(oracle):
     assert list(g.records["exit_code"]) == [6, 6, 6, 6]
 
 
+def same(a, b, f):
+    """Exact fields bit-for-bit; fsum / fabs within 1e-12 (their reduction tree
+    depends on the team size, which the auto scheduler picks per ensemble)."""
+    if f in ("fsum", "fabs"):
+        return abs(float(a) - float(b)) <= 1e-12 * max(abs(float(a)), 1e-300)
+    return a == b
+
+
 def test_solo_equals_ensemble():
     full = ens().run_text(text(LINES))
     for i, l in enumerate(LINES):
         solo = ens().run_text(text([l]))
         for f in FIELDS[1:]:
-            assert solo.records[0][f] == full.records[i][f], (i, f)
+            assert same(solo.records[0][f], full.records[i][f], f), (i, f)
         assert solo.stdout[0] == full.stdout[i]
         assert np.array_equal(solo.tallies[0], full.tallies[i])
 
@@ -57,13 +65,13 @@ def test_solo_equals_ensemble():
 def test_copies_and_permutation():
     r = ens().run_text(text([LINES[0]] * 37))
     for f in FIELDS[1:]:
-        assert np.all(r.records[f] == r.records[f][0])
+        assert all(same(x, r.records[f][0], f) for x in r.records[f])
     perm = [3, 0, 6, 2, 5, 1, 4]
     a = ens().run_text(text(LINES))
     b = ens().run_text(text([LINES[p] for p in perm]))
     for j, p in enumerate(perm):
         for f in FIELDS[1:]:
-            assert a.records[p][f] == b.records[j][f]
+            assert same(a.records[p][f], b.records[j][f], f)
 
 
 def test_sharded_launches_match_full():
@@ -76,7 +84,7 @@ def test_sharded_launches_match_full():
         for k in range(e.n):
             i = rank + k * G
             for f in FIELDS:
-                assert r.records[k][f] == full.records[i][f]
+                assert same(r.records[k][f], full.records[i][f], f)
             assert r.stdout[k] == full.stdout[i]
         e.close()
 

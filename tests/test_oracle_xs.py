@@ -27,6 +27,16 @@ def test_upstream_default_checksum_small(oracle):
 
 
 @pytest.mark.slow
+def test_upstream_history_checksum_small(oracle):
+    """History mode (NEXT 2): 500,000 particles x 34 dependent lookups."""
+    gold = json.load(open(os.path.join(GOLD, "xsbench_upstream_checksums.json")))["checksums"]
+    r = oracle.run_text("-s small -m history -G hash\n", app=oracle.APP_XSBENCH)
+    assert r.records[0]["exit_code"] == 0
+    assert int(r.records[0]["vhash"]) == gold["-s small -m history"]
+    assert r.records[0]["work"] == 500000 * 34
+
+
+@pytest.mark.slow
 def test_upstream_default_checksum_large(oracle):
     gold = json.load(open(os.path.join(GOLD, "xsbench_upstream_checksums.json")))["checksums"]
     r = oracle.run_text("-s large -m event -G hash\n", app=oracle.APP_XSBENCH)
@@ -117,7 +127,7 @@ def test_grid_types_agree_bitwise(oracle):
         assert recs[0][k] == recs[1][k] == recs[2][k]
 
 
-@pytest.mark.parametrize("line", ["-s medium", "-g 1", "-g", "-l -5", "-G sorted", "-m history", "-q 1",
+@pytest.mark.parametrize("line", ["-s medium", "-g 1", "-g", "-l -5", "-G sorted", "-m hist", "-q 1",
                                   "-g 12x", "-r -1", "-h 0"])
 def test_usage_errors(oracle, line):
     r = oracle.run_text(line + "\n", app=oracle.APP_XSBENCH)
