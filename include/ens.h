@@ -65,8 +65,10 @@ typedef enum {
   ENS_APP_ECHO = 1,
   ENS_APP_XSBENCH = 2,
   ENS_APP_RSBENCH = 3,
-  ENS_APP_AMGMK = 4
+  ENS_APP_AMGMK = 4,
+  ENS_APP_PAGERANK = 5
 } ens_app;
+#define ENS_N_APPS 6
 
 typedef struct ens_args ens_args;
 typedef struct ens_run ens_run;
@@ -189,8 +191,8 @@ int ens_run_phases(ens_run *r, uint64_t ns[ENS_PHASES]);
 typedef struct {
   int32_t n_instances;
   int32_t n_groups;        /* kernel launches (one per app present)            */
-  int32_t grid_blocks[5];  /* CTAs launched, per ens_app, 0 if absent            */
-  int32_t block_threads[5];
+  int32_t grid_blocks[ENS_N_APPS];  /* CTAs launched, per ens_app, 0 if absent   */
+  int32_t block_threads[ENS_N_APPS];
   int32_t kernel_launches; /* kernels per (re)launch                             */
   uint64_t arena_bytes;    /* per slot (max over groups)                         */
   uint64_t ws_bytes;
@@ -200,7 +202,7 @@ typedef struct {
   uint32_t stdout_bytes;   /* raw stdout bytes per instance                      */
   uint64_t h2d_bytes;      /* bytes copied host->device by ens_launch            */
   uint64_t d2h_bytes;      /* bytes copied device->host by the last ens_collect  */
-  int32_t team_ctas[5];    /* CTAs per team (cluster size), per ens_app           */
+  int32_t team_ctas[ENS_N_APPS];  /* CTAs per team (cluster size), per ens_app    */
 } ens_run_info;
 int ens_run_get_info(const ens_run *r, ens_run_info *info);
 

@@ -184,6 +184,7 @@ static uint32_t app_of_argv0(const std::string &a0) {
   if (b == "xsbench") return APP_XSBENCH;
   if (b == "rsbench") return APP_RSBENCH;
   if (b == "amgmk") return APP_AMGMK;
+  if (b == "pagerank") return APP_PAGERANK;
   return APP_BY_ARGV0;
 }
 
@@ -205,6 +206,7 @@ void run_isolated(uint32_t app, const std::vector<std::string> &argv, Instance &
     case APP_XSBENCH: run_xsbench(argv, inst); break;
     case APP_RSBENCH: run_rsbench(argv, inst); break;
     case APP_AMGMK: run_amgmk(argv, inst); break;
+    case APP_PAGERANK: run_pagerank(argv, inst); break;
     default: inst.rec.exit_code = 127; break;
   }
   inst.rec.flags |= kFlagDone;

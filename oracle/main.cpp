@@ -52,7 +52,7 @@ int main(int argc, char **argv) {
     else if (f == "-a") {
       std::string a = need();
       app = a == "echo" ? APP_ECHO : a == "xsbench" ? APP_XSBENCH : a == "rsbench" ? APP_RSBENCH
-          : a == "amgmk" ? APP_AMGMK : APP_BY_ARGV0;
+          : a == "amgmk" ? APP_AMGMK : a == "pagerank" ? APP_PAGERANK : APP_BY_ARGV0;
     } else {
       std::fprintf(stderr, "usage: ens_oracle -f file [-n N] [-j jobs] [-a app] [--argv0 name] [-o out.bin] [-q]\n");
       return 2;
@@ -70,7 +70,7 @@ int main(int argc, char **argv) {
   std::stringstream ss;
   ss << in.rdbuf();
   // explicit app without --argv0: the app name is argv[0] (reading Q3)
-  static const char *names[] = {"", "echo", "xsbench", "rsbench", "amgmk"};
+  static const char *names[] = {"", "echo", "xsbench", "rsbench", "amgmk", "pagerank"};
   if (!argv0 && app != APP_BY_ARGV0) argv0 = names[app];
   Args a = parse_args_text(ss.str(), argv0);
   if (n < 0) n = (long)a.lines.size();

@@ -44,7 +44,8 @@ constexpr uint32_t kFlagNomem = 1u << 1;
 constexpr uint32_t kFlagNotRun = 1u << 2;
 constexpr uint32_t kFlagDone = 1u << 3;
 
-enum App : uint32_t { APP_BY_ARGV0 = 0, APP_ECHO = 1, APP_XSBENCH = 2, APP_RSBENCH = 3, APP_AMGMK = 4 };
+enum App : uint32_t { APP_BY_ARGV0 = 0, APP_ECHO = 1, APP_XSBENCH = 2, APP_RSBENCH = 3, APP_AMGMK = 4,
+                      APP_PAGERANK = 5 };
 
 // ---- args file (Fig. 4, Fig. 5; readings Q1-Q4) -------
 struct Args {
@@ -75,6 +76,7 @@ void run_echo(const std::vector<std::string> &argv, Instance &inst);
 void run_xsbench(const std::vector<std::string> &argv, Instance &inst);
 void run_rsbench(const std::vector<std::string> &argv, Instance &inst);
 void run_amgmk(const std::vector<std::string> &argv, Instance &inst);
+void run_pagerank(const std::vector<std::string> &argv, Instance &inst);
 
 // one isolated run: dispatch on app (BY_ARGV0 → basename of argv[0])
 void run_isolated(uint32_t app, const std::vector<std::string> &argv, Instance &inst);

@@ -26,6 +26,9 @@ void fast_w(double zr, double zi, double *wr, double *wi);
 void init_tables(int small, int avg_poles, int avg_windows, uint64_t iseed, std::vector<int> &n_poles,
                  std::vector<int> &n_windows, std::vector<int> &win_start, std::vector<int> &win_end);
 }  // namespace rs_hooks
+namespace pr_hooks {
+void graph(long n, long avg, uint64_t gseed, std::vector<long> &deg, std::vector<long> &ptr, std::vector<long> &src);
+}
 namespace amg_hooks {
 void laplacian(long nx, long ny, long nz, std::vector<int> &row_ptr, std::vector<int> &col, std::vector<double> &val);
 void sweeps(long nx, long ny, long nz, long iters, std::vector<double> &u);
@@ -198,6 +201,17 @@ void oracle_amg_apply(long nx, long ny, long nz, const double *u, double *y) {
   std::vector<double> v(u, u + n), w;
   amg_hooks::apply(nx, ny, nz, v, w);
   std::memcpy(y, w.data(), (size_t)n * 8);
+}
+
+// ---- PageRank hooks ------------------------------------------------------------
+// in-edge CSR of the PR-2 graph; returns the edge count (arrays may be NULL to size)
+long oracle_pr_graph(long n, long avg, uint64_t gseed, long *deg, long *ptr, long *src) {
+  std::vector<long> d, p, s;
+  pr_hooks::graph(n, avg, gseed, d, p, s);
+  if (deg) std::memcpy(deg, d.data(), d.size() * sizeof(long));
+  if (ptr) std::memcpy(ptr, p.data(), p.size() * sizeof(long));
+  if (src) std::memcpy(src, s.data(), s.size() * sizeof(long));
+  return (long)s.size();
 }
 
 }  // extern "C"

@@ -18,8 +18,9 @@ ENS_EXIT_USAGE, ENS_EXIT_NOMEM, ENS_EXIT_NOTFOUND = 1, 12, 127
 ENS_RF_STDOUT_TRUNC, ENS_RF_NOMEM, ENS_RF_NOT_RUN, ENS_RF_DONE = 1, 2, 4, 8
 ENS_F_TIMESTAMPS, ENS_F_PHASES = 1, 2
 ENS_PHASES = 16
-ENS_APP_BY_ARGV0, ENS_APP_ECHO, ENS_APP_XSBENCH, ENS_APP_RSBENCH, ENS_APP_AMGMK = 0, 1, 2, 3, 4
-APP_IDS = {"auto": 0, "echo": 1, "xsbench": 2, "rsbench": 3, "amgmk": 4}
+ENS_APP_BY_ARGV0, ENS_APP_ECHO, ENS_APP_XSBENCH, ENS_APP_RSBENCH, ENS_APP_AMGMK, ENS_APP_PAGERANK = 0, 1, 2, 3, 4, 5
+ENS_N_APPS = 6
+APP_IDS = {"auto": 0, "echo": 1, "xsbench": 2, "rsbench": 3, "amgmk": 4, "pagerank": 5}
 ENS_TALLIES = 32
 ENS_MAX_ARGC = 128
 
@@ -47,12 +48,12 @@ class LaunchCfg(ctypes.Structure):
 
 class RunInfo(ctypes.Structure):
     _fields_ = [("n_instances", ctypes.c_int32), ("n_groups", ctypes.c_int32),
-                ("grid_blocks", ctypes.c_int32 * 5), ("block_threads", ctypes.c_int32 * 5),
+                ("grid_blocks", ctypes.c_int32 * ENS_N_APPS), ("block_threads", ctypes.c_int32 * ENS_N_APPS),
                 ("kernel_launches", ctypes.c_int32), ("arena_bytes", ctypes.c_uint64),
                 ("ws_bytes", ctypes.c_uint64), ("records_offset", ctypes.c_uint64),
                 ("tallies_offset", ctypes.c_uint64), ("stdout_offset", ctypes.c_uint64),
                 ("stdout_bytes", ctypes.c_uint32), ("h2d_bytes", ctypes.c_uint64),
-                ("d2h_bytes", ctypes.c_uint64), ("team_ctas", ctypes.c_int32 * 5)]
+                ("d2h_bytes", ctypes.c_uint64), ("team_ctas", ctypes.c_int32 * ENS_N_APPS)]
 
 
 def _load():

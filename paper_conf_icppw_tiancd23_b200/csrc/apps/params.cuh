@@ -13,7 +13,66 @@
 namespace ens {
 
 enum AppId : uint32_t { APP_BY_ARGV0 = 0, APP_ECHO = 1, APP_XSBENCH = 2, APP_RSBENCH = 3, APP_AMGMK = 4,
-                        APP_NOTFOUND = 5 /* internal: argv[0] names no app */ };
+                        APP_PAGERANK = 5, APP_NOTFOUND = 6 /* internal: argv[0] names no app */ };
+constexpr int kApps = 7;
+
+// ============================ Page-Rank-style ==============================
+struct PrParams {
+  long long n = 100000;
+  int avg = 8;
+  int iters = 10;
+  unsigned long long gseed = 42;
+};
+ENS_HD int pr_parse(int argc, const char *const *argv, PrParams &p) {
+  for (int i = 1; i < argc; i++) {
+    const char *f = argv[i];
+    if (i + 1 >= argc) return i;
+    const char *v = argv[i + 1];
+    long long x;
+    if (str_eq(f, "-n")) {
+      if (!parse_i64(v, &x) || x < 1 || x > (1LL << 24)) return i + 1;
+      p.n = x;
+    } else if (str_eq(f, "-e")) {
+      if (!parse_i64(v, &x) || x < 1 || x > 1024) return i + 1;
+      p.avg = (int)x;
+    } else if (str_eq(f, "-i")) {
+      if (!parse_i64(v, &x) || x < 0 || x > 100000) return i + 1;
+      p.iters = (int)x;
+    } else if (str_eq(f, "-R")) {
+      if (!parse_i64(v, &x) || x < 0) return i + 1;
+      p.gseed = (unsigned long long)x;
+    } else {
+      return i;
+    }
+    i++;
+  }
+  if (p.n * (2LL * p.avg - 1) > (1LL << 28)) return 0;  // edge-count cap (reading R-pr-range)
+  return -1;
+}
+struct PrLayout {
+  uint64_t deg, dstart, src_of_edge, tgt, in_ptr, cursor, in_e, r, r2, total;
+};
+ENS_HD PrLayout pr_layout(const PrParams &p) {
+  PrLayout L{};
+  const uint64_t n = (uint64_t)p.n, emax = (uint64_t)p.n * (uint64_t)(2 * p.avg - 1);
+  uint64_t o = 0;
+  auto take = [&](uint64_t bytes) {
+    const uint64_t at = o;
+    o = (o + bytes + 255) / 256 * 256;
+    return at;
+  };
+  L.deg = take(n * 4);
+  L.dstart = take((n + 8) * 4);
+  L.src_of_edge = take(emax * 4);
+  L.tgt = take(emax * 4);
+  L.in_ptr = take((n + 8) * 4);
+  L.cursor = take(n * 4);
+  L.in_e = take(emax * 4);
+  L.r = take(n * 8);
+  L.r2 = take(n * 8);
+  L.total = o;
+  return L;
+}
 
 // ============================ XSBench-style ================================
 enum { XS_UNIONIZED = 0, XS_NUCLIDE = 1, XS_HASH = 2 };

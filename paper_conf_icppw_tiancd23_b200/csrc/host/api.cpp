@@ -210,6 +210,7 @@ static uint32_t app_of_argv0(const char *a0) {
   if (!std::strcmp(b, "xsbench")) return APP_XSBENCH;
   if (!std::strcmp(b, "rsbench")) return APP_RSBENCH;
   if (!std::strcmp(b, "amgmk")) return APP_AMGMK;
+  if (!std::strcmp(b, "pagerank")) return APP_PAGERANK;
   return APP_NOTFOUND;
 }
 
@@ -224,7 +225,7 @@ static int threads_for(int32_t t) {
 // the whole workspace (0 = unlimited).
 static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, size_t mem_cap, Plan &P) {
   if (!a || !c) return fail(ENS_EINVAL, "ens_launch: NULL args or cfg");
-  if ((uint32_t)app > ENS_APP_AMGMK) return fail(ENS_EINVAL, "ens_launch: unknown app");
+  if ((uint32_t)app >= ENS_N_APPS) return fail(ENS_EINVAL, "ens_launch: unknown app");
   const int count = ens_args_count(a);
   const int64_t n = c->n_instances, first = c->first, stride = c->stride <= 0 ? 1 : c->stride;
   if (n < 0 || first < 0) return fail(ENS_EINVAL, "ens_launch: negative first / n_instances");
@@ -240,7 +241,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   if (e != cudaSuccess) return cuda_fail(e, "cudaDeviceGetAttribute");
 
   // group instances by app; shared memory per group (independent of team size)
-  Group g_by_app[6];
+  Group g_by_app[kApps];
   P.line_of_k.resize((size_t)n);
   for (int64_t k = 0; k < n; k++) {
     const uint32_t line = (uint32_t)(first + k * stride);
@@ -262,8 +263,8 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   // fewer instances than resident CTAs (the largest power of two <= 8 with
   // n_group * cs <= resident CTAs), or the cfg's team_ctas
   uint64_t need_arena = 0;
-  for (uint32_t ap : {(uint32_t)APP_XSBENCH, (uint32_t)APP_RSBENCH, (uint32_t)APP_AMGMK, (uint32_t)APP_ECHO,
-                      (uint32_t)APP_NOTFOUND}) {
+  for (uint32_t ap : {(uint32_t)APP_XSBENCH, (uint32_t)APP_RSBENCH, (uint32_t)APP_AMGMK, (uint32_t)APP_PAGERANK,
+                      (uint32_t)APP_ECHO, (uint32_t)APP_NOTFOUND}) {
     Group &g = g_by_app[ap];
     if (g.kmap.empty()) continue;
     g.T = std::min(T, app_max_threads(ap));

@@ -29,6 +29,8 @@ static const char *const kFmt[FMT_COUNT] = {
     /* FMT_RS_HDR    */ "RSBench-style HM=%s n_nuc=%d poles=%d windows=%d doppler=%d L=%ld seed=%lu\n",
     /* FMT_AMG       */ "AMGmk-style n=%d nnz=%d iters=%d maxerr=%.17g\n",
     /* FMT_XS_HIST   */ "XSBench-style history HM=%s n_iso=%d n_gp=%ld grid=%s particles=%ld L=%ld seed=%lu\n",
+    /* FMT_USAGE_PR  */ "usage: %s [-n nodes] [-e avg_degree] [-i iterations] [-R graph_seed]\n",
+    /* FMT_PR        */ "PageRank-style n=%ld edges=%ld iters=%ld top=%ld\n",
 };
 
 // Expand one format with its slots; returns false on malformed input.

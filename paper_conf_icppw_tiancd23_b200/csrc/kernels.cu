@@ -13,6 +13,7 @@
 
 #include "apps/amgmk.cuh"
 #include "apps/echo.cuh"
+#include "apps/pagerank.cuh"
 #include "apps/rsbench.cuh"
 #include "apps/xsbench.cuh"
 #include "kparams.h"
@@ -145,6 +146,7 @@ int app_max_threads(uint32_t app) {
     case APP_XSBENCH: return XsApp::kMaxT;
     case APP_RSBENCH: return RsApp::kMaxT;
     case APP_AMGMK: return AmgApp::kMaxT;
+    case APP_PAGERANK: return PrApp::kMaxT;
     case APP_NOTFOUND: return NotFoundApp::kMaxT;
   }
   return 32;
@@ -158,6 +160,7 @@ const void *kernel_ptr(uint32_t app, int T) {
     case APP_XSBENCH: return kernel_for<XsApp>(T);
     case APP_RSBENCH: return kernel_for<RsApp>(T);
     case APP_AMGMK: return kernel_for<AmgApp>(T);
+    case APP_PAGERANK: return kernel_for<PrApp>(T);
     case APP_NOTFOUND: return kernel_for<NotFoundApp>(T);
   }
   return nullptr;
@@ -170,6 +173,7 @@ bool app_size(uint32_t app, int argc, const char *const *argv, int T, int cs, ui
     case APP_XSBENCH: return XsApp::size(argc, argv, T, cs, arena, smem);
     case APP_RSBENCH: return RsApp::size(argc, argv, T, cs, arena, smem);
     case APP_AMGMK: return AmgApp::size(argc, argv, T, cs, arena, smem);
+    case APP_PAGERANK: return PrApp::size(argc, argv, T, cs, arena, smem);
     case APP_NOTFOUND: return NotFoundApp::size(argc, argv, T, cs, arena, smem);
   }
   *arena = 0;

@@ -20,6 +20,8 @@ enum FmtId : unsigned {
   FMT_RS_HDR = 9,     // RSBench-style header line
   FMT_AMG = 10,       // AMGmk-style result line
   FMT_XS_HIST = 11,   // XSBench-style history-mode header line
-  FMT_COUNT = 12
+  FMT_USAGE_PR = 12,  // pagerank usage line
+  FMT_PR = 13,        // Page-Rank-style result line
+  FMT_COUNT = 14
 };
 }  // namespace ens

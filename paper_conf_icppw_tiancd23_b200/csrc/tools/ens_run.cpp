@@ -44,7 +44,7 @@ int main(int argc, char **argv) {
     else if (f == "-a") {
       std::string a = val();
       app = a == "echo" ? ENS_APP_ECHO : a == "xsbench" ? ENS_APP_XSBENCH : a == "rsbench" ? ENS_APP_RSBENCH
-          : a == "amgmk" ? ENS_APP_AMGMK : ENS_APP_BY_ARGV0;
+          : a == "amgmk" ? ENS_APP_AMGMK : a == "pagerank" ? ENS_APP_PAGERANK : ENS_APP_BY_ARGV0;
     } else {
       std::fprintf(stderr, "usage: ens_run -f file [-n N] [-t T] [-a auto|echo|xsbench|rsbench|amgmk] [-g grid] "
                            "[--argv0 name] [--timestamps] [-q]\n");
@@ -55,7 +55,7 @@ int main(int argc, char **argv) {
     std::fprintf(stderr, "ens_run: -f is required\n");
     return 2;
   }
-  static const char *names[] = {nullptr, "echo", "xsbench", "rsbench", "amgmk"};
+  static const char *names[] = {nullptr, "echo", "xsbench", "rsbench", "amgmk", "pagerank"};
   if (!argv0 && app != ENS_APP_BY_ARGV0) argv0 = names[app];
   ens_args *a = nullptr;
   int rc = ens_load_args(file, argv0, &a);

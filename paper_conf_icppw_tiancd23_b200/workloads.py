@@ -61,7 +61,17 @@ def tstar(n=1024, seed0=1070):
     return c1(n, seed0)
 
 
-CONFIGS = {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5, "TSTAR": tstar}
+def pr(n=256):
+    """NEXT 3: Page-Rank-style instances (100k nodes, mean out-degree 8, 10 iterations)."""
+    return [f"pagerank -n 100000 -e 8 -i 10 -R {i}" for i in range(n)]
+
+
+def xs_history(n=64, particles=100000):
+    """NEXT 2: XSBench-style history mode (small), distinct seeds."""
+    return [f"xsbench -s small -m history -p {particles} -G unionized -r {1070 + i}" for i in range(n)]
+
+
+CONFIGS = {"C1": c1, "C2": c2, "C3": c3, "C4": c4, "C5": c5, "TSTAR": tstar, "PR": pr, "XSHIST": xs_history}
 
 
 def text(lines):

@@ -16,8 +16,9 @@ ORACLE_DIR = os.path.join(ROOT, "oracle")
 LIB_PATH = os.path.join(ORACLE_DIR, "liboracle.so")
 BIN_PATH = os.path.join(ORACLE_DIR, "ens_oracle")
 
-APP_BY_ARGV0, APP_ECHO, APP_XSBENCH, APP_RSBENCH, APP_AMGMK = 0, 1, 2, 3, 4
-APP_NAMES = {APP_ECHO: "echo", APP_XSBENCH: "xsbench", APP_RSBENCH: "rsbench", APP_AMGMK: "amgmk"}
+APP_BY_ARGV0, APP_ECHO, APP_XSBENCH, APP_RSBENCH, APP_AMGMK, APP_PAGERANK = 0, 1, 2, 3, 4, 5
+APP_NAMES = {APP_ECHO: "echo", APP_XSBENCH: "xsbench", APP_RSBENCH: "rsbench", APP_AMGMK: "amgmk",
+             APP_PAGERANK: "pagerank"}
 N_TALLIES = 32
 
 RECORD_DTYPE = np.dtype([
@@ -77,6 +78,7 @@ def lib():
                 "oracle_amg_csr": (None, [c_l, c_l, c_l, c_p, c_p, c_p]),
                 "oracle_amg_sweeps": (None, [c_l, c_l, c_l, c_l, c_p]),
                 "oracle_amg_apply": (None, [c_l, c_l, c_l, c_p, c_p]),
+                "oracle_pr_graph": (c_l, [c_l, c_l, c_u64, c_p, c_p, c_p]),
             }
             for name, (res, args) in sig.items():
                 f = getattr(L, name)
@@ -247,6 +249,16 @@ def amg_sweeps(nx, ny, nz, iters, u):
     u = np.array(u, dtype=np.float64, copy=True)
     lib().oracle_amg_sweeps(nx, ny, nz, iters, _ptr(u))
     return u
+
+
+def pr_graph(n, avg, gseed=42):
+    """PR-2 graph: out-degrees, in-edge CSR (ptr, src) in (source, edge) order."""
+    e = lib().oracle_pr_graph(n, avg, gseed, None, None, None)
+    deg = np.zeros(n, dtype=np.int64)
+    ptr = np.zeros(n + 1, dtype=np.int64)
+    src = np.zeros(max(e, 1), dtype=np.int64)
+    lib().oracle_pr_graph(n, avg, gseed, _ptr(deg), _ptr(ptr), _ptr(src))
+    return deg, ptr, src[:e]
 
 
 def amg_apply(nx, ny, nz, u):
