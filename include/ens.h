@@ -126,6 +126,14 @@ typedef struct {
                          4 or 8 (a thread-block cluster with distributed shared
                          memory); 0 = auto (largest power of two <= 8 with
                          n x team_ctas <= resident CTAs), ignored by other apps */
+  int32_t instances_per_cta; /* M, the paper's (N/M, M, 1) block mapping
+                         (P:393-404): M instances share one CTA, each on the
+                         row threadIdx.y of block_threads/M threads with its
+                         own arena slot and scheduler state.  1, 2, 4 or 8
+                         (rounded down to a power of two, and so that each
+                         instance keeps >= 32 threads); 0 = 1.  Applies to the
+                         bodies built for it (AMGmk, Page-Rank, echo, unknown
+                         programs) with team_ctas == 1; ignored by others.    */
 } ens_launch_cfg;
 
 /* Device bytes ens_launch needs for (app, a, c).  With c->grid_blocks == 0
@@ -203,6 +211,7 @@ typedef struct {
   uint64_t h2d_bytes;      /* bytes copied host->device by ens_launch            */
   uint64_t d2h_bytes;      /* bytes copied device->host by the last ens_collect  */
   int32_t team_ctas[ENS_N_APPS];  /* CTAs per team (cluster size), per ens_app    */
+  int32_t instances_per_cta[ENS_N_APPS]; /* M per ens_app (0 if absent)          */
 } ens_run_info;
 int ens_run_get_info(const ens_run *r, ens_run_info *info);
 

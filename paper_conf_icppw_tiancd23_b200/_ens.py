@@ -43,7 +43,7 @@ class LaunchCfg(ctypes.Structure):
     _fields_ = [("first", ctypes.c_int32), ("n_instances", ctypes.c_int32), ("stride", ctypes.c_int32),
                 ("grid_blocks", ctypes.c_int32), ("block_threads", ctypes.c_int32),
                 ("arena_bytes", ctypes.c_uint64), ("stdout_bytes", ctypes.c_uint32), ("flags", ctypes.c_uint32),
-                ("team_ctas", ctypes.c_int32)]
+                ("team_ctas", ctypes.c_int32), ("instances_per_cta", ctypes.c_int32)]
 
 
 class RunInfo(ctypes.Structure):
@@ -53,7 +53,8 @@ class RunInfo(ctypes.Structure):
                 ("ws_bytes", ctypes.c_uint64), ("records_offset", ctypes.c_uint64),
                 ("tallies_offset", ctypes.c_uint64), ("stdout_offset", ctypes.c_uint64),
                 ("stdout_bytes", ctypes.c_uint32), ("h2d_bytes", ctypes.c_uint64),
-                ("d2h_bytes", ctypes.c_uint64), ("team_ctas", ctypes.c_int32 * ENS_N_APPS)]
+                ("d2h_bytes", ctypes.c_uint64), ("team_ctas", ctypes.c_int32 * ENS_N_APPS),
+                ("instances_per_cta", ctypes.c_int32 * ENS_N_APPS)]
 
 
 def _load():
@@ -155,8 +156,10 @@ class Args:
             pass
 
 
-def make_cfg(n, first=0, stride=1, grid=0, threads=0, arena_bytes=0, stdout_bytes=0, flags=0, team_ctas=0):
-    return LaunchCfg(first, n, stride, grid, threads, arena_bytes, stdout_bytes, flags, team_ctas)
+def make_cfg(n, first=0, stride=1, grid=0, threads=0, arena_bytes=0, stdout_bytes=0, flags=0, team_ctas=0,
+             instances_per_cta=0):
+    return LaunchCfg(first, n, stride, grid, threads, arena_bytes, stdout_bytes, flags, team_ctas,
+                     instances_per_cta)
 
 
 def workspace_bytes(app, args, cfg):

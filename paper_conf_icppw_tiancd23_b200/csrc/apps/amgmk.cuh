@@ -19,6 +19,7 @@ struct AmgApp {
   static constexpr uint32_t kId = APP_AMGMK;
   static constexpr int kMaxT = 1024;  // 64 registers suffice
   static constexpr bool kTeam = false;
+  static constexpr bool kSub = true;  // runs as one of M instances per CTA (row threadIdx.y)
 
   __device__ static Result run(Ctx &c, int argc, char **argv) {
     Result R{};
@@ -78,7 +79,7 @@ struct AmgApp {
       }
       y[r] = 0.0;
     }
-    __syncthreads();
+    sub_sync();
 
     // ---- AMG-3: Jacobi sweeps and/or matvec -------------------------------
     for (int it = 0; it < p.iters; it++) {
@@ -94,7 +95,7 @@ struct AmgApp {
           }
           u2[r] = res / a0;
         }
-        __syncthreads();
+        sub_sync();
         double *t = u; u = u2; u2 = t;
       }
       if (p.kind == 1 || p.kind == 2) {
@@ -108,7 +109,7 @@ struct AmgApp {
           }
           y[r] = acc;
         }
-        __syncthreads();
+        sub_sync();
       }
     }
 

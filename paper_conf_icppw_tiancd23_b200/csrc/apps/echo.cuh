@@ -12,6 +12,7 @@ struct EchoApp {
   static constexpr uint32_t kId = APP_ECHO;
   static constexpr int kMaxT = 1024;
   static constexpr bool kTeam = false;
+  static constexpr bool kSub = true;
   __device__ static Result run(Ctx &c, int argc, char **argv) {
     Result R{};
     ens_printf(c, FMT_ECHO_ARGC, argc);
@@ -31,6 +32,7 @@ struct NotFoundApp {
   static constexpr uint32_t kId = APP_NOTFOUND;
   static constexpr int kMaxT = 1024;
   static constexpr bool kTeam = false;
+  static constexpr bool kSub = true;
   __device__ static Result run(Ctx &c, int argc, char **argv) {
     Result R{};
     ens_printf(c, FMT_NOTFOUND, argc > 0 ? (const char *)argv[0] : "");

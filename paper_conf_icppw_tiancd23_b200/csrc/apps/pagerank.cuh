@@ -23,6 +23,7 @@ struct PrApp {
   static constexpr uint32_t kId = APP_PAGERANK;
   static constexpr int kMaxT = 1024;
   static constexpr bool kTeam = false;
+  static constexpr bool kSub = true;
 
   __device__ static Result run(Ctx &c, int argc, char **argv) {
     Result R{};
@@ -68,7 +69,7 @@ struct PrApp {
         iptr[n] = 0;
       }
     }
-    __syncthreads();
+    sub_sync();
     global_exclusive_scan(dst, n + 1, c.sh);  // dst[u] = first edge of u; dst[n] = edges
     const long long E = dst[n];
     // ---- PR-2: targets, source by source (draw n + e + 1 for edge e) --------
@@ -83,12 +84,12 @@ struct PrApp {
         atomicAdd(&iptr[v], 1u);
       }
     }
-    __syncthreads();
+    sub_sync();
     global_exclusive_scan(iptr, n + 1, c.sh);  // in-edge offsets
     for (long long v = tid; v < n; v += T) cur[v] = iptr[v];
-    __syncthreads();
+    sub_sync();
     for (long long e = tid; e < E; e += T) ine[atomicAdd(&cur[tgt[e]], 1u)] = (uint32_t)e;
-    __syncthreads();
+    sub_sync();
     // per-target lists sorted by edge id == (source, edge) order; then sources
     for (long long v = tid; v < n; v += T) {
       const uint32_t lo = iptr[v], hi = iptr[v + 1];
@@ -107,7 +108,7 @@ struct PrApp {
     const double d = 0.85;
     const double base = (1.0 - d) / (double)n;
     for (long long v = tid; v < n; v += T) r[v] = 1.0 / (double)n;
-    __syncthreads();
+    sub_sync();
     for (int it = 0; it < p.iters; it++) {
       for (long long v = tid; v < n; v += T) {
         double acc = 0.0;
@@ -117,7 +118,7 @@ struct PrApp {
         }
         r2[v] = base + d * acc;
       }
-      __syncthreads();
+      sub_sync();
       double *t = r; r = r2; r2 = t;
     }
     // ---- PR-4 ---------------------------------------------------------------------
@@ -143,9 +144,9 @@ struct PrApp {
       const unsigned long long w = __shfl_xor_sync(0xffffffffu, cand, o);
       cand = w < cand ? w : cand;
     }
-    __syncthreads();
+    sub_sync();
     if ((tid & 31) == 0) c.sh->red_u[tid >> 5] = cand;
-    __syncthreads();
+    sub_sync();
     if (tid < 32) {
       unsigned long long m = tid < (T >> 5) ? c.sh->red_u[tid] : ~0ULL;
       for (int o = 16; o; o >>= 1) {
@@ -154,7 +155,7 @@ struct PrApp {
       }
       if (tid == 0) c.sh->red_u[0] = m;
     }
-    __syncthreads();
+    sub_sync();
     const long long topv = (long long)c.sh->red_u[0];
     R.vhash = bsum % 999983ULL;
     R.bitsum = bsum;

@@ -152,7 +152,7 @@ __device__ inline void global_exclusive_scan(uint32_t *a, long long n, Shared *s
       if (lane >= o) inc += t;
     }
     if (lane == 31) sh->red_u[w] = inc;
-    __syncthreads();
+    sub_sync();
     if (w == 0) {
       const unsigned long long t = lane < nw ? sh->red_u[lane] : 0ULL;
       unsigned long long ti = t;
@@ -163,7 +163,7 @@ __device__ inline void global_exclusive_scan(uint32_t *a, long long n, Shared *s
       if (lane < nw) sh->red_u[lane] = ti - t;                         // exclusive warp offsets
       if (lane == 31) sh->red_d[0] = __longlong_as_double((long long)ti);  // tile total
     }
-    __syncthreads();
+    sub_sync();
     uint32_t run = carry + (uint32_t)sh->red_u[w] + inc - sum;
     const uint32_t total = (uint32_t)__double_as_longlong(sh->red_d[0]);
 #pragma unroll
@@ -181,7 +181,7 @@ __device__ inline void global_exclusive_scan(uint32_t *a, long long n, Shared *s
         if (i0 + k < n) a[i0 + k] = v[k];
     }
     carry += total;
-    __syncthreads();
+    sub_sync();
   }
 }
 
@@ -214,6 +214,7 @@ struct XsApp {
   static constexpr int kMaxT = 512;
   static constexpr int kU = kXsU;
   static constexpr bool kTeam = true;  // splits nuclides and lookup batches over a cluster
+  static constexpr bool kSub = false;
 
   __device__ static Result run(Ctx &c, int argc, char **argv) {
     Result R{};

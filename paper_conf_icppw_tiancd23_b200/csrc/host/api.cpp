@@ -165,9 +165,13 @@ extern "C" void ens_args_free(ens_args *a) { delete a; }
 // ---------------------------------------------------------------------------
 struct Group {
   uint32_t app = 0;
-  int T = 0, grid = 0;  // grid = teams (arena slots); CTAs launched = grid * cs
+  int T = 0, grid = 0;  // grid = teams (arena slots); CTAs launched = grid * cs / m
   int cs = 1;           // CTAs per team (cluster size)
-  uint32_t smem = 0;
+  int m = 1;            // instances per CTA (block (T/m, m, 1)); m > 1 only with cs == 1
+  uint32_t smem = 0;    // app shared memory of one instance
+  uint32_t sub = 0;     // dynamic smem per instance row: scheduler state + app smem
+  size_t dyn() const { return (size_t)m * sub; }
+  int ctas() const { return grid * cs / m; }
   uint64_t arena = 0;
   std::vector<uint32_t> kmap;
   size_t kmap_off = 0;
@@ -235,6 +239,15 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   P.n = (int)n;
   P.stdout_cap = c->stdout_bytes ? (c->stdout_bytes + 7u) / 8u * 8u : 4096u;
   const int T = threads_for(c->block_threads);
+  if (c->instances_per_cta < 0) return fail(ENS_EINVAL, "ens_launch: negative instances_per_cta");
+  // M instances per CTA: power of two <= 8, >= 32 threads each
+  auto m_for = [&](uint32_t ap) {
+    const int Ta = std::min(T, app_max_threads(ap));
+    int m = 1;
+    if (app_sub_aware(ap))
+      while (m * 2 <= c->instances_per_cta && m < kMaxSubTeams && Ta / (m * 2) >= 32) m *= 2;
+    return m;
+  };
   int dev = 0, sms = 148;
   cudaError_t e = cudaGetDevice(&dev);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
@@ -253,7 +266,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     if (app == ENS_APP_BY_ARGV0) ap = argc > 0 ? app_of_argv0(argv[0]) : (uint32_t)APP_NOTFOUND;
     uint64_t ar = 0;
     uint32_t sm = 0;
-    app_size(ap, argc, argv, std::min(T, app_max_threads(ap)), 1, &ar, &sm);
+    app_size(ap, argc, argv, std::min(T, app_max_threads(ap)) / m_for(ap), 1, &ar, &sm);
     Group &g = g_by_app[ap];
     g.app = ap;
     g.smem = std::max(g.smem, sm);
@@ -268,35 +281,44 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     Group &g = g_by_app[ap];
     if (g.kmap.empty()) continue;
     g.T = std::min(T, app_max_threads(ap));
+    g.m = m_for(ap);
+    g.sub = sub_shared_bytes() + (g.smem + 15u) / 16u * 16u;
     int ctas = 0;
-    e = group_occupancy(ap, g.T, 1, g.smem, &ctas);
+    e = group_occupancy(ap, g.T, 1, g.dyn(), &ctas);
     if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor");
     if (ctas <= 0) return fail(ENS_EINVAL, "ens_launch: an instance needs more shared memory than one SM has");
     int cs = 1;
-    if (app_team_aware(ap)) {
+    if (g.m > 1) {  // teams are CTA rows: m slots per resident CTA, grid a multiple of m
+      int grid = c->grid_blocks ? c->grid_blocks * g.m : ctas * g.m;
+      const int64_t nn = (int64_t)g.kmap.size();
+      if (grid > nn) grid = (int)((nn + g.m - 1) / g.m * g.m);
+      g.grid = std::max(grid, g.m);
+    } else if (app_team_aware(ap)) {
       if (c->team_ctas > 0) {
         while (cs * 2 <= c->team_ctas && cs < kMaxTeamCtas) cs *= 2;
       } else if (!c->grid_blocks) {
         while (cs < kMaxTeamCtas && (int64_t)g.kmap.size() * cs * 2 <= ctas) cs *= 2;
       }
     }
-    int teams = ctas;
-    if (cs > 1) {
-      e = group_occupancy(ap, g.T, cs, g.smem, &teams);
-      if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters");
-      if (teams <= 0) cs = 1, teams = ctas;
+    if (g.m == 1) {
+      int teams = ctas;
+      if (cs > 1) {
+        e = group_occupancy(ap, g.T, cs, g.dyn(), &teams);
+        if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters");
+        if (teams <= 0) cs = 1, teams = ctas;
+      }
+      int grid = c->grid_blocks ? std::max(1, c->grid_blocks / cs) : teams;
+      grid = (int)std::min<int64_t>(grid, (int64_t)g.kmap.size());
+      g.grid = std::max(grid, 1);
     }
     g.cs = cs;
-    int grid = c->grid_blocks ? std::max(1, c->grid_blocks / cs) : teams;
-    grid = (int)std::min<int64_t>(grid, (int64_t)g.kmap.size());
-    g.grid = std::max(grid, 1);
     for (uint32_t k : g.kmap) {  // arena of this team size
       int argc;
       const char *const *argv;
       ens_args_get(a, (int)P.line_of_k[k], &argc, &argv);
       uint64_t ar = 0;
       uint32_t sm = 0;
-      app_size(ap, argc, argv, g.T, cs, &ar, &sm);
+      app_size(ap, argc, argv, g.T / g.m, cs, &ar, &sm);
       g.arena = std::max(g.arena, ar);
     }
     need_arena = std::max(need_arena, g.arena);
@@ -334,7 +356,11 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     if ((uint64_t)want > fit) {
       if (c->grid_blocks) return fail(ENS_ENOMEM, "ens_launch: grid_blocks x arena does not fit the workspace");
       want = (int)fit;
-      for (Group &g : P.groups) g.grid = std::min(g.grid, want);
+      for (Group &g : P.groups) {
+        g.grid = std::min(g.grid, want / g.m * g.m);  // whole CTAs of m slots
+        if (g.grid <= 0)
+          return fail(ENS_ENOMEM, "ens_launch: workspace cannot hold one CTA of instances_per_cta arena slots");
+      }
     }
   }
   P.slots = want;
@@ -383,7 +409,8 @@ static int enqueue(ens_run *r) {
     k.arena_bytes = P.arena_bytes;
     k.team_ctas = (uint32_t)g.cs;
     k.phases = (r->flags & ENS_F_PHASES) ? (unsigned long long *)(r->ws + P.o_phase) : nullptr;
-    cudaError_t e = launch_group(g.app, g.T, g.grid * g.cs, g.cs, g.smem, k, r->stream);
+    k.sub_stride = g.sub;
+    cudaError_t e = launch_group(g.app, g.T, g.m, g.ctas(), g.cs, g.dyn(), k, r->stream);
     if (e != cudaSuccess) return cuda_fail(e, "ens_kernel launch");
   }
   CU(cudaEventRecord(r->ev1, r->stream));
@@ -552,8 +579,9 @@ extern "C" int ens_run_get_info(const ens_run *r, ens_run_info *info) {
   info->n_groups = (int32_t)P.groups.size();
   for (const Group &g : P.groups) {
     const uint32_t ap = g.app == APP_NOTFOUND ? 0u : g.app;
-    info->grid_blocks[ap] = g.grid * g.cs;
+    info->grid_blocks[ap] = g.ctas();
     info->team_ctas[ap] = g.cs;
+    info->instances_per_cta[ap] = g.m;
     info->block_threads[ap] = g.T;
   }
   info->kernel_launches = (int32_t)P.groups.size();

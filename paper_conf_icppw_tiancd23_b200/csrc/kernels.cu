@@ -36,36 +36,48 @@ __device__ __forceinline__ uint32_t smid() {
 #define ENS_MINB_NUM 512
 #endif
 
+// Per-instance scheduler state, in dynamic shared memory: one copy per
+// instance running in the CTA (M = blockDim.y instances per CTA), followed
+// by that instance's app shared memory.
+struct SubShared {
+  Shared sh;
+  char *argv[ENS_MAX_ARGC + 1];
+  unsigned long long pos;
+  uint32_t j;
+};
+constexpr uint32_t kSubSharedBytes = (sizeof(SubShared) + 15) / 16 * 16;
+
+// T = threads per CTA (the launch bound); the instance runs on the CTA's row
+// threadIdx.y of blockDim.x threads (all of it when M = 1).
 template <class App, int T>
 __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T) : 1) ens_kernel(const KParams p) {
   extern __shared__ __align__(16) char dsmem[];
-  __shared__ char *s_argv[ENS_MAX_ARGC + 1];
-  __shared__ uint32_t s_j;
-  __shared__ unsigned long long s_pos;
-  __shared__ Shared sh;
-  const int tid = threadIdx.x;
-  const uint32_t cs = p.team_ctas;  // cluster dims (cs, 1, 1)
+  const int tid = threadIdx.x, B = blockDim.x, y = threadIdx.y, M = blockDim.y;
+  SubShared *ss = reinterpret_cast<SubShared *>(dsmem + (size_t)y * p.sub_stride);
+  Shared &sh = ss->sh;
+  char **s_argv = ss->argv;
+  const uint32_t cs = p.team_ctas;  // cluster dims (cs, 1, 1); M > 1 only with cs == 1
   const uint32_t cr = cs > 1 ? cooperative_groups::this_cluster().block_rank() : 0u;
-  char *const arena = p.arena_base + (size_t)(blockIdx.x / cs) * p.arena_bytes;
+  char *const arena = p.arena_base + ((size_t)(blockIdx.x / cs) * M + y) * p.arena_bytes;
   Ctx c;
   c.arena = arena;
   c.arena_cap = p.arena_bytes;
   c.out_cap = p.stdout_cap;
   c.sh = &sh;
-  c.smem = dsmem;
+  c.smem = reinterpret_cast<char *>(ss) + kSubSharedBytes;
   c.crank = cr;
   c.csize = cs;
   for (;;) {
-    if (tid == 0 && cr == 0) s_j = atomicAdd(p.counter, 1u);
+    if (tid == 0 && cr == 0) ss->j = atomicAdd(p.counter, 1u);
     team_sync(c);
-    const uint32_t j = cr == 0 ? s_j : *cta_shared(&s_j, 0);
+    const uint32_t j = cr == 0 ? ss->j : *cta_shared(&ss->j, 0);
     if (cs > 1) team_sync(c);  // every rank has read s_j before rank 0 may exit
     if (j >= p.n) break;       // team-uniform
     const uint32_t k = p.kmap[j];
     const uint32_t line = p.line_of_k[k];
     const uint32_t t0 = p.line_tok[line];
     const int argc = (int)(p.line_tok[line + 1] - t0);
-    for (int i = tid; i < argc; i += T) s_argv[i] = const_cast<char *>(p.blob) + p.tok_off[t0 + i];
+    for (int i = tid; i < argc; i += B) s_argv[i] = const_cast<char *>(p.blob) + p.tok_off[t0 + i];
     if (tid == 0) s_argv[argc] = nullptr;
     if (tid < 32) sh.tallies[tid] = 0;
     if (tid == 0) {
@@ -74,7 +86,7 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
     }
     uint64_t t_start = 0;
     if ((p.flags & ENS_F_TIMESTAMPS) && tid == 0) t_start = globaltimer();
-    __syncthreads();
+    sub_sync();
 
     c.k = k;
     c.id = line;
@@ -106,17 +118,17 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
         rec.t_start_ns = t_start;
         rec.t_end_ns = (p.flags & ENS_F_TIMESTAMPS) ? globaltimer() : 0ull;
         p.recs[k] = rec;
-        s_pos = atomicAdd(p.stdout_total, (unsigned long long)sh.out_len);
-        p.stdout_pos[k] = s_pos;
+        ss->pos = atomicAdd(p.stdout_total, (unsigned long long)sh.out_len);
+        p.stdout_pos[k] = ss->pos;
       }
-      __syncthreads();
+      sub_sync();
       {  // compact this instance's stdout (whole 8-B words)
         const unsigned long long *src = reinterpret_cast<const unsigned long long *>(c.out);
-        unsigned long long *dst = reinterpret_cast<unsigned long long *>(p.stdout_cmp + s_pos);
-        for (uint32_t w = tid; w < sh.out_len / 8; w += T) dst[w] = src[w];
+        unsigned long long *dst = reinterpret_cast<unsigned long long *>(p.stdout_cmp + ss->pos);
+        for (uint32_t w = tid; w < sh.out_len / 8; w += B) dst[w] = src[w];
       }
     }
-    team_sync(c);  // s_j, s_pos, s_argv, sh reused by the next instance
+    team_sync(c);  // j, pos, argv, sh reused by the next instance
   }
 }
 
@@ -153,6 +165,17 @@ int app_max_threads(uint32_t app) {
 }
 // whether the body splits its work over a multi-CTA team
 bool app_team_aware(uint32_t app) { return app == APP_XSBENCH ? XsApp::kTeam : false; }
+// whether the body can run as one of M instances per CTA (NEXT 1)
+bool app_sub_aware(uint32_t app) {
+  switch (app) {
+    case APP_ECHO: return EchoApp::kSub;
+    case APP_AMGMK: return AmgApp::kSub;
+    case APP_PAGERANK: return PrApp::kSub;
+    case APP_NOTFOUND: return NotFoundApp::kSub;
+  }
+  return false;
+}
+uint32_t sub_shared_bytes() { return kSubSharedBytes; }
 
 const void *kernel_ptr(uint32_t app, int T) {
   switch (app) {
@@ -186,14 +209,16 @@ static cudaError_t set_smem(const void *fn, size_t smem) {
   return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
 }
 
-cudaError_t launch_group(uint32_t app, int T, int grid, int cs, size_t smem, const KParams &p, cudaStream_t st) {
+// T = threads per CTA; m = instances per CTA: the block is (T/m, m, 1)
+cudaError_t launch_group(uint32_t app, int T, int m, int grid, int cs, size_t smem, const KParams &p,
+                         cudaStream_t st) {
   const void *fn = kernel_ptr(app, T);
   if (!fn) return cudaErrorInvalidValue;
   cudaError_t e = set_smem(fn, smem);
   if (e != cudaSuccess) return e;
   cudaLaunchConfig_t cfg{};
   cfg.gridDim = dim3((unsigned)grid);
-  cfg.blockDim = dim3((unsigned)T);
+  cfg.blockDim = dim3((unsigned)(T / m), (unsigned)m, 1u);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = st;
   cudaLaunchAttribute attr[1];

@@ -28,13 +28,17 @@ struct KParams {
   uint64_t arena_bytes;
   uint32_t team_ctas;         // CTAs per team (thread-block cluster size)
   unsigned long long *phases; // [ENS_PHASES] ns per phase (ENS_F_PHASES) or null
+  uint32_t sub_stride;        // dynamic smem bytes per instance slot of the CTA
 };
 
 const void *kernel_ptr(uint32_t app, int T);
 int app_max_threads(uint32_t app);
 bool app_team_aware(uint32_t app);
+bool app_sub_aware(uint32_t app);
+uint32_t sub_shared_bytes();
 bool app_size(uint32_t app, int argc, const char *const *argv, int T, int cs, uint64_t *arena, uint32_t *smem);
-cudaError_t launch_group(uint32_t app, int T, int grid, int cs, size_t smem, const KParams &p, cudaStream_t st);
+cudaError_t launch_group(uint32_t app, int T, int m, int grid, int cs, size_t smem, const KParams &p,
+                         cudaStream_t st);
 cudaError_t group_occupancy(uint32_t app, int T, int cs, size_t smem, int *teams);
 
 }  // namespace ens

@@ -95,6 +95,16 @@ ENS_HD uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 // per-instance context (identical copy in every thread of the block)
 // ---------------------------------------------------------------------------
 constexpr int kMaxTeamCtas = 8;  // portable thread-block-cluster size
+constexpr int kMaxSubTeams = 8;  // M instances per CTA (named barriers 1..8)
+
+// Barrier of the threads running this instance.  With M instances per CTA
+// (the paper's (N/M, M, 1) block) the
+// instance is the row threadIdx.y of the block and uses named barrier 1+y;
+// otherwise it is the whole CTA.
+__device__ __forceinline__ void sub_sync() {
+  if (blockDim.y > 1) asm volatile("bar.sync %0, %1;" ::"r"(1 + threadIdx.y), "r"(blockDim.x) : "memory");
+  else __syncthreads();
+}
 
 struct Shared {             // static shared memory of the scheduler
   uint32_t tallies[32];     // per-instance tallies (smem atomics)
@@ -148,7 +158,7 @@ __device__ __forceinline__ void phase_mark(Ctx &c, int k) {
 // scope, so global and shared writes before it are visible after it)
 __device__ __forceinline__ void team_sync(const Ctx &c) {
   if (c.csize > 1) cooperative_groups::this_cluster().sync();
-  else __syncthreads();
+  else sub_sync();
 }
 // `p` (a shared variable of this CTA) in the shared memory of team CTA `rank`
 template <class X>
@@ -229,27 +239,27 @@ __device__ __forceinline__ double warp_max_f64(double v) {  // NaN never wins
 __device__ inline unsigned long long block_sum_u64(Shared *sh, unsigned long long v) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
   v = warp_sum_u64(v);
-  __syncthreads();
+  sub_sync();
   if (lane == 0) sh->red_u[w] = v;
-  __syncthreads();
+  sub_sync();
   v = lane < nw ? sh->red_u[lane] : 0ULL;
   return warp_sum_u64(v);
 }
 __device__ inline double block_sum_f64(Shared *sh, double v) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
   v = warp_sum_f64(v);
-  __syncthreads();
+  sub_sync();
   if (lane == 0) sh->red_d[w] = v;
-  __syncthreads();
+  sub_sync();
   v = lane < nw ? sh->red_d[lane] : 0.0;
   return warp_sum_f64(v);
 }
 __device__ inline double block_max_f64(Shared *sh, double v) {
   const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
   v = warp_max_f64(v);
-  __syncthreads();
+  sub_sync();
   if (lane == 0) sh->red_d[w] = v;
-  __syncthreads();
+  sub_sync();
   v = lane < nw ? sh->red_d[lane] : v;
   return warp_max_f64(v);
 }

@@ -1,8 +1,8 @@
 // csrc/tools/ens_run.cpp — N5, the enhanced loader's command line (§3.2
 // P:422-436, Fig. 5c):
 //   ens_run -f <args file> [-n <num instances>] [-t <thread limit>]
-//           [-a auto|echo|xsbench|rsbench|amgmk] [-g grid] [--argv0 name]
-//           [--timestamps] [-q]
+//           [-a auto|echo|xsbench|rsbench|amgmk|pagerank] [-g grid]
+//           [-M instances per CTA] [--argv0 name] [--timestamps] [-q]
 // Runs the first n lines as one ensemble on the current GPU, prints every
 // instance's stdout in instance order, then one summary line on stderr.
 // (Multi-GPU runs go through the Python launcher, python -m
@@ -22,7 +22,7 @@ static int die(const char *what, int rc) {
 
 int main(int argc, char **argv) {
   const char *file = nullptr, *argv0 = nullptr;
-  int n = -1, t = 0, grid = 0;
+  int n = -1, t = 0, grid = 0, m = 0;
   bool quiet = false, ts = false;
   ens_app app = ENS_APP_BY_ARGV0;
   for (int i = 1; i < argc; i++) {
@@ -38,6 +38,7 @@ int main(int argc, char **argv) {
     else if (f == "-n") n = std::atoi(val());
     else if (f == "-t") t = std::atoi(val());
     else if (f == "-g") grid = std::atoi(val());
+    else if (f == "-M") m = std::atoi(val());
     else if (f == "--argv0") argv0 = val();
     else if (f == "--timestamps") ts = true;
     else if (f == "-q") quiet = true;
@@ -46,7 +47,8 @@ int main(int argc, char **argv) {
       app = a == "echo" ? ENS_APP_ECHO : a == "xsbench" ? ENS_APP_XSBENCH : a == "rsbench" ? ENS_APP_RSBENCH
           : a == "amgmk" ? ENS_APP_AMGMK : a == "pagerank" ? ENS_APP_PAGERANK : ENS_APP_BY_ARGV0;
     } else {
-      std::fprintf(stderr, "usage: ens_run -f file [-n N] [-t T] [-a auto|echo|xsbench|rsbench|amgmk] [-g grid] "
+      std::fprintf(stderr, "usage: ens_run -f file [-n N] [-t T] [-a auto|echo|xsbench|rsbench|amgmk|pagerank] [-g grid] "
+                           "[-M instances per CTA] "
                            "[--argv0 name] [--timestamps] [-q]\n");
       return 2;
     }
@@ -67,6 +69,7 @@ int main(int argc, char **argv) {
   cfg.stride = 1;
   cfg.grid_blocks = grid;
   cfg.block_threads = t;
+  cfg.instances_per_cta = m;
   cfg.flags = ts ? ENS_F_TIMESTAMPS : 0;
   ens_run *r = nullptr;
   rc = ens_launch(app, a, &cfg, nullptr, 0, nullptr, &r);

@@ -27,7 +27,8 @@ def main(argv=None):
     ap.add_argument("-f", required=True, help="arguments file: one instance command line per line")
     ap.add_argument("-n", type=int, default=None, help="number of instances (default: all lines)")
     ap.add_argument("-t", type=int, default=256, help="thread limit per instance (an upper bound)")
-    ap.add_argument("-a", default="auto", help="app: auto (argv[0] of each line), echo, xsbench, rsbench, amgmk")
+    ap.add_argument("-a", default="auto", help="app: auto (argv[0] of each line), echo, xsbench, rsbench, amgmk, pagerank")
+    ap.add_argument("-M", type=int, default=0, help="instances per CTA, the (N/M, M, 1) block mapping (P:393-404)")
     ap.add_argument("--argv0", default=None)
     ap.add_argument("-q", action="store_true", help="do not print the instances' stdout")
     a = ap.parse_args(argv)
@@ -44,7 +45,8 @@ def main(argv=None):
         print(f"ens_run: -n {n_total} > {len(args)} lines", file=sys.stderr)
         return 2
     n_local = D.shard_count(n_total, rank, world)
-    ens = Ensemble(args, app=a.a, n=n_local, first=rank, stride=world, threads=a.t).launch()
+    ens = Ensemble(args, app=a.a, n=n_local, first=rank, stride=world, threads=a.t,
+                   instances_per_cta=a.M).launch()
     torch.cuda.synchronize()
     ms = ens.elapsed_ms() if n_local else 0.0
     if world > 1:
