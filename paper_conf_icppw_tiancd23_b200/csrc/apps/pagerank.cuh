@@ -15,7 +15,7 @@
 #pragma once
 #include "../rt/device_rt.cuh"
 #include "params.cuh"
-#include "xsbench.cuh"  // global_exclusive_scan
+#include "../rt/scan.cuh"
 
 namespace ens {
 

@@ -284,7 +284,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     g.m = m_for(ap);
     g.sub = sub_shared_bytes() + (g.smem + 15u) / 16u * 16u;
     int ctas = 0;
-    e = group_occupancy(ap, g.T, 1, g.dyn(), &ctas);
+    e = group_occupancy(ap, g.T, g.m, 1, g.dyn(), &ctas);
     if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor");
     if (ctas <= 0) return fail(ENS_EINVAL, "ens_launch: an instance needs more shared memory than one SM has");
     int cs = 1;
@@ -303,7 +303,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     if (g.m == 1) {
       int teams = ctas;
       if (cs > 1) {
-        e = group_occupancy(ap, g.T, cs, g.dyn(), &teams);
+        e = group_occupancy(ap, g.T, 1, cs, g.dyn(), &teams);
         if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters");
         if (teams <= 0) cs = 1, teams = ctas;
       }

@@ -9,16 +9,29 @@
 // (memory = resident teams x arena, not NI x arena).
 // A team is one CTA, or (team-aware bodies, ensembles with fewer instances
 // than SMs) a thread-block cluster of up to 8 CTAs (see rt/device_rt.cuh).
+//
+// This file is compiled twice: as kernels.cu (ENS_SUB=0: one instance per
+// CTA row = the whole CTA, every host-side entry point) and as
+// kernels_sub.cu (ENS_SUB=1: the row kernels of the (N/M, M, 1) mapping for
+// the bodies built for it, see sub_sync in rt/device_rt.cuh).
 #include <cuda_runtime.h>
 
+#ifndef ENS_SUB
+#define ENS_SUB 0
+#endif
 #include "apps/amgmk.cuh"
 #include "apps/echo.cuh"
 #include "apps/pagerank.cuh"
+#if !ENS_SUB
 #include "apps/rsbench.cuh"
 #include "apps/xsbench.cuh"
+#endif
 #include "kparams.h"
 
 namespace ens {
+#if ENS_SUB
+namespace subk {  // row kernels: distinct symbols from the M = 1 kernels
+#endif
 
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
@@ -150,6 +163,19 @@ static const void *kernel_for(int T) {
   return nullptr;
 }
 
+#if ENS_SUB
+}  // namespace subk
+
+const void *kernel_ptr_sub(uint32_t app, int T) {
+  switch (app) {
+    case APP_ECHO: return subk::kernel_for<EchoApp>(T);
+    case APP_AMGMK: return subk::kernel_for<AmgApp>(T);
+    case APP_PAGERANK: return subk::kernel_for<PrApp>(T);
+    case APP_NOTFOUND: return subk::kernel_for<NotFoundApp>(T);
+  }
+  return nullptr;
+}
+#else
 // the largest block size an app's kernel is built for (the thread limit is an
 // upper bound)
 int app_max_threads(uint32_t app) {
@@ -212,7 +238,7 @@ static cudaError_t set_smem(const void *fn, size_t smem) {
 // T = threads per CTA; m = instances per CTA: the block is (T/m, m, 1)
 cudaError_t launch_group(uint32_t app, int T, int m, int grid, int cs, size_t smem, const KParams &p,
                          cudaStream_t st) {
-  const void *fn = kernel_ptr(app, T);
+  const void *fn = m > 1 ? kernel_ptr_sub(app, T) : kernel_ptr(app, T);
   if (!fn) return cudaErrorInvalidValue;
   cudaError_t e = set_smem(fn, smem);
   if (e != cudaSuccess) return e;
@@ -232,9 +258,9 @@ cudaError_t launch_group(uint32_t app, int T, int m, int grid, int cs, size_t sm
   return cudaLaunchKernelExC(&cfg, fn, args);
 }
 
-// resident teams (clusters of cs CTAs) on the whole device
-cudaError_t group_occupancy(uint32_t app, int T, int cs, size_t smem, int *teams) {
-  const void *fn = kernel_ptr(app, T);
+// resident teams (clusters of cs CTAs; CTAs when m > 1) on the whole device
+cudaError_t group_occupancy(uint32_t app, int T, int m, int cs, size_t smem, int *teams) {
+  const void *fn = m > 1 ? kernel_ptr_sub(app, T) : kernel_ptr(app, T);
   if (!fn) return cudaErrorInvalidValue;
   cudaError_t e = set_smem(fn, smem);
   if (e != cudaSuccess) return e;
@@ -259,5 +285,6 @@ cudaError_t group_occupancy(uint32_t app, int T, int cs, size_t smem, int *teams
   cfg.numAttrs = 1;
   return cudaOccupancyMaxActiveClusters(teams, fn, &cfg);
 }
+#endif  // !ENS_SUB
 
 }  // namespace ens

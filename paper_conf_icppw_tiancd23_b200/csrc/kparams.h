@@ -32,6 +32,7 @@ struct KParams {
 };
 
 const void *kernel_ptr(uint32_t app, int T);
+const void *kernel_ptr_sub(uint32_t app, int T);  // row kernels (m > 1), kernels_sub.cu
 int app_max_threads(uint32_t app);
 bool app_team_aware(uint32_t app);
 bool app_sub_aware(uint32_t app);
@@ -39,6 +40,6 @@ uint32_t sub_shared_bytes();
 bool app_size(uint32_t app, int argc, const char *const *argv, int T, int cs, uint64_t *arena, uint32_t *smem);
 cudaError_t launch_group(uint32_t app, int T, int m, int grid, int cs, size_t smem, const KParams &p,
                          cudaStream_t st);
-cudaError_t group_occupancy(uint32_t app, int T, int cs, size_t smem, int *teams);
+cudaError_t group_occupancy(uint32_t app, int T, int m, int cs, size_t smem, int *teams);
 
 }  // namespace ens

@@ -99,11 +99,31 @@ constexpr int kMaxSubTeams = 8;  // M instances per CTA (named barriers 1..8)
 
 // Barrier of the threads running this instance.  With M instances per CTA
 // (the paper's (N/M, M, 1) block) the
-// instance is the row threadIdx.y of the block and uses named barrier 1+y;
-// otherwise it is the whole CTA.
+// instance is the row threadIdx.y of the block and uses hardware barrier y;
+// otherwise it is the whole CTA.  The row variant is compiled separately
+// (ENS_SUB=1, kernels_sub.cu): ptxas reserves every barrier id a kernel
+// names, and the SM's barrier pool then caps resident CTAs (16 ids -> 4
+// CTAs/SM measured), so the M = 1 kernels only ever use barrier 0, and the
+// row kernels use the immediate ids 0..7 (8 ids, never a register id).
+#ifndef ENS_SUB
+#define ENS_SUB 0
+#endif
 __device__ __forceinline__ void sub_sync() {
-  if (blockDim.y > 1) asm volatile("bar.sync %0, %1;" ::"r"(1 + threadIdx.y), "r"(blockDim.x) : "memory");
-  else __syncthreads();
+#if ENS_SUB
+  const uint32_t n = blockDim.x;
+  switch (threadIdx.y) {
+    case 0: asm volatile("bar.sync 0, %0;" ::"r"(n) : "memory"); break;
+    case 1: asm volatile("bar.sync 1, %0;" ::"r"(n) : "memory"); break;
+    case 2: asm volatile("bar.sync 2, %0;" ::"r"(n) : "memory"); break;
+    case 3: asm volatile("bar.sync 3, %0;" ::"r"(n) : "memory"); break;
+    case 4: asm volatile("bar.sync 4, %0;" ::"r"(n) : "memory"); break;
+    case 5: asm volatile("bar.sync 5, %0;" ::"r"(n) : "memory"); break;
+    case 6: asm volatile("bar.sync 6, %0;" ::"r"(n) : "memory"); break;
+    default: asm volatile("bar.sync 7, %0;" ::"r"(n) : "memory"); break;
+  }
+#else
+  __syncthreads();
+#endif
 }
 
 struct Shared {             // static shared memory of the scheduler

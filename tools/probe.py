@@ -1,6 +1,6 @@
 """Time ensembles of arbitrary lines on the GPU (phase probes, not the bench).
 
-    python tools/probe.py "<line template with {i}>" N [threads] [reps] [--phases] [--team K]
+    python tools/probe.py "<line template with {i}>" N [threads] [reps] [--phases] [--team K] [--m M]
 
 Prints the best-of-reps CUDA-event time of the ensemble launch; with
 --phases also the per-phase device time (ENS_F_PHASES tracing), summed over
@@ -19,9 +19,10 @@ XS_PHASES = ["materials", "generate", "bucket scan", "scatter", "bucket sort", "
              "index sweep", "record permute", "hash column", "lookup sample+sort", "lookup gathers"]
 
 
-def probe(template, n, threads=512, reps=3, phases=False, team=0):
+def probe(template, n, threads=512, reps=3, phases=False, team=0, m=0):
     text = "".join(template.format(i=i) + "\n" for i in range(n))
-    e = Ensemble(Args.parse(text), app="auto", threads=threads, phases=phases, team_ctas=team).launch()
+    e = Ensemble(Args.parse(text), app="auto", threads=threads, phases=phases, team_ctas=team,
+                 instances_per_cta=m).launch()
     torch.cuda.synchronize()
     ts = []
     ph = None
@@ -48,8 +49,12 @@ if __name__ == "__main__":
     if "--team" in sys.argv:
         team = int(sys.argv[sys.argv.index("--team") + 1])
         args.remove(str(team))
-    t, ok, g, T, cs, ph = probe(args[0], int(args[1]), *(int(x) for x in args[2:]), phases=phases, team=team)
-    print(f"{t:9.3f} ms ok={ok} grid={g} T={T} team={cs} :: {args[0]} x{args[1]}", flush=True)
+    m = 0
+    if "--m" in sys.argv:
+        m = int(sys.argv[sys.argv.index("--m") + 1])
+        args.remove(str(m))
+    t, ok, g, T, cs, ph = probe(args[0], int(args[1]), *(int(x) for x in args[2:]), phases=phases, team=team, m=m)
+    print(f"{t:9.3f} ms ok={ok} grid={g} T={T} team={cs} m={m} :: {args[0]} x{args[1]}", flush=True)
     if ph:
         teams = max(max(g) // max(1, max(cs)), 1)
         for k, v in enumerate(ph):
