@@ -11,7 +11,7 @@ import os
 import numpy as np
 
 PKG_DIR = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(PKG_DIR, "libens.so")
+LIB_PATH = os.environ.get("ENS_LIB_PATH") or os.path.join(PKG_DIR, "libens.so")  # override: A/B builds
 
 ENS_OK, ENS_EINVAL, ENS_ENOENT, ENS_ENOMEM, ENS_ECUDA, ENS_ERANGE, ENS_EBUSY, ENS_EPARSE = 0, -1, -2, -3, -4, -5, -6, -7
 ENS_EXIT_USAGE, ENS_EXIT_NOMEM, ENS_EXIT_NOTFOUND = 1, 12, 127

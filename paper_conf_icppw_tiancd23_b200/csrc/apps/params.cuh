@@ -174,8 +174,23 @@ struct XsLayout {
   uint64_t chist;     // unionized: [n_chunks][n_iso] u32 owner counts per sweep chunk
   uint64_t index;     // unionized [n_u][n_iso] int32 / hash [n_iso][bins+1] XsHashEnt
   uint64_t hcol;      // hash: [cs][bins+1] int32 column being built
+  uint64_t lk_pe;     // event mode: [chunk] lookup energies sorted by (material, energy)
+  uint64_t lk_hist;   // event mode: [(12 << kb) + 1] u32 (material, energy) bucket counts -> cursors
   uint64_t total;
 };
+// Event-mode lookups are sampled, then bucket-sorted by (material, energy)
+// in chunks of at most 2^22 (upstream XSBench's GPU versions offer the same
+// material / energy sort; results per lookup are unchanged): a warp's lanes
+// then take neighbouring energies of one material, so they gather the same
+// index entries and record pairs.  kb = energy-bucket bits per material
+// (~2 lookups per bucket).
+constexpr long long kXsLkChunk = 1LL << 22;
+ENS_HD long long xs_lk_chunk(const XsParams &p) { return p.lookups < kXsLkChunk ? p.lookups : kXsLkChunk; }
+ENS_HD int xs_lk_bits(long long n_c) {
+  int kb = 0;
+  while (kb < 18 && (12LL << kb) * 2 < n_c) kb++;
+  return kb;
+}
 // hash index entry: the upstream index u_low = ig[b][i] plus E_i[u_low+1], so
 // a lookup knows from one 16-B load whether its energy lies in the first
 // record pair of the bin (a private accelerator; results are unchanged)
@@ -206,6 +221,11 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
     L.index = o; o = align_up(o + (uint64_t)p.n_iso * (p.bins + 1) * 16, 256);
     L.hcol = o; o = align_up(o + (uint64_t)cs * (p.bins + 1) * 4, 256);
   }
+  if (!p.history) {
+    const long long n_c = xs_lk_chunk(p);
+    L.lk_pe = o; o = align_up(o + (uint64_t)n_c * 8, 256);
+    L.lk_hist = o; o = align_up(o + ((12ULL << xs_lk_bits(n_c)) + 1) * 4, 256);
+  }
   L.total = o;
   return L;
 }
@@ -216,11 +236,8 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
 #endif
 constexpr int kXsU = ENS_XS_U;  // nuclide gathers in flight per lane
 constexpr int kXsMaxT = 512;  // XsApp::kMaxT
-// lookups per thread per material-sorted batch: enough that every thread
-// gets several fuel lookups (321 nuclides large / 34 small)
-ENS_HD int xs_batch_k(int n_iso) { return n_iso == 68 ? 8 : 24; }
 struct XsSmem {
-  uint32_t thr, nn, mats, concs, mcnt, nbkt, slot, total;
+  uint32_t thr, nn, mats, concs, mcnt, nbkt, total;
 };
 // T = the block size the instance runs with
 ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
@@ -231,11 +248,10 @@ ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   S.nn = o; o += 16 * 4;                  // num_nucs
   S.concs = o; o += 12 * mx * 8;          // concentrations
   S.mats = o; o += (uint32_t)align_up(12 * mx * 2, 16);  // nuclide ids (u16)
-  S.mcnt = o; o += 32 * 4;                // batch material counts / offsets
+  S.mcnt = o; o += 32 * 4;                // material counts / offsets of a lookup chunk
   S.nbkt = o;                             // per-nuclide sort buckets (hash / nuclide grids)
   if (p.grid != XS_UNIONIZED) o += (uint32_t)align_up((uint64_t)xs_nbn(p.n_gp) * 4, 16);
-  S.slot = o;                             // batch slots: energy (+ union index)
-  o += (uint32_t)xs_batch_k(p.n_iso) * (uint32_t)T * (p.grid == XS_UNIONIZED ? 12u : 8u);
+  (void)T;
   S.total = o;
   return S;
 }

@@ -873,91 +873,88 @@ struct XsApp {
   }
 
   // ---- XS-6..XS-10: lookups ----------------------------------------------
-  // Batches of K*T lookups: (A) every thread samples its K lookups (XS-6),
-  // the batch is counting-sorted by material into shared memory; (B) thread
-  // t takes sorted slots t, t+T, t+2T, ...: a warp's lanes share a material
-  // (same nuclide count: no divergence), every thread gets the same mix of
-  // materials (balanced), and each lane sums its lookup's nuclides in list
-  // order (XS-9's order, bit-exact), kU nuclides' gathers in flight at once.
+  // Per chunk of at most 2^22 lookups (XsLayout.lk_*): (A) every lookup is
+  // sampled (XS-6, lookup li draws 2li+1, 2li+2) and counted into its
+  // (material, energy) bucket; (B) one scan gives bucket offsets — material
+  // m starts at bucket m << kb; (C) lookups are re-sampled and their
+  // energies scattered to their bucket; (D) thread-per-slot over the sorted
+  // chunk: a warp's lanes share a material (same nuclide list, no
+  // divergence) and neighbouring energies (the same hash entries / record
+  // pairs, so one L1 line serves many lanes), and each lane sums its
+  // lookup's nuclides in list order (XS-9's order, bit-exact).  The order of
+  // lookups within a bucket (atomic) only permutes the fsum / fabs terms.
   template <int GRID>
   __device__ static __forceinline__ void lookups(Ctx &c, const XsParams &p, const XsLayout &L, const double *thr,
                                               const int *nn, const double *concs, const uint16_t *mats,
                                               Result &R) {
     const int tid = threadIdx.x, T = blockDim.x;
-    const int n_iso = p.n_iso, n_gp = p.n_gp, mx = xs_max_nucs(n_iso);
-    const long long n_u = (long long)n_iso * n_gp, nL = p.lookups;
+    const int n_iso = p.n_iso;
+    const long long n_u = (long long)n_iso * p.n_gp, nL = p.lookups;
     const double *recs = (const double *)(c.arena + L.recs);
     const int *ig = (const int *)(c.arena + L.index);
     const uint64_t *uA = (const uint64_t *)(c.arena + L.uenergy);
     const uint32_t *uf = (const uint32_t *)(c.arena + L.ufind);
+    double *lk_pe = (double *)(c.arena + L.lk_pe);
+    uint32_t *hist = (uint32_t *)(c.arena + L.lk_hist);
     const long long UB = xs_ubins(p);
     const XsSmem S = xs_smem(p, T);
-    const int K = xs_batch_k(n_iso);
-    double *slot_pe = (double *)(c.smem + S.slot);
-    int *slot_idx = (int *)(c.smem + S.slot + (size_t)K * T * 8);
-    uint32_t *mcnt = (uint32_t *)(c.smem + S.mcnt);  // [12] counts -> cursors, [16..28] offsets
+    uint32_t *mcnt = (uint32_t *)(c.smem + S.mcnt);  // [0..11] sampled counts, [16..28] material offsets
     const double du = 1.0 / p.bins;
+    const long long LC = xs_lk_chunk(p);
+    const int kb = xs_lk_bits(LC);
+    const long long NB = 12LL << kb;
+    const double bscale = (double)(1LL << kb);
+    const long long g0 = (long long)c.crank * T + tid, gs = (long long)c.csize * T;
+    const Affine JG = lcg_pow(2ULL * (uint64_t)gs);
     unsigned long long ver = 0, bsum = 0;
     double fsum = 0.0, fabs_ = 0.0;
-    const long long NBt = (long long)K * T;
-    const Affine JT = lcg_pow(2ULL * T);
-    for (long long b0 = (long long)c.crank * NBt; b0 < nL; b0 += NBt * c.csize) {  // batches striped over the team
-      const int nb = (int)((nL - b0 < NBt) ? nL - b0 : NBt);
-      if (tid < 12) mcnt[tid] = 0;
-      __syncthreads();
-      // (A1) count the batch's materials; lookup li = b0 + tid + r*T
-      const uint64_t s0 = lcg_pow(2ULL * (uint64_t)(b0 + tid))(p.seed);
+    if (tid < 12) mcnt[tid] = 0;
+    for (long long c0 = 0; c0 < nL; c0 += LC) {
+      const long long nc = nL - c0 < LC ? nL - c0 : LC;
+      for (long long b = g0; b <= NB; b += gs) hist[b] = 0u;
+      team_sync(c);
+      // (A) count
       {
-        uint64_t s = s0;
-        for (int r = 0; r < K; r++, s = JT(s)) {
-          if (tid + r * T >= nb) break;
-          uint64_t t = s;
-          (void)lcg_double(t);
-          atomicAdd(&mcnt[pick_mat_thr(thr, lcg_double(t))], 1u);
-        }
-      }
-      __syncthreads();
-      if (tid == 0) {  // offsets (material order 0..11) and cursors; tallies
-        uint32_t o = 0;
-        for (int m = 0; m < 12; m++) {
-          const uint32_t cm = mcnt[m];
-          mcnt[16 + m] = o;
-          c.sh->tallies[5 + m] += cm;
-          mcnt[m] = o;
-          o += cm;
-        }
-        mcnt[28] = o;
-      }
-      __syncthreads();
-      // (A2) re-sample, scatter energies (and union indices) to sorted slots
-      {
-        uint64_t s = s0;
-        for (int r = 0; r < K; r++, s = JT(s)) {
-          if (tid + r * T >= nb) break;
+        uint64_t s = lcg_pow(2ULL * (uint64_t)(c0 + g0))(p.seed);
+        for (long long li = g0; li < nc; li += gs, s = JG(s)) {
           uint64_t t = s;
           const double pe = lcg_double(t);
           const int mat = pick_mat_thr(thr, lcg_double(t));
-          const uint32_t pos = atomicAdd(&mcnt[mat], 1u);
-          slot_pe[pos] = pe;
-          if (GRID == XS_UNIONIZED) {  // == grid_search(u, pe, 0, n_u-1) (XS-7)
-            long long b = (long long)(pe * (double)UB);
-            if (b > UB - 1) b = UB - 1;
-            long long cc = ld_(uf + b);
-            while (cc < n_u - 1 && __longlong_as_double((long long)ld_(uA + cc + 1)) <= pe) cc++;
-            slot_idx[pos] = (int)(cc < n_u - 2 ? cc : n_u - 2);
-          }
+          long long eb = (long long)(pe * bscale);
+          eb = eb > (1LL << kb) - 1 ? (1LL << kb) - 1 : eb;
+          atomicAdd(&hist[((long long)mat << kb) + eb], 1u);
+          atomicAdd(&mcnt[mat], 1u);
         }
       }
-      __syncthreads();
+      team_sync(c);
+      // (B) bucket offsets (one CTA), material starts to every CTA's smem
+      if (c.crank == 0) global_exclusive_scan(hist, NB + 1, c.sh);
+      team_sync(c);
+      if (tid < 12) mcnt[16 + tid] = ld_(hist + ((long long)tid << kb));
+      if (tid == 12) mcnt[28] = (uint32_t)nc;
+      team_sync(c);  // every CTA has its offsets before (C) moves the cursors
+      // (C) scatter energies to their buckets (hist becomes bucket ends)
+      {
+        uint64_t s = lcg_pow(2ULL * (uint64_t)(c0 + g0))(p.seed);
+        for (long long li = g0; li < nc; li += gs, s = JG(s)) {
+          uint64_t t = s;
+          const double pe = lcg_double(t);
+          const int mat = pick_mat_thr(thr, lcg_double(t));
+          long long eb = (long long)(pe * bscale);
+          eb = eb > (1LL << kb) - 1 ? (1LL << kb) - 1 : eb;
+          lk_pe[atomicAdd(&hist[((long long)mat << kb) + eb], 1u)] = pe;
+        }
+      }
+      team_sync(c);
       phase_mark(c, 10);
-      // (B) thread-per-lookup over sorted slots
-      for (int sl = tid; sl < nb; sl += T) {
+      // (D) thread-per-lookup over the sorted chunk
+      for (long long sl = g0; sl < nc; sl += gs) {
         int mat = 0;
 #pragma unroll
-        for (int m = 1; m < 12; m++) mat += (sl >= (int)mcnt[16 + m]) ? 1 : 0;
-        const double pe = slot_pe[sl];
+        for (int m = 1; m < 12; m++) mat += (sl >= (long long)mcnt[16 + m]) ? 1 : 0;
+        const double pe = ld_(lk_pe + sl);
         int idx = 0;
-        if (GRID == XS_UNIONIZED) idx = slot_idx[sl];
+        if (GRID == XS_UNIONIZED) idx = union_idx(uf, uA, UB, n_u, pe);
         else if (GRID == XS_HASH) {
           const long long bb = (long long)(pe / du);
           idx = bb > p.bins - 1 ? p.bins - 1 : (int)bb;  // reading Q14
@@ -979,9 +976,10 @@ struct XsApp {
         fsum += m0; fsum += m1; fsum += m2; fsum += m3; fsum += m4;
         fabs_ += fabs(m0); fabs_ += fabs(m1); fabs_ += fabs(m2); fabs_ += fabs(m3); fabs_ += fabs(m4);
       }
-      __syncthreads();  // slots reused by the next batch
+      team_sync(c);  // lk_pe / hist reused by the next chunk
       phase_mark(c, 11);
     }
+    if (tid < 12) c.sh->tallies[5 + tid] += mcnt[tid];  // lookups this CTA sampled, per material
     ver = team_sum_u64(c, ver);
     bsum = team_sum_u64(c, bsum);
     fsum = team_sum_f64(c, fsum);

@@ -49,6 +49,14 @@ if __name__ == "__main__":
     if "--team" in sys.argv:
         team = int(sys.argv[sys.argv.index("--team") + 1])
         args.remove(str(team))
+    if "--l2fetch" in sys.argv:  # cudaLimitMaxL2FetchGranularity experiment
+        from cuda.bindings import runtime as rt
+        g = int(sys.argv[sys.argv.index("--l2fetch") + 1])
+        args.remove(str(g))
+        torch.cuda.init()
+        torch.zeros(1, device="cuda")
+        print("set", rt.cudaDeviceSetLimit(rt.cudaLimit.cudaLimitMaxL2FetchGranularity, g),
+              "get", rt.cudaDeviceGetLimit(rt.cudaLimit.cudaLimitMaxL2FetchGranularity), flush=True)
     m = 0
     if "--m" in sys.argv:
         m = int(sys.argv[sys.argv.index("--m") + 1])
