@@ -191,11 +191,12 @@ ENS_HD int xs_lk_bits(long long n_c) {
   while (kb < 18 && (12LL << kb) * 2 < n_c) kb++;
   return kb;
 }
-// hash index entry: the upstream index u_low = ig[b][i] plus E_i[u_low+1], so
-// a lookup knows from one 16-B load whether its energy lies in the first
-// record pair of the bin (a private accelerator; results are unchanged)
+// hash index entry: the upstream index u_low = ig[b][i], u_high = ig[b+1][i]
+// + 1 and E_i[u_low+1], so a lookup knows from one 16-B load its search range
+// and whether its energy lies in the first record pair of the bin (a private
+// accelerator; results are unchanged)
 struct XsHashEnt {
-  int u_low, pad;
+  int u_low, u_high;
   double e_next;
 };
 // cs = CTAs in the team: hash / nuclide grids give each CTA its own

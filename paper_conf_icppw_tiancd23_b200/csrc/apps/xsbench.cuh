@@ -418,11 +418,11 @@ struct XsApp {
         }
         if (tid == 0) col[p.bins] = n_gp - 2;
         __syncthreads();
-        for (int b = tid; b <= p.bins; b += T) {  // entries {u_low, E[u_low+1]}
+        for (int b = tid; b <= p.bins; b += T) {  // entries {u_low, u_high, E[u_low+1]}
           const int ul = col[b];
           XsHashEnt h;
           h.u_low = ul;
-          h.pad = 0;
+          h.u_high = (b < p.bins ? col[b + 1] : n_gp - 2) + 1;
           h.e_next = ld_(rec_i + 6 * (size_t)(ul + 1));
           ent[b] = h;
         }
@@ -701,6 +701,52 @@ struct XsApp {
     const uint16_t *mrow = mats + mat * mx;
     const double *crow = concs + mat * mx;
     double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
+    if constexpr (GRID == XS_HASH && kU == 1) {
+      // software-pipelined: nuclide j+1's index entry is in flight while
+      // nuclide j's record pair is gathered (two deep spills: measured slower)
+      const size_t hs = (size_t)p.bins + 1;
+      const XsHashEnt *hc = (const XsHashEnt *)ig + idx;
+      int4 hn = make_int4(0, 0, 0, 0);
+      if (nm > 0) hn = ld_(reinterpret_cast<const int4 *>(hc + (size_t)mrow[0] * hs));
+      for (int j = 0; j < nm; j++) {
+        const int4 h = hn;
+        const double *E = recs + (size_t)mrow[j] * n_gp * 6;
+        int lo = pe < __hiloint2double(h.w, h.z) ? h.x : h.x + 1;
+        const int uh = h.y;
+        const double2 *r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
+        double2 a0 = ld_(r2 + 0), a1 = ld_(r2 + 1), a2 = ld_(r2 + 2);
+        double2 b0 = ld_(r2 + 3), b1 = ld_(r2 + 4), b2 = ld_(r2 + 5);
+        if (j + 1 < nm) hn = ld_(reinterpret_cast<const int4 *>(hc + (size_t)mrow[j + 1] * hs));
+        while (pe >= b0.x && a0.x < pe && lo + 2 <= uh) {  // see the generic path below
+          lo++;
+          r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
+          a0 = b0; a1 = b1; a2 = b2;
+          b0 = ld_(r2 + 3); b1 = ld_(r2 + 4); b2 = ld_(r2 + 5);
+        }
+        if (!(a0.x < pe && pe < b0.x && lo + 1 <= uh)) {  // edges: upstream logic
+          const int u_low = h.x;
+          const double e_low = ld_(E + 6 * (size_t)u_low);
+          const double e_high = ld_(E + 6 * (size_t)uh);
+          int lower;
+          if (pe <= e_low) lower = 0;
+          else if (pe >= e_high) lower = n_gp - 1;
+          else lower = gs_recs(E, pe, u_low, uh);
+          const int l2 = lower == n_gp - 1 ? lower - 1 : lower;
+          r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)l2);
+          a0 = ld_(r2 + 0); a1 = ld_(r2 + 1); a2 = ld_(r2 + 2);
+          b0 = ld_(r2 + 3); b1 = ld_(r2 + 4); b2 = ld_(r2 + 5);
+        }
+        const double conc = crow[j];
+        const double f = (b0.x - pe) / (b0.x - a0.x);
+        m0 += (b0.y - f * (b0.y - a0.y)) * conc;
+        m1 += (b1.x - f * (b1.x - a1.x)) * conc;
+        m2 += (b1.y - f * (b1.y - a1.y)) * conc;
+        m3 += (b2.x - f * (b2.x - a2.x)) * conc;
+        m4 += (b2.y - f * (b2.y - a2.y)) * conc;
+      }
+      m[0] = m0; m[1] = m1; m[2] = m2; m[3] = m3; m[4] = m4;
+      return;
+    }
     for (int j0 = 0; j0 < nm; j0 += kU) {
       int nuc[kU], lo[kU], uh[kU];
       bool on[kU];
@@ -719,7 +765,7 @@ struct XsApp {
             const XsHashEnt *he = (const XsHashEnt *)ig + (size_t)nuc[u] * (p.bins + 1) + idx;
             const int4 h = ld_(reinterpret_cast<const int4 *>(he));
             const double e_next = __hiloint2double(h.w, h.z);
-            uh[u] = ld_(&he[1].u_low) + 1;
+            uh[u] = h.y;
             lo[u] = pe < e_next ? h.x : h.x + 1;
           } else if (GRID == XS_UNIONIZED) {
             const int k = ld_(ig + (size_t)idx * n_iso + nuc[u]);
