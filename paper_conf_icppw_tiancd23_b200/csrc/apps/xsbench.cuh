@@ -747,6 +747,27 @@ struct XsApp {
       m[0] = m0; m[1] = m1; m[2] = m2; m[3] = m3; m[4] = m4;
       return;
     }
+    if constexpr (GRID == XS_UNIONIZED && kU == 1) {  // same pipelining over the union row
+      const int *row = ig + (size_t)idx * n_iso;
+      int kn = nm > 0 ? ld_(row + mrow[0]) : 0;
+      for (int j = 0; j < nm; j++) {
+        const int k = kn;
+        if (j + 1 < nm) kn = ld_(row + mrow[j + 1]);
+        const int lo = (k == n_gp - 1) ? k - 1 : k;
+        const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)mrow[j] * n_gp + lo) * 6);
+        const double2 a0 = ld_(r2 + 0), a1 = ld_(r2 + 1), a2 = ld_(r2 + 2);
+        const double2 b0 = ld_(r2 + 3), b1 = ld_(r2 + 4), b2 = ld_(r2 + 5);
+        const double conc = crow[j];
+        const double f = (b0.x - pe) / (b0.x - a0.x);
+        m0 += (b0.y - f * (b0.y - a0.y)) * conc;
+        m1 += (b1.x - f * (b1.x - a1.x)) * conc;
+        m2 += (b1.y - f * (b1.y - a1.y)) * conc;
+        m3 += (b2.x - f * (b2.x - a2.x)) * conc;
+        m4 += (b2.y - f * (b2.y - a2.y)) * conc;
+      }
+      m[0] = m0; m[1] = m1; m[2] = m2; m[3] = m3; m[4] = m4;
+      return;
+    }
     for (int j0 = 0; j0 < nm; j0 += kU) {
       int nuc[kU], lo[kU], uh[kU];
       bool on[kU];
