@@ -166,8 +166,7 @@ constexpr int kXsSweepRows = 512;
 // arena layout (byte offsets, 256-B aligned)
 struct XsLayout {
   uint64_t recs;      // [n_iso][n_gp] x 48 B records, sorted per nuclide
-  uint64_t scratch;   // [n_u] x 48 B records in generation order
-  uint64_t keys;      // [n_u] x 16 B {energy bits, record id}, bucket-sorted
+  uint64_t keys;      // [n_u] (hash / nuclide: [cs][n_gp]) x 16 B {energy bits, record id}, bucket-sorted
   uint64_t bkt;       // [xs_buckets] u32 bucket counts -> offsets
   uint64_t uenergy;   // unionized: [n_u] sorted union energies (u64 bits)
   uint64_t ufind;     // unionized: [xs_ubins] u32 union search table (private accelerator)
@@ -208,7 +207,6 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
   // unionized: one sort of all n_u records; otherwise one nuclide at a time
   const uint64_t n_s = p.grid == XS_UNIONIZED ? n_u : (uint64_t)p.n_gp * (uint64_t)cs;
   L.recs = o; o = align_up(o + n_u * 48, 256);
-  L.scratch = o; o = align_up(o + n_s * 48, 256);
   L.keys = o; o = align_up(o + n_s * 16, 256);
   L.bkt = o;
   if (p.grid == XS_UNIONIZED) o = align_up(o + (uint64_t)xs_buckets(p) * 4, 256);
@@ -238,7 +236,7 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
 constexpr int kXsU = ENS_XS_U;  // nuclide gathers in flight per lane
 constexpr int kXsMaxT = 512;  // XsApp::kMaxT
 struct XsSmem {
-  uint32_t thr, nn, mats, concs, mcnt, nbkt, total;
+  uint32_t thr, nn, mats, concs, mcnt, jmp, nbkt, total;
 };
 // T = the block size the instance runs with
 ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
@@ -250,6 +248,7 @@ ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   S.concs = o; o += 12 * mx * 8;          // concentrations
   S.mats = o; o += (uint32_t)align_up(12 * mx * 2, 16);  // nuclide ids (u16)
   S.mcnt = o; o += 32 * 4;                // material counts / offsets of a lookup chunk
+  S.jmp = o; o += 4 * 64 * 16;            // LCG jump tables: A^(6 d 64^l), l < 4, d < 64
   S.nbkt = o;                             // per-nuclide sort buckets (hash / nuclide grids)
   if (p.grid != XS_UNIONIZED) o += (uint32_t)align_up((uint64_t)xs_nbn(p.n_gp) * 4, 16);
   (void)T;

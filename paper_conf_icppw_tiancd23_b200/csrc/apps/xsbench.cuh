@@ -6,11 +6,11 @@
 //
 // B200 design (results identical to the oracle):
 //  * init keeps shared memory small (material tables + bucket counters) so
-//    the L1 stays large for the lookup phase: each nuclide's records are
-//    generated into an L2-resident scratch (LCG jump constants), sorted by a
-//    bucket sort (energies are uniform in [0,1): counts -> scan -> scatter ->
-//    insertion sort of ~1.4-element buckets), then scattered once to their
-//    sorted position;
+//    the L1 stays large for the lookup phase: only {energy, record id} keys
+//    are sorted (energies are uniform in [0,1): counts -> scan -> scatter ->
+//    insertion sort of ~1.4-element buckets); each record is then written
+//    once, at its sorted position, its cross sections re-drawn from the LCG
+//    through jump tables (no generation-order copy);
 //  * the hash index grid is stored nuclide-major [n_iso][bins+1] (entry
 //    `bins` = n_gp-2, so u_high needs no branch) and built by a merge walk;
 //  * lookups run warp-cooperatively: lane = lookup for the sampling and the
@@ -181,6 +181,11 @@ struct XsApp {
 
     // ---- XS-2: materials, concentrations ---------------------------------
     hm_tables(n_iso, mx, thr, nn, concs, mats);
+    {  // LCG jump tables for XS-3's record draws (see jump6)
+      Affine *jt = (Affine *)(c.smem + S.jmp);
+      for (int x = threadIdx.x; x < 256; x += blockDim.x)
+        jt[x] = lcg_pow((6ULL * (uint64_t)(x & 63)) << (6 * (x >> 6)));
+    }
     __syncthreads();
     hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
     phase_mark(c, 0);
@@ -209,6 +214,27 @@ struct XsApp {
     ens_printf(c, FMT_VERIFY, (unsigned long long)R.vhash);
     R.exit_code = 0;
     return R;
+  }
+
+  // the LCG state s advanced by 6r draws (record r's draws are 6r+1..6r+6,
+  // XS-3), from the smem tables jt[64 l + d] = A^(6 d 64^l): four affine
+  // steps instead of a 6r-step walk (r < 2^24)
+  __device__ static __forceinline__ uint64_t jump6(const Affine *jt, uint32_t r, uint64_t s) {
+    s = jt[r & 63u](s);
+    s = jt[64 + ((r >> 6) & 63u)](s);
+    s = jt[128 + ((r >> 12) & 63u)](s);
+    return jt[192 + ((r >> 18) & 63u)](s);
+  }
+  // record r at dst: E (the key's energy, draw 6r+1) and draws 6r+2..6r+6
+  __device__ static __forceinline__ void put_record(const Affine *jt, uint32_t r, unsigned long long ebits,
+                                                    uint64_t gseed, double *dst) {
+    uint64_t t = lcg_next(jump6(jt, r, gseed));  // past the energy draw
+    const double x1 = lcg_double(t), x2 = lcg_double(t), x3 = lcg_double(t), x4 = lcg_double(t),
+                 x5 = lcg_double(t);
+    double2 *d = reinterpret_cast<double2 *>(dst);
+    d[0] = make_double2(__longlong_as_double((long long)ebits), x1);
+    d[1] = make_double2(x2, x3);
+    d[2] = make_double2(x4, x5);
   }
 
   // sort keys[lo, hi) by (energy, record id): <= 8 in registers, else in place
@@ -304,10 +330,11 @@ struct XsApp {
   }
 
   // ---- XS-3/4/5, hash and nuclide grids: one nuclide at a time -------------
-  // Nuclide i's n_gp records (draws 6r+1..6r+6, r = i*n_gp + j; XS-3) are
-  // generated into an L2-resident scratch, bucket-sorted by energy (XS-4:
-  // shared-memory counts -> scan -> scatter -> per-bucket sort), written to
-  // their sorted position, and (hash) the nuclide's index column is built as
+  // Nuclide i's n_gp energies (draw 6r+1 of record r = i*n_gp + j; XS-3)
+  // are bucket-sorted as {energy, j} keys in an L2-resident buffer (XS-4:
+  // shared-memory counts -> scan -> scatter -> per-bucket sort), each record
+  // is written once in sorted order (coalesced) with its draws 6r+2..6r+6
+  // re-generated, and (hash) the nuclide's index column is built as
   // a histogram of each energy's first bin followed by an inclusive scan
   // (XS-5: ig[i][b] = grid_search(E_i, b*du) = min(#{k>=1: E_k <= b*du}, n_gp-2)).
   __device__ static __noinline__ void init_nuc(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
@@ -315,58 +342,55 @@ struct XsApp {
     const int n_iso = p.n_iso, n_gp = p.n_gp;
     const int nbn = xs_nbn(n_gp);
     uint32_t *nb = (uint32_t *)(c.smem + S.nbkt);
+    const Affine *jt = (const Affine *)(c.smem + S.jmp);
     double *recs = (double *)(c.arena + L.recs);
-    double *scr = (double *)(c.arena + L.scratch);
     XsKey *keys = (XsKey *)(c.arena + L.keys);
     int *ig = (int *)(c.arena + L.index);
     const bool hash = p.grid == XS_HASH;
     const double du = 1.0 / p.bins;
-    const Affine J6T = lcg_pow(6ULL * T);
-    // this CTA takes nuclides crank, crank + csize, ... with its own scratch
-    scr += (size_t)c.crank * n_gp * 6;
+    const Affine J6T = lcg_pow(6ULL * T), J24T = lcg_pow(24ULL * T);
+    // this CTA takes nuclides crank, crank + csize, ... with its own keys
     keys += (size_t)c.crank * n_gp;
-    const Affine Jnuc = lcg_pow(6ULL * n_gp * c.csize);
-    uint64_t s_nuc = lcg_pow(6ULL * ((uint64_t)c.crank * n_gp + tid))(p.gseed);  // record (i*n_gp + tid)
     for (int i = (int)c.crank; i < n_iso; i += (int)c.csize) {
       int *col = (int *)(c.arena + L.hcol) + (size_t)c.crank * (p.bins + 1);  // this CTA's column
       XsHashEnt *ent = (XsHashEnt *)ig + (size_t)i * (p.bins + 1);
+      const uint32_t r0 = (uint32_t)i * (uint32_t)n_gp;  // record i*n_gp + j
       for (int b = tid; b < nbn; b += T) nb[b] = 0;
       if (hash)
         for (int b = tid; b <= p.bins; b += T) col[b] = 0;
       __syncthreads();
-      {  // generate + count
-        uint64_t s = s_nuc;
+      {  // count the energies' buckets (energy = draw 6r+1)
+        uint64_t s = jump6(jt, r0 + (uint32_t)tid, p.gseed);
         for (int j = tid; j < n_gp; j += T, s = J6T(s)) {
           uint64_t t = s;
-          double v[6];
-#pragma unroll
-          for (int f = 0; f < 6; f++) v[f] = lcg_double(t);
-          double2 *d = reinterpret_cast<double2 *>(scr + 6 * (size_t)j);
-          d[0] = make_double2(v[0], v[1]);
-          d[1] = make_double2(v[2], v[3]);
-          d[2] = make_double2(v[4], v[5]);
-          atomicAdd(&nb[bucket_of(v[0], j, n_gp, false, 0, nbn)], 1u);
+          atomicAdd(&nb[bucket_of(lcg_double(t), j, n_gp, false, 0, nbn)], 1u);
         }
-        s_nuc = Jnuc(s_nuc);
       }
       __syncthreads();
       phase_mark(c, 1);
       global_exclusive_scan(nb, nbn, c.sh);
       phase_mark(c, 2);
-      for (int j0 = tid; j0 < n_gp; j0 += 4 * T) {  // scatter {energy, j}
-        double e[4];
+      {  // scatter {energy, j}, the energies re-drawn, four atomics in flight
+        uint64_t s = jump6(jt, r0 + (uint32_t)tid, p.gseed);
+        for (int j0 = tid; j0 < n_gp; j0 += 4 * T, s = J24T(s)) {
+          double e[4];
+          uint64_t sq = s;
 #pragma unroll
-        for (int q = 0; q < 4; q++) e[q] = j0 + q * T < n_gp ? ld_(scr + 6 * (size_t)(j0 + q * T)) : 0.0;
+          for (int q = 0; q < 4; q++, sq = J6T(sq)) {
+            uint64_t t = sq;
+            e[q] = lcg_double(t);
+          }
 #pragma unroll
-        for (int q = 0; q < 4; q++) {
-          const int j = j0 + q * T;
-          if (j < n_gp) {
-            const uint32_t pos = atomicAdd(&nb[bucket_of(e[q], j, n_gp, false, 0, nbn)], 1u);
-            XsKey k;
-            k.key = dbits(e[q]);
-            k.idx = (unsigned)j;
-            k.pad = 0;
-            keys[pos] = k;
+          for (int q = 0; q < 4; q++) {
+            const int j = j0 + q * T;
+            if (j < n_gp) {
+              const uint32_t pos = atomicAdd(&nb[bucket_of(e[q], j, n_gp, false, 0, nbn)], 1u);
+              XsKey k;
+              k.key = dbits(e[q]);
+              k.idx = (unsigned)j;
+              k.pad = 0;
+              keys[pos] = k;
+            }
           }
         }
       }
@@ -375,31 +399,21 @@ struct XsApp {
       for (int b = tid; b < nbn; b += T) sort_bucket(keys, b ? nb[b - 1] : 0, nb[b]);
       __syncthreads();
       phase_mark(c, 4);
+      // records written in sorted order (coalesced), their draws re-generated
+      // from the jump tables; hash: each energy's first bin counted
       double *rec_i = recs + (size_t)i * n_gp * 6;
-      for (int k0 = tid; k0 < n_gp; k0 += 4 * T) {  // records to sorted position; bin histogram
-        unsigned jj[4];
-        unsigned long long kb[4];
+      for (int k0 = tid; k0 < n_gp; k0 += 2 * T) {
+        XsKey v[2];
 #pragma unroll
-        for (int q = 0; q < 4; q++) {
+        for (int q = 0; q < 2; q++)
+          if (k0 + q * T < n_gp) v[q] = keys[k0 + q * T];
+#pragma unroll
+        for (int q = 0; q < 2; q++) {
           const int k = k0 + q * T;
           if (k < n_gp) {
-            const XsKey v = keys[k];
-            jj[q] = v.idx;
-            kb[q] = v.key;
-          }
-        }
-#pragma unroll
-        for (int q = 0; q < 4; q++) {
-          const int k = k0 + q * T;
-          if (k < n_gp) {
-            const double2 *src = reinterpret_cast<const double2 *>(scr + 6 * (size_t)jj[q]);
-            double2 *dst = reinterpret_cast<double2 *>(rec_i + 6 * (size_t)k);
-            const double2 a = src[0], b = src[1], x = src[2];
-            dst[0] = a;
-            dst[1] = b;
-            dst[2] = x;
+            put_record(jt, r0 + v[q].idx, v[q].key, p.gseed, rec_i + 6 * (size_t)k);
             if (hash && k >= 1) {  // first bin b with E_k <= b*du
-              const double e = __longlong_as_double((long long)kb[q]);
+              const double e = __longlong_as_double((long long)v[q].key);
               long long bb = (long long)(e * p.bins);
               while (bb > 0 && (double)(bb - 1) * du >= e) bb--;
               while (bb < p.bins && (double)bb * du < e) bb++;
@@ -423,7 +437,7 @@ struct XsApp {
           XsHashEnt h;
           h.u_low = ul;
           h.u_high = (b < p.bins ? col[b + 1] : n_gp - 2) + 1;
-          h.e_next = ld_(rec_i + 6 * (size_t)(ul + 1));
+          h.e_next = __longlong_as_double((long long)keys[ul + 1].key);
           ent[b] = h;
         }
         __syncthreads();
@@ -432,46 +446,36 @@ struct XsApp {
     }
   }
 
-  // ---- XS-3/4/5: nuclide grid, sort, acceleration structure --------------
-  // One block-wide bucket sort of all n_u records replaces n_iso per-nuclide
-  // sorts: (G) generate every record (draws 6r+1..6r+6, XS-3) into scratch
-  // and count its bucket; (S) scan; (P) scatter {energy, record id}; (B)
-  // insertion-sort each ~2-element bucket.  Unionized buckets are by energy
-  // alone, so the sorted keys ARE the union (XS-5) and a nuclide's records in
-  // union order are its sorted records (XS-4); otherwise buckets are
-  // (nuclide, energy).  Ties are measure-zero (reading Q13) and broken by
-  // record id, deterministically.
+  // ---- XS-3/4/5, unionized grid: one block-wide sort of all records ------
+  // One bucket sort of all n_u records by energy replaces n_iso per-nuclide
+  // sorts and the union merge: (G) count each record's energy bucket (energy
+  // = draw 6r+1, XS-3); (S) scan; (P) scatter {energy, record id}; (B)
+  // insertion-sort each ~2-element bucket.  The sorted keys ARE the union
+  // (XS-5) and a nuclide's records in union order are its sorted records
+  // (XS-4).  Ties are measure-zero (reading Q13) and broken by record id.
+  // (U) union tables, (W) index sweep, (R) every record written once to its
+  // sorted position, its five cross sections re-drawn via the jump tables.
   __device__ static __noinline__ void init(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
     const int tid = threadIdx.x, T = blockDim.x;
     const int n_iso = p.n_iso, n_gp = p.n_gp;
     const long long n_u = (long long)n_iso * n_gp;
     const long long NB = xs_buckets(p);
     const int nbn = xs_nbn(n_gp);
+    const Affine *jt = (const Affine *)(c.smem + S.jmp);
     double *recs = (double *)(c.arena + L.recs);
-    double *scr = (double *)(c.arena + L.scratch);
     XsKey *keys = (XsKey *)(c.arena + L.keys);
     uint32_t *bkt = (uint32_t *)(c.arena + L.bkt);
     int *ig = (int *)(c.arena + L.index);
-    const bool uni = p.grid == XS_UNIONIZED;
+    const Affine J6T = lcg_pow(6ULL * T), J24T = lcg_pow(24ULL * T);
 
     for (long long b = tid; b < NB; b += T) bkt[b] = 0;
-    if (p.grid == XS_HASH)
-      for (long long x = tid; x < (long long)n_iso * (p.bins + 1); x += T) ig[x] = 0;
     __syncthreads();
-    // (G) generate + count
+    // (G) count
     {
-      const Affine J6T = lcg_pow(6ULL * T);
       uint64_t s = lcg_pow(6ULL * tid)(p.gseed);
       for (long long r = tid; r < n_u; r += T, s = J6T(s)) {
         uint64_t t = s;
-        double v[6];
-#pragma unroll
-        for (int f = 0; f < 6; f++) v[f] = lcg_double(t);
-        double2 *d = reinterpret_cast<double2 *>(scr + 6 * r);
-        d[0] = make_double2(v[0], v[1]);
-        d[1] = make_double2(v[2], v[3]);
-        d[2] = make_double2(v[4], v[5]);
-        atomicAdd(&bkt[bucket_of(v[0], r, n_gp, uni, NB, nbn)], 1u);
+        atomicAdd(&bkt[bucket_of(lcg_double(t), r, n_gp, true, NB, nbn)], 1u);
       }
     }
     __syncthreads();
@@ -479,156 +483,44 @@ struct XsApp {
     // (S) bucket offsets
     global_exclusive_scan(bkt, NB, c.sh);
     XS_STOP(2);
-    // (P) scatter
-    for (long long r0 = tid; r0 < n_u; r0 += 4LL * T) {  // 4 independent atomics in flight
-      double e[4];
-      uint32_t pos[4];
+    // (P) scatter, energies re-drawn, 4 independent atomics in flight
+    {
+      uint64_t s = lcg_pow(6ULL * tid)(p.gseed);
+      for (long long r0 = tid; r0 < n_u; r0 += 4LL * T, s = J24T(s)) {
+        double e[4];
+        uint32_t pos[4];
+        uint64_t sq = s;
 #pragma unroll
-      for (int q = 0; q < 4; q++) {
-        const long long r = r0 + (long long)q * T;
-        e[q] = r < n_u ? ld_(scr + 6 * r) : 0.0;
-      }
+        for (int q = 0; q < 4; q++, sq = J6T(sq)) {
+          uint64_t t = sq;
+          e[q] = lcg_double(t);
+        }
 #pragma unroll
-      for (int q = 0; q < 4; q++) {
-        const long long r = r0 + (long long)q * T;
-        if (r < n_u) pos[q] = atomicAdd(&bkt[bucket_of(e[q], r, n_gp, uni, NB, nbn)], 1u);
-      }
+        for (int q = 0; q < 4; q++) {
+          const long long r = r0 + (long long)q * T;
+          if (r < n_u) pos[q] = atomicAdd(&bkt[bucket_of(e[q], r, n_gp, true, NB, nbn)], 1u);
+        }
 #pragma unroll
-      for (int q = 0; q < 4; q++) {
-        const long long r = r0 + (long long)q * T;
-        if (r < n_u) {
-          XsKey k;
-          k.key = dbits(e[q]);
-          k.idx = (unsigned)r;
-          k.pad = 0;
-          keys[pos[q]] = k;
+        for (int q = 0; q < 4; q++) {
+          const long long r = r0 + (long long)q * T;
+          if (r < n_u) {
+            XsKey k;
+            k.key = dbits(e[q]);
+            k.idx = (unsigned)r;
+            k.pad = 0;
+            keys[pos[q]] = k;
+          }
         }
       }
     }
     __syncthreads();
     XS_STOP(3);
-    // (B) sort each bucket by (energy, record id); bkt[b] = end of bucket b.
-    // Buckets hold ~2 keys: up to 8 are sorted in registers, more in memory.
-    for (long long b = tid; b < NB; b += T) {
-      const long long lo = b ? (long long)bkt[b - 1] : 0, hi = (long long)bkt[b];
-      const int cnt = (int)(hi - lo);
-      if (cnt <= 1) continue;
-      if (cnt <= 8) {
-        unsigned long long kk[8];
-        unsigned ii[8];
-#pragma unroll
-        for (int q = 0; q < 8; q++)
-          if (q < cnt) {
-            const XsKey v = keys[lo + q];
-            kk[q] = v.key;
-            ii[q] = v.idx;
-          }
-#pragma unroll
-        for (int x = 1; x < 8; x++) {  // insertion sort, fully unrolled
-#pragma unroll
-          for (int y = x; y > 0; y--) {
-            if (x < cnt) {
-              const bool sw = kk[y - 1] > kk[y] || (kk[y - 1] == kk[y] && ii[y - 1] > ii[y]);
-              if (sw) {
-                const unsigned long long tk = kk[y - 1];
-                kk[y - 1] = kk[y];
-                kk[y] = tk;
-                const unsigned ti = ii[y - 1];
-                ii[y - 1] = ii[y];
-                ii[y] = ti;
-              }
-            }
-          }
-        }
-#pragma unroll
-        for (int q = 0; q < 8; q++)
-          if (q < cnt) {
-            XsKey v;
-            v.key = kk[q];
-            v.idx = ii[q];
-            v.pad = 0;
-            keys[lo + q] = v;
-          }
-      } else {
-        for (long long x = lo + 1; x < hi; x++) {
-          const XsKey v = keys[x];
-          long long y = x - 1;
-          while (y >= lo && (keys[y].key > v.key || (keys[y].key == v.key && keys[y].idx > v.idx))) {
-            keys[y + 1] = keys[y];
-            y--;
-          }
-          keys[y + 1] = v;
-        }
-      }
-    }
+    // (B) sort each bucket by (energy, record id); bkt[b] = end of bucket b
+    for (long long b = tid; b < NB; b += T) sort_bucket(keys, b ? (long long)bkt[b - 1] : 0, (long long)bkt[b]);
     __syncthreads();
-
     XS_STOP(4);
-    if (!uni) {
-      // (R) records to their sorted position: bucket order is nuclide-major
-      for (long long k = tid; k < n_u; k += T) {
-        const unsigned r = keys[k].idx;
-        const double2 *src = reinterpret_cast<const double2 *>(scr + 6 * (size_t)r);
-        double2 *dst = reinterpret_cast<double2 *>(recs + 6 * k);
-        const double2 a = src[0], b = src[1], e = src[2];
-        dst[0] = a;
-        dst[1] = b;
-        dst[2] = e;
-      }
-      if (p.grid != XS_HASH) {
-        __syncthreads();
-        return;
-      }
-    XS_STOP(5);
-      // (H) hash grid ig[i][b] = grid_search(E_i, b*du, 0, n_gp-1)
-      //      = min(#{k >= 1 : E_i[k] <= b*du}, n_gp-2): histogram of each
-      //      energy's first bin b_k (smallest b with E_k <= b*du), then a
-      //      per-nuclide prefix sum over the bins.
-      const double du = 1.0 / p.bins;
-      for (long long k = tid; k < n_u; k += T) {
-        const int i = (int)(k / n_gp), kk = (int)(k % n_gp);
-        if (kk == 0) continue;
-        const double e = __longlong_as_double((long long)keys[k].key);
-        long long b = (long long)(e * p.bins);
-        while (b > 0 && (double)(b - 1) * du >= e) b--;
-        while (b < p.bins && (double)b * du < e) b++;
-        if (b < p.bins) atomicAdd((unsigned *)&ig[(size_t)i * (p.bins + 1) + b], 1u);
-      }
-      __syncthreads();
-      {
-        const int lane = tid & 31, warp = tid >> 5, nw = T >> 5;
-        constexpr int R = 16;  // rows of 32 bins loaded per step (coalesced)
-        for (int i = warp; i < n_iso; i += nw) {
-          int *col = ig + (size_t)i * (p.bins + 1);
-          int carry = 0;  // inclusive prefix of all earlier bins
-          for (int b0 = 0; b0 < p.bins; b0 += 32 * R) {
-            int v[R];
-#pragma unroll
-            for (int q = 0; q < R; q++) {
-              const int b = b0 + 32 * q + lane;
-              v[q] = b < p.bins ? col[b] : 0;
-            }
-#pragma unroll
-            for (int q = 0; q < R; q++) {
-              int inc = v[q];
-              for (int o = 1; o < 32; o <<= 1) {
-                const int t = __shfl_up_sync(0xffffffffu, inc, o);
-                if (lane >= o) inc += t;
-              }
-              const int run = carry + inc;
-              const int b = b0 + 32 * q + lane;
-              if (b < p.bins) col[b] = run < n_gp - 2 ? run : n_gp - 2;
-              carry = __shfl_sync(0xffffffffu, run, 31);
-            }
-          }
-          if (lane == 0) col[p.bins] = n_gp - 2;
-        }
-      }
-      __syncthreads();
-      return;
-    }
 
-    // ---- unionized: keys[] is the union (XS-5); owner = record id / n_gp ----
+    // (U) keys[] is the union (XS-5); owner = record id / n_gp
     uint64_t *uA = (uint64_t *)(c.arena + L.uenergy);
     uint32_t *chist = (uint32_t *)(c.arena + L.chist);
     const long long nch = (n_u + kXsSweepRows - 1) / kXsSweepRows;
@@ -661,30 +553,22 @@ struct XsApp {
     }
     __syncthreads();
     XS_STOP(6);
-    // sweep: a warp per chunk, lanes own nuclides; row e of the index grid is
-    // clip(#{k>=1: E_i[k] <= u_e}, 0, n_gp-2) = clip(cnt_i(e) - 1, ...), and
-    // the owner's new count is the sorted position of that record (XS-4).
+    // (W) sweep: a warp per chunk, lanes own nuclides; row e of the index grid
+    // is clip(#{k>=1: E_i[k] <= u_e}, 0, n_gp-2) = clip(cnt_i(e) - 1, ...),
+    // and the owner's new count is the sorted position of that record (XS-4).
     if (n_iso <= 96) sweep<3>(keys, chist, ig, n_u, n_iso, n_gp, nch);
     else sweep<12>(keys, chist, ig, n_u, n_iso, n_gp, nch);
     __syncthreads();
     XS_STOP(7);
-    // records to their sorted positions (coalesced over the union order),
-    // four in flight per thread
-    for (long long e0 = tid; e0 < n_u; e0 += 4LL * T) {
-      XsKey k[4];
+    // (R) records to their sorted positions, keys read coalesced
+    for (long long e0 = tid; e0 < n_u; e0 += 2LL * T) {
+      XsKey k[2];
 #pragma unroll
-      for (int q = 0; q < 4; q++)
+      for (int q = 0; q < 2; q++)
         if (e0 + q * T < n_u) k[q] = keys[e0 + q * T];
 #pragma unroll
-      for (int q = 0; q < 4; q++)
-        if (e0 + q * T < n_u) {
-          const double2 *src = reinterpret_cast<const double2 *>(scr + 6 * (size_t)k[q].idx);
-          double2 *dst = reinterpret_cast<double2 *>(recs + 6 * (size_t)k[q].pad);
-          const double2 a = src[0], b = src[1], x = src[2];
-          dst[0] = a;
-          dst[1] = b;
-          dst[2] = x;
-        }
+      for (int q = 0; q < 2; q++)
+        if (e0 + q * T < n_u) put_record(jt, k[q].idx, k[q].key, p.gseed, recs + 6 * (size_t)k[q].pad);
     }
     __syncthreads();
     phase_mark(c, 8);
