@@ -190,13 +190,15 @@ ENS_HD int xs_lk_bits(long long n_c) {
   while (kb < 18 && (12LL << kb) * 2 < n_c) kb++;
   return kb;
 }
-// hash index entry: the upstream index u_low = ig[b][i], u_high = ig[b+1][i]
-// + 1 and E_i[u_low+1], so a lookup knows from one 16-B load its search range
-// and whether its energy lies in the first record pair of the bin (a private
-// accelerator; results are unchanged)
+// hash index entry (a private accelerator; results are unchanged): the
+// upstream index u_low = ig[b][i], u_high = ig[b+1][i] + 1 (n_gp <= 16384
+// fits 16 bits) and the energies E[u_low+1..u_low+6] quantized within bin b,
+// q = floor((E*bins - b) * 2^16) clamped to [0, 65535] (65535 also past the
+// grid).  q is monotone in E, so #{k: q(pe) > q_k} never exceeds the number
+// of those energies below pe: one 16-B load gives a bracket guess that is
+// exact unless two energies share a quantum, and it is always verified.
 struct XsHashEnt {
-  int u_low, u_high;
-  double e_next;
+  uint16_t u_low, u_high, q[6];
 };
 // cs = CTAs in the team: hash / nuclide grids give each CTA its own
 // per-nuclide scratch
@@ -230,10 +232,6 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
 }
 
 // dynamic shared memory layout: material tables + the sort's bucket counters
-#ifndef ENS_XS_U
-#define ENS_XS_U 1  // measured on B200: 1 beats 2 and 4 (register pressure)
-#endif
-constexpr int kXsU = ENS_XS_U;  // nuclide gathers in flight per lane
 constexpr int kXsMaxT = 512;  // XsApp::kMaxT
 struct XsSmem {
   uint32_t thr, nn, mats, concs, mcnt, jmp, nbkt, total;

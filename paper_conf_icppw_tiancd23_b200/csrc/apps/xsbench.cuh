@@ -152,7 +152,6 @@ struct XsApp {
   static constexpr uint32_t kId = APP_XSBENCH;
   // thread limit is an upper bound: 512 keeps 128 registers
   static constexpr int kMaxT = 512;
-  static constexpr int kU = kXsU;
   static constexpr bool kTeam = true;  // splits nuclides and lookup batches over a cluster
   static constexpr bool kSub = false;
 
@@ -432,12 +431,21 @@ struct XsApp {
         }
         if (tid == 0) col[p.bins] = n_gp - 2;
         __syncthreads();
-        for (int b = tid; b <= p.bins; b += T) {  // entries {u_low, u_high, E[u_low+1]}
+        for (int b = tid; b <= p.bins; b += T) {  // entries {u_low, u_high, q(E[u_low+1..u_low+6])}
           const int ul = col[b];
           XsHashEnt h;
-          h.u_low = ul;
-          h.u_high = (b < p.bins ? col[b + 1] : n_gp - 2) + 1;
-          h.e_next = __longlong_as_double((long long)keys[ul + 1].key);
+          h.u_low = (uint16_t)ul;
+          h.u_high = (uint16_t)((b < p.bins ? col[b + 1] : n_gp - 2) + 1);
+#pragma unroll
+          for (int k = 0; k < 6; k++) {
+            int q = 65535;
+            if (ul + 1 + k <= n_gp - 1) {
+              const double e = __longlong_as_double((long long)keys[ul + 1 + k].key);
+              const double x = (e * (double)p.bins - (double)b) * 65536.0;
+              q = x < 0.0 ? 0 : (x >= 65535.0 ? 65535 : (int)x);
+            }
+            h.q[k] = (uint16_t)q;
+          }
           ent[b] = h;
         }
         __syncthreads();
@@ -574,8 +582,27 @@ struct XsApp {
     phase_mark(c, 8);
   }
 
-  // XS-7..XS-9 for one lookup (energy pe, material mat, union / hash index
-  // idx): the macroscopic XS m[0..4], nuclides summed in list order.
+  // XS-8, XS-9 for one nuclide: interpolate the pair (a = low, b = high
+  // record: {E, total, elastic, absorption, fission, nu_fission}) at pe and
+  // add conc * micro to the five channels, in the oracle's operation order
+  __device__ static __forceinline__ void accumulate(double pe, double conc, const double2 &a0, const double2 &a1,
+                                                    const double2 &a2, const double2 &b0, const double2 &b1,
+                                                    const double2 &b2, double &m0, double &m1, double &m2,
+                                                    double &m3, double &m4) {
+    const double f = (b0.x - pe) / (b0.x - a0.x);
+    m0 += (b0.y - f * (b0.y - a0.y)) * conc;
+    m1 += (b1.x - f * (b1.x - a1.x)) * conc;
+    m2 += (b1.y - f * (b1.y - a1.y)) * conc;
+    m3 += (b2.x - f * (b2.x - a2.x)) * conc;
+    m4 += (b2.y - f * (b2.y - a2.y)) * conc;
+  }
+
+  // XS-7..XS-9 for one lookup (energy pe, material mat, union row / hash bin
+  // idx): the macroscopic XS m[0..4], nuclides summed in list order.  Each
+  // grid type is software-pipelined without holding future data in
+  // registers: index data a few nuclides ahead is prefetched into L1, the
+  // next nuclide's record pair is prefetched into L1 while this one's is
+  // gathered (a line's first touch goes to HBM).
   template <int GRID>
   __device__ static __forceinline__ void macro_lookup(const XsParams &p, const double *recs, const int *ig,
                                                       const int *nn, const double *concs, const uint16_t *mats,
@@ -585,30 +612,54 @@ struct XsApp {
     const uint16_t *mrow = mats + mat * mx;
     const double *crow = concs + mat * mx;
     double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
-    if constexpr (GRID == XS_HASH && kU == 1) {
-      // software-pipelined: nuclide j+1's index entry is in flight while
-      // nuclide j's record pair is gathered (two deep spills: measured slower)
+    auto pf_pair = [&](int j, int lo) {
+      const double *q = recs + ((size_t)mrow[j] * n_gp + lo) * 6;
+      prefetch_l1(q);
+      prefetch_l1(q + 11);
+    };
+    if constexpr (GRID == XS_HASH) {
+      // bracket guess from the entry's quantized energies (XsHashEnt): a
+      // lower bound on upstream's bracket, exact unless two energies share a
+      // 2^-16 bin quantum; verified on the gathered pair, walked / searched
+      // with upstream's logic otherwise
+      const int pq = (int)((pe * (double)p.bins - (double)idx) * 65536.0);
       const size_t hs = (size_t)p.bins + 1;
       const XsHashEnt *hc = (const XsHashEnt *)ig + idx;
-      int4 hn = make_int4(0, 0, 0, 0);
-      if (nm > 0) hn = ld_(reinterpret_cast<const int4 *>(hc + (size_t)mrow[0] * hs));
+      auto ent = [&](int j) { return reinterpret_cast<const uint4 *>(hc + (size_t)mrow[j] * hs); };
+      auto guess = [&](const uint4 &h) {
+        return (int)(h.x & 0xffffu) + (pq > (int)(h.y & 0xffffu)) + (pq > (int)(h.y >> 16)) +
+               (pq > (int)(h.z & 0xffffu)) + (pq > (int)(h.z >> 16)) + (pq > (int)(h.w & 0xffffu)) +
+               (pq > (int)(h.w >> 16));
+      };
+      const uint4 z = make_uint4(0, 0, 0, 0);
+      uint4 e0 = nm > 0 ? ld_(ent(0)) : z, e1 = nm > 1 ? ld_(ent(1)) : z, e2 = nm > 2 ? ld_(ent(2)) : z;
+      for (int k = 3; k < 6 && k < nm; k++) prefetch_l1(ent(k));
+      if (nm > 0) pf_pair(0, guess(e0));
+      if (nm > 1) pf_pair(1, guess(e1));
       for (int j = 0; j < nm; j++) {
-        const int4 h = hn;
+        const uint4 h = e0;
+        e0 = e1;
+        e1 = e2;
+        if (j + 3 < nm) e2 = ld_(ent(j + 3));
+        if (j + 6 < nm) prefetch_l1(ent(j + 6));
+        if (j + 2 < nm) pf_pair(j + 2, guess(e1));
         const double *E = recs + (size_t)mrow[j] * n_gp * 6;
-        int lo = pe < __hiloint2double(h.w, h.z) ? h.x : h.x + 1;
-        const int uh = h.y;
+        int lo = guess(h);
+        const int u_low = (int)(h.x & 0xffffu), uh = (int)(h.x >> 16);
+        lo = lo < uh - 1 ? lo : uh - 1;
         const double2 *r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
         double2 a0 = ld_(r2 + 0), a1 = ld_(r2 + 1), a2 = ld_(r2 + 2);
         double2 b0 = ld_(r2 + 3), b1 = ld_(r2 + 4), b2 = ld_(r2 + 5);
-        if (j + 1 < nm) hn = ld_(reinterpret_cast<const int4 *>(hc + (size_t)mrow[j + 1] * hs));
-        while (pe >= b0.x && a0.x < pe && lo + 2 <= uh) {  // see the generic path below
+        // lo is upstream's bracket (grid_search on [u_low, u_high], edge
+        // cases excluded) iff E[lo] < pe < E[lo+1] and lo+1 <= u_high;
+        // walk forward while pe is past the pair (a quantum collision)
+        while (pe >= b0.x && a0.x < pe && lo + 2 <= uh) {
           lo++;
           r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
           a0 = b0; a1 = b1; a2 = b2;
           b0 = ld_(r2 + 3); b1 = ld_(r2 + 4); b2 = ld_(r2 + 5);
         }
         if (!(a0.x < pe && pe < b0.x && lo + 1 <= uh)) {  // edges: upstream logic
-          const int u_low = h.x;
           const double e_low = ld_(E + 6 * (size_t)u_low);
           const double e_high = ld_(E + 6 * (size_t)uh);
           int lower;
@@ -620,119 +671,33 @@ struct XsApp {
           a0 = ld_(r2 + 0); a1 = ld_(r2 + 1); a2 = ld_(r2 + 2);
           b0 = ld_(r2 + 3); b1 = ld_(r2 + 4); b2 = ld_(r2 + 5);
         }
-        const double conc = crow[j];
-        const double f = (b0.x - pe) / (b0.x - a0.x);
-        m0 += (b0.y - f * (b0.y - a0.y)) * conc;
-        m1 += (b1.x - f * (b1.x - a1.x)) * conc;
-        m2 += (b1.y - f * (b1.y - a1.y)) * conc;
-        m3 += (b2.x - f * (b2.x - a2.x)) * conc;
-        m4 += (b2.y - f * (b2.y - a2.y)) * conc;
+        accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
       }
-      m[0] = m0; m[1] = m1; m[2] = m2; m[3] = m3; m[4] = m4;
-      return;
-    }
-    if constexpr (GRID == XS_UNIONIZED && kU == 1) {  // same pipelining over the union row
+    } else if constexpr (GRID == XS_UNIONIZED) {
+      // the union row idx holds every nuclide's bracket (XS-7)
       const int *row = ig + (size_t)idx * n_iso;
-      int kn = nm > 0 ? ld_(row + mrow[0]) : 0;
+      auto bracket = [&](int k) { return k == n_gp - 1 ? k - 1 : k; };
+      int k0 = nm > 0 ? ld_(row + mrow[0]) : 0, k1 = nm > 1 ? ld_(row + mrow[1]) : 0;
+      if (nm > 0) pf_pair(0, bracket(k0));
       for (int j = 0; j < nm; j++) {
-        const int k = kn;
-        if (j + 1 < nm) kn = ld_(row + mrow[j + 1]);
-        const int lo = (k == n_gp - 1) ? k - 1 : k;
-        const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)mrow[j] * n_gp + lo) * 6);
+        const int k = k0;
+        k0 = k1;
+        if (j + 2 < nm) k1 = ld_(row + mrow[j + 2]);
+        if (j + 1 < nm) pf_pair(j + 1, bracket(k0));
+        const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)mrow[j] * n_gp + bracket(k)) * 6);
         const double2 a0 = ld_(r2 + 0), a1 = ld_(r2 + 1), a2 = ld_(r2 + 2);
         const double2 b0 = ld_(r2 + 3), b1 = ld_(r2 + 4), b2 = ld_(r2 + 5);
-        const double conc = crow[j];
-        const double f = (b0.x - pe) / (b0.x - a0.x);
-        m0 += (b0.y - f * (b0.y - a0.y)) * conc;
-        m1 += (b1.x - f * (b1.x - a1.x)) * conc;
-        m2 += (b1.y - f * (b1.y - a1.y)) * conc;
-        m3 += (b2.x - f * (b2.x - a2.x)) * conc;
-        m4 += (b2.y - f * (b2.y - a2.y)) * conc;
+        accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
       }
-      m[0] = m0; m[1] = m1; m[2] = m2; m[3] = m3; m[4] = m4;
-      return;
-    }
-    for (int j0 = 0; j0 < nm; j0 += kU) {
-      int nuc[kU], lo[kU], uh[kU];
-      bool on[kU];
-      double2 a0[kU], a1[kU], a2[kU], b0v[kU], b1[kU], b2[kU];
-#pragma unroll
-      for (int u = 0; u < kU; u++) {  // XS-7 step 1: index entries
-        on[u] = j0 + u < nm;
-        nuc[u] = on[u] ? mrow[j0 + u] : 0;
-        lo[u] = 0;
-        uh[u] = 0;
-        if (on[u]) {
-          if (GRID == XS_HASH) {
-            // {u_low, E[u_low+1]} and the next bin's u_low: the bracket is
-            // u_low if pe < E[u_low+1], else (usually) u_low+1 — verified
-            // against the loaded pair below
-            const XsHashEnt *he = (const XsHashEnt *)ig + (size_t)nuc[u] * (p.bins + 1) + idx;
-            const int4 h = ld_(reinterpret_cast<const int4 *>(he));
-            const double e_next = __hiloint2double(h.w, h.z);
-            uh[u] = h.y;
-            lo[u] = pe < e_next ? h.x : h.x + 1;
-          } else if (GRID == XS_UNIONIZED) {
-            const int k = ld_(ig + (size_t)idx * n_iso + nuc[u]);
-            lo[u] = (k == n_gp - 1) ? k - 1 : k;
-          } else {
-            const int k = gs_recs(recs + (size_t)nuc[u] * n_gp * 6, pe, 0, n_gp - 1);
-            lo[u] = (k == n_gp - 1) ? k - 1 : k;
-          }
-        }
-      }
-#pragma unroll
-      for (int u = 0; u < kU; u++) {  // step 2: record pair at lo (hash: at u_low)
-        if (on[u]) {
-          const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)nuc[u] * n_gp + lo[u]) * 6);
-          a0[u] = ld_(r2 + 0); a1[u] = ld_(r2 + 1); a2[u] = ld_(r2 + 2);
-          b0v[u] = ld_(r2 + 3); b1[u] = ld_(r2 + 4); b2[u] = ld_(r2 + 5);
-        }
-      }
-      if (GRID == XS_HASH) {
-#pragma unroll
-        for (int u = 0; u < kU; u++) {
-          // the guess lo is exactly upstream's bracket (grid_search on
-          // [u_low, u_high], its edge cases excluded) iff E[lo] < pe <
-          // E[lo+1] and lo+1 <= u_high; otherwise the full upstream logic
-          // walk forward while pe is past the pair (one gather per step;
-          // the guess is short by more than one record for ~1 in 8)
-          while (on[u] && pe >= b0v[u].x && a0[u].x < pe && lo[u] + 2 <= uh[u]) {
-            lo[u]++;
-            const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)nuc[u] * n_gp + lo[u]) * 6);
-            a0[u] = b0v[u]; a1[u] = b1[u]; a2[u] = b2[u];
-            b0v[u] = ld_(r2 + 3); b1[u] = ld_(r2 + 4); b2[u] = ld_(r2 + 5);
-          }
-          if (on[u] && !(a0[u].x < pe && pe < b0v[u].x && lo[u] + 1 <= uh[u])) {  // edges: upstream logic
-            const double *E = recs + (size_t)nuc[u] * n_gp * 6;
-            const XsHashEnt *he = (const XsHashEnt *)ig + (size_t)nuc[u] * (p.bins + 1) + idx;
-            const int u_low = ld_(&he->u_low);
-            const int u_high = uh[u];
-            const double e_low = ld_(E + 6 * (size_t)u_low);
-            const double e_high = ld_(E + 6 * (size_t)u_high);
-            int lower;
-            if (pe <= e_low) lower = 0;
-            else if (pe >= e_high) lower = n_gp - 1;
-            else lower = gs_recs(E, pe, u_low, u_high);
-            const int l2 = lower == n_gp - 1 ? lower - 1 : lower;
-            const double2 *r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)l2);
-            a0[u] = ld_(r2 + 0); a1[u] = ld_(r2 + 1); a2[u] = ld_(r2 + 2);
-            b0v[u] = ld_(r2 + 3); b1[u] = ld_(r2 + 4); b2[u] = ld_(r2 + 5);
-          }
-        }
-      }
-#pragma unroll
-      for (int u = 0; u < kU; u++) {  // XS-8, XS-9 in nuclide order
-        if (on[u]) {
-          const double conc = crow[j0 + u];
-          // low = {E, total, elastic, absorption, fission, nu_fission}
-          const double f = (b0v[u].x - pe) / (b0v[u].x - a0[u].x);
-          m0 += (b0v[u].y - f * (b0v[u].y - a0[u].y)) * conc;
-          m1 += (b1[u].x - f * (b1[u].x - a1[u].x)) * conc;
-          m2 += (b1[u].y - f * (b1[u].y - a1[u].y)) * conc;
-          m3 += (b2[u].x - f * (b2[u].x - a2[u].x)) * conc;
-          m4 += (b2[u].y - f * (b2[u].y - a2[u].y)) * conc;
-        }
+    } else {
+      // nuclide grid: binary search of each nuclide's energies (XS-7)
+      for (int j = 0; j < nm; j++) {
+        const double *E = recs + (size_t)mrow[j] * n_gp * 6;
+        const int k = gs_recs(E, pe, 0, n_gp - 1);
+        const double2 *r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)(k == n_gp - 1 ? k - 1 : k));
+        const double2 a0 = ld_(r2 + 0), a1 = ld_(r2 + 1), a2 = ld_(r2 + 2);
+        const double2 b0 = ld_(r2 + 3), b1 = ld_(r2 + 4), b2 = ld_(r2 + 5);
+        accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
       }
     }
     m[0] = m0;

@@ -290,6 +290,9 @@ __device__ inline double block_max_f64(Shared *sh, double v) {
 template <class T>
 __device__ __forceinline__ T ld_(const T *p) { return *p; }
 
+// bring the line holding p into L1 without holding registers
+__device__ __forceinline__ void prefetch_l1(const void *p) { asm volatile("prefetch.global.L1 [%0];" ::"l"(p)); }
+
 __device__ __forceinline__ uint64_t dbits(double d) { return (uint64_t)__double_as_longlong(d); }
 
 // team reductions: block reduction, then CTA partials gathered in rank 0's
