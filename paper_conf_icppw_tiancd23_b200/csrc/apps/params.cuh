@@ -182,12 +182,12 @@ struct XsLayout {
 // material / energy sort; results per lookup are unchanged): a warp's lanes
 // then take neighbouring energies of one material, so they gather the same
 // index entries and record pairs.  kb = energy-bucket bits per material
-// (~2 lookups per bucket).
+// (~8 lookups per bucket).
 constexpr long long kXsLkChunk = 1LL << 22;
 ENS_HD long long xs_lk_chunk(const XsParams &p) { return p.lookups < kXsLkChunk ? p.lookups : kXsLkChunk; }
 ENS_HD int xs_lk_bits(long long n_c) {
   int kb = 0;
-  while (kb < 18 && (12LL << kb) * 2 < n_c) kb++;
+  while (kb < 18 && (12LL << kb) * 8 < n_c) kb++;
   return kb;
 }
 // hash index entry (a private accelerator; results are unchanged): the
@@ -231,6 +231,12 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
   return L;
 }
 
+// hash lookups: nuclides gathered per step (independent loads and divisions
+// in flight per lane)
+#ifndef ENS_XS_STEP
+#define ENS_XS_STEP 2
+#endif
+constexpr int kXsStep = ENS_XS_STEP;
 // dynamic shared memory layout: material tables + the sort's bucket counters
 constexpr int kXsMaxT = 512;  // XsApp::kMaxT
 struct XsSmem {

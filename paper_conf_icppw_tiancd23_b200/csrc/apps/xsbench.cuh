@@ -631,35 +631,33 @@ struct XsApp {
                (pq > (int)(h.z & 0xffffu)) + (pq > (int)(h.z >> 16)) + (pq > (int)(h.w & 0xffffu)) +
                (pq > (int)(h.w >> 16));
       };
-      const uint4 z = make_uint4(0, 0, 0, 0);
-      uint4 e0 = nm > 0 ? ld_(ent(0)) : z, e1 = nm > 1 ? ld_(ent(1)) : z, e2 = nm > 2 ? ld_(ent(2)) : z;
-      for (int k = 3; k < 6 && k < nm; k++) prefetch_l1(ent(k));
-      if (nm > 0) pf_pair(0, guess(e0));
-      if (nm > 1) pf_pair(1, guess(e1));
-      for (int j = 0; j < nm; j++) {
-        const uint4 h = e0;
-        e0 = e1;
-        e1 = e2;
-        if (j + 3 < nm) e2 = ld_(ent(j + 3));
-        if (j + 6 < nm) prefetch_l1(ent(j + 6));
-        if (j + 2 < nm) pf_pair(j + 2, guess(e1));
-        const double *E = recs + (size_t)mrow[j] * n_gp * 6;
+      // nuclide j's record pair at the guessed bracket
+      auto gather = [&](int j, const uint4 &h, double2 &a0, double2 &a1, double2 &a2, double2 &b0, double2 &b1,
+                        double2 &b2) {
+        const int uh = (int)(h.x >> 16);
         int lo = guess(h);
-        const int u_low = (int)(h.x & 0xffffu), uh = (int)(h.x >> 16);
         lo = lo < uh - 1 ? lo : uh - 1;
-        const double2 *r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
-        double2 a0 = ld_(r2 + 0), a1 = ld_(r2 + 1), a2 = ld_(r2 + 2);
-        double2 b0 = ld_(r2 + 3), b1 = ld_(r2 + 4), b2 = ld_(r2 + 5);
-        // lo is upstream's bracket (grid_search on [u_low, u_high], edge
-        // cases excluded) iff E[lo] < pe < E[lo+1] and lo+1 <= u_high;
-        // walk forward while pe is past the pair (a quantum collision)
+        const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)mrow[j] * n_gp + lo) * 6);
+        a0 = ld_(r2 + 0); a1 = ld_(r2 + 1); a2 = ld_(r2 + 2);
+        b0 = ld_(r2 + 3); b1 = ld_(r2 + 4); b2 = ld_(r2 + 5);
+        return 0;
+      };
+      // lo is upstream's bracket (grid_search on [u_low, u_high], edge cases
+      // excluded) iff E[lo] < pe < E[lo+1] and lo+1 <= u_high; walk forward
+      // while pe is past the pair (a quantum collision), else upstream logic
+      auto gather_fix = [&](int j, const uint4 &h, double2 &a0, double2 &a1, double2 &a2, double2 &b0,
+                            double2 &b1, double2 &b2) {
+        const double *E = recs + (size_t)mrow[j] * n_gp * 6;
+        const int u_low = (int)(h.x & 0xffffu), uh = (int)(h.x >> 16);
+        int lo = guess(h);
+        lo = lo < uh - 1 ? lo : uh - 1;
         while (pe >= b0.x && a0.x < pe && lo + 2 <= uh) {
           lo++;
-          r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
+          const double2 *w2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
           a0 = b0; a1 = b1; a2 = b2;
-          b0 = ld_(r2 + 3); b1 = ld_(r2 + 4); b2 = ld_(r2 + 5);
+          b0 = ld_(w2 + 3); b1 = ld_(w2 + 4); b2 = ld_(w2 + 5);
         }
-        if (!(a0.x < pe && pe < b0.x && lo + 1 <= uh)) {  // edges: upstream logic
+        if (!(a0.x < pe && pe < b0.x && lo + 1 <= uh)) {
           const double e_low = ld_(E + 6 * (size_t)u_low);
           const double e_high = ld_(E + 6 * (size_t)uh);
           int lower;
@@ -667,11 +665,60 @@ struct XsApp {
           else if (pe >= e_high) lower = n_gp - 1;
           else lower = gs_recs(E, pe, u_low, uh);
           const int l2 = lower == n_gp - 1 ? lower - 1 : lower;
-          r2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)l2);
-          a0 = ld_(r2 + 0); a1 = ld_(r2 + 1); a2 = ld_(r2 + 2);
-          b0 = ld_(r2 + 3); b1 = ld_(r2 + 4); b2 = ld_(r2 + 5);
+          const double2 *w2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)l2);
+          a0 = ld_(w2 + 0); a1 = ld_(w2 + 1); a2 = ld_(w2 + 2);
+          b0 = ld_(w2 + 3); b1 = ld_(w2 + 4); b2 = ld_(w2 + 5);
         }
-        accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
+        return 0;
+      };
+      // kXsStep nuclides per step (independent gathers and divisions in
+      // flight), accumulated in list order
+      constexpr int U = kXsStep;
+      const uint4 z = make_uint4(0, 0, 0, 0);
+      uint4 cur[U], nxt[U];
+#pragma unroll
+      for (int u = 0; u < U; u++) {
+        cur[u] = u < nm ? ld_(ent(u)) : z;
+        nxt[u] = U + u < nm ? ld_(ent(U + u)) : z;
+      }
+      for (int k = 2 * U; k < 4 * U && k < nm; k++) prefetch_l1(ent(k));
+#pragma unroll
+      for (int u = 0; u < U; u++)
+        if (u < nm) pf_pair(u, guess(cur[u]));
+      int j = 0;
+      for (; j + U <= nm; j += U) {
+        uint4 h[U];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+          h[u] = cur[u];
+          cur[u] = nxt[u];
+          if (j + 2 * U + u < nm) nxt[u] = ld_(ent(j + 2 * U + u));
+          if (j + 4 * U + u < nm) prefetch_l1(ent(j + 4 * U + u));
+          if (j + U + u < nm) pf_pair(j + U + u, guess(cur[u]));
+        }
+        double2 A[U][6];
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+          auto fix = gather(j + u, h[u], A[u][0], A[u][1], A[u][2], A[u][3], A[u][4], A[u][5]);
+          (void)fix;
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+          auto fix = gather_fix(j + u, h[u], A[u][0], A[u][1], A[u][2], A[u][3], A[u][4], A[u][5]);
+          (void)fix;
+        }
+#pragma unroll
+        for (int u = 0; u < U; u++)
+          accumulate(pe, crow[j + u], A[u][0], A[u][1], A[u][2], A[u][3], A[u][4], A[u][5], m0, m1, m2, m3, m4);
+      }
+#pragma unroll
+      for (int u = 0; u < U - 1; u++) {  // tail
+        if (j + u < nm) {
+          double2 a0, a1, a2, b0, b1, b2;
+          gather(j + u, cur[u], a0, a1, a2, b0, b1, b2);
+          gather_fix(j + u, cur[u], a0, a1, a2, b0, b1, b2);
+          accumulate(pe, crow[j + u], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
+        }
       }
     } else if constexpr (GRID == XS_UNIONIZED) {
       // the union row idx holds every nuclide's bracket (XS-7)
@@ -814,7 +861,7 @@ struct XsApp {
     uint32_t *hist = (uint32_t *)(c.arena + L.lk_hist);
     const long long UB = xs_ubins(p);
     const XsSmem S = xs_smem(p, T);
-    uint32_t *mcnt = (uint32_t *)(c.smem + S.mcnt);  // [0..11] sampled counts, [16..28] material offsets
+    uint32_t *mcnt = (uint32_t *)(c.smem + S.mcnt);  // [16..28] material offsets of the chunk
     const double du = 1.0 / p.bins;
     const long long LC = xs_lk_chunk(p);
     const int kb = xs_lk_bits(LC);
@@ -824,7 +871,6 @@ struct XsApp {
     const Affine JG = lcg_pow(2ULL * (uint64_t)gs);
     unsigned long long ver = 0, bsum = 0;
     double fsum = 0.0, fabs_ = 0.0;
-    if (tid < 12) mcnt[tid] = 0;
     for (long long c0 = 0; c0 < nL; c0 += LC) {
       const long long nc = nL - c0 < LC ? nL - c0 : LC;
       for (long long b = g0; b <= NB; b += gs) hist[b] = 0u;
@@ -839,7 +885,6 @@ struct XsApp {
           long long eb = (long long)(pe * bscale);
           eb = eb > (1LL << kb) - 1 ? (1LL << kb) - 1 : eb;
           atomicAdd(&hist[((long long)mat << kb) + eb], 1u);
-          atomicAdd(&mcnt[mat], 1u);
         }
       }
       team_sync(c);
@@ -849,6 +894,7 @@ struct XsApp {
       if (tid < 12) mcnt[16 + tid] = ld_(hist + ((long long)tid << kb));
       if (tid == 12) mcnt[28] = (uint32_t)nc;
       team_sync(c);  // every CTA has its offsets before (C) moves the cursors
+      if (c.crank == 0 && tid < 12) c.sh->tallies[5 + tid] += mcnt[17 + tid] - mcnt[16 + tid];  // per material
       // (C) scatter energies to their buckets (hist becomes bucket ends)
       {
         uint64_t s = lcg_pow(2ULL * (uint64_t)(c0 + g0))(p.seed);
@@ -895,7 +941,6 @@ struct XsApp {
       team_sync(c);  // lk_pe / hist reused by the next chunk
       phase_mark(c, 11);
     }
-    if (tid < 12) c.sh->tallies[5 + tid] += mcnt[tid];  // lookups this CTA sampled, per material
     ver = team_sum_u64(c, ver);
     bsum = team_sum_u64(c, bsum);
     fsum = team_sum_f64(c, fsum);
