@@ -181,7 +181,7 @@ def workload_lines(name, world):
     raise SystemExit(f"unknown workload {name}")
 
 
-THREADS = {"C2": 1024, "TSTAR": 512, "C1": 256, "C3": 256, "C4": 1024, "C5": 512}
+THREADS = {"C2": 512, "TSTAR": 512, "C1": 256, "C3": 256, "C4": 1024, "C5": 512}
 
 
 def time_ours(lines, world, rank, threads, steps, warmup, torch, dist_on, team_ctas=0):

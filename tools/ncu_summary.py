@@ -1,0 +1,119 @@
+"""Turn ncu output into the summaries committed under profiles/.
+
+    python tools/ncu_summary.py launches <ncu --csv log> <out.json> "<command>"
+        per-launch device times of `ncu --metrics gpu__time_duration.sum
+        --clock-control none --csv ...` (cold-cache, serialised)
+    python tools/ncu_summary.py full <report.ncu-rep> <out.txt> [workload]
+        key counters of one `ncu --set full` capture + warp-stall samples by
+        source line; with a workload name, also writes profiles/traffic.json
+        (dram__bytes_read.sum + dram__bytes_write.sum per launch, read by
+        bench.py as roofline.traffic)
+"""
+import collections
+import csv
+import io
+import json
+import os
+import re
+import subprocess
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+KEYS = [
+    "gpu__time_duration.sum", "dram__bytes_read.sum", "dram__bytes_write.sum",
+    "dram__throughput.avg.pct_of_peak_sustained_elapsed", "l1tex__t_sector_hit_rate.pct",
+    "lts__t_sector_hit_rate.pct", "l1tex__t_sectors_pipe_lsu_mem_global_op_ld.sum",
+    "lts__t_sectors_srcunit_tex_op_read.sum", "lts__t_sectors_srcunit_tex_op_write.sum",
+    "smsp__inst_executed.sum", "smsp__issue_active.avg.pct_of_peak_sustained_active",
+    "sm__warps_active.avg.per_cycle_active", "launch__registers_per_thread",
+    "launch__shared_mem_per_block_dynamic", "launch__grid_size", "launch__block_size",
+    "sm__pipe_fp64_cycles_active.avg.pct_of_peak_sustained_active",
+    "l1tex__throughput.avg.pct_of_peak_sustained_active",
+    "smsp__pcsamp_warps_issue_stalled_long_scoreboard", "smsp__pcsamp_warps_issue_stalled_wait",
+    "smsp__pcsamp_warps_issue_stalled_barrier", "smsp__pcsamp_warps_issue_stalled_selected",
+]
+
+UNIT = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}
+
+
+def launches(log, out, command):
+    text = open(log).read()
+    start = text.find('"ID"')
+    rows = list(csv.reader(io.StringIO(text[start:])))
+    hdr = rows[0]
+    i_id, i_k, i_g, i_b, i_n, i_u, i_v = (hdr.index(k) for k in ("ID", "Kernel Name", "Grid Size", "Block Size",
+                                                                   "Metric Name", "Metric Unit", "Metric Value"))
+    res = []
+    for r in rows[1:]:
+        if len(r) <= i_v or r[i_n] != "gpu__time_duration.sum":
+            continue
+        v = float(r[i_v].replace(",", ""))
+        scale = {"ns": 1, "us": 1e3, "usecond": 1e3, "ms": 1e6, "msecond": 1e6, "s": 1e9, "second": 1e9,
+                 "nsecond": 1}.get(r[i_u], 1)
+        res.append({"id": int(r[i_id]), "kernel": r[i_k], "grid": r[i_g], "block": r[i_b], "ns": v * scale})
+    total = sum(x["ns"] for x in res) or 1.0
+    by = collections.Counter()
+    for x in res:
+        by[x["kernel"]] += x["ns"]
+    json.dump({"command": command, "note": "cold-cache serialised per-launch device times (ncu); compare shares, "
+                                           "not absolute times, with the bench line",
+               "share_by_kernel": {k: v / total for k, v in by.most_common()}, "launches": res},
+              open(out, "w"), indent=1)
+    print(f"{len(res)} launches -> {out}")
+
+
+def full(rep, out, workload=None):
+    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
+    rows = list(csv.reader(raw.splitlines()))
+    hdr, units, vals = rows[0], rows[1], rows[2]
+    d = {hdr[i]: (vals[i], units[i]) for i in range(len(hdr))}
+    lines = [f"kernel: {d.get('Kernel Name', ('?',))[0]}  grid {d.get('Grid Size', ('?',))[0]} "
+             f"block {d.get('Block Size', ('?',))[0]}", "", "key counters (one launch):"]
+    for k in KEYS:
+        if k in d:
+            lines.append(f"  {k:58s} {d[k][0]:>22s} {d[k][1]}")
+    src = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
+                         capture_output=True, text=True).stdout
+    agg, tot, text, cur, hdr2 = collections.Counter(), 0, {}, None, None
+    for r in csv.reader(src.splitlines()):
+        if len(r) == 2 and r[0] == "File Path":
+            cur = r[1].split("/")[-1]
+            continue
+        if r and r[0] == "Line No":
+            hdr2 = r
+            continue
+        if hdr2 and len(r) >= 5 and r[0].isdigit():
+            try:
+                x = int(r[4] or 0)
+            except ValueError:
+                continue
+            key = (cur, int(r[0]))
+            agg[key] += x
+            tot += x
+            text[key] = r[1].strip()[:90]
+    lines += ["", f"warp-stall samples by source line (top 30 of {tot}):"]
+    for key, x in agg.most_common(30):
+        lines.append(f"  {100.0 * x / max(tot, 1):5.1f}%  {key[0]}:{key[1]}  {text[key]}")
+    open(out, "w").write("\n".join(lines) + "\n")
+    print(f"-> {out}")
+    if workload:
+        tb = 0.0
+        for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+            v, u = d[k]
+            tb += float(v.replace(",", "")) * UNIT.get(u, 1)
+        tp = os.path.join(ROOT, "profiles", "traffic.json")
+        t = json.load(open(tp)) if os.path.exists(tp) else {}
+        t[workload] = tb
+        t[f"_source_{workload}"] = (f"ncu --set full, {os.path.relpath(out, ROOT)}: dram__bytes_read.sum + "
+                                    f"dram__bytes_write.sum of one launch")
+        t.pop("_source", None)
+        json.dump(t, open(tp, "w"), indent=1)
+        print(f"traffic[{workload}] = {tb:.4g} B -> {tp}")
+
+
+if __name__ == "__main__":
+    if sys.argv[1] == "launches":
+        launches(sys.argv[2], sys.argv[3], sys.argv[4] if len(sys.argv) > 4 else "")
+    else:
+        full(sys.argv[2], sys.argv[3], sys.argv[4] if len(sys.argv) > 4 else None)
