@@ -139,6 +139,9 @@ ENS_HD int xs_parse(int argc, const char *const *argv, XsParams &p) {
 }
 
 ENS_HD int xs_max_nucs(int n_iso) { return n_iso == 68 ? 34 : 321; }
+// unionized index grid row stride: n_iso padded to 4 ints, so that a row is
+// written as 16-B vectors (the padding is never read)
+ENS_HD int xs_iso_pad(int n_iso) { return (n_iso + 3) & ~3; }
 ENS_HD int pow2_ceil(int n) {
   int p = 1;
   while (p < n) p <<= 1;
@@ -149,8 +152,22 @@ ENS_HD int pow2_ceil(int n) {
 // [0,1)): unionized by energy alone (the union order; each nuclide's order
 // is its subsequence), otherwise by (nuclide, energy).  Power-of-two bucket
 // counts keep floor(E * nb) exact.
+// Small unionized problems keep the sort's bucket counters (and after the
+// sort, the sweep's chunk owner counts) in shared memory: kXsSmemBkt u32,
+// ~2 keys per bucket.  0 = counters in the arena.
+constexpr int kXsSmemBkt = 32768;
+ENS_HD long long xs_smem_nb(const XsParams &p) {
+  if (p.grid != XS_UNIONIZED) return 0;
+  const long long n_u = (long long)p.n_iso * p.n_gp;
+  const long long nch = (n_u + 511) / 512;  // kXsSweepRows
+  if (n_u > 4LL * kXsSmemBkt || nch * p.n_iso > kXsSmemBkt) return 0;
+  long long nb = 1;
+  while (nb * 2 <= n_u / 2 && nb < kXsSmemBkt) nb *= 2;
+  return nb;
+}
 ENS_HD long long xs_buckets(const XsParams &p) {
   const long long n_u = (long long)p.n_iso * p.n_gp;
+  if (xs_smem_nb(p)) return xs_smem_nb(p);
   if (p.grid == XS_UNIONIZED) return pow2_ceil((int)((n_u + 1) / 2));
   return (long long)p.n_iso * (pow2_ceil(p.n_gp) / 2 > 0 ? pow2_ceil(p.n_gp) / 2 : 1);
 }
@@ -171,7 +188,7 @@ struct XsLayout {
   uint64_t uenergy;   // unionized: [n_u] sorted union energies (u64 bits)
   uint64_t ufind;     // unionized: [xs_ubins] u32 union search table (private accelerator)
   uint64_t chist;     // unionized: [n_chunks][n_iso] u32 owner counts per sweep chunk
-  uint64_t index;     // unionized [n_u][n_iso] int32 / hash [n_iso][bins+1] XsHashEnt
+  uint64_t index;     // unionized [n_u][xs_iso_pad] int32 / hash [n_iso][bins+1] XsHashEnt
   uint64_t hcol;      // hash: [cs][bins+1] int32 column being built
   uint64_t lk_pe;     // event mode: [chunk] lookup energies sorted by (material, energy)
   uint64_t lk_hist;   // event mode: [(12 << kb) + 1] u32 (material, energy) bucket counts -> cursors
@@ -217,7 +234,7 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
     L.uenergy = o; o = align_up(o + n_u * 8, 256);
     L.ufind = o; o = align_up(o + (uint64_t)xs_ubins(p) * 4, 256);
     L.chist = o; o = align_up(o + nch * (uint64_t)p.n_iso * 4, 256);
-    L.index = o; o = align_up(o + n_u * (uint64_t)p.n_iso * 4, 256);
+    L.index = o; o = align_up(o + n_u * (uint64_t)xs_iso_pad(p.n_iso) * 4, 256);
   } else if (p.grid == XS_HASH) {
     L.index = o; o = align_up(o + (uint64_t)p.n_iso * (p.bins + 1) * 16, 256);
     L.hcol = o; o = align_up(o + (uint64_t)cs * (p.bins + 1) * 4, 256);
@@ -240,7 +257,7 @@ constexpr int kXsStep = ENS_XS_STEP;
 // dynamic shared memory layout: material tables + the sort's bucket counters
 constexpr int kXsMaxT = 512;  // XsApp::kMaxT
 struct XsSmem {
-  uint32_t thr, nn, mats, concs, mcnt, jmp, nbkt, total;
+  uint32_t thr, nn, mats, concs, mcnt, jmp, nbkt, ubkt, total;
 };
 // T = the block size the instance runs with
 ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
@@ -253,9 +270,11 @@ ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   S.mats = o; o += (uint32_t)align_up(12 * mx * 2, 16);  // nuclide ids (u16)
   S.mcnt = o; o += 32 * 4;                // material counts / offsets of a lookup chunk
   S.jmp = o; o += 4 * 64 * 16;            // LCG jump tables: A^(6 d 64^l), l < 4, d < 64
-  S.nbkt = o;                             // per-nuclide sort buckets (hash / nuclide grids)
+  S.nbkt = o;  // per-nuclide sort buckets (hash / nuclide grids); unionized: per-warp sweep rows
   if (p.grid != XS_UNIONIZED) o += (uint32_t)align_up((uint64_t)xs_nbn(p.n_gp) * 4, 16);
-  (void)T;
+  else o += (uint32_t)(T / 32) * 2u * (uint32_t)xs_iso_pad(p.n_iso) * 4u;
+  S.ubkt = o;  // unionized, small: bucket counters, then chunk owner counts
+  if (xs_smem_nb(p)) o += (uint32_t)kXsSmemBkt * 4u;
   S.total = o;
   return S;
 }

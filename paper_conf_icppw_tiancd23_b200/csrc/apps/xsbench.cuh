@@ -286,44 +286,45 @@ struct XsApp {
     }
   }
 
-  // Unionized index grid sweep: a warp per chunk of union rows, lane l owns
-  // nuclides l, l+32, ... (NM = ceil(n_iso/32) of them, counts in registers);
-  // row e is ig[e][i] = clip(cnt_i(e) - 1, 0, n_gp-2) with cnt_i(e) =
-  // #{k: E_i[k] <= u_e}, and the owner's count before its increment is the
-  // sorted position of that record (stored in keys[e].pad).  Branch-free.
-  template <int NM>
-  __device__ static __forceinline__ void sweep(XsKey *keys, const uint32_t *chist, int *ig, long long n_u, int n_iso,
-                                               int n_gp, long long nch) {
+  // Unionized index grid sweep: a warp per chunk of union rows, the chunk's
+  // current row in the warp's shared memory: counts cnt_i(e) = #{k: E_i[k]
+  // <= u_e} and row values clip(cnt_i(e) - 1, 0, n_gp-2).  Each union row
+  // changes exactly one count (its owner's): the owner's lane updates it,
+  // then the warp copies the row out as 16-B vectors.  The owner's count
+  // before its increment is the sorted position of that record (stored in
+  // keys[e].pad).
+  __device__ static __forceinline__ void sweep(XsKey *keys, const uint32_t *chist, int *ig, int *sw, long long n_u,
+                                               int n_iso, int n_gp, long long nch) {
     const int tid = threadIdx.x, T = blockDim.x, lane = tid & 31, warp = tid >> 5, nw = T >> 5;
+    const int ip = xs_iso_pad(n_iso), ng4 = ip >> 2;
+    int *cnt = sw + (size_t)warp * 2 * ip, *val = cnt + ip;
+    auto clip = [&](int c) { const int v = c - 1; return v < 0 ? 0 : (v > n_gp - 2 ? n_gp - 2 : v); };
     for (long long ch = warp; ch < nch; ch += nw) {
       const long long e0 = ch * kXsSweepRows, e1 = (e0 + kXsSweepRows < n_u) ? e0 + kXsSweepRows : n_u;
-      int cnt[NM];
-#pragma unroll
-      for (int m = 0; m < NM; m++) {
-        const int i = lane + 32 * m;
-        cnt[m] = i < n_iso ? (int)chist[ch * n_iso + i] : 0;
+      for (int i = lane; i < ip; i += 32) {
+        const int c = i < n_iso ? (int)chist[ch * n_iso + i] : 0;
+        cnt[i] = c;
+        val[i] = clip(c);
       }
-      // owners of the next 32 rows are prefetched while this group is swept
-      int own_next = e0 + lane < e1 ? (int)(keys[e0 + lane].idx / (unsigned)n_gp) : -1;
+      __syncwarp();
+      // record ids of the next 32 rows are prefetched while this group is swept
+      unsigned id_next = e0 + lane < e1 ? keys[e0 + lane].idx : 0u;
       for (long long g = e0; g < e1; g += 32) {
-        const int own_cur = own_next;
-        own_next = g + 32 + lane < e1 ? (int)(keys[g + 32 + lane].idx / (unsigned)n_gp) : -1;
+        const int own_cur = (int)(id_next / (unsigned)n_gp);
+        id_next = g + 32 + lane < e1 ? keys[g + 32 + lane].idx : 0u;
         const int ng = (int)(e1 - g < 32 ? e1 - g : 32);
-        int *row = ig + (size_t)g * n_iso;
-        for (int sl = 0; sl < ng; sl++, row += n_iso) {
-          const int own = __shfl_sync(0xffffffffu, own_cur, sl);
-          int pos = -1;
-#pragma unroll
-          for (int m = 0; m < NM; m++) {
-            const int i = lane + 32 * m;
-            const int hit = own == i;
-            pos = hit ? i * n_gp + cnt[m] : pos;
-            cnt[m] += hit;
-            const int v = cnt[m] - 1;
-            if (i < n_iso) row[i] = v < 0 ? 0 : (v > n_gp - 2 ? n_gp - 2 : v);
+        int4 *row = reinterpret_cast<int4 *>(ig + (size_t)g * ip);
+        for (int sl = 0; sl < ng; sl++, row += ng4) {
+          if (lane == sl) {  // the row's owner
+            const int c = cnt[own_cur];
+            cnt[own_cur] = c + 1;
+            val[own_cur] = clip(c + 1);
+            keys[g + sl].pad = (unsigned)(own_cur * n_gp + c);
           }
-          if (pos >= 0) keys[g + sl].pad = (unsigned)pos;
+          __syncwarp();
+          for (int q = lane; q < ng4; q += 32) row[q] = reinterpret_cast<const int4 *>(val)[q];
         }
+        __syncwarp();
       }
     }
   }
@@ -472,9 +473,10 @@ struct XsApp {
     const Affine *jt = (const Affine *)(c.smem + S.jmp);
     double *recs = (double *)(c.arena + L.recs);
     XsKey *keys = (XsKey *)(c.arena + L.keys);
-    uint32_t *bkt = (uint32_t *)(c.arena + L.bkt);
+    const bool sm_bkt = xs_smem_nb(p) != 0;
+    uint32_t *bkt = sm_bkt ? (uint32_t *)(c.smem + S.ubkt) : (uint32_t *)(c.arena + L.bkt);
     int *ig = (int *)(c.arena + L.index);
-    const Affine J6T = lcg_pow(6ULL * T), J24T = lcg_pow(24ULL * T);
+    const Affine J6T = lcg_pow(6ULL * T);
 
     for (long long b = tid; b < NB; b += T) bkt[b] = 0;
     __syncthreads();
@@ -491,29 +493,33 @@ struct XsApp {
     // (S) bucket offsets
     global_exclusive_scan(bkt, NB, c.sh);
     XS_STOP(2);
-    // (P) scatter, energies re-drawn, 4 independent atomics in flight
+    // (P) scatter, energies re-drawn, kQ independent atomics in flight (the
+    // returned cursor is an L2 round trip)
     {
+      constexpr int kQ = 8;
+      const Affine JQT = lcg_pow(6ULL * kQ * T);
       uint64_t s = lcg_pow(6ULL * tid)(p.gseed);
-      for (long long r0 = tid; r0 < n_u; r0 += 4LL * T, s = J24T(s)) {
-        double e[4];
-        uint32_t pos[4];
+      for (long long r0 = tid; r0 < n_u; r0 += (long long)kQ * T, s = JQT(s)) {
+        unsigned long long eb[kQ];
+        uint32_t pos[kQ];
         uint64_t sq = s;
 #pragma unroll
-        for (int q = 0; q < 4; q++, sq = J6T(sq)) {
+        for (int q = 0; q < kQ; q++, sq = J6T(sq)) {
           uint64_t t = sq;
-          e[q] = lcg_double(t);
+          eb[q] = dbits(lcg_double(t));
         }
 #pragma unroll
-        for (int q = 0; q < 4; q++) {
+        for (int q = 0; q < kQ; q++) {
           const long long r = r0 + (long long)q * T;
-          if (r < n_u) pos[q] = atomicAdd(&bkt[bucket_of(e[q], r, n_gp, true, NB, nbn)], 1u);
+          if (r < n_u)
+            pos[q] = atomicAdd(&bkt[bucket_of(__longlong_as_double((long long)eb[q]), r, n_gp, true, NB, nbn)], 1u);
         }
 #pragma unroll
-        for (int q = 0; q < 4; q++) {
+        for (int q = 0; q < kQ; q++) {
           const long long r = r0 + (long long)q * T;
           if (r < n_u) {
             XsKey k;
-            k.key = dbits(e[q]);
+            k.key = eb[q];
             k.idx = (unsigned)r;
             k.pad = 0;
             keys[pos[q]] = k;
@@ -530,27 +536,29 @@ struct XsApp {
 
     // (U) keys[] is the union (XS-5); owner = record id / n_gp
     uint64_t *uA = (uint64_t *)(c.arena + L.uenergy);
-    uint32_t *chist = (uint32_t *)(c.arena + L.chist);
+    uint32_t *chist = sm_bkt ? bkt : (uint32_t *)(c.arena + L.chist);  // the sort's counters are dead
     const long long nch = (n_u + kXsSweepRows - 1) / kXsSweepRows;
     uint32_t *uf = (uint32_t *)(c.arena + L.ufind);
     const long long UB = xs_ubins(p);
     for (long long x = tid; x < nch * n_iso; x += T) chist[x] = 0;
-    for (long long b = tid; b < UB; b += T) uf[b] = 0;
     __syncthreads();
     XS_STOP(5);
-    for (long long e = tid; e < n_u; e += T) {  // union energies, chunk owner counts,
-      const XsKey k = keys[e];                   // search-table histogram
-      uA[e] = k.key;
+    // first bin b with u <= b / UB (UB a power of two: exact)
+    auto bfirst = [&](unsigned long long bits) {
+      const double x = __longlong_as_double((long long)bits) * (double)UB;
+      long long bk = (long long)x;
+      if ((double)bk < x) bk++;
+      return bk < UB ? bk : UB;
+    };
+    for (long long e = tid; e < n_u; e += T) {  // union energies, chunk owner counts, search table:
+      const XsKey k = keys[e];                   // ufind[b] = #{k >= 1 : u_k <= b / UB} = e on
+      uA[e] = k.key;                             // [b_e, b_e+1) (b_0 := 0, b_n_u := UB)
       atomicAdd(&chist[(e / kXsSweepRows) * n_iso + k.idx / n_gp], 1u);
-      if (e >= 1) {  // first bin b with u_e <= b / UB (UB a power of two: exact)
-        const double x = __longlong_as_double((long long)k.key) * (double)UB;
-        long long bk = (long long)x;
-        if ((double)bk < x) bk++;
-        if (bk < UB) atomicAdd(&uf[bk], 1u);
-      }
+      const long long lo = e == 0 ? 0 : bfirst(k.key);
+      const long long hi = e + 1 < n_u ? bfirst(keys[e + 1].key) : UB;
+      for (long long b = lo; b < hi; b++) uf[b] = (uint32_t)e;
     }
     __syncthreads();
-    global_exclusive_scan<true>(uf, UB, c.sh);  // ufind[b] = #{k >= 1 : u_k <= b / UB}
     for (int i = tid; i < n_iso; i += T) {  // exclusive scan over chunks per owner
       uint32_t run = 0;
       for (long long ch = 0; ch < nch; ch++) {
@@ -564,8 +572,7 @@ struct XsApp {
     // (W) sweep: a warp per chunk, lanes own nuclides; row e of the index grid
     // is clip(#{k>=1: E_i[k] <= u_e}, 0, n_gp-2) = clip(cnt_i(e) - 1, ...),
     // and the owner's new count is the sorted position of that record (XS-4).
-    if (n_iso <= 96) sweep<3>(keys, chist, ig, n_u, n_iso, n_gp, nch);
-    else sweep<12>(keys, chist, ig, n_u, n_iso, n_gp, nch);
+    sweep(keys, chist, ig, (int *)(c.smem + S.nbkt), n_u, n_iso, n_gp, nch);
     __syncthreads();
     XS_STOP(7);
     // (R) records to their sorted positions, keys read coalesced
@@ -722,7 +729,7 @@ struct XsApp {
       }
     } else if constexpr (GRID == XS_UNIONIZED) {
       // the union row idx holds every nuclide's bracket (XS-7)
-      const int *row = ig + (size_t)idx * n_iso;
+      const int *row = ig + (size_t)idx * xs_iso_pad(n_iso);
       auto bracket = [&](int k) { return k == n_gp - 1 ? k - 1 : k; };
       int k0 = nm > 0 ? ld_(row + mrow[0]) : 0, k1 = nm > 1 ? ld_(row + mrow[1]) : 0;
       if (nm > 0) pf_pair(0, bracket(k0));
