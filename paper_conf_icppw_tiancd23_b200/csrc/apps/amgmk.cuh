@@ -33,7 +33,7 @@ struct AmgApp {
     }
     const AmgLayout L = amg_layout(p);
     if (L.total > c.arena_cap) {
-      if (threadIdx.x == 0) c.sh->flags |= 2u;
+      if (threadIdx.x == 0) ens_sh(c)->flags |= 2u;
       R.exit_code = ENS_EXIT_NOMEM;
       return R;
     }
@@ -125,10 +125,10 @@ struct AmgApp {
       const double e = fabs(v - (p.kind == 0 ? 1.0 : ld_(f + r)));
       if (e > mxe) mxe = e;
     }
-    bsum = block_sum_u64(c.sh, bsum);
-    fsum = block_sum_f64(c.sh, fsum);
-    fabs_ = block_sum_f64(c.sh, fabs_);
-    mxe = block_max_f64(c.sh, mxe);
+    bsum = block_sum_u64(ens_sh(c), bsum);
+    fsum = block_sum_f64(ens_sh(c), fsum);
+    fabs_ = block_sum_f64(ens_sh(c), fabs_);
+    mxe = block_max_f64(ens_sh(c), mxe);
     R.vhash = bsum % 999983ULL;
     R.bitsum = bsum;
     R.fsum = fsum;

@@ -37,7 +37,7 @@ struct PrApp {
     }
     const PrLayout L = pr_layout(p);
     if (L.total > c.arena_cap) {
-      if (threadIdx.x == 0) c.sh->flags |= 2u;
+      if (threadIdx.x == 0) ens_sh(c)->flags |= 2u;
       R.exit_code = ENS_EXIT_NOMEM;
       return R;
     }
@@ -70,7 +70,7 @@ struct PrApp {
       }
     }
     sub_sync();
-    global_exclusive_scan(dst, n + 1, c.sh);  // dst[u] = first edge of u; dst[n] = edges
+    global_exclusive_scan(dst, n + 1, ens_sh(c));  // dst[u] = first edge of u; dst[n] = edges
     const long long E = dst[n];
     // ---- PR-2: targets, source by source (draw n + e + 1 for edge e) --------
     for (long long u = tid; u < n; u += T) {
@@ -85,7 +85,7 @@ struct PrApp {
       }
     }
     sub_sync();
-    global_exclusive_scan(iptr, n + 1, c.sh);  // in-edge offsets
+    global_exclusive_scan(iptr, n + 1, ens_sh(c));  // in-edge offsets
     for (long long v = tid; v < n; v += T) cur[v] = iptr[v];
     sub_sync();
     for (long long e = tid; e < E; e += T) ine[atomicAdd(&cur[tgt[e]], 1u)] = (uint32_t)e;
@@ -135,28 +135,28 @@ struct PrApp {
         top = v;
       }
     }
-    bsum = block_sum_u64(c.sh, bsum);
-    fsum = block_sum_f64(c.sh, fsum);
-    fabs_ = block_sum_f64(c.sh, fabs_);
-    const double bmax = block_max_f64(c.sh, best);
+    bsum = block_sum_u64(ens_sh(c), bsum);
+    fsum = block_sum_f64(ens_sh(c), fsum);
+    fabs_ = block_sum_f64(ens_sh(c), fabs_);
+    const double bmax = block_max_f64(ens_sh(c), best);
     unsigned long long cand = (best == bmax) ? (unsigned long long)top : ~0ULL;
     for (int o = 16; o; o >>= 1) {
       const unsigned long long w = __shfl_xor_sync(0xffffffffu, cand, o);
       cand = w < cand ? w : cand;
     }
     sub_sync();
-    if ((tid & 31) == 0) c.sh->red_u[tid >> 5] = cand;
+    if ((tid & 31) == 0) ens_sh(c)->red_u[tid >> 5] = cand;
     sub_sync();
     if (tid < 32) {
-      unsigned long long m = tid < (T >> 5) ? c.sh->red_u[tid] : ~0ULL;
+      unsigned long long m = tid < (T >> 5) ? ens_sh(c)->red_u[tid] : ~0ULL;
       for (int o = 16; o; o >>= 1) {
         const unsigned long long w = __shfl_xor_sync(0xffffffffu, m, o);
         m = w < m ? w : m;
       }
-      if (tid == 0) c.sh->red_u[0] = m;
+      if (tid == 0) ens_sh(c)->red_u[0] = m;
     }
     sub_sync();
-    const long long topv = (long long)c.sh->red_u[0];
+    const long long topv = (long long)ens_sh(c)->red_u[0];
     R.vhash = bsum % 999983ULL;
     R.bitsum = bsum;
     R.fsum = fsum;

@@ -180,6 +180,29 @@ ENS_HD long long xs_ubins(const XsParams &p) { return pow2_ceil((int)(((long lon
 // union-sweep chunks (rows per chunk) for the index grid
 constexpr int kXsSweepRows = 512;
 
+// Unionized init, warp path (n_gp <= kXsWarpGp): a warp sorts one nuclide at
+// a time in its own shared memory and writes the nuclide's records, its
+// sorted energies and, per union value chunk, how many of its energies lie
+// below the chunk; then a warp per value chunk [ch/NC, (ch+1)/NC) gathers the
+// chunk's energies from the sorted runs, sorts them in shared memory and
+// writes the union energies, the search table and the index rows of the
+// chunk.  NC = ubins / kXsBinsPerChunk (powers of two: chunk and bin bounds
+// are exact), so a chunk holds 64..128 union energies on average; one that
+// exceeds kXsChunkCap (never seen: ~10 sigma) sends the instance to the
+// block-wide path.
+constexpr int kXsWarpGp = 1024;
+constexpr int kXsNucBkt = 512;  // per-nuclide sort buckets
+constexpr uint32_t kXsNucScr = kXsWarpGp * 6 + kXsNucBkt * 4;  // bytes per warp: u32 keys, u16 j, counters
+constexpr int kXsBinsPerChunk = 64;   // search-table bins per union chunk
+constexpr int kXsChunkCap = 256;      // union energies a warp sorts at once
+constexpr int kXsChunkFb = 256;       // fine sort buckets per union chunk
+constexpr uint32_t kXsUniScr = kXsChunkCap * 20 + kXsChunkFb * 4;  // bytes per chunk warp
+ENS_HD bool xs_warp_union(const XsParams &p) { return p.grid == XS_UNIONIZED && p.n_gp <= kXsWarpGp; }
+ENS_HD long long xs_uchunks(const XsParams &p) {
+  const long long ub = xs_ubins(p);
+  return ub > kXsBinsPerChunk ? ub / kXsBinsPerChunk : 1;
+}
+
 // arena layout (byte offsets, 256-B aligned)
 struct XsLayout {
   uint64_t recs;      // [n_iso][n_gp] x 48 B records, sorted per nuclide
@@ -188,6 +211,7 @@ struct XsLayout {
   uint64_t uenergy;   // unionized: [n_u] sorted union energies (u64 bits)
   uint64_t ufind;     // unionized: [xs_ubins] u32 union search table (private accelerator)
   uint64_t chist;     // unionized: [n_chunks][n_iso] u32 owner counts per sweep chunk
+  uint64_t ustart;    // unionized, warp path: [NC+1][iso_pad] i32 #{k: E_i[k] < ch/NC}
   uint64_t index;     // unionized [n_u][xs_iso_pad] int32 / hash [n_iso][bins+1] XsHashEnt
   uint64_t hcol;      // hash: [cs][bins+1] int32 column being built
   uint64_t lk_pe;     // event mode: [chunk] lookup energies sorted by (material, energy)
@@ -234,6 +258,7 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
     L.uenergy = o; o = align_up(o + n_u * 8, 256);
     L.ufind = o; o = align_up(o + (uint64_t)xs_ubins(p) * 4, 256);
     L.chist = o; o = align_up(o + nch * (uint64_t)p.n_iso * 4, 256);
+    if (xs_warp_union(p)) { L.ustart = o; o = align_up(o + (uint64_t)xs_iso_pad(p.n_iso) * (xs_uchunks(p) + 1) * 4, 256); }
     L.index = o; o = align_up(o + n_u * (uint64_t)xs_iso_pad(p.n_iso) * 4, 256);
   } else if (p.grid == XS_HASH) {
     L.index = o; o = align_up(o + (uint64_t)p.n_iso * (p.bins + 1) * 16, 256);
@@ -275,6 +300,11 @@ ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   else o += (uint32_t)(T / 32) * 2u * (uint32_t)xs_iso_pad(p.n_iso) * 4u;
   S.ubkt = o;  // unionized, small: bucket counters, then chunk owner counts
   if (xs_smem_nb(p)) o += (uint32_t)kXsSmemBkt * 4u;
+  // unionized warp path: kXsWarpScr per warp, overlaying nbkt / ubkt
+  if (xs_warp_union(p)) {
+    const uint32_t need = (uint32_t)(T / 32) * (kXsNucScr > kXsUniScr ? kXsNucScr : kXsUniScr);
+    if (S.nbkt + need > o) o = S.nbkt + need;
+  }
   S.total = o;
   return S;
 }

@@ -167,21 +167,21 @@ struct XsApp {
     }
     const XsLayout L = xs_layout(p, c.csize);
     if (L.total > c.arena_cap) {
-      if (threadIdx.x == 0) c.sh->flags |= 2u;  // ENS_RF_NOMEM
+      if (threadIdx.x == 0) ens_sh(c)->flags |= 2u;  // ENS_RF_NOMEM
       R.exit_code = ENS_EXIT_NOMEM;
       return R;
     }
     const int n_iso = p.n_iso, mx = xs_max_nucs(n_iso);
     const XsSmem S = xs_smem(p, blockDim.x);
-    double *thr = (double *)(c.smem + S.thr);
-    int *nn = (int *)(c.smem + S.nn);
-    double *concs = (double *)(c.smem + S.concs);
-    uint16_t *mats = (uint16_t *)(c.smem + S.mats);
+    double *thr = (double *)(ens_smem(c) + S.thr);
+    int *nn = (int *)(ens_smem(c) + S.nn);
+    double *concs = (double *)(ens_smem(c) + S.concs);
+    uint16_t *mats = (uint16_t *)(ens_smem(c) + S.mats);
 
     // ---- XS-2: materials, concentrations ---------------------------------
     hm_tables(n_iso, mx, thr, nn, concs, mats);
     {  // LCG jump tables for XS-3's record draws (see jump6)
-      Affine *jt = (Affine *)(c.smem + S.jmp);
+      Affine *jt = (Affine *)(ens_smem(c) + S.jmp);
       for (int x = threadIdx.x; x < 256; x += blockDim.x)
         jt[x] = lcg_pow((6ULL * (uint64_t)(x & 63)) << (6 * (x >> 6)));
     }
@@ -189,7 +189,8 @@ struct XsApp {
     hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
     phase_mark(c, 0);
     if (p.grid == XS_UNIONIZED) {
-      if (c.crank == 0) init(c, p, L, S);  // one CTA builds the union
+      if (c.crank == 0 && !(xs_warp_union(p) && init_warp(c, p, L, S)))
+        init(c, p, L, S);  // one CTA builds the union
     } else {
       init_nuc(c, p, L, S);  // nuclides striped over the team's CTAs
     }
@@ -341,8 +342,8 @@ struct XsApp {
     const int tid = threadIdx.x, T = blockDim.x;
     const int n_iso = p.n_iso, n_gp = p.n_gp;
     const int nbn = xs_nbn(n_gp);
-    uint32_t *nb = (uint32_t *)(c.smem + S.nbkt);
-    const Affine *jt = (const Affine *)(c.smem + S.jmp);
+    uint32_t *nb = (uint32_t *)(ens_smem(c) + S.nbkt);
+    const Affine *jt = (const Affine *)(ens_smem(c) + S.jmp);
     double *recs = (double *)(c.arena + L.recs);
     XsKey *keys = (XsKey *)(c.arena + L.keys);
     int *ig = (int *)(c.arena + L.index);
@@ -368,7 +369,7 @@ struct XsApp {
       }
       __syncthreads();
       phase_mark(c, 1);
-      global_exclusive_scan(nb, nbn, c.sh);
+      global_exclusive_scan(nb, nbn, ens_sh(c));
       phase_mark(c, 2);
       {  // scatter {energy, j}, the energies re-drawn, four atomics in flight
         uint64_t s = jump6(jt, r0 + (uint32_t)tid, p.gseed);
@@ -425,7 +426,7 @@ struct XsApp {
       __syncthreads();
       phase_mark(c, 8);
       if (hash) {
-        global_exclusive_scan<true>((uint32_t *)col, p.bins, c.sh);
+        global_exclusive_scan<true>((uint32_t *)col, p.bins, ens_sh(c));
         for (int b = tid; b < p.bins; b += T) {
           const int v = col[b];
           if (v > n_gp - 2) col[b] = n_gp - 2;
@@ -470,11 +471,11 @@ struct XsApp {
     const long long n_u = (long long)n_iso * n_gp;
     const long long NB = xs_buckets(p);
     const int nbn = xs_nbn(n_gp);
-    const Affine *jt = (const Affine *)(c.smem + S.jmp);
+    const Affine *jt = (const Affine *)(ens_smem(c) + S.jmp);
     double *recs = (double *)(c.arena + L.recs);
     XsKey *keys = (XsKey *)(c.arena + L.keys);
     const bool sm_bkt = xs_smem_nb(p) != 0;
-    uint32_t *bkt = sm_bkt ? (uint32_t *)(c.smem + S.ubkt) : (uint32_t *)(c.arena + L.bkt);
+    uint32_t *bkt = sm_bkt ? (uint32_t *)(ens_smem(c) + S.ubkt) : (uint32_t *)(c.arena + L.bkt);
     int *ig = (int *)(c.arena + L.index);
     const Affine J6T = lcg_pow(6ULL * T);
 
@@ -491,7 +492,7 @@ struct XsApp {
     __syncthreads();
     XS_STOP(1);
     // (S) bucket offsets
-    global_exclusive_scan(bkt, NB, c.sh);
+    global_exclusive_scan(bkt, NB, ens_sh(c));
     XS_STOP(2);
     // (P) scatter, energies re-drawn, kQ independent atomics in flight (the
     // returned cursor is an L2 round trip)
@@ -572,7 +573,7 @@ struct XsApp {
     // (W) sweep: a warp per chunk, lanes own nuclides; row e of the index grid
     // is clip(#{k>=1: E_i[k] <= u_e}, 0, n_gp-2) = clip(cnt_i(e) - 1, ...),
     // and the owner's new count is the sorted position of that record (XS-4).
-    sweep(keys, chist, ig, (int *)(c.smem + S.nbkt), n_u, n_iso, n_gp, nch);
+    sweep(keys, chist, ig, (int *)(ens_smem(c) + S.nbkt), n_u, n_iso, n_gp, nch);
     __syncthreads();
     XS_STOP(7);
     // (R) records to their sorted positions, keys read coalesced
@@ -587,6 +588,369 @@ struct XsApp {
     }
     __syncthreads();
     phase_mark(c, 8);
+  }
+
+  // ---- XS-3/4/5, unionized grid, warp path (n_gp <= kXsWarpGp) -----------
+  // (N) a warp per nuclide, in its own shared memory: energies (draw 6r+1 of
+  // record r = i*n_gp + j, XS-3) are bucket-sorted by (energy, j) (XS-4),
+  // each record is written once at its sorted position (coalesced; its five
+  // cross sections re-drawn through the jump tables), the sorted energies go
+  // to `ecmp` and ustart[i][ch] = #{k: chunk(E_i[k]) < ch} marks where each
+  // union value chunk begins in the nuclide's run.  (U) a warp per chunk
+  // gathers the chunk's energies from the n_iso runs, sorts them by (energy,
+  // nuclide) — the union order of the block-wide sort (reading Q13) — and
+  // writes the union energies, the chunk's search-table bins and the chunk's
+  // index rows (the nuclides' counts start at ustart[.][ch] and one count
+  // steps per row: lanes hold the counts of four nuclides each in registers
+  // and store a row as 16-B vectors).  Returns false if a chunk held more
+  // than kXsChunkCap energies (the caller then runs the block-wide path).
+  __device__ static __forceinline__ int nuc_bkt(double e) {
+    const int b = (int)(e * (double)kXsNucBkt);
+    return b < kXsNucBkt - 1 ? b : kXsNucBkt - 1;
+  }
+  __device__ static __forceinline__ long long uchunk(double e, long long NC) {
+    const long long ch = (long long)(e * (double)NC);
+    return ch < NC - 1 ? ch : NC - 1;
+  }
+  __device__ static __forceinline__ int chunk_fb(double e, long long ch, long long NC) {
+    const int b = (int)((e * (double)NC - (double)ch) * (double)kXsChunkFb);
+    return b < 0 ? 0 : (b < kXsChunkFb - 1 ? b : kXsChunkFb - 1);
+  }
+  // exclusive prefix sum of cnt[0..N) (shared), by one warp, N = 32 * V
+  template <int V>
+  __device__ static __forceinline__ void warp_scan_smem(uint32_t *cnt, int lane) {
+    uint32_t v[V], sum = 0;
+#pragma unroll
+    for (int q = 0; q < V; q++) {
+      v[q] = cnt[lane * V + q];
+      sum += v[q];
+    }
+    uint32_t inc = sum;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      const uint32_t t = __shfl_up_sync(0xffffffffu, inc, o);
+      if (lane >= o) inc += t;
+    }
+    uint32_t run = inc - sum;
+#pragma unroll
+    for (int q = 0; q < V; q++) {
+      cnt[lane * V + q] = run;
+      run += v[q];
+    }
+  }
+  // insertion sort of (E bits, tag) pairs in [lo, hi) (shared memory)
+  __device__ static __forceinline__ void isort_pairs(unsigned long long *E, uint16_t *t, int lo, int hi) {
+    for (int x = lo + 1; x < hi; x++) {
+      const unsigned long long ve = E[x];
+      const uint16_t vt = t[x];
+      int y = x - 1;
+      while (y >= lo && (E[y] > ve || (E[y] == ve && t[y] > vt))) {
+        E[y + 1] = E[y];
+        t[y + 1] = t[y];
+        y--;
+      }
+      E[y + 1] = ve;
+      t[y + 1] = vt;
+    }
+  }
+  // 16-B store to global memory
+  __device__ static __forceinline__ void st_v4(int *p, int x, int y, int z, int w) {
+    asm volatile("st.global.v4.s32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(x), "r"(y), "r"(z), "r"(w) : "memory");
+  }
+  __device__ static __forceinline__ int clip0(int v, int hi) { return v < 0 ? 0 : (v > hi ? hi : v); }
+  // one index row: step the lane's counts by the row's owner, store them
+  template <int Q, bool CLIP>
+  __device__ static __forceinline__ void row_step(int own, const int (&qb)[Q], int4 (&c)[Q], int *row, int hi) {
+#pragma unroll
+    for (int k = 0; k < Q; k++) {
+      // c[k].{x,y,z,w} += (own == qb[k] + {0,1,2,3}): predicated adds (no branch)
+      asm("{ .reg .pred p0, p1, p2, p3; .reg .s32 d;\n\t"
+          "sub.s32 d, %4, %5;\n\t"
+          "setp.eq.s32 p0, d, 0; setp.eq.s32 p1, d, 1; setp.eq.s32 p2, d, 2; setp.eq.s32 p3, d, 3;\n\t"
+          "@p0 add.s32 %0, %0, 1; @p1 add.s32 %1, %1, 1; @p2 add.s32 %2, %2, 1; @p3 add.s32 %3, %3, 1; }"
+          : "+r"(c[k].x), "+r"(c[k].y), "+r"(c[k].z), "+r"(c[k].w)
+          : "r"(own), "r"(qb[k]));
+      if (CLIP) st_v4(row + qb[k], clip0(c[k].x, hi), clip0(c[k].y, hi), clip0(c[k].z, hi), clip0(c[k].w, hi));
+      else st_v4(row + qb[k], c[k].x, c[k].y, c[k].z, c[k].w);
+    }
+  }
+  // index rows e0 .. e0+m-1 of one union chunk.  Lane holds, for k < Q, the
+  // counts of the four nuclides of quad (lane + 32k) mod ip/4 (quads past
+  // the row are duplicates: every lane stores, duplicates store equal data),
+  // minus one; row r steps the count of its owner Ou[r] and is stored as
+  // ip/4 16-B vectors.  ua / ub = the chunk's and the next chunk's rows of
+  // ustart: when no count of the chunk can leave [1, n_gp-1], the row
+  // values need no clipping (almost every chunk).
+  template <int Q, bool CLIP>
+  __device__ static __forceinline__ void chunk_rows(const uint16_t *Ou, int m, int *row, int ip, int hi,
+                                                    const int (&qb)[Q], int4 (&c)[Q]) {
+    int r = 0;
+    for (; r + 4 <= m; r += 4) {
+      const uint2 o4 = *reinterpret_cast<const uint2 *>(Ou + r);
+      row_step<Q, CLIP>((int)(o4.x & 0xffffu), qb, c, row, hi);
+      row_step<Q, CLIP>((int)(o4.x >> 16), qb, c, row + ip, hi);
+      row_step<Q, CLIP>((int)(o4.y & 0xffffu), qb, c, row + 2 * ip, hi);
+      row_step<Q, CLIP>((int)(o4.y >> 16), qb, c, row + 3 * ip, hi);
+      row += 4 * ip;
+    }
+    for (; r < m; r++, row += ip) row_step<Q, CLIP>((int)Ou[r], qb, c, row, hi);
+  }
+  template <int Q>
+  __device__ static __forceinline__ void chunk_sweep(const uint16_t *Ou, int m, int *ig, long long e0, int ip,
+                                                     int n_gp, int lane, const int *ua) {
+    const int ng4 = ip >> 2;
+    int qb[Q];
+    int4 c[Q];
+    bool inner = true;
+#pragma unroll
+    for (int k = 0; k < Q; k++) {
+      qb[k] = 4 * ((lane + 32 * k) % ng4);
+      const int4 v = ld_(reinterpret_cast<const int4 *>(ua + qb[k]));
+      const int4 w = ld_(reinterpret_cast<const int4 *>(ua + ip + qb[k]));
+      c[k] = make_int4(v.x - 1, v.y - 1, v.z - 1, v.w - 1);
+      inner = inner && v.x >= 1 && v.y >= 1 && v.z >= 1 && v.w >= 1 && w.x <= n_gp - 1 && w.y <= n_gp - 1 &&
+              w.z <= n_gp - 1 && w.w <= n_gp - 1;
+    }
+    int *row = ig + (size_t)e0 * ip;
+    if (__all_sync(0xffffffffu, inner)) chunk_rows<Q, false>(Ou, m, row, ip, n_gp - 2, qb, c);
+    else chunk_rows<Q, true>(Ou, m, row, ip, n_gp - 2, qb, c);
+  }
+  // energy draw (6r+1) of record r and its 32-bit sort key (the LCG state's
+  // top bits: monotone in the energy)
+  __device__ static __forceinline__ double rec_energy(const Affine *jt, uint32_t r, uint64_t gseed) {
+    uint64_t t = jump6(jt, r, gseed);
+    return lcg_double(t);
+  }
+  // insertion sort of (key, j) in [lo, hi) by (energy, j): keys order the
+  // energies except on equal keys, where the energies are re-drawn
+  __device__ static __forceinline__ void isort_keys(uint32_t *K, uint16_t *J, int lo, int hi, const Affine *jt,
+                                                    uint32_t r0, uint64_t gseed) {
+    for (int x = lo + 1; x < hi; x++) {
+      const uint32_t vk = K[x];
+      const uint16_t vj = J[x];
+      int y = x - 1;
+      for (; y >= lo; y--) {
+        const uint32_t yk = K[y];
+        bool after;  // element y sorts after the inserted one
+        if (yk != vk) after = yk > vk;
+        else {
+          const double ey = rec_energy(jt, r0 + J[y], gseed), ev = rec_energy(jt, r0 + vj, gseed);
+          after = ey > ev || (ey == ev && J[y] > vj);
+        }
+        if (!after) break;
+        K[y + 1] = yk;
+        J[y + 1] = J[y];
+      }
+      K[y + 1] = vk;
+      J[y + 1] = vj;
+    }
+  }
+
+  // (U) of init_warp: warp per union chunk.  NI = nuclide slots per lane
+  // (lane + 32z), Q = index-row quads per lane.  Each chunk's ustart rows are
+  // loaded one chunk ahead (registers) so their latency overlaps the
+  // previous chunk's rows.  Returns 1 if a chunk exceeded kXsChunkCap.
+  template <int NI, int Q>
+  __device__ static __noinline__ unsigned union_chunks(Ctx &c, const XsParams &p, const XsLayout &L,
+                                                       const XsSmem &S) {
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const int n_iso = p.n_iso, n_gp = p.n_gp, ip = xs_iso_pad(n_iso);
+    const int NC = (int)xs_uchunks(p);
+    const long long UB = xs_ubins(p), BPC = UB / NC;
+    const unsigned long long *ecmp = (const unsigned long long *)(c.arena + L.keys);
+    const int *ust = (const int *)(c.arena + L.ustart);
+    uint64_t *uA = (uint64_t *)(c.arena + L.uenergy);
+    uint32_t *uf = (uint32_t *)(c.arena + L.ufind);
+    int *ig = (int *)(c.arena + L.index);
+    char *scr = ens_smem(c) + S.nbkt + (size_t)warp * kXsUniScr;
+    unsigned long long *Eu = (unsigned long long *)scr;
+    unsigned long long *Eg = Eu + kXsChunkCap;  // gathered, unsorted
+    uint16_t *Ou = (uint16_t *)(scr + kXsChunkCap * 16);
+    uint16_t *Og = Ou + kXsChunkCap;
+    uint32_t *fc = (uint32_t *)(scr + kXsChunkCap * 20);
+    unsigned ovf = 0;
+    int an[NI], bn[NI];
+    auto load = [&](int ch) {
+#pragma unroll
+      for (int z = 0; z < NI; z++) {
+        const int i = lane + 32 * z;
+        an[z] = i < n_iso ? ld_(ust + (size_t)ch * ip + i) : 0;
+        bn[z] = i < n_iso ? ld_(ust + (size_t)(ch + 1) * ip + i) : 0;
+      }
+    };
+    if (warp < NC) load(warp);
+    for (int ch = warp; ch < NC; ch += nw) {
+      // run of nuclide i in this chunk: ecmp[i][a .. a + len); offsets by a warp scan
+      int a[NI], len[NI], o[NI];
+      int e0l = 0, tot = 0;
+#pragma unroll
+      for (int z = 0; z < NI; z++) {
+        a[z] = an[z];
+        len[z] = bn[z] - an[z];
+      }
+      if (ch + nw < NC) load(ch + nw);
+#pragma unroll
+      for (int z = 0; z < NI; z++) {
+        int inc = len[z];
+#pragma unroll
+        for (int d = 1; d < 32; d <<= 1) {
+          const int t = __shfl_up_sync(0xffffffffu, inc, d);
+          if (lane >= d) inc += t;
+        }
+        o[z] = tot + inc - len[z];
+        tot += __shfl_sync(0xffffffffu, inc, 31);
+        e0l += a[z];
+      }
+      const long long e0 = (long long)warp_sum_u64((unsigned long long)e0l);
+      const int m = tot;
+      if (m > kXsChunkCap) {
+        ovf = 1;
+        continue;
+      }
+      for (int b = lane; b < kXsChunkFb; b += 32) fc[b] = 0;
+      phase_mark(c, 12);
+      // gather: lane per nuclide, its run copied to its offset (the first
+      // four elements of every run in one batch of loads)
+#pragma unroll
+      for (int z = 0; z < NI; z++) {
+        const int i = lane + 32 * z;
+        const unsigned long long *src = ecmp + (size_t)i * n_gp + a[z];
+        unsigned long long v[4];
+#pragma unroll
+        for (int x = 0; x < 4; x++)
+          if (x < len[z]) v[x] = ld_(src + x);
+#pragma unroll
+        for (int x = 0; x < 4; x++)
+          if (x < len[z]) {
+            Eg[o[z] + x] = v[x];
+            Og[o[z] + x] = (uint16_t)i;
+          }
+        for (int x = 4; x < len[z]; x++) {
+          Eg[o[z] + x] = ld_(src + x);
+          Og[o[z] + x] = (uint16_t)i;
+        }
+      }
+      __syncwarp();
+      for (int x = lane; x < m; x += 32) atomicAdd(&fc[chunk_fb(__longlong_as_double((long long)Eg[x]), ch, NC)], 1u);
+      __syncwarp();
+      warp_scan_smem<kXsChunkFb / 32>(fc, lane);
+      __syncwarp();
+      for (int x = lane; x < m; x += 32) {
+        const unsigned long long eb = Eg[x];
+        const uint32_t pos = atomicAdd(&fc[chunk_fb(__longlong_as_double((long long)eb), ch, NC)], 1u);
+        Eu[pos] = eb;
+        Ou[pos] = Og[x];
+      }
+      __syncwarp();
+      phase_mark(c, 13);
+      for (int b = lane; b < kXsChunkFb; b += 32) isort_pairs(Eu, Ou, b ? (int)fc[b - 1] : 0, (int)fc[b]);
+      __syncwarp();
+      phase_mark(c, 14);
+      for (int r = lane; r < m; r += 32) uA[e0 + r] = Eu[r];
+      // search table: uf[b] = #{k >= 1: u_k <= b / UB}, b in this chunk's bins
+      for (long long b = ch * BPC + lane; b < (ch + 1) * BPC; b += 32) {
+        const unsigned long long vb = dbits((double)b / (double)UB);
+        int lo = 0, hi = m;  // first r with Eu[r] > vb
+        while (lo < hi) {
+          const int mid = (lo + hi) >> 1;
+          if (Eu[mid] <= vb) lo = mid + 1;
+          else hi = mid;
+        }
+        const long long v = e0 + lo - 1;
+        uf[b] = (uint32_t)(v > 0 ? v : 0);
+      }
+      phase_mark(c, 15);
+      chunk_sweep<Q>(Ou, m, ig, e0, ip, n_gp, lane, ust + (size_t)ch * ip);
+      __syncwarp();
+      phase_mark(c, 9);
+    }
+    return ovf;
+  }
+
+  __device__ static __noinline__ bool init_warp(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
+    const int tid = threadIdx.x, T = blockDim.x, lane = tid & 31, warp = tid >> 5, nw = T >> 5;
+    const int n_iso = p.n_iso, n_gp = p.n_gp, ip = xs_iso_pad(n_iso);
+    const int NC = (int)xs_uchunks(p);
+    const Affine *jt = (const Affine *)(ens_smem(c) + S.jmp);
+    double *recs = (double *)(c.arena + L.recs);
+    unsigned long long *ecmp = (unsigned long long *)(c.arena + L.keys);  // [n_iso][n_gp] sorted energies
+    int *ust = (int *)(c.arena + L.ustart);                                 // [NC+1][ip]
+    const Affine J32 = lcg_pow(6ULL * 32ULL);
+    const uint64_t gseed = p.gseed;
+
+    // (N) nuclides, a warp each
+    for (int x = tid; x < (NC + 1) * (ip - n_iso); x += T)
+      ust[(x / (ip - n_iso)) * ip + n_iso + x % (ip - n_iso)] = 0;  // pad columns
+    {
+      char *scr = ens_smem(c) + S.nbkt + (size_t)warp * kXsNucScr;
+      uint32_t *K = (uint32_t *)scr;
+      uint16_t *J = (uint16_t *)(scr + kXsWarpGp * 4);
+      uint32_t *cnt = (uint32_t *)(scr + kXsWarpGp * 6);
+      for (int i = warp; i < n_iso; i += nw) {
+        const uint32_t r0 = (uint32_t)i * (uint32_t)n_gp;
+        for (int b = lane; b < kXsNucBkt; b += 32) cnt[b] = 0;
+        __syncwarp();
+        {
+          uint64_t s = jump6(jt, r0 + (uint32_t)lane, gseed);
+          for (int j = lane; j < n_gp; j += 32, s = J32(s)) atomicAdd(&cnt[(uint32_t)(lcg_next(s) >> 31) >> 23], 1u);
+        }
+        __syncwarp();
+        phase_mark(c, 1);
+        warp_scan_smem<kXsNucBkt / 32>(cnt, lane);
+        __syncwarp();
+        {
+          uint64_t s = jump6(jt, r0 + (uint32_t)lane, gseed);
+          for (int j = lane; j < n_gp; j += 32, s = J32(s)) {
+            const uint32_t key = (uint32_t)(lcg_next(s) >> 31);
+            const uint32_t pos = atomicAdd(&cnt[key >> 23], 1u);
+            K[pos] = key;
+            J[pos] = (uint16_t)j;
+          }
+        }
+        __syncwarp();
+        phase_mark(c, 2);
+        for (int b = lane; b < kXsNucBkt; b += 32) isort_keys(K, J, b ? (int)cnt[b - 1] : 0, (int)cnt[b], jt, r0, gseed);
+        __syncwarp();
+        phase_mark(c, 3);
+        // records at their sorted positions (coalesced), sorted energies, and
+        // ustart[ch][i] = k for the chunks ch in (chunk(E[k-1]), chunk(E[k])]
+        double *rec_i = recs + (size_t)r0 * 6;
+        int carry = -1;
+#pragma unroll 2
+        for (int k0 = 0; k0 < n_gp; k0 += 32) {
+          const int k = k0 + lane;
+          int chk = NC;
+          if (k < n_gp) {
+            uint64_t t = jump6(jt, r0 + J[k], gseed);
+            const double e = lcg_double(t), x1 = lcg_double(t), x2 = lcg_double(t), x3 = lcg_double(t),
+                         x4 = lcg_double(t), x5 = lcg_double(t);
+            double2 *d = reinterpret_cast<double2 *>(rec_i + 6 * (size_t)k);
+            d[0] = make_double2(e, x1);
+            d[1] = make_double2(x2, x3);
+            d[2] = make_double2(x4, x5);
+            ecmp[(size_t)r0 + k] = dbits(e);
+            chk = (int)uchunk(e, NC);
+          }
+          int prev = __shfl_up_sync(0xffffffffu, chk, 1);
+          if (lane == 0) prev = carry;
+          if (k < n_gp)
+            for (int ch = prev + 1; ch <= chk; ch++) ust[ch * ip + i] = k;
+          if (k == n_gp - 1)
+            for (int ch = chk + 1; ch <= NC; ch++) ust[ch * ip + i] = n_gp;
+          carry = __shfl_sync(0xffffffffu, chk, 31);
+        }
+        __syncwarp();
+        phase_mark(c, 5);
+      }
+    }
+    __syncthreads();
+    phase_mark(c, 6);
+
+    // (U) union chunks, a warp each
+    const unsigned ovf = ip <= 128 ? union_chunks<3, 1>(c, p, L, S) : union_chunks<12, 3>(c, p, L, S);
+    const int bad = __syncthreads_or((int)ovf);
+    phase_mark(c, 8);
+    return !bad;
   }
 
   // XS-8, XS-9 for one nuclide: interpolate the pair (a = low, b = high
@@ -824,8 +1188,8 @@ struct XsApp {
           fabs_ += fabs(m[x]);
         }
         ver += (unsigned long long)(am + 1);
-        atomicAdd(&c.sh->tallies[am], 1u);
-        atomicAdd(&c.sh->tallies[5 + mat], 1u);
+        atomicAdd(&ens_sh(c)->tallies[am], 1u);
+        atomicAdd(&ens_sh(c)->tallies[5 + mat], 1u);
         s = fwd[n_forward](s);
         pe = lcg_double(s);
         mat = pick_mat_thr(thr, lcg_double(s));
@@ -868,7 +1232,7 @@ struct XsApp {
     uint32_t *hist = (uint32_t *)(c.arena + L.lk_hist);
     const long long UB = xs_ubins(p);
     const XsSmem S = xs_smem(p, T);
-    uint32_t *mcnt = (uint32_t *)(c.smem + S.mcnt);  // [16..28] material offsets of the chunk
+    uint32_t *mcnt = (uint32_t *)(ens_smem(c) + S.mcnt);  // [16..28] material offsets of the chunk
     const double du = 1.0 / p.bins;
     const long long LC = xs_lk_chunk(p);
     const int kb = xs_lk_bits(LC);
@@ -896,12 +1260,12 @@ struct XsApp {
       }
       team_sync(c);
       // (B) bucket offsets (one CTA), material starts to every CTA's smem
-      if (c.crank == 0) global_exclusive_scan(hist, NB + 1, c.sh);
+      if (c.crank == 0) global_exclusive_scan(hist, NB + 1, ens_sh(c));
       team_sync(c);
       if (tid < 12) mcnt[16 + tid] = ld_(hist + ((long long)tid << kb));
       if (tid == 12) mcnt[28] = (uint32_t)nc;
       team_sync(c);  // every CTA has its offsets before (C) moves the cursors
-      if (c.crank == 0 && tid < 12) c.sh->tallies[5 + tid] += mcnt[17 + tid] - mcnt[16 + tid];  // per material
+      if (c.crank == 0 && tid < 12) ens_sh(c)->tallies[5 + tid] += mcnt[17 + tid] - mcnt[16 + tid];  // per material
       // (C) scatter energies to their buckets (hist becomes bucket ends)
       {
         uint64_t s = lcg_pow(2ULL * (uint64_t)(c0 + g0))(p.seed);
@@ -940,7 +1304,7 @@ struct XsApp {
         if (m3 > mxv) { mxv = m3; am = 3; }
         if (m4 > mxv) { mxv = m4; am = 4; }
         ver += (unsigned long long)(am + 1);
-        atomicAdd(&c.sh->tallies[am], 1u);
+        atomicAdd(&ens_sh(c)->tallies[am], 1u);
         bsum += dbits(m0) + dbits(m1) + dbits(m2) + dbits(m3) + dbits(m4);
         fsum += m0; fsum += m1; fsum += m2; fsum += m3; fsum += m4;
         fabs_ += fabs(m0); fabs_ += fabs(m1); fabs_ += fabs(m2); fabs_ += fabs(m3); fabs_ += fabs(m4);

@@ -76,8 +76,8 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
   c.arena = arena;
   c.arena_cap = p.arena_bytes;
   c.out_cap = p.stdout_cap;
-  c.sh = &sh;
-  c.smem = reinterpret_cast<char *>(ss) + kSubSharedBytes;
+  c.sh_off = (uint32_t)((size_t)y * p.sub_stride);  // ss: &ss->sh == ss
+  c.smem_off = c.sh_off + kSubSharedBytes;
   c.crank = cr;
   c.csize = cs;
   for (;;) {

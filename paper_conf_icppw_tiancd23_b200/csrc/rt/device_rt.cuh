@@ -153,12 +153,19 @@ struct Ctx {
   uint64_t arena_cap;
   char *out;           // this instance's raw stdout buffer
   uint32_t out_cap;
-  Shared *sh;
-  char *smem;          // dynamic shared memory of the app
+  uint32_t sh_off;     // scheduler state (Shared) and the app's dynamic
+  uint32_t smem_off;   // shared memory: byte offsets in the dynamic smem
   uint32_t crank, csize;  // CTA rank in the team, team CTAs
   unsigned long long *phases;  // tracing: ns per phase, or null
   unsigned long long t_mark;   // tracing: last mark (team thread 0)
 };
+
+// The instance's shared memory, addressed from the dynamic shared-memory
+// symbol: pointers derived from it stay in the shared window after a Ctx
+// crosses a call, so accesses compile to LDS/STS/ATOMS, not generic LD/ST.
+extern __shared__ __align__(16) char ens_dsmem[];
+__device__ __forceinline__ char *ens_smem(const Ctx &c) { return ens_dsmem + c.smem_off; }
+__device__ __forceinline__ Shared *ens_sh(const Ctx &c) { return reinterpret_cast<Shared *>(ens_dsmem + c.sh_off); }
 
 __device__ __forceinline__ unsigned long long gtimer() {
   unsigned long long t;
@@ -207,9 +214,9 @@ __device__ inline void out_write(Ctx &c, unsigned fmt, const OutArg *args, int n
   uint32_t payload = 0;
   for (int i = 0; i < n; i++) payload += args[i].kind == 3 ? 8u + (uint32_t)align_up(str_len(args[i].s), 8) : 8u;
   uint32_t need = 8u + payload;
-  uint32_t len = c.sh->out_len;
+  uint32_t len = ens_sh(c)->out_len;
   if (len + need > c.out_cap) {
-    c.sh->flags |= 1u;  // ENS_RF_STDOUT_TRUNC
+    ens_sh(c)->flags |= 1u;  // ENS_RF_STDOUT_TRUNC
     return;
   }
   unsigned long long *w = reinterpret_cast<unsigned long long *>(c.out + len);
@@ -227,7 +234,7 @@ __device__ inline void out_write(Ctx &c, unsigned fmt, const OutArg *args, int n
       *w++ = args[i].u;
     }
   }
-  c.sh->out_len = len + need;
+  ens_sh(c)->out_len = len + need;
 }
 
 template <class... A>
@@ -299,24 +306,24 @@ __device__ __forceinline__ uint64_t dbits(double d) { return (uint64_t)__double_
 // shared memory and summed in rank order (deterministic); result valid in
 // rank 0 (in every thread of it).
 __device__ inline unsigned long long team_sum_u64(Ctx &c, unsigned long long v) {
-  v = block_sum_u64(c.sh, v);
+  v = block_sum_u64(ens_sh(c), v);
   if (c.csize == 1) return v;
-  if (threadIdx.x == 0) *cta_shared(&c.sh->team_u[c.crank], 0) = v;
+  if (threadIdx.x == 0) *cta_shared(&ens_sh(c)->team_u[c.crank], 0) = v;
   team_sync(c);
   unsigned long long t = 0;
   if (c.crank == 0)
-    for (uint32_t r = 0; r < c.csize; r++) t += c.sh->team_u[r];
+    for (uint32_t r = 0; r < c.csize; r++) t += ens_sh(c)->team_u[r];
   team_sync(c);
   return t;
 }
 __device__ inline double team_sum_f64(Ctx &c, double v) {
-  v = block_sum_f64(c.sh, v);
+  v = block_sum_f64(ens_sh(c), v);
   if (c.csize == 1) return v;
-  if (threadIdx.x == 0) *cta_shared(&c.sh->team_d[c.crank], 0) = v;
+  if (threadIdx.x == 0) *cta_shared(&ens_sh(c)->team_d[c.crank], 0) = v;
   team_sync(c);
   double t = 0.0;
   if (c.crank == 0)
-    for (uint32_t r = 0; r < c.csize; r++) t += c.sh->team_d[r];
+    for (uint32_t r = 0; r < c.csize; r++) t += ens_sh(c)->team_d[r];
   team_sync(c);
   return t;
 }
