@@ -196,7 +196,7 @@ constexpr uint32_t kXsNucScr = kXsWarpGp * 6 + kXsNucBkt * 4;  // bytes per warp
 constexpr int kXsBinsPerChunk = 64;   // search-table bins per union chunk
 constexpr int kXsChunkCap = 256;      // union energies a warp sorts at once
 constexpr int kXsChunkFb = 256;       // fine sort buckets per union chunk
-constexpr uint32_t kXsUniScr = kXsChunkCap * 20 + kXsChunkFb * 4;  // bytes per chunk warp
+constexpr uint32_t kXsUniScr = kXsChunkCap * 30 + kXsChunkFb * 4;  // bytes per chunk warp (2 gather buffers)
 ENS_HD bool xs_warp_union(const XsParams &p) { return p.grid == XS_UNIONIZED && p.n_gp <= kXsWarpGp; }
 ENS_HD long long xs_uchunks(const XsParams &p) {
   const long long ub = xs_ubins(p);

@@ -653,9 +653,10 @@ struct XsApp {
       t[y + 1] = vt;
     }
   }
-  // 16-B store to global memory
+  // 16-B store to global memory, evict-first (the index grid streams past L2,
+  // which keeps the init's scratch — sorted energies, ustart — resident)
   __device__ static __forceinline__ void st_v4(int *p, int x, int y, int z, int w) {
-    asm volatile("st.global.v4.s32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(x), "r"(y), "r"(z), "r"(w) : "memory");
+    asm volatile("st.global.cs.v4.s32 [%0], {%1, %2, %3, %4};" ::"l"(p), "r"(x), "r"(y), "r"(z), "r"(w) : "memory");
   }
   __device__ static __forceinline__ int clip0(int v, int hi) { return v < 0 ? 0 : (v > hi ? hi : v); }
   // one index row: step the lane's counts by the row's owner, store them
@@ -763,11 +764,11 @@ struct XsApp {
     uint32_t *uf = (uint32_t *)(c.arena + L.ufind);
     int *ig = (int *)(c.arena + L.index);
     char *scr = ens_smem(c) + S.nbkt + (size_t)warp * kXsUniScr;
-    unsigned long long *Eu = (unsigned long long *)scr;
-    unsigned long long *Eg = Eu + kXsChunkCap;  // gathered, unsorted
-    uint16_t *Ou = (uint16_t *)(scr + kXsChunkCap * 16);
-    uint16_t *Og = Ou + kXsChunkCap;
-    uint32_t *fc = (uint32_t *)(scr + kXsChunkCap * 20);
+    unsigned long long *Eu = (unsigned long long *)scr;          // sorted chunk
+    unsigned long long *Eg0 = Eu + kXsChunkCap;                  // gathered, unsorted (2 buffers)
+    uint16_t *Ou = (uint16_t *)(scr + kXsChunkCap * 24);
+    uint16_t *Og0 = Ou + kXsChunkCap;
+    uint32_t *fc = (uint32_t *)(scr + kXsChunkCap * 30);
     unsigned ovf = 0;
     int an[NI], bn[NI];
     auto load = [&](int ch) {
@@ -778,59 +779,66 @@ struct XsApp {
         bn[z] = i < n_iso ? ld_(ust + (size_t)(ch + 1) * ip + i) : 0;
       }
     };
-    if (warp < NC) load(warp);
-    for (int ch = warp; ch < NC; ch += nw) {
-      // run of nuclide i in this chunk: ecmp[i][a .. a + len); offsets by a warp scan
-      int a[NI], len[NI], o[NI];
+    // stage a chunk: its runs ecmp[i][an .. bn) copied asynchronously
+    // (cp.async) to gather buffer `buf` at their prefix offsets; sets the
+    // chunk's size and first union row
+    int m_n = 0;
+    long long e0_n = 0;
+    auto stage = [&](int buf) {
       int e0l = 0, tot = 0;
+      unsigned long long *Eg = Eg0 + buf * kXsChunkCap;
+      uint16_t *Og = Og0 + buf * kXsChunkCap;
+      int o[NI];
 #pragma unroll
       for (int z = 0; z < NI; z++) {
-        a[z] = an[z];
-        len[z] = bn[z] - an[z];
-      }
-      if (ch + nw < NC) load(ch + nw);
-#pragma unroll
-      for (int z = 0; z < NI; z++) {
-        int inc = len[z];
+        const int len = bn[z] - an[z];
+        int inc = len;
 #pragma unroll
         for (int d = 1; d < 32; d <<= 1) {
           const int t = __shfl_up_sync(0xffffffffu, inc, d);
           if (lane >= d) inc += t;
         }
-        o[z] = tot + inc - len[z];
+        o[z] = tot + inc - len;
         tot += __shfl_sync(0xffffffffu, inc, 31);
-        e0l += a[z];
+        e0l += an[z];
       }
-      const long long e0 = (long long)warp_sum_u64((unsigned long long)e0l);
-      const int m = tot;
-      if (m > kXsChunkCap) {
-        ovf = 1;
-        continue;
-      }
-      for (int b = lane; b < kXsChunkFb; b += 32) fc[b] = 0;
-      phase_mark(c, 12);
-      // gather: lane per nuclide, its run copied to its offset (the first
-      // four elements of every run in one batch of loads)
+      e0_n = (long long)warp_sum_u64((unsigned long long)e0l);
+      m_n = tot;
+      if (tot <= kXsChunkCap) {
 #pragma unroll
-      for (int z = 0; z < NI; z++) {
-        const int i = lane + 32 * z;
-        const unsigned long long *src = ecmp + (size_t)i * n_gp + a[z];
-        unsigned long long v[4];
-#pragma unroll
-        for (int x = 0; x < 4; x++)
-          if (x < len[z]) v[x] = ld_(src + x);
-#pragma unroll
-        for (int x = 0; x < 4; x++)
-          if (x < len[z]) {
-            Eg[o[z] + x] = v[x];
+        for (int z = 0; z < NI; z++) {
+          const int i = lane + 32 * z;
+          const unsigned long long *src = ecmp + (size_t)i * n_gp + an[z];
+          for (int x = 0; x < bn[z] - an[z]; x++) {
+            const uint32_t dst = (uint32_t)__cvta_generic_to_shared(Eg + o[z] + x);
+            asm volatile("cp.async.ca.shared.global [%0], [%1], 8;" ::"r"(dst), "l"(src + x) : "memory");
             Og[o[z] + x] = (uint16_t)i;
           }
-        for (int x = 4; x < len[z]; x++) {
-          Eg[o[z] + x] = ld_(src + x);
-          Og[o[z] + x] = (uint16_t)i;
         }
       }
+      asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+    int buf = 0;
+    if (warp < NC) {
+      load(warp);
+      stage(0);
+    }
+    for (int ch = warp; ch < NC; ch += nw, buf ^= 1) {
+      const int m = m_n;
+      const long long e0 = e0_n;
+      if (ch + nw < NC) load(ch + nw);
+      asm volatile("cp.async.wait_all;" ::: "memory");
       __syncwarp();
+      if (m > kXsChunkCap) {
+        ovf = 1;
+        if (ch + nw < NC) stage(buf ^ 1);
+        continue;
+      }
+      const unsigned long long *Eg = Eg0 + buf * kXsChunkCap;
+      const uint16_t *Og = Og0 + buf * kXsChunkCap;
+      for (int b = lane; b < kXsChunkFb; b += 32) fc[b] = 0;
+      __syncwarp();
+      phase_mark(c, 12);
       for (int x = lane; x < m; x += 32) atomicAdd(&fc[chunk_fb(__longlong_as_double((long long)Eg[x]), ch, NC)], 1u);
       __syncwarp();
       warp_scan_smem<kXsChunkFb / 32>(fc, lane);
@@ -860,10 +868,12 @@ struct XsApp {
         uf[b] = (uint32_t)(v > 0 ? v : 0);
       }
       phase_mark(c, 15);
+      if (ch + nw < NC) stage(buf ^ 1);  // the next chunk's gather overlaps this chunk's rows
       chunk_sweep<Q>(Ou, m, ig, e0, ip, n_gp, lane, ust + (size_t)ch * ip);
       __syncwarp();
       phase_mark(c, 9);
     }
+    asm volatile("cp.async.wait_all;" ::: "memory");
     return ovf;
   }
 
@@ -925,9 +935,9 @@ struct XsApp {
             const double e = lcg_double(t), x1 = lcg_double(t), x2 = lcg_double(t), x3 = lcg_double(t),
                          x4 = lcg_double(t), x5 = lcg_double(t);
             double2 *d = reinterpret_cast<double2 *>(rec_i + 6 * (size_t)k);
-            d[0] = make_double2(e, x1);
-            d[1] = make_double2(x2, x3);
-            d[2] = make_double2(x4, x5);
+            __stcs(d, make_double2(e, x1));  // evict-first, like the index rows
+            __stcs(d + 1, make_double2(x2, x3));
+            __stcs(d + 2, make_double2(x4, x5));
             ecmp[(size_t)r0 + k] = dbits(e);
             chk = (int)uchunk(e, NC);
           }
