@@ -198,6 +198,8 @@ constexpr int kXsChunkCap = 256;      // union energies a warp sorts at once
 constexpr int kXsChunkFb = 256;       // fine sort buckets per union chunk
 constexpr uint32_t kXsUniScr = kXsChunkCap * 30 + kXsChunkFb * 4;  // bytes per chunk warp (2 gather buffers)
 ENS_HD bool xs_warp_union(const XsParams &p) { return p.grid == XS_UNIONIZED && p.n_gp <= kXsWarpGp; }
+// warps of a CTA with warp-path scratch (larger blocks leave the rest idle in the init)
+ENS_HD int xs_warp_scr_warps(int T) { return T / 32 < 16 ? T / 32 : 16; }
 ENS_HD long long xs_uchunks(const XsParams &p) {
   const long long ub = xs_ubins(p);
   return ub > kXsBinsPerChunk ? ub / kXsBinsPerChunk : 1;
@@ -282,7 +284,7 @@ constexpr int kXsStep = ENS_XS_STEP;
 // dynamic shared memory layout: material tables + the sort's bucket counters
 constexpr int kXsMaxT = 512;  // XsApp::kMaxT
 struct XsSmem {
-  uint32_t thr, nn, mats, concs, mcnt, jmp, nbkt, ubkt, total;
+  uint32_t thr, nn, mats, concs, mcnt, jmp, nbkt, ubkt, nkey, total;
 };
 // T = the block size the instance runs with
 ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
@@ -300,9 +302,12 @@ ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   else o += (uint32_t)(T / 32) * 2u * (uint32_t)xs_iso_pad(p.n_iso) * 4u;
   S.ubkt = o;  // unionized, small: bucket counters, then chunk owner counts
   if (xs_smem_nb(p)) o += (uint32_t)kXsSmemBkt * 4u;
+  // hash / nuclide grids: one nuclide's u32 sort keys and u16 record indices
+  S.nkey = o;
+  if (p.grid != XS_UNIONIZED) o += (uint32_t)align_up((uint64_t)p.n_gp * 6, 16);
   // unionized warp path: kXsWarpScr per warp, overlaying nbkt / ubkt
   if (xs_warp_union(p)) {
-    const uint32_t need = (uint32_t)(T / 32) * (kXsNucScr > kXsUniScr ? kXsNucScr : kXsUniScr);
+    const uint32_t need = (uint32_t)xs_warp_scr_warps(T) * (kXsNucScr > kXsUniScr ? kXsNucScr : kXsUniScr);
     if (S.nbkt + need > o) o = S.nbkt + need;
   }
   S.total = o;

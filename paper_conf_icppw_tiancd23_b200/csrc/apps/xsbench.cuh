@@ -151,6 +151,8 @@ __device__ __forceinline__ long long bucket_of(double e, long long r, int n_gp, 
 struct XsApp {
   static constexpr uint32_t kId = APP_XSBENCH;
   // thread limit is an upper bound: 512 keeps 128 registers
+  // (measured: a 1024-thread build at 64 registers spills and runs C2's
+  // lookups 1.8x slower)
   static constexpr int kMaxT = 512;
   static constexpr bool kTeam = true;  // splits nuclides and lookup batches over a cluster
   static constexpr bool kSub = false;
@@ -231,10 +233,10 @@ struct XsApp {
     uint64_t t = lcg_next(jump6(jt, r, gseed));  // past the energy draw
     const double x1 = lcg_double(t), x2 = lcg_double(t), x3 = lcg_double(t), x4 = lcg_double(t),
                  x5 = lcg_double(t);
-    double2 *d = reinterpret_cast<double2 *>(dst);
-    d[0] = make_double2(__longlong_as_double((long long)ebits), x1);
-    d[1] = make_double2(x2, x3);
-    d[2] = make_double2(x4, x5);
+    double2 *d = reinterpret_cast<double2 *>(dst);  // evict-first: the tables stream past L2
+    __stcs(d, make_double2(__longlong_as_double((long long)ebits), x1));
+    __stcs(d + 1, make_double2(x2, x3));
+    __stcs(d + 2, make_double2(x4, x5));
   }
 
   // sort keys[lo, hi) by (energy, record id): <= 8 in registers, else in place
@@ -335,9 +337,8 @@ struct XsApp {
   // are bucket-sorted as {energy, j} keys in an L2-resident buffer (XS-4:
   // shared-memory counts -> scan -> scatter -> per-bucket sort), each record
   // is written once in sorted order (coalesced) with its draws 6r+2..6r+6
-  // re-generated, and (hash) the nuclide's index column is built as
-  // a histogram of each energy's first bin followed by an inclusive scan
-  // (XS-5: ig[i][b] = grid_search(E_i, b*du) = min(#{k>=1: E_k <= b*du}, n_gp-2)).
+  // re-generated, and (hash) the nuclide's index column is built by a merge
+  // walk over the sorted energies, each bin written once (XS-5: ig[i][b] = grid_search(E_i, b*du) = min(#{k>=1: E_k <= b*du}, n_gp-2)).
   __device__ static __noinline__ void init_nuc(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
     const int tid = threadIdx.x, T = blockDim.x;
     const int n_iso = p.n_iso, n_gp = p.n_gp;
@@ -345,110 +346,136 @@ struct XsApp {
     uint32_t *nb = (uint32_t *)(ens_smem(c) + S.nbkt);
     const Affine *jt = (const Affine *)(ens_smem(c) + S.jmp);
     double *recs = (double *)(c.arena + L.recs);
-    XsKey *keys = (XsKey *)(c.arena + L.keys);
+    unsigned long long *ekey = (unsigned long long *)(c.arena + L.keys);  // sorted energies (this CTA's)
+    uint32_t *K = (uint32_t *)(ens_smem(c) + S.nkey);                     // sort keys, then
+    uint16_t *J = (uint16_t *)(ens_smem(c) + S.nkey + (size_t)n_gp * 4);  // record indices j
     int *ig = (int *)(c.arena + L.index);
     const bool hash = p.grid == XS_HASH;
+    int kbits = 0;
+    while ((1 << kbits) < nbn) kbits++;
+    auto nkey_bkt = [&](uint32_t key) { return kbits ? (int)(key >> (32 - kbits)) : 0; };
     const double du = 1.0 / p.bins;
     const Affine J6T = lcg_pow(6ULL * T), J24T = lcg_pow(24ULL * T);
-    // this CTA takes nuclides crank, crank + csize, ... with its own keys
-    keys += (size_t)c.crank * n_gp;
+    // this CTA takes nuclides crank, crank + csize, ... with its own scratch
+    ekey += (size_t)c.crank * n_gp;
     for (int i = (int)c.crank; i < n_iso; i += (int)c.csize) {
       int *col = (int *)(c.arena + L.hcol) + (size_t)c.crank * (p.bins + 1);  // this CTA's column
       XsHashEnt *ent = (XsHashEnt *)ig + (size_t)i * (p.bins + 1);
       const uint32_t r0 = (uint32_t)i * (uint32_t)n_gp;  // record i*n_gp + j
       for (int b = tid; b < nbn; b += T) nb[b] = 0;
-      if (hash)
-        for (int b = tid; b <= p.bins; b += T) col[b] = 0;
       __syncthreads();
-      {  // count the energies' buckets (energy = draw 6r+1)
+      {  // count the energies' buckets (energy = draw 6r+1; bucket = top bits of its sort key)
         uint64_t s = jump6(jt, r0 + (uint32_t)tid, p.gseed);
-        for (int j = tid; j < n_gp; j += T, s = J6T(s)) {
-          uint64_t t = s;
-          atomicAdd(&nb[bucket_of(lcg_double(t), j, n_gp, false, 0, nbn)], 1u);
-        }
+        for (int j = tid; j < n_gp; j += T, s = J6T(s)) atomicAdd(&nb[nkey_bkt((uint32_t)(lcg_next(s) >> 31))], 1u);
       }
       __syncthreads();
       phase_mark(c, 1);
       global_exclusive_scan(nb, nbn, ens_sh(c));
       phase_mark(c, 2);
-      {  // scatter {energy, j}, the energies re-drawn, four atomics in flight
+      {  // scatter {key, j} in shared memory, four atomics in flight
         uint64_t s = jump6(jt, r0 + (uint32_t)tid, p.gseed);
         for (int j0 = tid; j0 < n_gp; j0 += 4 * T, s = J24T(s)) {
-          double e[4];
+          uint32_t key[4];
           uint64_t sq = s;
 #pragma unroll
-          for (int q = 0; q < 4; q++, sq = J6T(sq)) {
-            uint64_t t = sq;
-            e[q] = lcg_double(t);
-          }
+          for (int q = 0; q < 4; q++, sq = J6T(sq)) key[q] = (uint32_t)(lcg_next(sq) >> 31);
 #pragma unroll
           for (int q = 0; q < 4; q++) {
             const int j = j0 + q * T;
             if (j < n_gp) {
-              const uint32_t pos = atomicAdd(&nb[bucket_of(e[q], j, n_gp, false, 0, nbn)], 1u);
-              XsKey k;
-              k.key = dbits(e[q]);
-              k.idx = (unsigned)j;
-              k.pad = 0;
-              keys[pos] = k;
+              const uint32_t pos = atomicAdd(&nb[nkey_bkt(key[q])], 1u);
+              K[pos] = key[q];
+              J[pos] = (uint16_t)j;
             }
           }
         }
       }
       __syncthreads();
       phase_mark(c, 3);
-      for (int b = tid; b < nbn; b += T) sort_bucket(keys, b ? nb[b - 1] : 0, nb[b]);
+      for (int b = tid; b < nbn; b += T) isort_keys(K, J, b ? (int)nb[b - 1] : 0, (int)nb[b], jt, r0, p.gseed);
       __syncthreads();
       phase_mark(c, 4);
-      // records written in sorted order (coalesced), their draws re-generated
-      // from the jump tables; hash: each energy's first bin counted
+      // records written in sorted order (coalesced, evict-first), their draws
+      // re-generated from the jump tables; the sorted energies to `ekey`
       double *rec_i = recs + (size_t)i * n_gp * 6;
-      for (int k0 = tid; k0 < n_gp; k0 += 2 * T) {
-        XsKey v[2];
-#pragma unroll
-        for (int q = 0; q < 2; q++)
-          if (k0 + q * T < n_gp) v[q] = keys[k0 + q * T];
-#pragma unroll
-        for (int q = 0; q < 2; q++) {
-          const int k = k0 + q * T;
-          if (k < n_gp) {
-            put_record(jt, r0 + v[q].idx, v[q].key, p.gseed, rec_i + 6 * (size_t)k);
-            if (hash && k >= 1) {  // first bin b with E_k <= b*du
-              const double e = __longlong_as_double((long long)v[q].key);
-              long long bb = (long long)(e * p.bins);
-              while (bb > 0 && (double)(bb - 1) * du >= e) bb--;
-              while (bb < p.bins && (double)bb * du < e) bb++;
-              if (bb < p.bins) atomicAdd((unsigned *)&col[bb], 1u);
-            }
-          }
-        }
+#pragma unroll 2
+      for (int k = tid; k < n_gp; k += T) {
+        uint64_t t = jump6(jt, r0 + J[k], p.gseed);
+        const double e = lcg_double(t), x1 = lcg_double(t), x2 = lcg_double(t), x3 = lcg_double(t),
+                     x4 = lcg_double(t), x5 = lcg_double(t);
+        double2 *d = reinterpret_cast<double2 *>(rec_i + 6 * (size_t)k);
+        __stcs(d, make_double2(e, x1));
+        __stcs(d + 1, make_double2(x2, x3));
+        __stcs(d + 2, make_double2(x4, x5));
+        ekey[k] = dbits(e);
       }
       __syncthreads();
       phase_mark(c, 8);
       if (hash) {
-        global_exclusive_scan<true>((uint32_t *)col, p.bins, ens_sh(c));
-        for (int b = tid; b < p.bins; b += T) {
-          const int v = col[b];
-          if (v > n_gp - 2) col[b] = n_gp - 2;
+        // column by a merge walk over the sorted energies: bin b's count
+        // #{k >= 1: E_k <= b*du} is k on [bfirst(E_k), bfirst(E_k+1)) (0
+        // before bfirst(E_1)); each bin is written once, clamped to n_gp-2
+        auto bfirst = [&](double e) {  // first bin b with e <= b*du (bins if none)
+          long long bb = (long long)(e * p.bins);
+          while (bb > 0 && (double)(bb - 1) * du >= e) bb--;
+          while (bb < p.bins && (double)bb * du < e) bb++;
+          return (int)bb;
+        };
+        constexpr int U = 4;  // independent iterations per thread (loads first)
+        for (int k0 = tid; k0 < n_gp; k0 += U * T) {
+          unsigned long long ek[U], ek1[U];
+#pragma unroll
+          for (int u = 0; u < U; u++) {
+            const int k = k0 + u * T;
+            ek[u] = k < n_gp ? ld_(ekey + k) : 0ull;
+            ek1[u] = k + 1 < n_gp ? ld_(ekey + k + 1) : 0ull;
+          }
+#pragma unroll
+          for (int u = 0; u < U; u++) {
+            const int k = k0 + u * T;
+            if (k < n_gp) {
+              const int lo = k == 0 ? 0 : bfirst(__longlong_as_double((long long)ek[u]));
+              const int hi = k + 1 < n_gp ? bfirst(__longlong_as_double((long long)ek1[u])) : p.bins;
+              const int v = k < n_gp - 2 ? k : n_gp - 2;
+              for (int b = lo; b < hi; b++) col[b] = v;
+            }
+          }
         }
         if (tid == 0) col[p.bins] = n_gp - 2;
         __syncthreads();
-        for (int b = tid; b <= p.bins; b += T) {  // entries {u_low, u_high, q(E[u_low+1..u_low+6])}
-          const int ul = col[b];
-          XsHashEnt h;
-          h.u_low = (uint16_t)ul;
-          h.u_high = (uint16_t)((b < p.bins ? col[b + 1] : n_gp - 2) + 1);
+        for (int b0 = tid; b0 <= p.bins; b0 += U * T) {  // entries {u_low, u_high, q(E[u_low+1..u_low+6])}
+          int ul[U], uh[U];
 #pragma unroll
-          for (int k = 0; k < 6; k++) {
-            int q = 65535;
-            if (ul + 1 + k <= n_gp - 1) {
-              const double e = __longlong_as_double((long long)keys[ul + 1 + k].key);
-              const double x = (e * (double)p.bins - (double)b) * 65536.0;
-              q = x < 0.0 ? 0 : (x >= 65535.0 ? 65535 : (int)x);
-            }
-            h.q[k] = (uint16_t)q;
+          for (int u = 0; u < U; u++) {
+            const int b = b0 + u * T;
+            ul[u] = b <= p.bins ? ld_(col + b) : 0;
+            uh[u] = b < p.bins ? ld_(col + b + 1) : n_gp - 2;
           }
-          ent[b] = h;
+          unsigned long long e6[U][6];
+#pragma unroll
+          for (int u = 0; u < U; u++)
+#pragma unroll
+            for (int k = 0; k < 6; k++)
+              e6[u][k] = ul[u] + 1 + k <= n_gp - 1 && b0 + u * T <= p.bins ? ld_(ekey + ul[u] + 1 + k) : 0ull;
+#pragma unroll
+          for (int u = 0; u < U; u++) {
+            const int b = b0 + u * T;
+            if (b > p.bins) continue;
+            XsHashEnt h;
+            h.u_low = (uint16_t)ul[u];
+            h.u_high = (uint16_t)(uh[u] + 1);
+#pragma unroll
+            for (int k = 0; k < 6; k++) {
+              int q = 65535;
+              if (ul[u] + 1 + k <= n_gp - 1) {
+                const double e = __longlong_as_double((long long)e6[u][k]);
+                const double x = (e * (double)p.bins - (double)b) * 65536.0;
+                q = x < 0.0 ? 0 : (x >= 65535.0 ? 65535 : (int)x);
+              }
+              h.q[k] = (uint16_t)q;
+            }
+            __stcs(reinterpret_cast<uint4 *>(ent + b), *reinterpret_cast<const uint4 *>(&h));
+          }
         }
         __syncthreads();
         phase_mark(c, 9);
@@ -754,9 +781,10 @@ struct XsApp {
   template <int NI, int Q>
   __device__ static __noinline__ unsigned union_chunks(Ctx &c, const XsParams &p, const XsLayout &L,
                                                        const XsSmem &S) {
-    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = xs_warp_scr_warps((int)blockDim.x);
     const int n_iso = p.n_iso, n_gp = p.n_gp, ip = xs_iso_pad(n_iso);
     const int NC = (int)xs_uchunks(p);
+    if (warp >= nw) return 0;
     const long long UB = xs_ubins(p), BPC = UB / NC;
     const unsigned long long *ecmp = (const unsigned long long *)(c.arena + L.keys);
     const int *ust = (const int *)(c.arena + L.ustart);
@@ -878,7 +906,7 @@ struct XsApp {
   }
 
   __device__ static __noinline__ bool init_warp(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
-    const int tid = threadIdx.x, T = blockDim.x, lane = tid & 31, warp = tid >> 5, nw = T >> 5;
+    const int tid = threadIdx.x, T = blockDim.x, lane = tid & 31, warp = tid >> 5, nw = xs_warp_scr_warps(T);
     const int n_iso = p.n_iso, n_gp = p.n_gp, ip = xs_iso_pad(n_iso);
     const int NC = (int)xs_uchunks(p);
     const Affine *jt = (const Affine *)(ens_smem(c) + S.jmp);
@@ -896,7 +924,7 @@ struct XsApp {
       uint32_t *K = (uint32_t *)scr;
       uint16_t *J = (uint16_t *)(scr + kXsWarpGp * 4);
       uint32_t *cnt = (uint32_t *)(scr + kXsWarpGp * 6);
-      for (int i = warp; i < n_iso; i += nw) {
+      for (int i = warp; i < n_iso && warp < nw; i += nw) {
         const uint32_t r0 = (uint32_t)i * (uint32_t)n_gp;
         for (int b = lane; b < kXsNucBkt; b += 32) cnt[b] = 0;
         __syncwarp();
