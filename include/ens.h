@@ -56,7 +56,10 @@ enum {
 /* ens_launch_cfg.flags */
 enum {
   ENS_F_TIMESTAMPS = 1u << 0, /* fill smid / t_start_ns / t_end_ns in records  */
-  ENS_F_PHASES = 1u << 1      /* accumulate per-phase device time (tracing)    */
+  ENS_F_PHASES = 1u << 1,     /* accumulate per-phase device time (tracing)    */
+  ENS_F_GENERIC = 1u << 2     /* bodies take their general paths only (no fast
+                                 paths such as XS's warp-per-nuclide unionized
+                                 init): results are identical — for testing   */
 };
 #define ENS_PHASES 16
 

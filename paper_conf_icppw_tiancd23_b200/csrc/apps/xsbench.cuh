@@ -191,7 +191,7 @@ struct XsApp {
     hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
     phase_mark(c, 0);
     if (p.grid == XS_UNIONIZED) {
-      if (c.crank == 0 && !(xs_warp_union(p) && init_warp(c, p, L, S)))
+      if (c.crank == 0 && !(xs_warp_union(p) && !(c.flags & ENS_F_GENERIC) && init_warp(c, p, L, S)))
         init(c, p, L, S);  // one CTA builds the union
     } else {
       init_nuc(c, p, L, S);  // nuclides striped over the team's CTAs

@@ -105,6 +105,7 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
     c.id = line;
     c.out = p.stdout_base + (size_t)k * p.stdout_cap;
     c.phases = p.phases;
+    c.flags = p.flags;
     phase_mark(c, -1);
     Result r{};
     if (App::kTeam || cr == 0) r = App::run(c, argc, s_argv);

@@ -156,6 +156,7 @@ struct Ctx {
   uint32_t sh_off;     // scheduler state (Shared) and the app's dynamic
   uint32_t smem_off;   // shared memory: byte offsets in the dynamic smem
   uint32_t crank, csize;  // CTA rank in the team, team CTAs
+  uint32_t flags;              // launch flags (ENS_F_*)
   unsigned long long *phases;  // tracing: ns per phase, or null
   unsigned long long t_mark;   // tracing: last mark (team thread 0)
 };

@@ -111,3 +111,30 @@ def test_cluster_team_parity(oracle, team):
              RS_CASES[0], AMG_CASES[1], "echo team"]
     g, o = run_both(oracle, lines, threads=128, team_ctas=team)
     assert_parity(g, o)
+
+
+# unionized init: warp path (n_gp <= 1024) at its edges, the block-wide path
+# just past it, large (89 quads per index row) and history mode; each also
+# with ENS_F_GENERIC (the block-wide path forced) — both equal the oracle
+WARP_UNION_CASES = [
+    "xsbench -s small -g 1024 -l 3000 -G unionized -r 21",
+    "xsbench -s small -g 1025 -l 3000 -G unionized -r 22",
+    "xsbench -s large -g 1000 -l 3000 -G unionized -r 23",
+    "xsbench -s small -g 3 -l 1000 -G unionized -r 24",
+    "xsbench -s small -g 500 -m history -p 300 -l 20 -G unionized -r 25",
+]
+
+
+@pytest.mark.parametrize("generic", [False, True])
+@pytest.mark.parametrize("line", WARP_UNION_CASES)
+def test_xs_union_paths(oracle, line, generic):
+    g, o = run_both(oracle, [line], generic=generic)
+    assert_parity(g, o)
+
+
+@pytest.mark.parametrize("threads", [32, 64, 128, 512])
+def test_xs_warp_union_threads(oracle, threads):
+    """The warp path with 1..16 warps per team (T=32 runs every nuclide and chunk on one warp)."""
+    lines = ["xsbench -s small -g 300 -l 2000 -G unionized -r 26", "xsbench -s large -g 64 -l 500 -G unionized -r 27"]
+    g, o = run_both(oracle, lines, threads=threads)
+    assert_parity(g, o)
