@@ -15,8 +15,12 @@ import torch  # noqa: E402
 from paper_conf_icppw_tiancd23_b200 import Args  # noqa: E402
 from paper_conf_icppw_tiancd23_b200.ensemble import Ensemble  # noqa: E402
 
-XS_PHASES = ["materials", "generate", "bucket scan", "scatter", "bucket sort", "clear tables", "union tables",
-             "index sweep", "record permute", "hash column", "lookup sample+sort", "lookup gathers"]
+XS_PHASES = [  # phase ids by init path: block-wide unionized / hash+nuclide (init_nuc) / warp path (init_warp)
+    "materials", "count", "scan | warp: scan+scatter", "scatter | warp: bucket sort", "bucket sort",
+    "clear tables | warp: records+ustart", "union tables | warp: wait for nuclides", "index sweep",
+    "record permute | warp: wait for chunks", "hash column | warp: index rows", "lookup sample+sort",
+    "lookup gathers", "warp: chunk setup", "warp: chunk gather+count+scatter", "warp: chunk sort",
+    "warp: union energies + search table"]
 
 
 def probe(template, n, threads=512, reps=3, phases=False, team=0, m=0):
