@@ -94,6 +94,50 @@ def algorithmic_bytes(lines, recs, tallies):
     return total
 
 
+# RS-3 algorithmic FP64 work, counted from the formulas as written (each +, -, *, /, sqrt, sin,
+# cos, atan = 1 op; complex ops expanded textbook-style: c_mul 6, c_div 11, c_add/c_sub 2):
+# per nuclide visited: window 2, sigT factors 41, background 3, sigE 1, macro 8 = 55;
+# per pole term: doppler |Z| >= 6 (asymptotic) 76, doppler |Z| < 6 (Abrarov, 11 cexp) 766,
+# no doppler 43.  Bytes: 64-B pole + 1-B l per term, 32-B window + 32-B K0RS per nuclide.
+RS_FLOPS_NUC, RS_FLOPS_FAR, RS_FLOPS_NEAR, RS_FLOPS_NODOPP = 55, 76, 766, 43
+RS_BYTES_TERM, RS_BYTES_NUC = 65, 64
+
+
+def rs_work(lines, recs, tallies):
+    """(algorithmic FP64 ops, algorithmic bytes) of the RS instances of one launch, from the
+    per-instance work counters (tallies[24..26]: pole terms, Abrarov-branch terms) and material
+    tallies (nuclides visited)."""
+    flops = byts = 0
+    for k, line in enumerate(lines):
+        t = line.split()
+        if t[0] != "rsbench" or recs[k]["exit_code"] != 0:
+            continue
+        n_nuc = 355 if ("-s" in t and t[t.index("-s") + 1] == "large") else 68
+        nn = XS_NUM_NUCS[n_nuc]
+        tal = tallies[k]
+        nucs = sum(int(tal[5 + m]) * nn[m] for m in range(12))
+        terms = int(tal[24]) | (int(tal[25]) << 32)
+        near = int(tal[26])
+        if "-d" in t:
+            f_terms = RS_FLOPS_NODOPP * terms
+        else:
+            f_terms = RS_FLOPS_FAR * (terms - near) + RS_FLOPS_NEAR * near
+        flops += RS_FLOPS_NUC * nucs + f_terms
+        byts += RS_BYTES_NUC * nucs + RS_BYTES_TERM * terms
+    return flops, byts
+
+
+def measured_peak_fp64():
+    """FP64 FLOP/s (DFMA = 2) measured now by the DFMA microbenchmark (csrc/tools/fp64_peak.cu)."""
+    import ctypes
+    lib = ctypes.CDLL(os.path.join(ROOT, "paper_conf_icppw_tiancd23_b200", "libens_tools.so"))
+    fl, ms = ctypes.c_double(), ctypes.c_float()
+    rc = lib.ens_tool_fp64_peak(None, 5, ctypes.byref(fl), ctypes.byref(ms))
+    if rc != 0:
+        raise RuntimeError(f"fp64 peak microbenchmark failed: cuda error {rc}")
+    return fl.value
+
+
 def measured_peak_hbm():
     p = os.path.join(ROOT, "MEASURED_PEAKS.json")
     try:
@@ -346,9 +390,19 @@ def main():
     ms_max = float(t.item())
     local_lines = lines[rank::world]
     algo = algorithmic_bytes(local_lines, res.records, res.tallies)
+    rs_flops, rs_bytes = rs_work(local_lines, res.records, res.tallies)
+    algo += rs_bytes
     kern_ms = sum(per_ms) / len(per_ms)
     peak, peak_kind = measured_peak_hbm()
     achieved = algo / (kern_ms * 1e-3) / 1e9
+    fp64 = None
+    if rs_flops:
+        fp64_peak = measured_peak_fp64() / 1e12
+        fp64 = {"achieved": rs_flops / (kern_ms * 1e-3) / 1e12, "peak": fp64_peak, "unit": "TFLOP/s",
+                "frac": rs_flops / (kern_ms * 1e-3) / 1e12 / fp64_peak, "algorithmic_flops_per_launch": rs_flops,
+                "peak_kind": "measured now: DFMA microbenchmark (csrc/tools/fp64_peak.cu), DFMA = 2 FLOP; the "
+                             "RS body is built --fmad=false, so its mul/add arithmetic issues 1 FLOP per DP "
+                             "instruction and tops out at half of this"}
     lookups_local = int(res.records["work"].sum())
     tt = torch.tensor([lookups_local, algo], dtype=torch.float64, device="cuda")
     if dist_on:
@@ -413,6 +467,15 @@ def main():
                                       f"(team of {max(info.team_ctas)} CTAs)",
                             "algorithmic_bytes_per_launch": algo, "kernel_ms": kern_ms},
                "clocks": clocks, "all_exit_ok": ok}
+        if fp64 is not None:
+            hbm_part = {k: out["roofline"][k] for k in ("bound", "achieved", "peak", "unit", "frac")}
+            if all(l.split()[0] == "rsbench" for l in local_lines):
+                # RS-only launch: the FP64 pipe is the roofline (reading Q18)
+                out["roofline"].update({"bound": "alu", "achieved": fp64["achieved"], "peak": fp64["peak"],
+                                        "unit": "TFLOP/s", "frac": fp64["frac"], "peak_kind": fp64["peak_kind"],
+                                        "algorithmic_flops_per_launch": rs_flops, "hbm": hbm_part})
+            else:
+                out["roofline"]["fp64"] = fp64
         if traffic and traffic < 0.5 * algo:
             out["roofline"]["note"] = (
                 "algorithmic bytes (SURVEY 8(d): every lookup's 16-B bracket, 4-B index entries and 96-B record "

@@ -368,8 +368,19 @@ struct RsLayout {
   uint64_t pole_l;     // [total_poles] u8 l_value
   uint64_t windows;    // [total_windows] x 32 B {T, A, F, (start,end)}
   uint64_t k0rs;       // [n_nuc][4] double
+  uint64_t lk_e;       // [chunk] lookup energies sorted by (material, energy)
+  uint64_t lk_hist;    // [(12 << kb) + 1] u32 (material, energy) bucket counts -> cursors
   uint64_t total;
 };
+// RS-3 lookups run in chunks sorted by (material, energy) (a private
+// schedule: every lookup's result is unchanged), ~8 lookups per bucket
+constexpr long long kRsLkChunk = 1LL << 20;
+ENS_HD long long rs_lk_chunk(const RsParams &p) { return p.lookups < kRsLkChunk ? p.lookups : kRsLkChunk; }
+ENS_HD int rs_lk_bits(long long n_c) {
+  int kb = 0;
+  while (kb < 16 && (12LL << kb) * 8 < n_c) kb++;
+  return kb;
+}
 ENS_HD RsLayout rs_layout(const RsParams &p) {
   RsLayout L{};
   const uint64_t tp = (uint64_t)p.avg_poles * p.n_nuc, tw = (uint64_t)p.avg_windows * p.n_nuc;
@@ -380,11 +391,14 @@ ENS_HD RsLayout rs_layout(const RsParams &p) {
   L.pole_l = o; o = align_up(o + tp, 256);
   L.windows = o; o = align_up(o + tw * 32, 256);
   L.k0rs = o; o = align_up(o + p.n_nuc * 32ULL, 256);
+  const long long n_c = rs_lk_chunk(p);
+  L.lk_e = o; o = align_up(o + (uint64_t)n_c * 8, 256);
+  L.lk_hist = o; o = align_up(o + ((12ULL << rs_lk_bits(n_c)) + 1) * 4, 256);
   L.total = o;
   return L;
 }
 struct RsSmem {
-  uint32_t thr, nn, concs, mats, npol, nwin, total;
+  uint32_t thr, nn, concs, mats, npol, nwin, mcnt, total;
 };
 ENS_HD RsSmem rs_smem(const RsParams &p) {
   RsSmem S{};
@@ -396,6 +410,7 @@ ENS_HD RsSmem rs_smem(const RsParams &p) {
   S.mats = o; o += (uint32_t)align_up(12 * mx * 2, 16);
   S.npol = o; o += (uint32_t)align_up((p.n_nuc + 1) * 4, 16);   // pole counts -> offsets
   S.nwin = o; o += (uint32_t)align_up((p.n_nuc + 1) * 4, 16);   // window counts -> offsets
+  S.mcnt = o; o += 64;                                            // sorted chunk: material starts [13]
   S.total = o;
   return S;
 }

@@ -174,6 +174,7 @@ struct Group {
   int ctas() const { return grid * cs / m; }
   uint64_t arena = 0;
   std::vector<uint32_t> kmap;
+  std::vector<double> cost;  // app_cost per kmap entry (schedule only)
   size_t kmap_off = 0;
 };
 
@@ -271,6 +272,20 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     g.app = ap;
     g.smem = std::max(g.smem, sm);
     g.kmap.push_back((uint32_t)k);
+    g.cost.push_back(app_cost(ap, argc, argv));
+  }
+  // longest-first instance queue (LPT): teams pull the heavy instances first
+  // and the light ones fill the tail (results are schedule-independent, Q5)
+  for (Group &g : g_by_app) {
+    if (g.kmap.size() < 2) continue;
+    std::vector<uint32_t> ord(g.kmap.size());
+    for (size_t x = 0; x < ord.size(); x++) ord[x] = (uint32_t)x;
+    std::stable_sort(ord.begin(), ord.end(), [&](uint32_t u, uint32_t v) { return g.cost[u] > g.cost[v]; });
+    std::vector<uint32_t> km(ord.size());
+    std::vector<double> co(ord.size());
+    for (size_t x = 0; x < ord.size(); x++) km[x] = g.kmap[ord[x]], co[x] = g.cost[ord[x]];
+    g.kmap.swap(km);
+    g.cost.swap(co);
   }
   // team size: team-aware bodies get a cluster of cs CTAs when the group has
   // fewer instances than resident CTAs (the largest power of two <= 8 with
@@ -298,6 +313,12 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
         while (cs * 2 <= c->team_ctas && cs < kMaxTeamCtas) cs *= 2;
       } else if (!c->grid_blocks) {
         while (cs < kMaxTeamCtas && (int64_t)g.kmap.size() * cs * 2 <= ctas) cs *= 2;
+        // uneven ensembles: a team large enough that the heaviest instance
+        // ends within one CTA's fair share of the total work
+        double tot = 0.0, mx = 0.0;
+        for (double w : g.cost) tot += w, mx = std::max(mx, w);
+        const double fair = tot / (double)std::min<int64_t>((int64_t)ctas, (int64_t)g.kmap.size());
+        while (cs < kMaxTeamCtas && mx > 1.5 * fair * cs) cs *= 2;
       }
     }
     if (g.m == 1) {

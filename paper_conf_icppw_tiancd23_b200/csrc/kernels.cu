@@ -191,7 +191,43 @@ int app_max_threads(uint32_t app) {
   return 32;
 }
 // whether the body splits its work over a multi-CTA team
-bool app_team_aware(uint32_t app) { return app == APP_XSBENCH ? XsApp::kTeam : false; }
+bool app_team_aware(uint32_t app) {
+  return app == APP_XSBENCH ? XsApp::kTeam : app == APP_RSBENCH ? RsApp::kTeam : false;
+}
+// host-side work estimate of one instance (relative units: dependent loads /
+// pole terms / row or edge updates), for the schedule only: the instance
+// queue is ordered longest-first and the team size covers the heaviest
+// instance.  Results never depend on it (reading Q5).
+double app_cost(uint32_t app, int argc, const char *const *argv) {
+  switch (app) {
+    case APP_XSBENCH: {
+      XsParams p;
+      if (xs_parse(argc, argv, p) >= 0) return 1.0;
+      const double nucs = p.n_iso == 68 ? 15.49 : 55.38, n_u = (double)p.n_iso * p.n_gp;
+      const double lk = p.history ? (double)p.particles * (double)p.lookups : (double)p.lookups;
+      return lk * nucs + n_u * (p.grid == XS_UNIONIZED ? p.n_iso / 8.0 : 2.0);
+    }
+    case APP_RSBENCH: {
+      RsParams p;
+      if (rs_parse(argc, argv, p) >= 0) return 1.0;
+      const double ppw = (double)p.avg_poles / p.avg_windows, per_term = p.doppler ? 1.0 : 0.6;
+      return (double)p.lookups * 15.49 * (4.0 + (ppw > 1.0 ? ppw - 1.0 : 0.0) * per_term) +
+             (double)p.avg_poles * p.n_nuc;
+    }
+    case APP_AMGMK: {
+      AmgParams p;
+      if (amg_parse(argc, argv, p) >= 0) return 1.0;
+      const double n = (double)p.nx * p.ny * p.nz;
+      return 7.0 * n * (p.iters + 1);
+    }
+    case APP_PAGERANK: {
+      PrParams p;
+      if (pr_parse(argc, argv, p) >= 0) return 1.0;
+      return (double)p.n * (p.avg + 1) * (p.iters + 1);
+    }
+  }
+  return 1.0;
+}
 // whether the body can run as one of M instances per CTA (NEXT 1)
 bool app_sub_aware(uint32_t app) {
   switch (app) {

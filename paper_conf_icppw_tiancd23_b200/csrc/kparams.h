@@ -35,6 +35,7 @@ const void *kernel_ptr(uint32_t app, int T);
 const void *kernel_ptr_sub(uint32_t app, int T);  // row kernels (m > 1), kernels_sub.cu
 int app_max_threads(uint32_t app);
 bool app_team_aware(uint32_t app);
+double app_cost(uint32_t app, int argc, const char *const *argv);
 bool app_sub_aware(uint32_t app);
 uint32_t sub_shared_bytes();
 bool app_size(uint32_t app, int argc, const char *const *argv, int T, int cs, uint64_t *arena, uint32_t *smem);

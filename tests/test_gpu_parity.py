@@ -138,3 +138,23 @@ def test_xs_warp_union_threads(oracle, threads):
     lines = ["xsbench -s small -g 300 -l 2000 -G unionized -r 26", "xsbench -s large -g 64 -l 500 -G unionized -r 27"]
     g, o = run_both(oracle, lines, threads=threads)
     assert_parity(g, o)
+
+
+RS_UNEVEN = [f"rsbench -s small -l {L} -p {P} -w {W}{d} -r {i + 1}"
+             for i, (L, P, W, d) in enumerate([(3000, 400, 10, ""), (200, 50, 25, ""), (100, 20, 10, " -d"),
+                                               (1500, 100, 50, " -d"), (50, 10, 5, ""), (700, 300, 30, "")])]
+
+
+@pytest.mark.parametrize("team", [0, 1, 2, 8])
+def test_rs_team_parity(oracle, team):
+    """RS is team-aware: a cluster of CTAs stripes the pole/window draws and the sorted lookup
+    batches; the auto team (0) sizes it for the heaviest instance of an uneven ensemble and the
+    queue is longest-first.  Every team size and order gives the oracle's results."""
+    g, o = run_both(oracle, RS_CASES + RS_UNEVEN, threads=256, team_ctas=team)
+    assert_parity(g, o)
+
+
+def test_rs_chunk_boundary(oracle):
+    """More lookups than one sorted chunk (kRsLkChunk = 2^20): chunks are sampled in order."""
+    g, o = run_both(oracle, ["rsbench -s small -l 1100000 -p 10 -w 10 -r 9", RS_CASES[0]])
+    assert_parity(g, o)

@@ -64,3 +64,33 @@ def test_verification_invariants(oracle, extra):
 def test_usage_errors(oracle, line):
     r = oracle.run_text(line + "\n", app=oracle.APP_RSBENCH)
     assert r.records[0]["exit_code"] == 1 and b"usage: rsbench" in r.stdout[0]
+
+
+@pytest.mark.parametrize("extra", ["", "-d"])
+def test_pole_term_counter(oracle, extra):
+    """tallies[24..25] = pole terms evaluated (the RS roofline's work unit): recomputed from the
+    window table (RS-2.5) and the lookup stream (RS-3: E, mat; window = (int)(E / (1/n_win)),
+    poles [start, end)); tallies[26] (Abrarov branch) is 0 without doppler and <= terms with it."""
+    L, P, W, seed = 300, 40, 8, 3
+    r = oracle.run_text(f"-s small -l {L} -p {P} -w {W} {extra} -r {seed}\n", app=oracle.APP_RSBENCH)
+    tal = r.tallies[0]
+    npol, nwin, ws, we = oracle.rs_tables(1, P, W)
+    woff = np.concatenate([[0], np.cumsum(nwin)])
+    num, mats = oracle.xs_materials(68)
+    want = 0
+    for i in range(L):
+        s = oracle.lcg_ff(seed, 2 * i)
+        E, s = oracle.lcg_double(s)
+        mat, s = oracle.pick_mat(s)
+        for j in range(num[mat]):
+            nuc = mats[mat, j]
+            w = int(E / (1.0 / nwin[nuc]))
+            if w == nwin[nuc]:
+                w -= 1
+            want += int(we[woff[nuc] + w] - ws[woff[nuc] + w])
+    got = int(tal[24]) | (int(tal[25]) << 32)
+    assert got == want and want > 0
+    if extra == "-d":
+        assert int(tal[26]) == 0
+    else:
+        assert 0 <= int(tal[26]) <= got
