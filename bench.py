@@ -478,10 +478,10 @@ def main():
                 out["roofline"]["fp64"] = fp64
         if traffic and traffic < 0.5 * algo:
             out["roofline"]["note"] = (
-                "algorithmic bytes (SURVEY 8(d): every lookup's 16-B bracket, 4-B index entries and 96-B record "
-                "pairs) exceed the DRAM traffic ncu measures: the lookups are sorted by (material, energy), so "
-                "neighbouring lanes share entries and pairs through L1/L2; dram_gbs is the HBM rate actually "
-                "moved, and the kernel is issue/latency bound (profiles/ncu_c2_r1e.txt)")
+                "algorithmic bytes (SURVEY 8(d): per lookup the XS bracket, index entries and record pairs, or "
+                "the RS windows and poles) exceed the DRAM traffic ncu measures: lookups run in (material, "
+                "energy)-sorted batches, so neighbouring lanes share entries, pairs and poles through L1/L2; "
+                "dram_gbs is the HBM rate actually moved (profiles/ncu_*_r1*.txt)")
         if world_note:
             out["note"] = world_note
         if world == 1:

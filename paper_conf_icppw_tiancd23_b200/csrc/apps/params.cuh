@@ -156,8 +156,11 @@ ENS_HD int pow2_ceil(int n) {
 // sort, the sweep's chunk owner counts) in shared memory: kXsSmemBkt u32,
 // ~2 keys per bucket.  0 = counters in the arena.
 constexpr int kXsSmemBkt = 32768;
+ENS_HD bool xs_warp_union(const XsParams &p);
 ENS_HD long long xs_smem_nb(const XsParams &p) {
-  if (p.grid != XS_UNIONIZED) return 0;
+  // the warp path's problems keep the block-wide fallback's counters in the
+  // arena: its shared memory then fits two CTAs per SM at T <= 256
+  if (p.grid != XS_UNIONIZED || xs_warp_union(p)) return 0;
   const long long n_u = (long long)p.n_iso * p.n_gp;
   const long long nch = (n_u + 511) / 512;  // kXsSweepRows
   if (n_u > 4LL * kXsSmemBkt || nch * p.n_iso > kXsSmemBkt) return 0;
