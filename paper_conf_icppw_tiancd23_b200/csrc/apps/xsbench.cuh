@@ -414,13 +414,21 @@ struct XsApp {
       if (hash) {
         // column by a merge walk over the sorted energies: bin b's count
         // #{k >= 1: E_k <= b*du} is k on [bfirst(E_k), bfirst(E_k+1)) (0
-        // before bfirst(E_1)); each bin is written once, clamped to n_gp-2
+        // before bfirst(E_1)); each bin is written once, clamped to n_gp-2.
+        // When it fits, the column and each energy's quantization key fk =
+        // bin(E) << 16 | q(E within its bin) live in the shared memory the
+        // sort no longer needs (the 16-B entries then take no global loads);
+        // otherwise the column goes to this CTA's arena scratch.
         auto bfirst = [&](double e) {  // first bin b with e <= b*du (bins if none)
           long long bb = (long long)(e * p.bins);
           while (bb > 0 && (double)(bb - 1) * du >= e) bb--;
           while (bb < p.bins && (double)bb * du < e) bb++;
           return (int)bb;
         };
+        const uint32_t col_b = (uint32_t)align_up((uint64_t)(p.bins + 1) * 4, 16);
+        const bool sm_col = col_b + (uint32_t)n_gp * 4u <= S.total - S.nbkt && p.bins < 65536;
+        int *colp = sm_col ? (int *)(ens_smem(c) + S.nbkt) : col;
+        uint32_t *fk = (uint32_t *)(ens_smem(c) + S.nbkt + col_b);
         constexpr int U = 4;  // independent iterations per thread (loads first)
         for (int k0 = tid; k0 < n_gp; k0 += U * T) {
           unsigned long long ek[U], ek1[U];
@@ -434,15 +442,45 @@ struct XsApp {
           for (int u = 0; u < U; u++) {
             const int k = k0 + u * T;
             if (k < n_gp) {
-              const int lo = k == 0 ? 0 : bfirst(__longlong_as_double((long long)ek[u]));
+              const double e = __longlong_as_double((long long)ek[u]);
+              const int lo = k == 0 ? 0 : bfirst(e);
               const int hi = k + 1 < n_gp ? bfirst(__longlong_as_double((long long)ek1[u])) : p.bins;
               const int v = k < n_gp - 2 ? k : n_gp - 2;
-              for (int b = lo; b < hi; b++) col[b] = v;
+              for (int b = lo; b < hi; b++) colp[b] = v;
+              if (sm_col) {  // the entry pass's (e * bins - b) * 2^16 at b = bin(e), as integers
+                const double y = e * (double)p.bins;
+                int be = (int)y;
+                be = be < p.bins ? be : p.bins;
+                const double x = (y - (double)be) * 65536.0;
+                const int q = x < 0.0 ? 0 : (x >= 65535.0 ? 65535 : (int)x);
+                fk[k] = ((uint32_t)be << 16) | (uint32_t)q;
+              }
             }
           }
         }
-        if (tid == 0) col[p.bins] = n_gp - 2;
+        if (tid == 0) colp[p.bins] = n_gp - 2;
         __syncthreads();
+        if (sm_col) {
+          // entries {u_low, u_high, q(E[u_low+1..u_low+6])} from shared memory:
+          // q = 0 below bin b, 65535 above it or past the grid
+          for (int b = tid; b <= p.bins; b += T) {
+            const int ul = colp[b], uh = b < p.bins ? colp[b + 1] : n_gp - 2;
+            XsHashEnt h;
+            h.u_low = (uint16_t)ul;
+            h.u_high = (uint16_t)(uh + 1);
+#pragma unroll
+            for (int k = 0; k < 6; k++) {
+              int q = 65535;
+              if (ul + 1 + k <= n_gp - 1) {
+                const uint32_t f = fk[ul + 1 + k];
+                const int fb = (int)(f >> 16);
+                q = fb == b ? (int)(f & 0xffffu) : (fb > b ? 65535 : 0);
+              }
+              h.q[k] = (uint16_t)q;
+            }
+            __stcs(reinterpret_cast<uint4 *>(ent + b), *reinterpret_cast<const uint4 *>(&h));
+          }
+        } else {
         for (int b0 = tid; b0 <= p.bins; b0 += U * T) {  // entries {u_low, u_high, q(E[u_low+1..u_low+6])}
           int ul[U], uh[U];
 #pragma unroll
@@ -476,6 +514,7 @@ struct XsApp {
             }
             __stcs(reinterpret_cast<uint4 *>(ent + b), *reinterpret_cast<const uint4 *>(&h));
           }
+        }
         }
         __syncthreads();
         phase_mark(c, 9);

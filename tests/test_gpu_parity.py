@@ -24,6 +24,9 @@ XS_CASES = [
     "xsbench -s large -g 40 -l 2000 -G unionized -r 5",
     "xsbench -s large -g 200 -l 2000 -G hash -h 500 -r 6",
     "xsbench -s small -g 16384 -l 2000 -G hash -h 100 -r 4",
+    # hash column in shared memory (fits) vs the arena scratch (bins >= 2^16)
+    "xsbench -s small -g 11303 -l 3000 -G hash -h 10000 -r 13",
+    "xsbench -s small -g 3000 -l 2000 -G hash -h 70000 -r 12",
 ]
 
 RS_CASES = [
