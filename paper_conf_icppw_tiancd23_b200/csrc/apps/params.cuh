@@ -240,9 +240,10 @@ ENS_HD int xs_lk_bits(long long n_c) {
 // upstream index u_low = ig[b][i], u_high = ig[b+1][i] + 1 (n_gp <= 16384
 // fits 16 bits) and the energies E[u_low+1..u_low+6] quantized within bin b,
 // q = floor((E*bins - b) * 2^16) clamped to [0, 65535] (65535 also past the
-// grid).  q is monotone in E, so #{k: q(pe) > q_k} never exceeds the number
-// of those energies below pe: one 16-B load gives a bracket guess that is
-// exact unless two energies share a quantum, and it is always verified.
+// grid), stored as q >> 1 (15 bits: the lookup compares six at once, SWAR).
+// q is monotone in E, so #{k: q(pe) > q_k} never exceeds the number of those
+// energies below pe: one 16-B load gives a bracket guess that is exact
+// unless two energies share a quantum, and it is always verified.
 struct XsHashEnt {
   uint16_t u_low, u_high, q[6];
 };

@@ -476,7 +476,7 @@ struct XsApp {
                 const int fb = (int)(f >> 16);
                 q = fb == b ? (int)(f & 0xffffu) : (fb > b ? 65535 : 0);
               }
-              h.q[k] = (uint16_t)q;
+              h.q[k] = (uint16_t)(q >> 1);  // 15-bit quanta (SWAR compare in guess)
             }
             __stcs(reinterpret_cast<uint4 *>(ent + b), *reinterpret_cast<const uint4 *>(&h));
           }
@@ -510,7 +510,7 @@ struct XsApp {
                 const double x = (e * (double)p.bins - (double)b) * 65536.0;
                 q = x < 0.0 ? 0 : (x >= 65535.0 ? 65535 : (int)x);
               }
-              h.q[k] = (uint16_t)q;
+              h.q[k] = (uint16_t)(q >> 1);  // 15-bit quanta (SWAR compare in guess)
             }
             __stcs(reinterpret_cast<uint4 *>(ent + b), *reinterpret_cast<const uint4 *>(&h));
           }
@@ -1074,10 +1074,15 @@ struct XsApp {
       const size_t hs = (size_t)p.bins + 1;
       const XsHashEnt *hc = (const XsHashEnt *)ig + idx;
       auto ent = [&](int j) { return reinterpret_cast<const uint4 *>(hc + (size_t)mrow[j] * hs); };
+      // #{k: pq15 > q_k} over the six 15-bit quanta by a SWAR compare: per
+      // halfword 0x8000 + pq15 - q - 1 keeps bit 15 iff pq15 > q (no borrow
+      // or carry crosses halves), one popcount for all six
+      const uint32_t pq15 = (uint32_t)(pq < 0 ? 0 : (pq >> 1 > 32767 ? 32767 : pq >> 1));
+      const uint32_t P = (pq15 | (pq15 << 16) | 0x80008000u) - 0x00010001u;
       auto guess = [&](const uint4 &h) {
-        return (int)(h.x & 0xffffu) + (pq > (int)(h.y & 0xffffu)) + (pq > (int)(h.y >> 16)) +
-               (pq > (int)(h.z & 0xffffu)) + (pq > (int)(h.z >> 16)) + (pq > (int)(h.w & 0xffffu)) +
-               (pq > (int)(h.w >> 16));
+        const uint32_t m = 0x80008000u;
+        const uint32_t x = ((P - h.y) & m) | (((P - h.z) & m) >> 1) | (((P - h.w) & m) >> 2);
+        return (int)(h.x & 0xffffu) + __popc(x);
       };
       // nuclide j's record pair at the guessed bracket
       auto gather = [&](int j, const uint4 &h, double2 &a0, double2 &a1, double2 &a2, double2 &b0, double2 &b1,
