@@ -1061,7 +1061,7 @@ struct XsApp {
     const double *crow = concs + mat * mx;
     double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
     auto pf_pair = [&](int j, int lo) {
-      const double *q = recs + ((size_t)mrow[j] * n_gp + lo) * 6;
+      const double *q = recs + ((uint32_t)mrow[j] * (uint32_t)n_gp + (uint32_t)lo) * 6u;  // < 2^32 (n_u <= 355 * 16384)
       prefetch_l1(q);
       prefetch_l1(q + 11);
     };
@@ -1073,7 +1073,8 @@ struct XsApp {
       const int pq = (int)((pe * (double)p.bins - (double)idx) * 65536.0);
       const size_t hs = (size_t)p.bins + 1;
       const XsHashEnt *hc = (const XsHashEnt *)ig + idx;
-      auto ent = [&](int j) { return reinterpret_cast<const uint4 *>(hc + (size_t)mrow[j] * hs); };
+      const uint32_t hs32 = (uint32_t)p.bins + 1u;  // entry index < 355 * (10^7 + 1) < 2^32
+      auto ent = [&](int j) { return reinterpret_cast<const uint4 *>(hc + (uint32_t)mrow[j] * hs32); };
       // #{k: pq15 > q_k} over the six 15-bit quanta by a SWAR compare: per
       // halfword 0x8000 + pq15 - q - 1 keeps bit 15 iff pq15 > q (no borrow
       // or carry crosses halves), one popcount for all six
@@ -1090,7 +1091,7 @@ struct XsApp {
         const int uh = (int)(h.x >> 16);
         int lo = guess(h);
         lo = lo < uh - 1 ? lo : uh - 1;
-        const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)mrow[j] * n_gp + lo) * 6);
+        const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((uint32_t)mrow[j] * (uint32_t)n_gp + (uint32_t)lo) * 6u);
         a0 = ld_(r2 + 0); a1 = ld_(r2 + 1); a2 = ld_(r2 + 2);
         b0 = ld_(r2 + 3); b1 = ld_(r2 + 4); b2 = ld_(r2 + 5);
         return 0;
@@ -1100,7 +1101,7 @@ struct XsApp {
       // while pe is past the pair (a quantum collision), else upstream logic
       auto gather_fix = [&](int j, const uint4 &h, double2 &a0, double2 &a1, double2 &a2, double2 &b0,
                             double2 &b1, double2 &b2) {
-        const double *E = recs + (size_t)mrow[j] * n_gp * 6;
+        const double *E = recs + (uint32_t)mrow[j] * (uint32_t)n_gp * 6u;
         const int u_low = (int)(h.x & 0xffffu), uh = (int)(h.x >> 16);
         int lo = guess(h);
         lo = lo < uh - 1 ? lo : uh - 1;
