@@ -419,11 +419,11 @@ struct XsApp {
         // bin(E) << 16 | q(E within its bin) live in the shared memory the
         // sort no longer needs (the 16-B entries then take no global loads);
         // otherwise the column goes to this CTA's arena scratch.
-        auto bfirst = [&](double e) {  // first bin b with e <= b*du (bins if none)
-          long long bb = (long long)(e * p.bins);
+        auto bfirst = [&](double e) {  // first bin b with e <= b*du (bins if none; bins <= 10^7: int)
+          int bb = (int)(e * p.bins);
           while (bb > 0 && (double)(bb - 1) * du >= e) bb--;
           while (bb < p.bins && (double)bb * du < e) bb++;
-          return (int)bb;
+          return bb;
         };
         const uint32_t col_b = (uint32_t)align_up((uint64_t)(p.bins + 1) * 4, 16);
         const bool sm_col = col_b + (uint32_t)n_gp * 4u <= S.total - S.nbkt && p.bins < 65536;
