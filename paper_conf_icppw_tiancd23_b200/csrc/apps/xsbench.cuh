@@ -128,7 +128,7 @@ __device__ __forceinline__ long long gs_u64(const uint64_t *A, double q, long lo
 #ifdef ENS_XS_STOP  // profiling builds only: stop init after phase k
 #define XS_STOP(k) do { if (ENS_XS_STOP == (k)) { __syncthreads(); return; } } while (0)
 #else
-#define XS_STOP(k) phase_mark(c, (k))  // tracing (ENS_F_PHASES): end of init phase k
+#define XS_STOP(k) phase_mark_if(trc, c, (k))  // tracing (ENS_F_PHASES): end of init phase k
 #endif
 
 struct XsKey {
@@ -340,6 +340,7 @@ struct XsApp {
   // re-generated, and (hash) the nuclide's index column is built by a merge
   // walk over the sorted energies, each bin written once (XS-5: ig[i][b] = grid_search(E_i, b*du) = min(#{k>=1: E_k <= b*du}, n_gp-2)).
   __device__ static __noinline__ void init_nuc(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
+    const bool trc = tracing(c);  // tracing (ENS_F_PHASES) thread, cached
     const int tid = threadIdx.x, T = blockDim.x;
     const int n_iso = p.n_iso, n_gp = p.n_gp;
     const int nbn = xs_nbn(n_gp);
@@ -369,9 +370,9 @@ struct XsApp {
         for (int j = tid; j < n_gp; j += T, s = J6T(s)) atomicAdd(&nb[nkey_bkt((uint32_t)(lcg_next(s) >> 31))], 1u);
       }
       __syncthreads();
-      phase_mark(c, 1);
+      phase_mark_if(trc, c, 1);
       global_exclusive_scan(nb, nbn, ens_sh(c));
-      phase_mark(c, 2);
+      phase_mark_if(trc, c, 2);
       {  // scatter {key, j} in shared memory, four atomics in flight
         uint64_t s = jump6(jt, r0 + (uint32_t)tid, p.gseed);
         for (int j0 = tid; j0 < n_gp; j0 += 4 * T, s = J24T(s)) {
@@ -391,10 +392,10 @@ struct XsApp {
         }
       }
       __syncthreads();
-      phase_mark(c, 3);
+      phase_mark_if(trc, c, 3);
       for (int b = tid; b < nbn; b += T) isort_keys(K, J, b ? (int)nb[b - 1] : 0, (int)nb[b], jt, r0, p.gseed);
       __syncthreads();
-      phase_mark(c, 4);
+      phase_mark_if(trc, c, 4);
       // records written in sorted order (coalesced, evict-first), their draws
       // re-generated from the jump tables; the sorted energies to `ekey`
       double *rec_i = recs + (size_t)i * n_gp * 6;
@@ -410,7 +411,7 @@ struct XsApp {
         ekey[k] = dbits(e);
       }
       __syncthreads();
-      phase_mark(c, 8);
+      phase_mark_if(trc, c, 8);
       if (hash) {
         // column by a merge walk over the sorted energies: bin b's count
         // #{k >= 1: E_k <= b*du} is k on [bfirst(E_k), bfirst(E_k+1)) (0
@@ -517,7 +518,7 @@ struct XsApp {
         }
         }
         __syncthreads();
-        phase_mark(c, 9);
+        phase_mark_if(trc, c, 9);
       }
     }
   }
@@ -532,6 +533,7 @@ struct XsApp {
   // (U) union tables, (W) index sweep, (R) every record written once to its
   // sorted position, its five cross sections re-drawn via the jump tables.
   __device__ static __noinline__ void init(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
+    const bool trc = tracing(c);  // tracing (ENS_F_PHASES) thread, cached
     const int tid = threadIdx.x, T = blockDim.x;
     const int n_iso = p.n_iso, n_gp = p.n_gp;
     const long long n_u = (long long)n_iso * n_gp;
@@ -653,7 +655,7 @@ struct XsApp {
         if (e0 + q * T < n_u) put_record(jt, k[q].idx, k[q].key, p.gseed, recs + 6 * (size_t)k[q].pad);
     }
     __syncthreads();
-    phase_mark(c, 8);
+    phase_mark_if(trc, c, 8);
   }
 
   // ---- XS-3/4/5, unionized grid, warp path (n_gp <= kXsWarpGp) -----------
@@ -820,6 +822,7 @@ struct XsApp {
   template <int NI, int Q>
   __device__ static __noinline__ unsigned union_chunks(Ctx &c, const XsParams &p, const XsLayout &L,
                                                        const XsSmem &S) {
+    const bool trc = tracing(c);  // tracing (ENS_F_PHASES) thread, cached
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5, nw = xs_warp_scr_warps((int)blockDim.x);
     const int n_iso = p.n_iso, n_gp = p.n_gp, ip = xs_iso_pad(n_iso);
     const int NC = (int)xs_uchunks(p);
@@ -905,7 +908,7 @@ struct XsApp {
       const uint16_t *Og = Og0 + buf * kXsChunkCap;
       for (int b = lane; b < kXsChunkFb; b += 32) fc[b] = 0;
       __syncwarp();
-      phase_mark(c, 12);
+      phase_mark_if(trc, c, 12);
       for (int x = lane; x < m; x += 32) atomicAdd(&fc[chunk_fb(__longlong_as_double((long long)Eg[x]), ch, NC)], 1u);
       __syncwarp();
       warp_scan_smem<kXsChunkFb / 32>(fc, lane);
@@ -917,10 +920,10 @@ struct XsApp {
         Ou[pos] = Og[x];
       }
       __syncwarp();
-      phase_mark(c, 13);
+      phase_mark_if(trc, c, 13);
       for (int b = lane; b < kXsChunkFb; b += 32) isort_pairs(Eu, Ou, b ? (int)fc[b - 1] : 0, (int)fc[b]);
       __syncwarp();
-      phase_mark(c, 14);
+      phase_mark_if(trc, c, 14);
       for (int r = lane; r < m; r += 32) uA[e0 + r] = Eu[r];
       // search table: uf[b] = #{k >= 1: u_k <= b / UB}, b in this chunk's bins
       for (long long b = ch * BPC + lane; b < (ch + 1) * BPC; b += 32) {
@@ -934,17 +937,18 @@ struct XsApp {
         const long long v = e0 + lo - 1;
         uf[b] = (uint32_t)(v > 0 ? v : 0);
       }
-      phase_mark(c, 15);
+      phase_mark_if(trc, c, 15);
       if (ch + nw < NC) stage(buf ^ 1);  // the next chunk's gather overlaps this chunk's rows
       chunk_sweep<Q>(Ou, m, ig, e0, ip, n_gp, lane, ust + (size_t)ch * ip);
       __syncwarp();
-      phase_mark(c, 9);
+      phase_mark_if(trc, c, 9);
     }
     asm volatile("cp.async.wait_all;" ::: "memory");
     return ovf;
   }
 
   __device__ static __noinline__ bool init_warp(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
+    const bool trc = tracing(c);  // tracing (ENS_F_PHASES) thread, cached
     const int tid = threadIdx.x, T = blockDim.x, lane = tid & 31, warp = tid >> 5, nw = xs_warp_scr_warps(T);
     const int n_iso = p.n_iso, n_gp = p.n_gp, ip = xs_iso_pad(n_iso);
     const int NC = (int)xs_uchunks(p);
@@ -972,7 +976,7 @@ struct XsApp {
           for (int j = lane; j < n_gp; j += 32, s = J32(s)) atomicAdd(&cnt[(uint32_t)(lcg_next(s) >> 31) >> 23], 1u);
         }
         __syncwarp();
-        phase_mark(c, 1);
+        phase_mark_if(trc, c, 1);
         warp_scan_smem<kXsNucBkt / 32>(cnt, lane);
         __syncwarp();
         {
@@ -985,10 +989,10 @@ struct XsApp {
           }
         }
         __syncwarp();
-        phase_mark(c, 2);
+        phase_mark_if(trc, c, 2);
         for (int b = lane; b < kXsNucBkt; b += 32) isort_keys(K, J, b ? (int)cnt[b - 1] : 0, (int)cnt[b], jt, r0, gseed);
         __syncwarp();
-        phase_mark(c, 3);
+        phase_mark_if(trc, c, 3);
         // records at their sorted positions (coalesced), sorted energies, and
         // ustart[ch][i] = k for the chunks ch in (chunk(E[k-1]), chunk(E[k])]
         double *rec_i = recs + (size_t)r0 * 6;
@@ -1017,16 +1021,16 @@ struct XsApp {
           carry = __shfl_sync(0xffffffffu, chk, 31);
         }
         __syncwarp();
-        phase_mark(c, 5);
+        phase_mark_if(trc, c, 5);
       }
     }
     __syncthreads();
-    phase_mark(c, 6);
+    phase_mark_if(trc, c, 6);
 
     // (U) union chunks, a warp each
     const unsigned ovf = ip <= 128 ? union_chunks<3, 1>(c, p, L, S) : union_chunks<12, 3>(c, p, L, S);
     const int bad = __syncthreads_or((int)ovf);
-    phase_mark(c, 8);
+    phase_mark_if(trc, c, 8);
     return !bad;
   }
 
@@ -1304,6 +1308,7 @@ struct XsApp {
   __device__ static __forceinline__ void lookups(Ctx &c, const XsParams &p, const XsLayout &L, const double *thr,
                                               const int *nn, const double *concs, const uint16_t *mats,
                                               Result &R) {
+    const bool trc = tracing(c);  // tracing (ENS_F_PHASES) thread, cached
     const int tid = threadIdx.x, T = blockDim.x;
     const int n_iso = p.n_iso;
     const long long n_u = (long long)n_iso * p.n_gp, nL = p.lookups;
@@ -1362,7 +1367,7 @@ struct XsApp {
         }
       }
       team_sync(c);
-      phase_mark(c, 10);
+      phase_mark_if(trc, c, 10);
       // (D) thread-per-lookup over the sorted chunk
       for (long long sl = g0; sl < nc; sl += gs) {
         int mat = 0;
@@ -1393,7 +1398,7 @@ struct XsApp {
         fabs_ += fabs(m0); fabs_ += fabs(m1); fabs_ += fabs(m2); fabs_ += fabs(m3); fabs_ += fabs(m4);
       }
       team_sync(c);  // lk_pe / hist reused by the next chunk
-      phase_mark(c, 11);
+      phase_mark_if(trc, c, 11);
     }
     ver = team_sum_u64(c, ver);
     bsum = team_sum_u64(c, bsum);

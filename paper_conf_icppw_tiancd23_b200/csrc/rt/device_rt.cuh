@@ -173,6 +173,9 @@ __device__ __forceinline__ unsigned long long gtimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
+// tracing: is this the thread that marks phases?  Hot loops test a cached
+// copy (phase_mark_if): the Ctx lives in local memory across calls
+__device__ __forceinline__ bool tracing(const Ctx &c) { return c.phases && threadIdx.x == 0 && c.crank == 0; }
 // tracing: charge the time since the last mark to phase k (team thread 0)
 __device__ __forceinline__ void phase_mark(Ctx &c, int k) {
   if (c.phases && threadIdx.x == 0 && c.crank == 0) {
@@ -180,6 +183,9 @@ __device__ __forceinline__ void phase_mark(Ctx &c, int k) {
     if (k >= 0) atomicAdd(&c.phases[k], now - c.t_mark);
     c.t_mark = now;
   }
+}
+__device__ __forceinline__ void phase_mark_if(bool on, Ctx &c, int k) {
+  if (on) phase_mark(c, k);
 }
 
 // barrier of the whole team (cluster barrier: release/acquire at cluster
