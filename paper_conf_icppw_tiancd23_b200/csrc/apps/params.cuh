@@ -194,11 +194,18 @@ constexpr int kXsSweepRows = 512;
 // exceeds kXsChunkCap (never seen: ~10 sigma) sends the instance to the
 // block-wide path.
 constexpr int kXsWarpGp = 1024;
-constexpr int kXsNucBkt = 512;  // per-nuclide sort buckets
+#ifndef ENS_XS_NUC_BKT_BITS
+#define ENS_XS_NUC_BKT_BITS 9
+#endif
+constexpr int kXsNucBktBits = ENS_XS_NUC_BKT_BITS;
+constexpr int kXsNucBkt = 1 << kXsNucBktBits;  // per-nuclide sort buckets (top bits of the 32-bit key)
 constexpr uint32_t kXsNucScr = kXsWarpGp * 6 + kXsNucBkt * 4;  // bytes per warp: u32 keys, u16 j, counters
 constexpr int kXsBinsPerChunk = 64;   // search-table bins per union chunk
 constexpr int kXsChunkCap = 256;      // union energies a warp sorts at once
-constexpr int kXsChunkFb = 256;       // fine sort buckets per union chunk
+#ifndef ENS_XS_CHUNK_FB
+#define ENS_XS_CHUNK_FB 32
+#endif
+constexpr int kXsChunkFb = ENS_XS_CHUNK_FB;  // fine sort buckets per union chunk
 constexpr uint32_t kXsUniScr = kXsChunkCap * 30 + kXsChunkFb * 4;  // bytes per chunk warp (2 gather buffers)
 ENS_HD bool xs_warp_union(const XsParams &p) { return p.grid == XS_UNIONIZED && p.n_gp <= kXsWarpGp; }
 // warps of a CTA with warp-path scratch (larger blocks leave the rest idle in the init)

@@ -926,8 +926,9 @@ struct XsApp {
       phase_mark_if(trc, c, 14);
       for (int r = lane; r < m; r += 32) uA[e0 + r] = Eu[r];
       // search table: uf[b] = #{k >= 1: u_k <= b / UB}, b in this chunk's bins
+      const double inv_ub = 1.0 / (double)UB;  // UB a power of two: b * inv_ub == b / UB exactly
       for (long long b = ch * BPC + lane; b < (ch + 1) * BPC; b += 32) {
-        const unsigned long long vb = dbits((double)b / (double)UB);
+        const unsigned long long vb = dbits((double)b * inv_ub);
         int lo = 0, hi = m;  // first r with Eu[r] > vb
         while (lo < hi) {
           const int mid = (lo + hi) >> 1;
@@ -973,7 +974,7 @@ struct XsApp {
         __syncwarp();
         {
           uint64_t s = jump6(jt, r0 + (uint32_t)lane, gseed);
-          for (int j = lane; j < n_gp; j += 32, s = J32(s)) atomicAdd(&cnt[(uint32_t)(lcg_next(s) >> 31) >> 23], 1u);
+          for (int j = lane; j < n_gp; j += 32, s = J32(s)) atomicAdd(&cnt[(uint32_t)(lcg_next(s) >> 31) >> (32 - kXsNucBktBits)], 1u);
         }
         __syncwarp();
         phase_mark_if(trc, c, 1);
@@ -983,7 +984,7 @@ struct XsApp {
           uint64_t s = jump6(jt, r0 + (uint32_t)lane, gseed);
           for (int j = lane; j < n_gp; j += 32, s = J32(s)) {
             const uint32_t key = (uint32_t)(lcg_next(s) >> 31);
-            const uint32_t pos = atomicAdd(&cnt[key >> 23], 1u);
+            const uint32_t pos = atomicAdd(&cnt[key >> (32 - kXsNucBktBits)], 1u);
             K[pos] = key;
             J[pos] = (uint16_t)j;
           }
