@@ -174,7 +174,13 @@ ENS_HD long long xs_buckets(const XsParams &p) {
   if (p.grid == XS_UNIONIZED) return pow2_ceil((int)((n_u + 1) / 2));
   return (long long)p.n_iso * (pow2_ceil(p.n_gp) / 2 > 0 ? pow2_ceil(p.n_gp) / 2 : 1);
 }
-ENS_HD int xs_nbn(int n_gp) { return pow2_ceil(n_gp) / 2 > 0 ? pow2_ceil(n_gp) / 2 : 1; }
+// per-nuclide sort buckets of the hash / nuclide init (~ENS_XS_NBN_DIV / 2 keys each)
+#ifndef ENS_XS_NBN_DIV
+#define ENS_XS_NBN_DIV 2
+#endif
+ENS_HD int xs_nbn(int n_gp) {
+  return pow2_ceil(n_gp) / ENS_XS_NBN_DIV > 0 ? pow2_ceil(n_gp) / ENS_XS_NBN_DIV : 1;
+}
 // bins of the union search table: ufind[b] = #{k >= 1 : u_k <= b / ubins}
 // (power of two, ~1 union energy per bin), so the union position of energy
 // p is ufind[floor(p * ubins)] plus a short forward scan — the same index as
@@ -315,7 +321,15 @@ ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   if (xs_smem_nb(p)) o += (uint32_t)kXsSmemBkt * 4u;
   // hash / nuclide grids: one nuclide's u32 sort keys and u16 record indices
   S.nkey = o;
-  if (p.grid != XS_UNIONIZED) o += (uint32_t)align_up((uint64_t)p.n_gp * 6, 16);
+  if (p.grid != XS_UNIONIZED) {
+    o += (uint32_t)align_up((uint64_t)p.n_gp * 6, 16);
+    // the hash column + quantization keys reuse [nbkt, total) after the sort;
+    // grow the region by up to 16 KB so that they fit (else arena scratch)
+    if (p.grid == XS_HASH) {
+      const uint64_t need = align_up((uint64_t)(p.bins + 1) * 4, 16) + (uint64_t)p.n_gp * 4, have = o - S.nbkt;
+      if (need > have && need - have <= 16384) o = S.nbkt + (uint32_t)align_up(need, 16);
+    }
+  }
   // unionized warp path: kXsWarpScr per warp, overlaying nbkt / ubkt
   if (xs_warp_union(p)) {
     const uint32_t need = (uint32_t)xs_warp_scr_warps(T) * (kXsNucScr > kXsUniScr ? kXsNucScr : kXsUniScr);
