@@ -2,7 +2,7 @@
 """bench.py — ensemble execution on B200: instances/s, lookups/s, HBM roofline.
 
     python bench.py [--gpus N] [--steps K] [--warmup W] [--impl ours|reference]
-                    [--workload C2|TSTAR|C1|C3|C4|C5] [--no-extras]
+                    [--workload C2|C2U|TSTAR|C1|C3|C4|C5] [--no-extras]
 
 One step = one pass of the whole hot path over one
 batch: every instance of the workload launched as ONE persistent ensemble
@@ -211,6 +211,9 @@ def workload_lines(name, world):
     if name == "C2":
         return W.c2(64 * world), "C2: 64 x XSBench-style large (355 nuclides, 11303 gridpoints, hash 10000 bins, " \
                                  "1M lookups) per GPU, distinct seeds; weak scaling by instance id"
+    if name == "C2U":
+        lines = [l.replace("-G hash -h 10000", "-G unionized") for l in W.c2(24 * world)]
+        return lines, "C2u: 24 x XSBench-style large unionized (5.92 GB of tables each; 1M lookups) per GPU"
     if name == "TSTAR":
         return W.tstar(1024 * world), "TSTAR: 1024 x XSBench-style small (68 nuclides, 1000 gridpoints, unionized, " \
                                       "10k lookups) per GPU"
@@ -225,7 +228,7 @@ def workload_lines(name, world):
     raise SystemExit(f"unknown workload {name}")
 
 
-THREADS = {"C2": 512, "TSTAR": 512, "C1": 256, "C3": 256, "C4": 1024, "C5": 512}
+THREADS = {"C2": 512, "C2U": 512, "TSTAR": 512, "C1": 256, "C3": 256, "C4": 1024, "C5": 512}
 
 
 def time_ours(lines, world, rank, threads, steps, warmup, torch, dist_on, team_ctas=0):

@@ -191,8 +191,10 @@ struct XsApp {
     hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
     phase_mark(c, 0);
     if (p.grid == XS_UNIONIZED) {
-      if (c.crank == 0 && !(xs_warp_union(p) && !(c.flags & ENS_F_GENERIC) && init_warp(c, p, L, S)))
-        init(c, p, L, S);  // one CTA builds the union
+      const bool warp_path = xs_warp_union(p) && !(c.flags & ENS_F_GENERIC);
+      if (!warp_path && !xs_smem_nb(p)) init(c, p, L, S, c.csize > 1);  // block-wide, striped over the team
+      else if (c.crank == 0 && !(warp_path && init_warp(c, p, L, S)))
+        init(c, p, L, S, false);  // one CTA builds the union (shared-memory counters / warp-path overflow)
     } else {
       init_nuc(c, p, L, S);  // nuclides striped over the team's CTAs
     }
@@ -297,12 +299,12 @@ struct XsApp {
   // before its increment is the sorted position of that record (stored in
   // keys[e].pad).
   __device__ static __forceinline__ void sweep(XsKey *keys, const uint32_t *chist, int *ig, int *sw, long long n_u,
-                                               int n_iso, int n_gp, long long nch) {
+                                               int n_iso, int n_gp, long long nch, int crank, int csize) {
     const int tid = threadIdx.x, T = blockDim.x, lane = tid & 31, warp = tid >> 5, nw = T >> 5;
     const int ip = xs_iso_pad(n_iso), ng4 = ip >> 2;
     int *cnt = sw + (size_t)warp * 2 * ip, *val = cnt + ip;
     auto clip = [&](int c) { const int v = c - 1; return v < 0 ? 0 : (v > n_gp - 2 ? n_gp - 2 : v); };
-    for (long long ch = warp; ch < nch; ch += nw) {
+    for (long long ch = warp + (long long)crank * nw; ch < nch; ch += (long long)nw * csize) {
       const long long e0 = ch * kXsSweepRows, e1 = (e0 + kXsSweepRows < n_u) ? e0 + kXsSweepRows : n_u;
       for (int i = lane; i < ip; i += 32) {
         const int c = i < n_iso ? (int)chist[ch * n_iso + i] : 0;
@@ -532,9 +534,17 @@ struct XsApp {
   // (XS-4).  Ties are measure-zero (reading Q13) and broken by record id.
   // (U) union tables, (W) index sweep, (R) every record written once to its
   // sorted position, its five cross sections re-drawn via the jump tables.
-  __device__ static __noinline__ void init(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
+  __device__ static __noinline__ void init(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S,
+                                          bool team) {
     const bool trc = tracing(c);  // tracing (ENS_F_PHASES) thread, cached
     const int tid = threadIdx.x, T = blockDim.x;
+    // team: the cluster's CTAs stripe every pass (cluster barrier between
+    // passes; the counters live in the arena); else this CTA runs it alone
+    const long long g0 = team ? (long long)c.crank * T + tid : tid, GS = team ? (long long)c.csize * T : T;
+    auto sync = [&]() {
+      if (team) team_sync(c);
+      else __syncthreads();
+    };
     const int n_iso = p.n_iso, n_gp = p.n_gp;
     const long long n_u = (long long)n_iso * n_gp;
     const long long NB = xs_buckets(p);
@@ -545,30 +555,31 @@ struct XsApp {
     const bool sm_bkt = xs_smem_nb(p) != 0;
     uint32_t *bkt = sm_bkt ? (uint32_t *)(ens_smem(c) + S.ubkt) : (uint32_t *)(c.arena + L.bkt);
     int *ig = (int *)(c.arena + L.index);
-    const Affine J6T = lcg_pow(6ULL * T);
+    const Affine J6T = lcg_pow(6ULL * (uint64_t)GS);
 
-    for (long long b = tid; b < NB; b += T) bkt[b] = 0;
-    __syncthreads();
+    for (long long b = g0; b < NB; b += GS) bkt[b] = 0;
+    sync();
     // (G) count
     {
-      uint64_t s = lcg_pow(6ULL * tid)(p.gseed);
-      for (long long r = tid; r < n_u; r += T, s = J6T(s)) {
+      uint64_t s = lcg_pow(6ULL * (uint64_t)g0)(p.gseed);
+      for (long long r = g0; r < n_u; r += GS, s = J6T(s)) {
         uint64_t t = s;
         atomicAdd(&bkt[bucket_of(lcg_double(t), r, n_gp, true, NB, nbn)], 1u);
       }
     }
-    __syncthreads();
+    sync();
     XS_STOP(1);
     // (S) bucket offsets
-    global_exclusive_scan(bkt, NB, ens_sh(c));
+    if (!team || c.crank == 0) global_exclusive_scan(bkt, NB, ens_sh(c));
+    if (team) team_sync(c);
     XS_STOP(2);
     // (P) scatter, energies re-drawn, kQ independent atomics in flight (the
     // returned cursor is an L2 round trip)
     {
       constexpr int kQ = 8;
-      const Affine JQT = lcg_pow(6ULL * kQ * T);
-      uint64_t s = lcg_pow(6ULL * tid)(p.gseed);
-      for (long long r0 = tid; r0 < n_u; r0 += (long long)kQ * T, s = JQT(s)) {
+      const Affine JQT = lcg_pow(6ULL * kQ * (uint64_t)GS);
+      uint64_t s = lcg_pow(6ULL * (uint64_t)g0)(p.gseed);
+      for (long long r0 = g0; r0 < n_u; r0 += (long long)kQ * GS, s = JQT(s)) {
         unsigned long long eb[kQ];
         uint32_t pos[kQ];
         uint64_t sq = s;
@@ -579,13 +590,13 @@ struct XsApp {
         }
 #pragma unroll
         for (int q = 0; q < kQ; q++) {
-          const long long r = r0 + (long long)q * T;
+          const long long r = r0 + (long long)q * GS;
           if (r < n_u)
             pos[q] = atomicAdd(&bkt[bucket_of(__longlong_as_double((long long)eb[q]), r, n_gp, true, NB, nbn)], 1u);
         }
 #pragma unroll
         for (int q = 0; q < kQ; q++) {
-          const long long r = r0 + (long long)q * T;
+          const long long r = r0 + (long long)q * GS;
           if (r < n_u) {
             XsKey k;
             k.key = eb[q];
@@ -596,11 +607,11 @@ struct XsApp {
         }
       }
     }
-    __syncthreads();
+    sync();
     XS_STOP(3);
     // (B) sort each bucket by (energy, record id); bkt[b] = end of bucket b
-    for (long long b = tid; b < NB; b += T) sort_bucket(keys, b ? (long long)bkt[b - 1] : 0, (long long)bkt[b]);
-    __syncthreads();
+    for (long long b = g0; b < NB; b += GS) sort_bucket(keys, b ? (long long)bkt[b - 1] : 0, (long long)bkt[b]);
+    sync();
     XS_STOP(4);
 
     // (U) keys[] is the union (XS-5); owner = record id / n_gp
@@ -609,8 +620,8 @@ struct XsApp {
     const long long nch = (n_u + kXsSweepRows - 1) / kXsSweepRows;
     uint32_t *uf = (uint32_t *)(c.arena + L.ufind);
     const long long UB = xs_ubins(p);
-    for (long long x = tid; x < nch * n_iso; x += T) chist[x] = 0;
-    __syncthreads();
+    for (long long x = g0; x < nch * n_iso; x += GS) chist[x] = 0;
+    sync();
     XS_STOP(5);
     // first bin b with u <= b / UB (UB a power of two: exact)
     auto bfirst = [&](unsigned long long bits) {
@@ -619,7 +630,7 @@ struct XsApp {
       if ((double)bk < x) bk++;
       return bk < UB ? bk : UB;
     };
-    for (long long e = tid; e < n_u; e += T) {  // union energies, chunk owner counts, search table:
+    for (long long e = g0; e < n_u; e += GS) {  // union energies, chunk owner counts, search table:
       const XsKey k = keys[e];                   // ufind[b] = #{k >= 1 : u_k <= b / UB} = e on
       uA[e] = k.key;                             // [b_e, b_e+1) (b_0 := 0, b_n_u := UB)
       atomicAdd(&chist[(e / kXsSweepRows) * n_iso + k.idx / n_gp], 1u);
@@ -627,8 +638,8 @@ struct XsApp {
       const long long hi = e + 1 < n_u ? bfirst(keys[e + 1].key) : UB;
       for (long long b = lo; b < hi; b++) uf[b] = (uint32_t)e;
     }
-    __syncthreads();
-    for (int i = tid; i < n_iso; i += T) {  // exclusive scan over chunks per owner
+    sync();
+    for (long long i = g0; i < n_iso; i += GS) {  // exclusive scan over chunks per owner
       uint32_t run = 0;
       for (long long ch = 0; ch < nch; ch++) {
         const uint32_t v = chist[ch * n_iso + i];
@@ -636,25 +647,26 @@ struct XsApp {
         run += v;
       }
     }
-    __syncthreads();
+    sync();
     XS_STOP(6);
     // (W) sweep: a warp per chunk, lanes own nuclides; row e of the index grid
     // is clip(#{k>=1: E_i[k] <= u_e}, 0, n_gp-2) = clip(cnt_i(e) - 1, ...),
     // and the owner's new count is the sorted position of that record (XS-4).
-    sweep(keys, chist, ig, (int *)(ens_smem(c) + S.nbkt), n_u, n_iso, n_gp, nch);
-    __syncthreads();
+    sweep(keys, chist, ig, (int *)(ens_smem(c) + S.nbkt), n_u, n_iso, n_gp, nch, team ? (int)c.crank : 0,
+          team ? (int)c.csize : 1);
+    sync();
     XS_STOP(7);
     // (R) records to their sorted positions, keys read coalesced
-    for (long long e0 = tid; e0 < n_u; e0 += 2LL * T) {
+    for (long long e0 = g0; e0 < n_u; e0 += 2LL * GS) {
       XsKey k[2];
 #pragma unroll
       for (int q = 0; q < 2; q++)
-        if (e0 + q * T < n_u) k[q] = keys[e0 + q * T];
+        if (e0 + q * GS < n_u) k[q] = keys[e0 + q * GS];
 #pragma unroll
       for (int q = 0; q < 2; q++)
-        if (e0 + q * T < n_u) put_record(jt, k[q].idx, k[q].key, p.gseed, recs + 6 * (size_t)k[q].pad);
+        if (e0 + q * GS < n_u) put_record(jt, k[q].idx, k[q].key, p.gseed, recs + 6 * (size_t)k[q].pad);
     }
-    __syncthreads();
+    sync();
     phase_mark_if(trc, c, 8);
   }
 

@@ -161,3 +161,14 @@ def test_rs_chunk_boundary(oracle):
     """More lookups than one sorted chunk (kRsLkChunk = 2^20): chunks are sampled in order."""
     g, o = run_both(oracle, ["rsbench -s small -l 1100000 -p 10 -w 10 -r 9", RS_CASES[0]])
     assert_parity(g, o)
+
+
+@pytest.mark.parametrize("team", [1, 2, 8])
+def test_xs_blockwide_union_team(oracle, team):
+    """The block-wide unionized init (n_gp > 1024, counters in the arena) is striped over the
+    team's CTAs (cluster barriers between passes): same union, index grid and records."""
+    lines = ["xsbench -s small -g 2000 -l 2000 -G unionized -r 31",
+             "xsbench -s large -g 1100 -l 1000 -G unionized -r 32",
+             "xsbench -s small -g 1500 -l 1000 -G unionized -r 33"]
+    g, o = run_both(oracle, lines, threads=256, team_ctas=team)
+    assert_parity(g, o)
