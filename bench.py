@@ -308,7 +308,11 @@ def time_e2e(lines, world, rank, threads, steps, torch, dist_on):
     return dt / steps, h2d, d2h
 
 
-def cpu_oracle_sample(lines, budget_s=20.0, max_instances=None):
+# host memory per oracle instance caps the sample: a large unionized XS instance holds 5.9 GB
+ORACLE_MAX_INSTANCES = {"C2U": 1}
+
+
+def cpu_oracle_sample(lines, budget_s=20.0, max_instances=None, cap=None):
     """The oracle as it stands on this host: a bounded sample of the workload's instances —
     the first k lines, one per core, k grown x4 while a pass takes under budget_s / 8."""
     sys.path.insert(0, os.path.join(ROOT, "tests"))
@@ -316,13 +320,14 @@ def cpu_oracle_sample(lines, budget_s=20.0, max_instances=None):
     oracle_lib.build()
     cores = os.cpu_count() or 1
     k = max(1, min(max_instances or cores, len(lines)))
+    cap = cap or len(lines)
     while True:
         t0 = time.perf_counter()
         r = oracle_lib.run_text("".join(l + "\n" for l in lines[:k]), jobs=min(cores, k))
         dt = time.perf_counter() - t0
-        if dt >= budget_s / 8 or k >= len(lines):
+        if dt >= budget_s / 8 or k >= min(len(lines), cap):
             break
-        k = min(len(lines), 4 * k)
+        k = min(len(lines), cap, 4 * k)
     work = int(r.records["work"].sum())
     return {"instances": k, "seconds": dt, "cores": min(cores, k), "work": work}
 
@@ -353,7 +358,8 @@ def main():
         cores = os.cpu_count() or 1
         per = []
         for s in range(a.steps):
-            r = cpu_oracle_sample(lines, max_instances=min(cores, len(lines), 16))
+            r = cpu_oracle_sample(lines, max_instances=min(cores, len(lines), 16, ORACLE_MAX_INSTANCES.get(a.workload, 16)),
+                                  cap=ORACLE_MAX_INSTANCES.get(a.workload))
             per.append(r)
         inst = sum(r["instances"] for r in per)
         sec = sum(r["seconds"] for r in per)
@@ -413,7 +419,13 @@ def main():
     lookups_total = float(tt[0].item())
     ok = bool((res.records["exit_code"] == 0).all())
 
-    # e2e through the C ABI from host buffers
+    # e2e through the C ABI from host buffers (the device-resident ensemble's
+    # workspace is released first: both would not fit for C2U's 145 GB)
+    info_kl, info_bt, info_gb, info_tc = (int(info.kernel_launches), max(info.block_threads), max(info.grid_blocks),
+                                          max(info.team_ctas))
+    ens.close()
+    ens = None
+    torch.cuda.empty_cache()
     e2e_s, h2d, d2h = time_e2e(lines, world, rank, threads, max(2, min(a.steps, 5)), torch, dist_on)
     te = torch.tensor([e2e_s], dtype=torch.float64, device="cuda")
     if dist_on:
@@ -461,13 +473,12 @@ def main():
                "lookups_per_s": lookups_total / (ms_max * 1e-3),
                "e2e": {"value": len(lines) / e2e_s, "unit": "instances/s", "h2d_bytes_per_step": h2d,
                        "d2h_bytes_per_step": d2h},
-               "gpu_launches": int(info.kernel_launches) * a.steps,
+               "gpu_launches": info_kl * a.steps,
                "roofline": {"bound": "hbm", "achieved": achieved, "peak": peak, "unit": "GB/s",
                             "frac": achieved / peak, "traffic": traffic, "peak_kind": peak_kind,
                             "dram_gbs": traffic / (kern_ms * 1e-3) / 1e9 if traffic else None,
                             "dram_frac": traffic / (kern_ms * 1e-3) / 1e9 / peak if traffic else None,
-                            "kernel": f"ens_kernel<App,{max(info.block_threads)}> x {max(info.grid_blocks)} CTAs "
-                                      f"(team of {max(info.team_ctas)} CTAs)",
+                            "kernel": f"ens_kernel<App,{info_bt}> x {info_gb} CTAs (team of {info_tc} CTAs)",
                             "algorithmic_bytes_per_launch": algo, "kernel_ms": kern_ms},
                "clocks": clocks, "all_exit_ok": ok}
         if fp64 is not None:
@@ -488,7 +499,9 @@ def main():
         if world_note:
             out["note"] = world_note
         if world == 1:
-            cb = cpu_oracle_sample(lines, max_instances=min(os.cpu_count() or 1, 16, len(lines)))
+            cb = cpu_oracle_sample(lines, max_instances=min(os.cpu_count() or 1, 16, len(lines),
+                                                             ORACLE_MAX_INSTANCES.get(a.workload, 16)),
+                                   cap=ORACLE_MAX_INSTANCES.get(a.workload))
             out["cpu_baseline"] = {"value": cb["instances"] / cb["seconds"], "unit": "instances/s",
                                    "cores": cb["cores"], "kind": "oracle",
                                    "sample": f"first {cb['instances']} instances of the workload (full size) "
