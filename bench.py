@@ -454,6 +454,25 @@ def main():
                                      "T1_cluster_team_ms": solo2_ms / 2,
                                      "value_vs_cluster_team_T1": (solo2_ms / 2) * len(lines) / ms,
                                      "paper_context": "51x at 64 instances on A100 40GB (P:44-45, P:639-640)"}
+        # XSBench's own convention times the lookup phase alone: the same launch with
+        # ENS_F_PHASES tracing gives each team's device time in the lookup phases
+        # (sample+sort, gathers); every team runs one instance concurrently here
+        from paper_conf_icppw_tiancd23_b200 import Args as _Args, workloads as _W
+        from paper_conf_icppw_tiancd23_b200.ensemble import Ensemble as _Ens
+        pe = _Ens(_Args.parse(_W.text(lines)), app="auto", threads=threads, phases=True).launch()
+        torch.cuda.synchronize()
+        pe.relaunch()
+        torch.cuda.synchronize()
+        ph = pe.run.phases_ns()
+        pinfo = pe.info()
+        teams = max(1, max(pinfo.grid_blocks) // max(1, max(pinfo.team_ctas)))
+        lk_ms = (ph[10] + ph[11]) / teams / 1e6
+        in_ms = sum(ph[k] for k in range(10)) / teams / 1e6
+        pe.close()
+        extras["phases_per_team_ms"] = {"init": in_ms, "lookups": lk_ms,
+                                        "lookup_phase_rate": lookups_total / (lk_ms * 1e-3),
+                                        "note": "XSBench convention (lookup phase only), from ENS_F_PHASES tracing "
+                                                "of one warm launch: lookups / mean team lookup-phase time"}
         # north-star target launch: >= 1024 XSBench-style instances per B200 at >= 60% HBM
         tl, _ = workload_lines("TSTAR", 1)
         t_ens, t_res, t_info, t_ms, t_per, _ = time_ours(tl, 1, 0, THREADS["TSTAR"], 5, 3, torch, False)
