@@ -1195,16 +1195,37 @@ struct XsApp {
       // the union row idx holds every nuclide's bracket (XS-7)
       const int *row = ig + (size_t)idx * xs_iso_pad(n_iso);
       auto bracket = [&](int k) { return k == n_gp - 1 ? k - 1 : k; };
-      int k0 = nm > 0 ? ld_(row + mrow[0]) : 0, k1 = nm > 1 ? ld_(row + mrow[1]) : 0;
-      if (nm > 0) pf_pair(0, bracket(k0));
-      for (int j = 0; j < nm; j++) {
-        const int k = k0;
-        k0 = k1;
-        if (j + 2 < nm) k1 = ld_(row + mrow[j + 2]);
-        if (j + 1 < nm) pf_pair(j + 1, bracket(k0));
-        const double2 *r2 = reinterpret_cast<const double2 *>(recs + ((size_t)mrow[j] * n_gp + bracket(k)) * 6);
-        const double2 a0 = ld_(r2 + 0), a1 = ld_(r2 + 1), a2 = ld_(r2 + 2);
-        const double2 b0 = ld_(r2 + 3), b1 = ld_(r2 + 4), b2 = ld_(r2 + 5);
+      // two nuclides per step (both pairs' loads in flight before either is
+      // used), accumulated in list order; index entries two steps ahead,
+      // pair prefetches one step ahead
+      auto pair = [&](int j, int k) {
+        return reinterpret_cast<const double2 *>(recs + ((uint32_t)mrow[j] * (uint32_t)n_gp + (uint32_t)k) * 6u);
+      };
+      int ia = nm > 0 ? ld_(row + mrow[0]) : 0, ib = nm > 1 ? ld_(row + mrow[1]) : 0;
+      int na = nm > 2 ? ld_(row + mrow[2]) : 0, nb = nm > 3 ? ld_(row + mrow[3]) : 0;
+      if (nm > 0) pf_pair(0, bracket(ia));
+      if (nm > 1) pf_pair(1, bracket(ib));
+      int j = 0;
+      for (; j + 2 <= nm; j += 2) {
+        const int ka = bracket(ia), kb = bracket(ib);
+        ia = na;
+        ib = nb;
+        if (j + 4 < nm) na = ld_(row + mrow[j + 4]);
+        if (j + 5 < nm) nb = ld_(row + mrow[j + 5]);
+        if (j + 2 < nm) pf_pair(j + 2, bracket(ia));
+        if (j + 3 < nm) pf_pair(j + 3, bracket(ib));
+        const double2 *ra = pair(j, ka), *rb = pair(j + 1, kb);
+        const double2 a0 = ld_(ra + 0), a1 = ld_(ra + 1), a2 = ld_(ra + 2);
+        const double2 b0 = ld_(ra + 3), b1 = ld_(ra + 4), b2 = ld_(ra + 5);
+        const double2 c0 = ld_(rb + 0), c1 = ld_(rb + 1), c2 = ld_(rb + 2);
+        const double2 d0 = ld_(rb + 3), d1 = ld_(rb + 4), d2 = ld_(rb + 5);
+        accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
+        accumulate(pe, crow[j + 1], c0, c1, c2, d0, d1, d2, m0, m1, m2, m3, m4);
+      }
+      if (j < nm) {
+        const double2 *ra = pair(j, bracket(ia));
+        const double2 a0 = ld_(ra + 0), a1 = ld_(ra + 1), a2 = ld_(ra + 2);
+        const double2 b0 = ld_(ra + 3), b1 = ld_(ra + 4), b2 = ld_(ra + 5);
         accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
       }
     } else {
