@@ -776,9 +776,21 @@ struct XsApp {
     }
     for (; r < m; r++, row += ip) row_step<Q, CLIP>((int)Ou[r], qb, c, row, hi);
   }
+  // the lane's ustart quads of a chunk (rows ch and ch+1), loaded ahead of
+  // the chunk's sort so that their latency is hidden
+  template <int Q>
+  __device__ static __forceinline__ void sweep_quads(const int *ua, int ip, int lane, int4 (&v)[Q], int4 (&w)[Q]) {
+    const int ng4 = ip >> 2;
+#pragma unroll
+    for (int k = 0; k < Q; k++) {
+      const int qb = 4 * ((lane + 32 * k) % ng4);
+      v[k] = ld_(reinterpret_cast<const int4 *>(ua + qb));
+      w[k] = ld_(reinterpret_cast<const int4 *>(ua + ip + qb));
+    }
+  }
   template <int Q>
   __device__ static __forceinline__ void chunk_sweep(const uint16_t *Ou, int m, int *ig, long long e0, int ip,
-                                                     int n_gp, int lane, const int *ua) {
+                                                     int n_gp, int lane, const int4 (&vq)[Q], const int4 (&wq)[Q]) {
     const int ng4 = ip >> 2;
     int qb[Q];
     int4 c[Q];
@@ -786,8 +798,7 @@ struct XsApp {
 #pragma unroll
     for (int k = 0; k < Q; k++) {
       qb[k] = 4 * ((lane + 32 * k) % ng4);
-      const int4 v = ld_(reinterpret_cast<const int4 *>(ua + qb[k]));
-      const int4 w = ld_(reinterpret_cast<const int4 *>(ua + ip + qb[k]));
+      const int4 v = vq[k], w = wq[k];
       c[k] = make_int4(v.x - 1, v.y - 1, v.z - 1, v.w - 1);
       inner = inner && v.x >= 1 && v.y >= 1 && v.z >= 1 && v.w >= 1 && w.x <= n_gp - 1 && w.y <= n_gp - 1 &&
               w.z <= n_gp - 1 && w.w <= n_gp - 1;
@@ -918,6 +929,8 @@ struct XsApp {
       }
       const unsigned long long *Eg = Eg0 + buf * kXsChunkCap;
       const uint16_t *Og = Og0 + buf * kXsChunkCap;
+      int4 vq[Q], wq[Q];  // this chunk's ustart quads, in flight during the sort
+      sweep_quads<Q>(ust + (size_t)ch * ip, ip, lane, vq, wq);
       for (int b = lane; b < kXsChunkFb; b += 32) fc[b] = 0;
       __syncwarp();
       phase_mark_if(trc, c, 12);
@@ -952,7 +965,7 @@ struct XsApp {
       }
       phase_mark_if(trc, c, 15);
       if (ch + nw < NC) stage(buf ^ 1);  // the next chunk's gather overlaps this chunk's rows
-      chunk_sweep<Q>(Ou, m, ig, e0, ip, n_gp, lane, ust + (size_t)ch * ip);
+      chunk_sweep<Q>(Ou, m, ig, e0, ip, n_gp, lane, vq, wq);
       __syncwarp();
       phase_mark_if(trc, c, 9);
     }
