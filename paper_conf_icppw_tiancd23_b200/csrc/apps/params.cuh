@@ -185,7 +185,12 @@ ENS_HD int xs_nbn(int n_gp) {
 // (power of two, ~1 union energy per bin), so the union position of energy
 // p is ufind[floor(p * ubins)] plus a short forward scan — the same index as
 // XS-7's binary search, in two dependent loads instead of ~17
-ENS_HD long long xs_ubins(const XsParams &p) { return pow2_ceil((int)(((long long)p.n_iso * p.n_gp + 1) / 2)); }
+#ifndef ENS_XS_UB_MUL
+#define ENS_XS_UB_MUL 1
+#endif
+ENS_HD long long xs_ubins(const XsParams &p) {
+  return (long long)pow2_ceil((int)(((long long)p.n_iso * p.n_gp + 1) / 2)) * ENS_XS_UB_MUL;
+}
 // union-sweep chunks (rows per chunk) for the index grid
 constexpr int kXsSweepRows = 512;
 
@@ -206,7 +211,7 @@ constexpr int kXsWarpGp = 1024;
 constexpr int kXsNucBktBits = ENS_XS_NUC_BKT_BITS;
 constexpr int kXsNucBkt = 1 << kXsNucBktBits;  // per-nuclide sort buckets (top bits of the 32-bit key)
 constexpr uint32_t kXsNucScr = kXsWarpGp * 6 + kXsNucBkt * 4;  // bytes per warp: u32 keys, u16 j, counters
-constexpr int kXsBinsPerChunk = 64;   // search-table bins per union chunk
+constexpr int kXsBinsPerChunk = 64 * ENS_XS_UB_MUL;   // search-table bins per union chunk
 constexpr int kXsChunkCap = 256;      // union energies a warp sorts at once
 #ifndef ENS_XS_CHUNK_FB
 #define ENS_XS_CHUNK_FB 32
