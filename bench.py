@@ -228,7 +228,7 @@ def workload_lines(name, world):
     raise SystemExit(f"unknown workload {name}")
 
 
-THREADS = {"C2": 512, "C2U": 512, "TSTAR": 512, "C1": 256, "C3": 256, "C4": 1024, "C5": 512}
+THREADS = {"C2": 512, "C2U": 512, "TSTAR": 512, "C1": 256, "C3": 256, "C4": 1024, "C5": 1024}
 
 
 def time_ours(lines, world, rank, threads, steps, warmup, torch, dist_on, team_ctas=0):
@@ -340,6 +340,7 @@ def main():
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="C2")
     ap.add_argument("--no-extras", action="store_true", help="skip the TSTAR / solo side measurements")
+    ap.add_argument("--threads", type=int, default=0, help="thread limit per team (default: per workload)")
     a = ap.parse_args()
     world, rank, local = dist_env()
     if a.gpus != world and world == 1:
@@ -347,7 +348,7 @@ def main():
     else:
         world_note = None
     lines, wl_desc = workload_lines(a.workload, world)
-    threads = THREADS.get(a.workload, 256)
+    threads = a.threads or THREADS.get(a.workload, 256)
     n_local = len(range(rank, len(lines), world))
     config = {"workload": wl_desc, "instances_per_gpu": n_local, "instances_total": len(lines),
               "block_threads": threads, "l2": "inputs larger than L2 (per-instance tables >> 126 MB in total)",
