@@ -25,6 +25,9 @@ namespace rs_hooks {
 void fast_w(double zr, double zi, double *wr, double *wi);
 void init_tables(int small, int avg_poles, int avg_windows, uint64_t iseed, std::vector<int> &n_poles,
                  std::vector<int> &n_windows, std::vector<int> &win_start, std::vector<int> &win_end);
+void dump_and_micro(int small, int avg_poles, int avg_windows, uint64_t iseed, int doppler, int n,
+                    const int *nucs, const double *Es, double *micro, std::vector<double> &poles,
+                    std::vector<double> &wins, std::vector<double> &k0rs);
 }  // namespace rs_hooks
 namespace pr_hooks {
 void graph(long n, long avg, uint64_t gseed, std::vector<long> &deg, std::vector<long> &ptr, std::vector<long> &src);
@@ -162,6 +165,20 @@ void oracle_xs_set_conc_seed(uint64_t s) { xs_hooks::set_conc_seed(s); }
 
 // ---- RS hooks ----------------------------------------------------------------
 void oracle_rs_fast_w(double zr, double zi, double *wr, double *wi) { rs_hooks::fast_w(zr, zi, wr, wi); }
+// RS-3 micro cross sections at n (nuc, E) points plus the flattened tables
+// (9 doubles per pole, 3 per window, 4 K0RS per nuclide); returns 0, or -1
+// if a table exceeds its capacity (in doubles)
+int oracle_rs_micro(int small, int avg_poles, int avg_windows, uint64_t iseed, int doppler, int n, const int *nucs,
+                    const double *Es, double *micro, double *poles, long pcap, double *wins, long wcap,
+                    double *k0rs, long kcap) {
+  std::vector<double> p, w, k;
+  rs_hooks::dump_and_micro(small, avg_poles, avg_windows, iseed, doppler, n, nucs, Es, micro, p, w, k);
+  if ((long)p.size() > pcap || (long)w.size() > wcap || (long)k.size() > kcap) return -1;
+  std::memcpy(poles, p.data(), p.size() * 8);
+  std::memcpy(wins, w.data(), w.size() * 8);
+  std::memcpy(k0rs, k.data(), k.size() * 8);
+  return 0;
+}
 // returns total windows; arrays sized n_nuc (n_poles, n_windows) and total windows
 int oracle_rs_tables(int small, int avg_poles, int avg_windows, uint64_t iseed, int *n_poles, int *n_windows,
                      int *win_start, int *win_end, int cap) {

@@ -74,6 +74,8 @@ def lib():
                 "oracle_xs_set_conc_seed": (None, [c_u64]),
                 "oracle_rs_fast_w": (None, [c_d, c_d, c_p, c_p]),
                 "oracle_rs_tables": (c_i, [c_i, c_i, c_i, c_u64, c_p, c_p, c_p, c_p, c_i]),
+                "oracle_rs_micro": (c_i, [c_i, c_i, c_i, c_u64, c_i, c_i, c_p, c_p, c_p, c_p, c_l, c_p, c_l,
+                                          c_p, c_l]),
                 "oracle_amg_nnz": (c_l, [c_l, c_l, c_l]),
                 "oracle_amg_csr": (None, [c_l, c_l, c_l, c_p, c_p, c_p]),
                 "oracle_amg_sweeps": (None, [c_l, c_l, c_l, c_l, c_p]),
@@ -233,6 +235,24 @@ def rs_tables(small, avg_poles, avg_windows, iseed=42):
                                _ptr(ws), _ptr(we), cap)
     assert k >= 0
     return npol, nwin, ws[:k], we[:k]
+
+
+def rs_micro(small, avg_poles, avg_windows, doppler, nucs, Es, iseed=42):
+    """RS-3 micro xs (sigT, sigA, sigF, sigE) at (nucs[k], Es[k]) and the tables
+    (poles: n x 9 = EA, RT, RA, RF as (re, im), l; windows: m x 3 = T, A, F;
+    K0RS: n_nuc x 4), all from one RS-2 init."""
+    n_nuc = 68 if small else 355
+    nucs = np.ascontiguousarray(nucs, dtype=np.int32)
+    Es = np.ascontiguousarray(Es, dtype=np.float64)
+    micro = np.zeros((len(nucs), 4))
+    poles = np.zeros((avg_poles * n_nuc, 9))
+    wins = np.zeros((avg_windows * n_nuc, 3))
+    k0 = np.zeros((n_nuc, 4))
+    rc = lib().oracle_rs_micro(1 if small else 0, avg_poles, avg_windows, iseed, doppler, len(nucs), _ptr(nucs),
+                               _ptr(Es), _ptr(micro), _ptr(poles), poles.size, _ptr(wins), wins.size, _ptr(k0),
+                               k0.size)
+    assert rc == 0
+    return micro, poles, wins, k0
 
 
 def amg_csr(nx, ny, nz):
