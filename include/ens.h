@@ -182,7 +182,11 @@ typedef struct {
  * (cap bytes) with stdout_off[k]..stdout_off[k+1] the bytes of instance k
  * (stdout_off has n+1 entries).  stdout_buf == NULL: only stdout_off is
  * filled (to size a buffer); cap too small: ENS_ERANGE with stdout_off
- * filled.  Blocks on the stream.                                              */
+ * filled.  Blocks until this run's kernels are done (its end event, not the
+ * whole stream: a launch queued behind it keeps running while this one is
+ * collected; copies use a non-blocking stream).  The first call after a (re)launch copies
+ * and formats; later calls for the same launch return the same result from
+ * the run's host copy (tallies are copied on the first call that asks).      */
 int ens_collect(ens_run *r, ens_record *recs, uint32_t *tallies, char *stdout_buf, size_t cap,
                 uint64_t *stdout_off);
 
@@ -212,7 +216,7 @@ typedef struct {
   uint64_t stdout_offset;  /* byte offset of the raw stdout buffers              */
   uint32_t stdout_bytes;   /* raw stdout bytes per instance                      */
   uint64_t h2d_bytes;      /* bytes copied host->device by ens_launch            */
-  uint64_t d2h_bytes;      /* bytes copied device->host by the last ens_collect  */
+  uint64_t d2h_bytes;      /* bytes copied device->host collecting the last launch */
   int32_t team_ctas[ENS_N_APPS];  /* CTAs per team (cluster size), per ens_app    */
   int32_t instances_per_cta[ENS_N_APPS]; /* M per ens_app (0 if absent)          */
 } ens_run_info;
@@ -223,7 +227,7 @@ int ens_run_get_info(const ens_run *r, ens_run_info *info);
  * length (needed size) or <0; writes at most cap bytes.                       */
 long ens_format_stdout(uint32_t app, const void *raw, size_t raw_len, char *out, size_t cap);
 
-void ens_run_free(ens_run *r); /* synchronises the stream, then frees           */
+void ens_run_free(ens_run *r); /* waits for the run's own work, then frees      */
 const char *ens_strerror(int err);
 const char *ens_last_error(void);
 const char *ens_version(void);

@@ -15,6 +15,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -200,6 +201,15 @@ struct ens_run {
   bool owns_ws = false;
   cudaStream_t stream = nullptr;
   char *h_stage = nullptr;
+  size_t h_stage_cap = 0;
+  // S10 result of this launch, formatted once (ens_collect is called twice by
+  // callers that size their stdout buffer first); cleared by enqueue
+  bool collected = false, have_tal = false;
+  int bad = 0;
+  std::vector<ens_record> c_recs;
+  std::vector<uint32_t> c_tal;
+  std::vector<uint64_t> c_off;
+  std::string c_text;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   uint32_t flags = 0;
   bool launched = false;
@@ -207,6 +217,74 @@ struct ens_run {
 };
 
 static size_t al(size_t x) { return (x + 255) / 256 * 256; }
+
+// Pinned staging buffers are pooled for the process: cudaHostAlloc /
+// cudaFreeHost cost milliseconds each (page pinning and unmapping), which a
+// per-launch buffer would pay on every ens_launch.  A buffer returns to the
+// pool in ens_run_free, after the stream (and so its H2D copy) is done.
+namespace {
+std::mutex g_pin_mu;
+std::vector<std::pair<size_t, char *>> g_pin_free;
+constexpr size_t kPinPoolMax = 8;
+
+cudaError_t pin_get(size_t bytes, char **p, size_t *cap) {
+  {
+    std::lock_guard<std::mutex> lk(g_pin_mu);
+    size_t best = g_pin_free.size();
+    for (size_t i = 0; i < g_pin_free.size(); i++)
+      if (g_pin_free[i].first >= bytes && (best == g_pin_free.size() || g_pin_free[i].first < g_pin_free[best].first))
+        best = i;
+    if (best < g_pin_free.size()) {
+      *cap = g_pin_free[best].first;
+      *p = g_pin_free[best].second;
+      g_pin_free.erase(g_pin_free.begin() + (long)best);
+      return cudaSuccess;
+    }
+  }
+  size_t c = 64 << 10;
+  while (c < bytes) c *= 2;
+  cudaError_t e = cudaHostAlloc((void **)p, c, cudaHostAllocDefault);
+  *cap = e == cudaSuccess ? c : 0;
+  return e;
+}
+
+// Device->host result copies go through a non-blocking stream of their own
+// (one per device), after the run's end event: a run is collected without
+// waiting for work queued behind it on the launch stream (e.g. the next
+// launch, or the legacy default stream's implicit synchronisation).
+cudaError_t d2h_copy(void *dst, const void *src, size_t bytes) {
+  static std::mutex mu;
+  static cudaStream_t streams[64] = {};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64) return cudaMemcpy(dst, src, bytes, cudaMemcpyDeviceToHost);
+  cudaStream_t st;
+  {
+    std::lock_guard<std::mutex> lk(mu);
+    if (!streams[dev]) {
+      e = cudaStreamCreateWithFlags(&streams[dev], cudaStreamNonBlocking);
+      if (e != cudaSuccess) return e;
+    }
+    st = streams[dev];
+  }
+  e = cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToHost, st);
+  if (e != cudaSuccess) return e;
+  return cudaStreamSynchronize(st);
+}
+
+void pin_put(char *p, size_t cap) {
+  if (!p) return;
+  {
+    std::lock_guard<std::mutex> lk(g_pin_mu);
+    if (g_pin_free.size() < kPinPoolMax) {
+      g_pin_free.emplace_back(cap, p);
+      return;
+    }
+  }
+  cudaFreeHost(p);
+}
+}  // namespace
 
 static uint32_t app_of_argv0(const char *a0) {
   const char *b = std::strrchr(a0, '/');
@@ -406,6 +484,7 @@ extern "C" int ens_workspace_bytes(ens_app app, const ens_args *a, const ens_lau
 
 static int enqueue(ens_run *r) {
   const Plan &P = r->P;
+  r->collected = r->have_tal = false;
   CU(cudaMemsetAsync(r->ws + P.o_ctr, 0, P.zeroed_end - P.o_ctr, r->stream));
   CU(cudaEventRecord(r->ev0, r->stream));
   for (size_t gi = 0; gi < P.groups.size(); gi++) {
@@ -478,7 +557,7 @@ extern "C" int ens_launch(ens_app app, const ens_args *a, const ens_launch_cfg *
   *out = r;
   if (P.n == 0) return ENS_OK;
   // one pinned staging buffer, one H2D copy
-  e = cudaHostAlloc((void **)&r->h_stage, P.staged, cudaHostAllocDefault);
+  e = pin_get(P.staged, &r->h_stage, &r->h_stage_cap);
   if (e != cudaSuccess) {
     *out = nullptr;
     ens_run_free(r);
@@ -523,43 +602,83 @@ extern "C" int ens_collect(ens_run *r, ens_record *recs, uint32_t *tallies, char
     if (stdout_off) stdout_off[0] = 0;
     return ENS_OK;
   }
-  CU(cudaStreamSynchronize(r->stream));
-  CU(cudaGetLastError());
-  r->d2h = 0;
-  // counters | records | stdout positions: one copy
-  std::vector<char> zb(P.zeroed_end - P.o_ctr);
-  CU(cudaMemcpy(zb.data(), r->ws + P.o_ctr, zb.size(), cudaMemcpyDeviceToHost));
-  r->d2h += zb.size();
-  const uint64_t total = *(const uint64_t *)(zb.data() + 8 * P.groups.size());
-  std::vector<ens_record> R((size_t)n);
-  std::memcpy(R.data(), zb.data() + (P.o_recs - P.o_ctr), (size_t)n * sizeof(ens_record));
-  const uint64_t *pos = (const uint64_t *)(zb.data() + (P.o_pos - P.o_ctr));
-  if (tallies) {
-    CU(cudaMemcpy(tallies, r->ws + P.o_tal, (size_t)n * ENS_TALLIES * 4, cudaMemcpyDeviceToHost));
-    r->d2h += (size_t)n * ENS_TALLIES * 4;
-  }
-  std::vector<uint64_t> cmp((size_t)(total + 7) / 8 + 1);
-  if (total) CU(cudaMemcpy(cmp.data(), r->ws + P.o_cmp, (size_t)total, cudaMemcpyDeviceToHost));
-  r->d2h += total;
-  std::string text;
-  std::vector<uint64_t> off((size_t)n + 1, 0);
-  int bad = 0;
-  for (int k = 0; k < n; k++) {
-    ens_record &x = R[(size_t)k];
-    if (!(x.flags & ENS_RF_DONE)) {  // never completed
-      std::memset(&x, 0, sizeof x);
-      x.instance = P.line_of_k[(size_t)k];
-      x.flags = ENS_RF_NOT_RUN;
-    } else if (x.stdout_len) {
-      const size_t before = text.size();
-      if (pos[k] + x.stdout_len > total || format_raw((const char *)cmp.data() + pos[k], x.stdout_len, text) < 0) {
-        bad++;
-        text.resize(before);
-      }
-      x.stdout_len = (uint32_t)(text.size() - before);
+  if (!r->collected) {
+    CU(cudaEventSynchronize(r->ev1));
+    CU(cudaGetLastError());
+    r->d2h = 0;
+    // counters | records | stdout positions | tallies (contiguous: o_tal ==
+    // zeroed_end): one copy into a pooled pinned buffer, then the compacted
+    // raw stdout: a second copy
+    const size_t head = P.o_tal + (size_t)n * ENS_TALLIES * 4 - P.o_ctr;
+    char *hb = nullptr;
+    size_t hb_cap = 0;
+    CU(pin_get(head, &hb, &hb_cap));
+    cudaError_t ce = d2h_copy(hb, r->ws + P.o_ctr, head);
+    if (ce != cudaSuccess) {
+      pin_put(hb, hb_cap);
+      return cuda_fail(ce, "ens_collect: D2H");
     }
-    off[(size_t)k + 1] = text.size();
+    r->d2h += head;
+    const uint64_t total = *(const uint64_t *)(hb + 8 * P.groups.size());
+    std::vector<ens_record> &R = r->c_recs;
+    R.resize((size_t)n);
+    std::memcpy(R.data(), hb + (P.o_recs - P.o_ctr), (size_t)n * sizeof(ens_record));
+    std::vector<uint64_t> posv((size_t)n);
+    std::memcpy(posv.data(), hb + (P.o_pos - P.o_ctr), (size_t)n * 8);
+    const uint64_t *pos = posv.data();
+    r->c_tal.resize((size_t)n * ENS_TALLIES);
+    std::memcpy(r->c_tal.data(), hb + (P.o_tal - P.o_ctr), (size_t)n * ENS_TALLIES * 4);
+    r->have_tal = true;
+    const char *cmp = hb;
+    if (total > hb_cap) {
+      pin_put(hb, hb_cap);
+      hb = nullptr;
+      ce = pin_get(total, &hb, &hb_cap);
+      if (ce != cudaSuccess) return cuda_fail(ce, "ens_collect: cudaHostAlloc");
+      cmp = hb;
+    }
+    if (total) ce = d2h_copy(hb, r->ws + P.o_cmp, (size_t)total);
+    if (ce != cudaSuccess) {
+      pin_put(hb, hb_cap);
+      return cuda_fail(ce, "ens_collect: D2H stdout");
+    }
+    r->d2h += total;
+    std::string &text = r->c_text;
+    text.clear();
+    std::vector<uint64_t> &off = r->c_off;
+    off.assign((size_t)n + 1, 0);
+    int bad = 0;
+    for (int k = 0; k < n; k++) {
+      ens_record &x = R[(size_t)k];
+      if (!(x.flags & ENS_RF_DONE)) {  // never completed
+        std::memset(&x, 0, sizeof x);
+        x.instance = P.line_of_k[(size_t)k];
+        x.flags = ENS_RF_NOT_RUN;
+      } else if (x.stdout_len) {
+        const size_t before = text.size();
+        if (pos[k] + x.stdout_len > total || format_raw(cmp + pos[k], x.stdout_len, text) < 0) {
+          bad++;
+          text.resize(before);
+        }
+        x.stdout_len = (uint32_t)(text.size() - before);
+      }
+      off[(size_t)k + 1] = text.size();
+    }
+    pin_put(hb, hb_cap);
+    r->bad = bad;
+    r->collected = true;
   }
+  if (tallies && !r->have_tal) {
+    r->c_tal.resize((size_t)n * ENS_TALLIES);
+    CU(d2h_copy(r->c_tal.data(), r->ws + P.o_tal, (size_t)n * ENS_TALLIES * 4));
+    r->d2h += (size_t)n * ENS_TALLIES * 4;
+    r->have_tal = true;
+  }
+  if (tallies) std::memcpy(tallies, r->c_tal.data(), r->c_tal.size() * 4);
+  const std::vector<ens_record> &R = r->c_recs;
+  const std::vector<uint64_t> &off = r->c_off;
+  const std::string &text = r->c_text;
+  const int bad = r->bad;
   if (recs) std::memcpy(recs, R.data(), R.size() * sizeof(ens_record));
   if (stdout_off) std::memcpy(stdout_off, off.data(), off.size() * 8);
   if (bad) return fail(ENS_ECUDA, "ens_collect: malformed device stdout records");
@@ -628,9 +747,12 @@ extern "C" long ens_format_stdout(uint32_t app, const void *raw, size_t raw_len,
 
 extern "C" void ens_run_free(ens_run *r) {
   if (!r) return;
-  if (r->launched) cudaStreamSynchronize(r->stream);
+  if (r->launched)
+    cudaEventSynchronize(r->ev1);  // the run's own work (H2D, kernels) is done
+  else if (r->h_stage)
+    cudaStreamSynchronize(r->stream);  // a failed enqueue may leave the H2D in flight
   if (r->owns_ws && r->ws) cudaFree(r->ws);
-  if (r->h_stage) cudaFreeHost(r->h_stage);
+  pin_put(r->h_stage, r->h_stage_cap);
   if (r->ev0) cudaEventDestroy(r->ev0);
   if (r->ev1) cudaEventDestroy(r->ev1);
   delete r;

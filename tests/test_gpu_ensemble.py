@@ -115,3 +115,27 @@ def test_timestamps_and_smid():
     assert np.all(r.records["t_end_ns"] >= r.records["t_start_ns"])
     assert np.all(r.records["t_start_ns"] > 0)
     assert len(set(r.records["smid"].tolist())) > 16
+
+
+def test_runs_in_flight_on_one_stream():
+    """Two launches queued on one stream with their own workspaces: collecting the first
+    waits for its own run only (end event), while the second is still queued or running;
+    both equal a solo sequential run, and collect is idempotent (second call = cached)."""
+    import torch
+    from paper_conf_icppw_tiancd23_b200 import Args, _ens
+    lines = LINES[:5] * 6
+    args = Args.parse(text(lines))
+    cfg = _ens.make_cfg(len(lines))
+    ws = _ens.workspace_bytes("auto", args, cfg)
+    bufs = [torch.empty(ws, dtype=torch.uint8, device="cuda") for _ in range(2)]
+    stream = torch.cuda.current_stream().cuda_stream
+    want = ens().run_text(text(lines))
+    runs = [_ens.Run.launch("auto", args, cfg, b.data_ptr(), ws, stream, keep=b) for b in bufs]
+    for run in runs:
+        for _ in range(2):
+            got = run.collect()
+            for f in FIELDS:
+                assert all(same(got.records[k][f], want.records[k][f], f) for k in range(len(lines))), f
+            assert got.stdout == want.stdout
+            assert np.array_equal(got.tallies, want.tallies)
+        run.close()
