@@ -57,9 +57,14 @@ enum {
 enum {
   ENS_F_TIMESTAMPS = 1u << 0, /* fill smid / t_start_ns / t_end_ns in records  */
   ENS_F_PHASES = 1u << 1,     /* accumulate per-phase device time (tracing)    */
-  ENS_F_GENERIC = 1u << 2     /* bodies take their general paths only (no fast
+  ENS_F_GENERIC = 1u << 2,    /* bodies take their general paths only (no fast
                                  paths such as XS's warp-per-nuclide unionized
                                  init): results are identical — for testing   */
+  ENS_F_SERIAL = 1u << 3      /* mixed-app ensembles: launch the per-app kernels
+                                 one after another on one shared arena (the
+                                 default gives each its own arena region, when
+                                 they fit, and runs them concurrently on forked
+                                 streams so one's tail overlaps the next)      */
 };
 #define ENS_PHASES 16
 

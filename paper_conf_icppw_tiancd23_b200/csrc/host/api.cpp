@@ -177,6 +177,7 @@ struct Group {
   std::vector<uint32_t> kmap;
   std::vector<double> cost;  // app_cost per kmap entry (schedule only)
   size_t kmap_off = 0;
+  size_t arena_off = 0;  // this group's arena region (offset from o_arena)
 };
 
 struct Plan {  // workspace layout (byte offsets) and groups
@@ -184,6 +185,7 @@ struct Plan {  // workspace layout (byte offsets) and groups
   uint32_t stdout_cap = 4096;
   uint64_t arena_bytes = 0;
   int slots = 0;
+  bool concurrent = false;  // groups on forked streams, each with its own arena region
   std::vector<Group> groups;
   std::vector<uint32_t> line_of_k;
   // staged (H2D) part
@@ -211,6 +213,7 @@ struct ens_run {
   std::vector<uint64_t> c_off;
   std::string c_text;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
+  std::vector<cudaEvent_t> ev_join;  // concurrent groups: one per forked group
   uint32_t flags = 0;
   bool launched = false;
   uint64_t d2h = 0;
@@ -271,6 +274,24 @@ cudaError_t d2h_copy(void *dst, const void *src, size_t bytes) {
   e = cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToHost, st);
   if (e != cudaSuccess) return e;
   return cudaStreamSynchronize(st);
+}
+
+// Forked launch streams for concurrent groups: (device, index) -> a
+// non-blocking stream, created once per process.
+cudaError_t aux_stream(size_t i, cudaStream_t *out) {
+  static std::mutex mu;
+  static cudaStream_t streams[64][ENS_N_APPS] = {};
+  int dev = 0;
+  cudaError_t e = cudaGetDevice(&dev);
+  if (e != cudaSuccess) return e;
+  if (dev < 0 || dev >= 64 || i >= (size_t)ENS_N_APPS) return cudaErrorInvalidValue;
+  std::lock_guard<std::mutex> lk(mu);
+  if (!streams[dev][i]) {
+    e = cudaStreamCreateWithFlags(&streams[dev][i], cudaStreamNonBlocking);
+    if (e != cudaSuccess) return e;
+  }
+  *out = streams[dev][i];
+  return cudaSuccess;
 }
 
 void pin_put(char *p, size_t cap) {
@@ -464,6 +485,21 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   }
   P.slots = want;
   P.total = o + (size_t)want * P.arena_bytes;
+  // several groups: give each its own arena region (slots x arena_bytes) so
+  // their kernels may run concurrently, when that fits the workspace cap
+  if (P.groups.size() > 1 && !(c->flags & ENS_F_SERIAL)) {
+    size_t off = 0;
+    for (const Group &g : P.groups) off += (size_t)g.grid * P.arena_bytes;
+    if (!mem_cap || o + off <= mem_cap) {
+      off = 0;
+      for (Group &g : P.groups) {
+        g.arena_off = off;
+        off += (size_t)g.grid * P.arena_bytes;
+      }
+      P.concurrent = true;
+      P.total = o + off;
+    }
+  }
   return ENS_OK;
 }
 
@@ -505,13 +541,22 @@ static int enqueue(ens_run *r) {
     k.stdout_base = r->ws + P.o_out;
     k.stdout_cmp = r->ws + P.o_cmp;
     k.stdout_cap = P.stdout_cap;
-    k.arena_base = r->ws + P.o_arena;
     k.arena_bytes = P.arena_bytes;
     k.team_ctas = (uint32_t)g.cs;
     k.phases = (r->flags & ENS_F_PHASES) ? (unsigned long long *)(r->ws + P.o_phase) : nullptr;
     k.sub_stride = g.sub;
-    cudaError_t e = launch_group(g.app, g.T, g.m, g.ctas(), g.cs, g.dyn(), k, r->stream);
+    k.arena_base = r->ws + P.o_arena + g.arena_off;
+    cudaStream_t st = r->stream;
+    if (P.concurrent && gi > 0) {  // fork: group gi on an aux stream after ev0
+      CU(aux_stream(gi - 1, &st));
+      CU(cudaStreamWaitEvent(st, r->ev0, 0));
+    }
+    cudaError_t e = launch_group(g.app, g.T, g.m, g.ctas(), g.cs, g.dyn(), k, st);
     if (e != cudaSuccess) return cuda_fail(e, "ens_kernel launch");
+    if (P.concurrent && gi > 0) {  // join back into the launch stream
+      CU(cudaEventRecord(r->ev_join[gi - 1], st));
+      CU(cudaStreamWaitEvent(r->stream, r->ev_join[gi - 1], 0));
+    }
   }
   CU(cudaEventRecord(r->ev1, r->stream));
   r->launched = true;
@@ -550,6 +595,12 @@ extern "C" int ens_launch(ens_app app, const ens_args *a, const ens_launch_cfg *
   }
   cudaError_t e = cudaEventCreate(&r->ev0);
   if (e == cudaSuccess) e = cudaEventCreate(&r->ev1);
+  if (P.concurrent)
+    for (size_t gi = 1; gi < P.groups.size() && e == cudaSuccess; gi++) {
+      cudaEvent_t ej = nullptr;
+      e = cudaEventCreateWithFlags(&ej, cudaEventDisableTiming);
+      if (e == cudaSuccess) r->ev_join.push_back(ej);
+    }
   if (e != cudaSuccess) {
     ens_run_free(r);
     return cuda_fail(e, "cudaEventCreate");
@@ -755,6 +806,7 @@ extern "C" void ens_run_free(ens_run *r) {
   pin_put(r->h_stage, r->h_stage_cap);
   if (r->ev0) cudaEventDestroy(r->ev0);
   if (r->ev1) cudaEventDestroy(r->ev1);
+  for (cudaEvent_t ej : r->ev_join) cudaEventDestroy(ej);
   delete r;
 }
 

@@ -139,3 +139,16 @@ def test_runs_in_flight_on_one_stream():
             assert got.stdout == want.stdout
             assert np.array_equal(got.tallies, want.tallies)
         run.close()
+
+
+def test_concurrent_groups_equal_serial():
+    """A mixed-app ensemble runs its per-app kernels concurrently on forked streams, each
+    with its own arena region; ENS_F_SERIAL runs them one after another on one shared
+    arena: the records, tallies and stdout are the same."""
+    lines = LINES * 9
+    a = ens().run_text(text(lines))
+    b = ens().run_text(text(lines), serial=True)
+    for f in FIELDS:
+        assert all(same(a.records[k][f], b.records[k][f], f) for k in range(len(lines))), f
+    assert a.stdout == b.stdout
+    assert np.array_equal(a.tallies, b.tallies)
