@@ -76,7 +76,12 @@ ENS_HD PrLayout pr_layout(const PrParams &p) {
 
 // ============================ XSBench-style ================================
 enum { XS_UNIONIZED = 0, XS_NUCLIDE = 1, XS_HASH = 2 };
-constexpr int kXsMaxGp = 16384;  // per-nuclide sort fits one SM's shared memory
+// -g range (reading R-xs-range): 2 <= n_gp <= 2^16, the oracle's bound since
+// its first commit; every per-nuclide grid index then fits 16 bits
+constexpr int kXsMaxGp = 65536;
+// hash / nuclide init: one nuclide's sort keys (6 B each) and bucket counters
+// sit in shared memory up to this n_gp, in per-CTA arena scratch above it
+constexpr int kXsSmemGp = 16384;
 
 struct XsParams {
   int n_iso = 355;
@@ -181,6 +186,15 @@ ENS_HD long long xs_buckets(const XsParams &p) {
 ENS_HD int xs_nbn(int n_gp) {
   return pow2_ceil(n_gp) / ENS_XS_NBN_DIV > 0 ? pow2_ceil(n_gp) / ENS_XS_NBN_DIV : 1;
 }
+// hash / nuclide grids: the per-nuclide sort runs in shared memory
+ENS_HD bool xs_nuc_smem(const XsParams &p) { return p.n_gp <= kXsSmemGp; }
+// bytes of per-CTA arena scratch of the per-nuclide sort when it does not fit
+// shared memory: [nbn] u32 counters | [n_gp] u32 keys | [n_gp] u16 record ids
+ENS_HD uint64_t xs_nscr_bytes(const XsParams &p) {
+  if (p.grid == XS_UNIONIZED || xs_nuc_smem(p)) return 0;
+  return align_up((uint64_t)xs_nbn(p.n_gp) * 4, 256) + align_up((uint64_t)p.n_gp * 4, 256) +
+         align_up((uint64_t)p.n_gp * 2, 256);
+}
 // bins of the union search table: ufind[b] = #{k >= 1 : u_k <= b / ubins}
 // (power of two, ~1 union energy per bin), so the union position of energy
 // p is ufind[floor(p * ubins)] plus a short forward scan — the same index as
@@ -237,6 +251,7 @@ struct XsLayout {
   uint64_t ustart;    // unionized, warp path: [NC+1][iso_pad] i32 #{k: E_i[k] < ch/NC}
   uint64_t index;     // unionized [n_u][xs_iso_pad] int32 / hash [n_iso][bins+1] XsHashEnt
   uint64_t hcol;      // hash: [cs][bins+1] int32 column being built
+  uint64_t nscr;      // hash / nuclide, n_gp > kXsSmemGp: [cs] x xs_nscr_bytes per-nuclide sort scratch
   uint64_t lk_pe;     // event mode: [chunk] lookup energies sorted by (material, energy)
   uint64_t lk_hist;   // event mode: [(12 << kb) + 1] u32 (material, energy) bucket counts -> cursors
   uint64_t total;
@@ -255,8 +270,8 @@ ENS_HD int xs_lk_bits(long long n_c) {
   return kb;
 }
 // hash index entry (a private accelerator; results are unchanged): the
-// upstream index u_low = ig[b][i], u_high = ig[b+1][i] + 1 (n_gp <= 16384
-// fits 16 bits) and the energies E[u_low+1..u_low+6] quantized within bin b,
+// upstream index u_low = ig[b][i], u_high = ig[b+1][i] + 1 (n_gp <= 65536:
+// u_high <= n_gp - 1 fits 16 bits) and the energies E[u_low+1..u_low+6] quantized within bin b,
 // q = floor((E*bins - b) * 2^16) clamped to [0, 65535] (65535 also past the
 // grid), stored as q >> 1 (15 bits: the lookup compares six at once, SWAR).
 // q is monotone in E, so #{k: q(pe) > q_k} never exceeds the number of those
@@ -288,6 +303,7 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
     L.index = o; o = align_up(o + (uint64_t)p.n_iso * (p.bins + 1) * 16, 256);
     L.hcol = o; o = align_up(o + (uint64_t)cs * (p.bins + 1) * 4, 256);
   }
+  if (p.grid != XS_UNIONIZED) { L.nscr = o; o = align_up(o + (uint64_t)cs * xs_nscr_bytes(p), 256); }
   if (!p.history) {
     const long long n_c = xs_lk_chunk(p);
     L.lk_pe = o; o = align_up(o + (uint64_t)n_c * 8, 256);
@@ -318,15 +334,15 @@ ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   S.concs = o; o += 12 * mx * 8;          // concentrations
   S.mats = o; o += (uint32_t)align_up(12 * mx * 2, 16);  // nuclide ids (u16)
   S.mcnt = o; o += 32 * 4;                // material counts / offsets of a lookup chunk
-  S.jmp = o; o += 4 * 64 * 16;            // LCG jump tables: A^(6 d 64^l), l < 4, d < 64
+  S.jmp = o; o += 5 * 64 * 16;            // LCG jump tables: A^(6 d 64^l), l < 5, d < 64
   S.nbkt = o;  // per-nuclide sort buckets (hash / nuclide grids); unionized: per-warp sweep rows
-  if (p.grid != XS_UNIONIZED) o += (uint32_t)align_up((uint64_t)xs_nbn(p.n_gp) * 4, 16);
+  if (p.grid != XS_UNIONIZED) o += xs_nuc_smem(p) ? (uint32_t)align_up((uint64_t)xs_nbn(p.n_gp) * 4, 16) : 0u;
   else o += (uint32_t)(T / 32) * 2u * (uint32_t)xs_iso_pad(p.n_iso) * 4u;
   S.ubkt = o;  // unionized, small: bucket counters, then chunk owner counts
   if (xs_smem_nb(p)) o += (uint32_t)kXsSmemBkt * 4u;
   // hash / nuclide grids: one nuclide's u32 sort keys and u16 record indices
   S.nkey = o;
-  if (p.grid != XS_UNIONIZED) {
+  if (p.grid != XS_UNIONIZED && xs_nuc_smem(p)) {
     o += (uint32_t)align_up((uint64_t)p.n_gp * 6, 16);
     // the hash column + quantization keys reuse [nbkt, total) after the sort;
     // grow the region by up to 16 KB so that they fit (else arena scratch)

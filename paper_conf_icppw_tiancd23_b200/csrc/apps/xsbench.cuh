@@ -184,7 +184,7 @@ struct XsApp {
     hm_tables(n_iso, mx, thr, nn, concs, mats);
     {  // LCG jump tables for XS-3's record draws (see jump6)
       Affine *jt = (Affine *)(ens_smem(c) + S.jmp);
-      for (int x = threadIdx.x; x < 256; x += blockDim.x)
+      for (int x = threadIdx.x; x < 320; x += blockDim.x)
         jt[x] = lcg_pow((6ULL * (uint64_t)(x & 63)) << (6 * (x >> 6)));
     }
     __syncthreads();
@@ -222,12 +222,15 @@ struct XsApp {
 
   // the LCG state s advanced by 6r draws (record r's draws are 6r+1..6r+6,
   // XS-3), from the smem tables jt[64 l + d] = A^(6 d 64^l): four affine
-  // steps instead of a 6r-step walk (r < 2^24)
+  // steps instead of a 6r-step walk, a fifth for r >= 2^24 (n_u <= 355 *
+  // 65536 < 2^30)
   __device__ static __forceinline__ uint64_t jump6(const Affine *jt, uint32_t r, uint64_t s) {
     s = jt[r & 63u](s);
     s = jt[64 + ((r >> 6) & 63u)](s);
     s = jt[128 + ((r >> 12) & 63u)](s);
-    return jt[192 + ((r >> 18) & 63u)](s);
+    s = jt[192 + ((r >> 18) & 63u)](s);
+    if (r >> 24) s = jt[256 + ((r >> 24) & 63u)](s);
+    return s;
   }
   // record r at dst: E (the key's energy, draw 6r+1) and draws 6r+2..6r+6
   __device__ static __forceinline__ void put_record(const Affine *jt, uint32_t r, unsigned long long ebits,
@@ -341,17 +344,27 @@ struct XsApp {
   // is written once in sorted order (coalesced) with its draws 6r+2..6r+6
   // re-generated, and (hash) the nuclide's index column is built by a merge
   // walk over the sorted energies, each bin written once (XS-5: ig[i][b] = grid_search(E_i, b*du) = min(#{k>=1: E_k <= b*du}, n_gp-2)).
-  __device__ static __noinline__ void init_nuc(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
+  // SMK: the sort's keys and counters in shared memory (n_gp <= kXsSmemGp),
+  // else in this CTA's arena scratch (L2 atomics; the same algorithm)
+  __device__ static void init_nuc(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
+    if (xs_nuc_smem(p)) init_nuc_t<true>(c, p, L, S);
+    else init_nuc_t<false>(c, p, L, S);
+  }
+  template <bool SMK>
+  __device__ static __noinline__ void init_nuc_t(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
     const bool trc = tracing(c);  // tracing (ENS_F_PHASES) thread, cached
     const int tid = threadIdx.x, T = blockDim.x;
     const int n_iso = p.n_iso, n_gp = p.n_gp;
     const int nbn = xs_nbn(n_gp);
-    uint32_t *nb = (uint32_t *)(ens_smem(c) + S.nbkt);
+    char *gscr = c.arena + L.nscr + (size_t)c.crank * xs_nscr_bytes(p);
+    uint32_t *nb = SMK ? (uint32_t *)(ens_smem(c) + S.nbkt) : (uint32_t *)gscr;
     const Affine *jt = (const Affine *)(ens_smem(c) + S.jmp);
     double *recs = (double *)(c.arena + L.recs);
     unsigned long long *ekey = (unsigned long long *)(c.arena + L.keys);  // sorted energies (this CTA's)
-    uint32_t *K = (uint32_t *)(ens_smem(c) + S.nkey);                     // sort keys, then
-    uint16_t *J = (uint16_t *)(ens_smem(c) + S.nkey + (size_t)n_gp * 4);  // record indices j
+    const size_t kofs = SMK ? 0 : align_up((uint64_t)nbn * 4, 256);
+    uint32_t *K = SMK ? (uint32_t *)(ens_smem(c) + S.nkey) : (uint32_t *)(gscr + kofs);  // sort keys, then
+    uint16_t *J = SMK ? (uint16_t *)(ens_smem(c) + S.nkey + (size_t)n_gp * 4)            // record indices j
+                      : (uint16_t *)(gscr + kofs + align_up((uint64_t)n_gp * 4, 256));
     int *ig = (int *)(c.arena + L.index);
     const bool hash = p.grid == XS_HASH;
     int kbits = 0;

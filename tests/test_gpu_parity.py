@@ -27,6 +27,16 @@ XS_CASES = [
     # hash column in shared memory (fits) vs the arena scratch (bins >= 2^16)
     "xsbench -s small -g 11303 -l 3000 -G hash -h 10000 -r 13",
     "xsbench -s small -g 3000 -l 2000 -G hash -h 70000 -r 12",
+    # n_gp above the shared-memory per-nuclide sort (kXsSmemGp = 16384): keys and
+    # counters in arena scratch; up to the -g bound 65536 (reading R-xs-range)
+    "xsbench -s small -g 20000 -l 3000 -G hash -h 1000 -r 21",
+    "xsbench -s small -g 20000 -l 3000 -G nuclide -r 22",
+    "xsbench -s small -g 20000 -l 3000 -G unionized -r 23",
+    "xsbench -s small -g 65536 -l 2000 -G hash -h 5000 -r 24",
+    "xsbench -s small -g 65536 -l 2000 -G unionized -r 25",
+    "xsbench -s small -g 16385 -l 1000 -m history -p 20 -G hash -h 300 -r 26",
+    # r >= 2^24 records (the fifth jump-table level): 355 * 50000 = 17.75 M records
+    "xsbench -s large -g 50000 -l 1000 -G hash -h 2000 -r 27",
 ]
 
 RS_CASES = [
@@ -51,6 +61,7 @@ MISC_CASES = [
     "echo a b  c",
     "nosuchapp -x 1",
     "xsbench -g 1",
+    "xsbench -g 65537",
     "xsbench -s tiny",
     "xsbench -l",
     "rsbench -q",

@@ -128,8 +128,19 @@ def test_grid_types_agree_bitwise(oracle):
 
 
 @pytest.mark.parametrize("line", ["-s medium", "-g 1", "-g", "-l -5", "-G sorted", "-m hist", "-q 1",
-                                  "-g 12x", "-r -1", "-h 0"])
+                                  "-g 12x", "-r -1", "-h 0", "-g 65537"])
 def test_usage_errors(oracle, line):
     r = oracle.run_text(line + "\n", app=oracle.APP_XSBENCH)
     assert r.records[0]["exit_code"] == 1
     assert b"invalid argument" in r.stdout[0] and b"usage: xsbench" in r.stdout[0]
+
+
+def test_gp_range_upper_bound(oracle):
+    """Reading R-xs-range: -g up to 2^16 is a valid line (the oracle's bound since its first
+    commit); a run at the bound keeps the XS-10 invariants."""
+    L = 300
+    r = oracle.run_text(f"-s small -g 65536 -l {L} -G hash -h 100 -r 5\n", app=oracle.APP_XSBENCH)
+    rec, tal = r.records[0], r.tallies[0]
+    assert rec["exit_code"] == 0 and rec["work"] == L
+    ver = sum((c + 1) * int(tal[c]) for c in range(5))
+    assert L <= ver <= 5 * L and int(rec["vhash"]) == ver % 999983
