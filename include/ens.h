@@ -142,6 +142,17 @@ typedef struct {
                          instance keeps >= 32 threads); 0 = 1.  Applies to the
                          bodies built for it (AMGmk, Page-Rank, echo, unknown
                          programs) with team_ctas == 1; ignored by others.    */
+  uint32_t dump_rows; /* element-wise result dump (testing): 0 = off; else each
+                         instance writes up to dump_rows result rows of 8
+                         doubles {key, material, v[0..4], argmax} into the
+                         workspace, read back with ens_collect_dump.  XS / RS
+                         event lookups: one row per lookup (key = its energy,
+                         v = the macroscopic cross sections of XS-9 / RS-3,
+                         argmax of XS-10 / RS-3), in the kernel's (sorted)
+                         lookup order, the first dump_rows slots; AMG: rows
+                         0..dump_rows-1 of the reported vector (key = row
+                         index, v[0] = value, argmax = -1).  Unwritten rows
+                         are all zero.  Results never depend on it.           */
 } ens_launch_cfg;
 
 /* Device bytes ens_launch needs for (app, a, c).  With c->grid_blocks == 0
@@ -194,6 +205,13 @@ typedef struct {
  * the run's host copy (tallies are copied on the first call that asks).      */
 int ens_collect(ens_run *r, ens_record *recs, uint32_t *tallies, char *stdout_buf, size_t cap,
                 uint64_t *stdout_off);
+
+/* Element-wise dump of the last (re)launch (cfg.dump_rows > 0): copies
+ * n x dump_rows x 8 doubles (row layout: see ens_launch_cfg.dump_rows), for
+ * record slot k at out + k*dump_rows*8.  cap = doubles available at out;
+ * ENS_ERANGE if smaller, ENS_EINVAL if the run was launched without a dump.
+ * Blocks until the run's kernels are done.                                   */
+int ens_collect_dump(ens_run *r, double *out, size_t cap);
 
 /* CUDA-event time of the last (re)launch's kernels, in ms.                   */
 int ens_run_elapsed_ms(ens_run *r, float *ms);

@@ -164,6 +164,7 @@ void run_amgmk(const std::vector<std::string> &argv, Instance &inst) {
     fabs_ += std::fabs(R[(size_t)i]);
     double e = std::fabs(R[(size_t)i] - (in.kind == 0 ? 1.0 : f[(size_t)i]));
     if (e > maxerr) maxerr = e;
+    if ((size_t)i < inst.dump_cap) note_result(inst, (double)i, 0, &R[(size_t)i], 1, -1);
   }
   inst.rec.vhash = bitsum % 999983ULL;
   inst.rec.bitsum = bitsum;

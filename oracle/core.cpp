@@ -1,5 +1,6 @@
 // oracle/core.cpp — TEST INFRASTRUCTURE ONLY (see oracle.hpp header).
 // Args-file loader, shared primitives, echo body, instance dispatch.
+#include <cmath>
 #include "oracle.hpp"
 
 #include <cstdarg>
@@ -160,6 +161,20 @@ bool parse_long(const std::string &s, long long *v) {
   return true;
 }
 
+void note_result(Instance &inst, double key, int mat, const double *v, int nv, int argmax) {
+  if (argmax >= 0 && nv > 1) {  // argmax margin: v[argmax] minus the largest other channel
+    double second = -1.0 / 0.0;
+    for (int c = 0; c < nv; c++)
+      if (c != argmax && v[c] > second) second = v[c];
+    const double m = (v[argmax] - second) / std::fabs(v[argmax]);
+    if (m < inst.min_margin) inst.min_margin = m;
+  }
+  if (inst.dump.size() / 8 >= inst.dump_cap) return;
+  double row[8] = {key, (double)mat, 0, 0, 0, 0, 0, (double)argmax};
+  for (int c = 0; c < nv && c < 5; c++) row[2 + c] = v[c];
+  inst.dump.insert(inst.dump.end(), row, row + 8);
+}
+
 uint64_t dbits(double d) {
   uint64_t u;
   std::memcpy(&u, &d, 8);
@@ -189,7 +204,9 @@ static uint32_t app_of_argv0(const std::string &a0) {
 }
 
 void run_isolated(uint32_t app, const std::vector<std::string> &argv, Instance &inst) {
+  const size_t dump_cap = inst.dump_cap;  // the caller's request survives the reset
   inst = Instance();
+  inst.dump_cap = dump_cap;
   if (app == APP_BY_ARGV0) {
     app = argv.empty() ? (uint32_t)APP_BY_ARGV0 : app_of_argv0(argv[0]);
     if (app == APP_BY_ARGV0) {

@@ -61,7 +61,17 @@ struct Instance {
   Record rec{};
   uint32_t tallies[kTallies] = {0};
   std::string out;  // stdout bytes
+  // Element-wise results (tests only): the first dump_cap result vectors of
+  // the run as rows of 8 doubles {key, material, v[0..4], argmax}: XS / RS
+  // lookups in index order (key = the lookup's energy), AMG rows of the
+  // reported vector (key = row index).  min_margin = the smallest relative
+  // argmax margin (max - runner-up) / |max| over every lookup (XS-10 / RS-3).
+  size_t dump_cap = 0;
+  std::vector<double> dump;
+  double min_margin = 1.0 / 0.0;
 };
+// append one dump row (if dump_cap allows) and fold the lookup's argmax margin
+void note_result(Instance &inst, double key, int mat, const double *v, int nv, int argmax);
 
 // LCG of SURVEY.md §8(c) "Shared primitives" (upstream XSBench/RSBench).
 uint64_t lcg_step(uint64_t s);

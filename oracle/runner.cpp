@@ -23,6 +23,7 @@ void set_conc_seed(uint64_t s);
 }  // namespace xs_hooks
 namespace rs_hooks {
 void fast_w(double zr, double zi, double *wr, double *wi);
+double trig_eval(int kind, double x);
 void init_tables(int small, int avg_poles, int avg_windows, uint64_t iseed, std::vector<int> &n_poles,
                  std::vector<int> &n_windows, std::vector<int> &win_start, std::vector<int> &win_end);
 void dump_and_micro(int small, int avg_poles, int avg_windows, uint64_t iseed, int doppler, int n,
@@ -42,9 +43,10 @@ struct Run {
   std::vector<Instance> inst;
 };
 
-Run *run_ensemble(const Args &args, uint32_t app, long n, int jobs) {
+Run *run_ensemble(const Args &args, uint32_t app, long n, int jobs, size_t dump_cap) {
   Run *r = new Run();
   r->inst.resize((size_t)n);
+  for (Instance &I : r->inst) I.dump_cap = dump_cap;
   std::atomic<long> next(0);
   auto worker = [&]() {
     for (;;) {
@@ -62,6 +64,7 @@ Run *run_ensemble(const Args &args, uint32_t app, long n, int jobs) {
   for (auto &t : th) t.join();
   return r;
 }
+Run *run_ensemble(const Args &args, uint32_t app, long n, int jobs) { return run_ensemble(args, app, n, jobs, 0); }
 
 }  // namespace oracle
 
@@ -78,6 +81,21 @@ void *oracle_run(const char *text, size_t len, const char *argv0, uint32_t app, 
   if (n > (long)a.lines.size()) return nullptr;
   return run_ensemble(a, app, n, jobs);
 }
+// the same with element-wise dumps of the first dump_cap results per instance
+void *oracle_run_dump(const char *text, size_t len, const char *argv0, uint32_t app, long n, int jobs,
+                      long dump_cap) {
+  Args a = parse_args_text(std::string(text, len), argv0);
+  if (n < 0) n = (long)a.lines.size();
+  if (n > (long)a.lines.size() || dump_cap < 0) return nullptr;
+  return run_ensemble(a, app, n, jobs, (size_t)dump_cap);
+}
+// dump rows of instance i (8 doubles each) into out (may be NULL); returns the row count
+long oracle_dump(void *h, long i, double *out) {
+  const std::vector<double> &d = ((Run *)h)->inst[(size_t)i].dump;
+  if (out) std::memcpy(out, d.data(), d.size() * 8);
+  return (long)(d.size() / 8);
+}
+double oracle_margin(void *h, long i) { return ((Run *)h)->inst[(size_t)i].min_margin; }
 long oracle_count(void *h) { return (long)((Run *)h)->inst.size(); }
 void oracle_records(void *h, Record *out) {
   Run *r = (Run *)h;
@@ -165,6 +183,10 @@ void oracle_xs_set_conc_seed(uint64_t s) { xs_hooks::set_conc_seed(s); }
 
 // ---- RS hooks ----------------------------------------------------------------
 void oracle_rs_fast_w(double zr, double zi, double *wr, double *wi) { rs_hooks::fast_w(zr, zi, wr, wi); }
+// RS-3's sin (kind 0), cos (1), atan (2) at n points (reading R-rs-trig)
+void oracle_rs_trig(int kind, long n, const double *x, double *y) {
+  for (long k = 0; k < n; k++) y[k] = rs_hooks::trig_eval(kind, x[k]);
+}
 // RS-3 micro cross sections at n (nuc, E) points plus the flattened tables
 // (9 doubles per pole, 3 per window, 4 K0RS per nuclide); returns 0, or -1
 // if a table exceeds its capacity (in doubles)

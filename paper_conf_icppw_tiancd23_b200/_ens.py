@@ -43,7 +43,8 @@ class LaunchCfg(ctypes.Structure):
     _fields_ = [("first", ctypes.c_int32), ("n_instances", ctypes.c_int32), ("stride", ctypes.c_int32),
                 ("grid_blocks", ctypes.c_int32), ("block_threads", ctypes.c_int32),
                 ("arena_bytes", ctypes.c_uint64), ("stdout_bytes", ctypes.c_uint32), ("flags", ctypes.c_uint32),
-                ("team_ctas", ctypes.c_int32), ("instances_per_cta", ctypes.c_int32)]
+                ("team_ctas", ctypes.c_int32), ("instances_per_cta", ctypes.c_int32),
+                ("dump_rows", ctypes.c_uint32)]
 
 
 class RunInfo(ctypes.Structure):
@@ -75,6 +76,7 @@ def _load():
         "ens_launch": (i, [i, p, ctypes.POINTER(LaunchCfg), p, sz, p, pp]),
         "ens_run_relaunch": (i, [p, p]),
         "ens_collect": (i, [p, p, p, p, sz, p]),
+        "ens_collect_dump": (i, [p, p, sz]),
         "ens_run_elapsed_ms": (i, [p, ctypes.POINTER(ctypes.c_float)]),
         "ens_run_phases": (i, [p, ctypes.POINTER(ctypes.c_uint64)]),
         "ens_run_get_info": (i, [p, ctypes.POINTER(RunInfo)]),
@@ -93,7 +95,8 @@ def _load():
 
 lib = _load()
 EXPORTED = ["ens_load_args", "ens_parse_args", "ens_expand_args", "ens_args_count", "ens_args_get", "ens_args_free",
-            "ens_workspace_bytes", "ens_launch", "ens_run_relaunch", "ens_collect", "ens_run_elapsed_ms",
+            "ens_workspace_bytes", "ens_launch", "ens_run_relaunch", "ens_collect", "ens_collect_dump",
+            "ens_run_elapsed_ms",
             "ens_run_phases",
             "ens_run_get_info", "ens_format_stdout", "ens_run_free", "ens_strerror", "ens_last_error",
             "ens_version"]
@@ -157,9 +160,9 @@ class Args:
 
 
 def make_cfg(n, first=0, stride=1, grid=0, threads=0, arena_bytes=0, stdout_bytes=0, flags=0, team_ctas=0,
-             instances_per_cta=0):
+             instances_per_cta=0, dump_rows=0):
     return LaunchCfg(first, n, stride, grid, threads, arena_bytes, stdout_bytes, flags, team_ctas,
-                     instances_per_cta)
+                     instances_per_cta, dump_rows)
 
 
 def workspace_bytes(app, args, cfg):
@@ -210,6 +213,13 @@ class Run:
         else:
             _check("ens_collect", lib.ens_collect(self._h, rp, tp, None, 0, op))
         return Collected(recs, tal, outs)
+
+    def collect_dump(self, dump_rows):
+        """Element-wise result rows [n, dump_rows, 8] (launched with dump_rows > 0)."""
+        d = np.zeros((self.n, dump_rows, 8))
+        _check("ens_collect_dump", lib.ens_collect_dump(self._h, d.ctypes.data_as(ctypes.c_void_p) if d.size else None,
+                                                        d.size))
+        return d
 
     def elapsed_ms(self):
         ms = ctypes.c_float()

@@ -124,6 +124,7 @@ struct AmgApp {
       fabs_ += fabs(v);
       const double e = fabs(v - (p.kind == 0 ? 1.0 : ld_(f + r)));
       if (e > mxe) mxe = e;
+      if (c.dump) dump_row(c.dump, c.dump_rows, r, (double)r, 0, &v, 1, -1);
     }
     bsum = block_sum_u64(ens_sh(c), bsum);
     fsum = block_sum_f64(ens_sh(c), fsum);

@@ -1429,6 +1429,8 @@ struct XsApp {
       team_sync(c);
       phase_mark_if(trc, c, 10);
       // (D) thread-per-lookup over the sorted chunk
+      double *const dmp = c.dump;
+      const uint32_t drows = c.dump_rows;
       for (long long sl = g0; sl < nc; sl += gs) {
         int mat = 0;
 #pragma unroll
@@ -1453,6 +1455,7 @@ struct XsApp {
         if (m4 > mxv) { mxv = m4; am = 4; }
         ver += (unsigned long long)(am + 1);
         atomicAdd(&ens_sh(c)->tallies[am], 1u);
+        if (dmp) dump_row(dmp, drows, c0 + sl, pe, mat, mv, 5, am);
         bsum += dbits(m0) + dbits(m1) + dbits(m2) + dbits(m3) + dbits(m4);
         fsum += m0; fsum += m1; fsum += m2; fsum += m3; fsum += m4;
         fabs_ += fabs(m0); fabs_ += fabs(m1); fabs_ += fabs(m2); fabs_ += fabs(m3); fabs_ += fabs(m4);

@@ -191,7 +191,8 @@ struct Plan {  // workspace layout (byte offsets) and groups
   // staged (H2D) part
   size_t o_blob = 0, o_tok = 0, o_line = 0, o_lok = 0, o_kmap = 0, staged = 0;
   // zeroed part: counters (n_groups + 1 u64 stdout total), recs, pos
-  size_t o_ctr = 0, o_recs = 0, o_pos = 0, o_phase = 0, zeroed_end = 0;
+  size_t o_ctr = 0, o_recs = 0, o_pos = 0, o_phase = 0, o_dump = 0, zeroed_end = 0;
+  uint32_t dump_rows = 0;
   size_t o_tal = 0, o_out = 0, o_cmp = 0, o_arena = 0, total = 0;
 };
 
@@ -463,6 +464,8 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   P.o_recs = o; o = al(o + (size_t)n * sizeof(ens_record));
   P.o_pos = o; o = al(o + (size_t)n * 8);
   P.o_phase = o; o = al(o + ENS_PHASES * 8);
+  P.dump_rows = c->dump_rows;
+  P.o_dump = o; o = al(o + (size_t)n * c->dump_rows * 64);  // unwritten rows read as zero
   P.zeroed_end = o;
   P.o_tal = o; o = al(o + (size_t)n * ENS_TALLIES * 4);
   P.o_out = o; o = al(o + (size_t)n * P.stdout_cap);
@@ -546,6 +549,8 @@ static int enqueue(ens_run *r) {
     k.phases = (r->flags & ENS_F_PHASES) ? (unsigned long long *)(r->ws + P.o_phase) : nullptr;
     k.sub_stride = g.sub;
     k.arena_base = r->ws + P.o_arena + g.arena_off;
+    k.dump = P.dump_rows ? (double *)(r->ws + P.o_dump) : nullptr;
+    k.dump_rows = P.dump_rows;
     cudaStream_t st = r->stream;
     if (P.concurrent && gi > 0) {  // fork: group gi on an aux stream after ev0
       CU(aux_stream(gi - 1, &st));
@@ -737,6 +742,18 @@ extern "C" int ens_collect(ens_run *r, ens_record *recs, uint32_t *tallies, char
     if (cap < text.size()) return fail(ENS_ERANGE, "ens_collect: stdout buffer too small");
     std::memcpy(stdout_buf, text.data(), text.size());
   }
+  return ENS_OK;
+}
+
+extern "C" int ens_collect_dump(ens_run *r, double *out, size_t cap) {
+  if (!r || (!out && cap)) return fail(ENS_EINVAL, "ens_collect_dump: NULL");
+  const Plan &P = r->P;
+  if (!P.dump_rows) return fail(ENS_EINVAL, "ens_collect_dump: launched with dump_rows = 0");
+  const size_t want = (size_t)P.n * P.dump_rows * 8;
+  if (cap < want) return fail(ENS_ERANGE, "ens_collect_dump: cap < n x dump_rows x 8");
+  if (P.n == 0 || !r->launched) return ENS_OK;
+  CU(cudaEventSynchronize(r->ev1));
+  CU(d2h_copy(out, r->ws + P.o_dump, want * 8));
   return ENS_OK;
 }
 

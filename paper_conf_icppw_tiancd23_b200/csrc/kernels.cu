@@ -106,6 +106,8 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
     c.out = p.stdout_base + (size_t)k * p.stdout_cap;
     c.phases = p.phases;
     c.flags = p.flags;
+    c.dump = p.dump ? p.dump + (size_t)k * p.dump_rows * 8 : nullptr;
+    c.dump_rows = p.dump_rows;
     phase_mark(c, -1);
     Result r{};
     if (App::kTeam || cr == 0) r = App::run(c, argc, s_argv);

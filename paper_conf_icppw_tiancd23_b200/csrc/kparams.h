@@ -29,6 +29,8 @@ struct KParams {
   uint32_t team_ctas;         // CTAs per team (thread-block cluster size)
   unsigned long long *phases; // [ENS_PHASES] ns per phase (ENS_F_PHASES) or null
   uint32_t sub_stride;        // dynamic smem bytes per instance slot of the CTA
+  double *dump;               // [n_instances][dump_rows][8] element-wise results, or null
+  uint32_t dump_rows;
 };
 
 const void *kernel_ptr(uint32_t app, int T);

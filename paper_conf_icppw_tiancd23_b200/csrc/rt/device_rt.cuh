@@ -159,7 +159,21 @@ struct Ctx {
   uint32_t flags;              // launch flags (ENS_F_*)
   unsigned long long *phases;  // tracing: ns per phase, or null
   unsigned long long t_mark;   // tracing: last mark (team thread 0)
+  double *dump;                // element-wise dump rows of this instance (testing), or null
+  uint32_t dump_rows;
 };
+// element-wise dump (ens_launch_cfg.dump_rows): row `slot` = {key, mat,
+// v[0..nv), argmax}, zero-padded to 8 doubles
+__device__ __forceinline__ void dump_row(double *dump, uint32_t rows, long long slot, double key, int mat,
+                                         const double *v, int nv, int argmax) {
+  if (!dump || slot < 0 || slot >= (long long)rows) return;
+  double *d = dump + (size_t)slot * 8;
+  d[0] = key;
+  d[1] = (double)mat;
+#pragma unroll
+  for (int q = 0; q < 5; q++) d[2 + q] = q < nv ? v[q] : 0.0;
+  d[7] = (double)argmax;
+}
 
 // The instance's shared memory, addressed from the dynamic shared-memory
 // symbol: pointers derived from it stay in the shared window after a Ctx

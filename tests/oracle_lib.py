@@ -51,6 +51,9 @@ def lib():
             sig = {
                 "oracle_run": (c_p, [ctypes.c_char_p, c_sz, ctypes.c_char_p, c_u32, c_l, c_i]),
                 "oracle_count": (c_l, [c_p]),
+                "oracle_run_dump": (c_p, [ctypes.c_char_p, c_sz, ctypes.c_char_p, c_u32, c_l, c_i, c_l]),
+                "oracle_dump": (c_l, [c_p, c_l, c_p]),
+                "oracle_margin": (c_d, [c_p, c_l]),
                 "oracle_records": (None, [c_p, c_p]),
                 "oracle_tallies": (None, [c_p, c_p]),
                 "oracle_stdout_len": (c_sz, [c_p, c_l]),
@@ -73,6 +76,7 @@ def lib():
                 "oracle_xs_materials": (c_i, [c_i, c_p, c_p, c_p]),
                 "oracle_xs_set_conc_seed": (None, [c_u64]),
                 "oracle_rs_fast_w": (None, [c_d, c_d, c_p, c_p]),
+                "oracle_rs_trig": (None, [c_i, c_l, c_p, c_p]),
                 "oracle_rs_tables": (c_i, [c_i, c_i, c_i, c_u64, c_p, c_p, c_p, c_p, c_i]),
                 "oracle_rs_micro": (c_i, [c_i, c_i, c_i, c_u64, c_i, c_i, c_p, c_p, c_p, c_p, c_l, c_p, c_l,
                                           c_p, c_l]),
@@ -103,8 +107,11 @@ class OracleRun:
         self.stdout = stdout
 
 
-def run_text(text, app=APP_BY_ARGV0, argv0=None, n=-1, jobs=None):
-    """Run the ensemble defined by args-file `text` on the CPU oracle."""
+def run_text(text, app=APP_BY_ARGV0, argv0=None, n=-1, jobs=None, dump=0):
+    """Run the ensemble defined by args-file `text` on the CPU oracle.  dump > 0 also
+    returns, per instance, its first `dump` result rows (8 doubles: key, material,
+    v[0..4], argmax; see oracle.hpp Instance) in .dumps and the minimum relative
+    argmax margin in .margins."""
     L = lib()
     if isinstance(text, str):
         text = text.encode()
@@ -113,7 +120,7 @@ def run_text(text, app=APP_BY_ARGV0, argv0=None, n=-1, jobs=None):
     a0 = argv0.encode() if argv0 else None
     if jobs is None:
         jobs = os.cpu_count() or 1
-    h = L.oracle_run(text, len(text), a0, app, n, jobs)
+    h = L.oracle_run_dump(text, len(text), a0, app, n, jobs, dump) if dump else L.oracle_run(text, len(text), a0, app, n, jobs)
     if not h:
         raise ValueError("oracle_run: n larger than the number of lines")
     try:
@@ -129,7 +136,17 @@ def run_text(text, app=APP_BY_ARGV0, argv0=None, n=-1, jobs=None):
             b = ctypes.create_string_buffer(ln + 1)
             L.oracle_stdout(h, i, b)
             outs.append(b.raw[:ln])
-        return OracleRun(recs, tal, outs)
+        run = OracleRun(recs, tal, outs)
+        if dump:
+            run.dumps, run.margins = [], np.zeros(cnt)
+            for i in range(cnt):
+                k = L.oracle_dump(h, i, None)
+                d = np.zeros((k, 8))
+                if k:
+                    L.oracle_dump(h, i, _ptr(d))
+                run.dumps.append(d)
+                run.margins[i] = L.oracle_margin(h, i)
+        return run
     finally:
         L.oracle_free(h)
 
@@ -222,6 +239,14 @@ def rs_fast_w(z):
     wr, wi = ctypes.c_double(), ctypes.c_double()
     lib().oracle_rs_fast_w(z.real, z.imag, ctypes.byref(wr), ctypes.byref(wi))
     return complex(wr.value, wi.value)
+
+
+def rs_trig(kind, x):
+    """RS-3's sin / cos / atan (kind 'sin' | 'cos' | 'atan'; reading R-rs-trig) at the points x."""
+    x = np.ascontiguousarray(x, dtype=np.float64)
+    y = np.zeros_like(x)
+    lib().oracle_rs_trig({"sin": 0, "cos": 1, "atan": 2}[kind], x.size, _ptr(x), _ptr(y))
+    return y
 
 
 def rs_tables(small, avg_poles, avg_windows, iseed=42):
