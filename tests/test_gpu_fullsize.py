@@ -70,3 +70,45 @@ def test_c4_sampled(oracle):
     r = run_cfg(lines, 1024)
     assert np.all(r.records["exit_code"] == 0)
     check_sample(oracle, lines, r, [0, 1, 777, 1023])
+
+
+def test_c2_full_elementwise_sample(oracle):
+    """C2 at bench size and launch config: the first 20000 sorted lookup slots of two instances,
+    element by element (bit-exact) against the oracle's per-lookup rows (all 1M, by energy)."""
+    from paper_conf_icppw_tiancd23_b200 import workloads
+    lines = workloads.c2()
+    rows = 20000
+    r = run_cfg(lines, 512, dump_rows=rows)
+    for i in (0, 63):
+        o = oracle.run_text(lines[i] + "\n", dump=1000000)
+        od = o.dumps[0]
+        gd = r.dump[i]
+        gd = gd[~np.all(gd == 0, axis=1)]
+        assert len(gd) == rows
+        pos = np.searchsorted(od[:, 0], gd[:, 0], sorter=np.argsort(od[:, 0]))
+        srt = od[np.argsort(od[:, 0])]
+        hit = srt[pos]
+        assert np.array_equal(hit[:, 0], gd[:, 0]) and np.array_equal(hit[:, 1], gd[:, 1])
+        assert np.array_equal(hit[:, 2:8].view(np.uint64), gd[:, 2:8].view(np.uint64))
+
+
+def test_c5_full_sampled(oracle):
+    """C5: 4096 mixed lines (XS / XS / RS / AMG) at the bench's thread limit, concurrent per-app
+    groups on forked streams with separate arena regions; 16 sampled instances spanning the
+    three apps, the queue's head and tail, against the oracle."""
+    from paper_conf_icppw_tiancd23_b200 import workloads
+    lines = workloads.c5()
+    r = run_cfg(lines, 1024)
+    assert np.all(r.records["exit_code"] == 0)
+    assert np.all(r.records["instance"] == np.arange(4096))
+    check_sample(oracle, lines, r, [0, 1, 2, 3, 1021, 1022, 1023, 1024, 2046, 2047, 2048, 2049, 4092, 4093, 4094, 4095])
+
+
+def test_c2u_full_sampled(oracle):
+    """C2u: 24 x large unionized (5.92 GB of tables each; 142 GB of slot arenas), 1M lookups,
+    the bench launch; the first and last instance against the oracle."""
+    from paper_conf_icppw_tiancd23_b200 import workloads
+    lines = [l.replace("-G hash -h 10000", "-G unionized") for l in workloads.c2(24)]
+    r = run_cfg(lines, 512)
+    assert np.all(r.records["exit_code"] == 0)
+    check_sample(oracle, lines, r, [0, 23])

@@ -21,7 +21,8 @@ GOLD = os.path.join(os.path.dirname(__file__), "golden")
 def test_history_default_matches_upstream(size, grid):
     from paper_conf_icppw_tiancd23_b200.ensemble import run_text
     if size == "large" and grid == "unionized":
-        pytest.skip("5.9 GB per instance; covered by the hash grid (same bracket)")
+        pytest.skip("the 500k-particle default is 17M dependent lookups on 5.9 GB of tables; "
+                    "test_history_large_unionized_reduced covers this grid against the oracle")
     gold = json.load(open(os.path.join(GOLD, "xsbench_upstream_checksums.json")))["checksums"]
     r = run_text(f"xsbench -s {size} -m history -G {grid}\n", app="auto", threads=512)
     assert r.records[0]["exit_code"] == 0
@@ -38,5 +39,16 @@ def test_history_parity(oracle, team):
              "xsbench -s small -m history -p 0 -g 10"]
     text = "".join(l + "\n" for l in lines)
     g = run_text(text, app="auto", threads=256, team_ctas=team)
+    o = oracle.run_text(text)
+    assert_parity(g, o)
+
+
+def test_history_large_unionized_reduced(oracle):
+    """Large unionized history (5.9 GB of tables) at reduced particle counts, against the oracle."""
+    from paper_conf_icppw_tiancd23_b200.ensemble import run_text
+    lines = ["xsbench -s large -m history -G unionized -p 3000 -r 1070",
+             "xsbench -s large -m history -G unionized -p 1500 -l 20 -r 1071"]
+    text = "".join(l + "\n" for l in lines)
+    g = run_text(text, app="auto", threads=512)
     o = oracle.run_text(text)
     assert_parity(g, o)
