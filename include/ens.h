@@ -60,11 +60,25 @@ enum {
   ENS_F_GENERIC = 1u << 2,    /* bodies take their general paths only (no fast
                                  paths such as XS's warp-per-nuclide unionized
                                  init): results are identical — for testing   */
-  ENS_F_SERIAL = 1u << 3      /* mixed-app ensembles: launch the per-app kernels
+  ENS_F_SERIAL = 1u << 3,     /* mixed-app ensembles: launch the per-app kernels
                                  one after another on one shared arena (the
                                  default gives each its own arena region, when
                                  they fit, and runs them concurrently on forked
                                  streams so one's tail overlaps the next)      */
+  ENS_F_FUSED = 1u << 4,      /* run every instance start to finish inside the
+                                 one ensemble kernel (the paper's mapping)     */
+  ENS_F_SPLIT_PHASES = 1u << 5 /* run XSBench-style event-mode instances whose
+                                 lookups fit one sorted chunk (<= 2^22) in
+                                 SPLIT PHASES: the ensemble kernel builds every
+                                 instance's tables and sorted lookups in an
+                                 arena slot of its own, then a second
+                                 persistent kernel spreads all instances'
+                                 lookup batches over every SM and writes their
+                                 records.  Default (neither flag): split when
+                                 the group has fewer instances than resident
+                                 CTAs and enough lookup batches to fill every
+                                 SM, and one slot per instance fits the
+                                 workspace.  Results are identical either way. */
 };
 #define ENS_PHASES 16
 

@@ -313,6 +313,35 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
   return L;
 }
 
+// ---- split phases (ENS_F_FUSED off): XS event-mode instances whose lookups
+// fit one sorted chunk run as two kernels.  The ensemble kernel (phase 1:
+// one team per instance, as always) builds the tables and the sorted lookup
+// chunk in a per-INSTANCE arena and writes an XsDesc; phase 2 is a
+// persistent kernel over every SM whose CTAs pull lookup batches ("items":
+// kXsItemLookups consecutive sorted slots of one instance) from one queue,
+// so all instances' lookups share every SM; the CTA finishing an instance's
+// last item writes its record and stdout.  Per-lookup results are unchanged.
+constexpr long long kXsItemLookups = 4096;
+ENS_HD bool xs_split_ok(const XsParams &p) { return !p.history && p.lookups > 0 && p.lookups <= kXsLkChunk; }
+ENS_HD long long xs_items(const XsParams &p) {
+  return xs_split_ok(p) ? (p.lookups + kXsItemLookups - 1) / kXsItemLookups : 0;
+}
+struct XsDesc {            // written by phase 1 (team rank 0, thread 0), read by phase 2
+  uint64_t recs, index, uenergy, ufind, lk_pe;  // device addresses in the instance's arena
+  uint64_t lookups, seed, t_start;
+  long long ubins;
+  uint32_t mcnt[13];       // material starts in the sorted chunk, mcnt[12] = lookups
+  int32_t n_iso, n_gp, grid, bins;
+  uint32_t k, line;        // record slot, instance id
+  uint32_t item0, n_items; // this instance's items in the phase-2 queue
+  uint32_t pad[2];
+};
+struct XsItemPart {        // one phase-2 item's partial results (summed in item order)
+  unsigned long long ver, bsum;
+  double fsum, fabs;
+  uint32_t am[5], pad[3];
+};
+
 // hash lookups: nuclides gathered per step (independent loads and divisions
 // in flight per lane)
 #ifndef ENS_XS_STEP

@@ -199,6 +199,31 @@ struct XsApp {
       init_nuc(c, p, L, S);  // nuclides striped over the team's CTAs
     }
     team_sync(c);
+    if (c.desc && xs_split_ok(p)) {  // split phases: sort the lookups, hand them to phase 2
+      uint32_t *mcnt = (uint32_t *)(ens_smem(c) + S.mcnt);
+      lookup_sort(c, p, L, thr, 0, p.lookups);
+      if (c.crank == 0 && threadIdx.x == 0) {
+        XsDesc *d = reinterpret_cast<XsDesc *>(c.desc);
+        d->recs = (uint64_t)(c.arena + L.recs);
+        d->index = (uint64_t)(c.arena + L.index);
+        d->uenergy = (uint64_t)(c.arena + L.uenergy);
+        d->ufind = (uint64_t)(c.arena + L.ufind);
+        d->lk_pe = (uint64_t)(c.arena + L.lk_pe);
+        d->lookups = (uint64_t)p.lookups;
+        d->seed = p.seed;
+        d->ubins = xs_ubins(p);
+        for (int m = 0; m < 13; m++) d->mcnt[m] = mcnt[16 + m];
+        d->n_iso = p.n_iso;
+        d->n_gp = p.n_gp;
+        d->grid = p.grid;
+        d->bins = p.bins;
+        d->k = c.k;
+        d->line = c.id;
+        d->t_start = c.t_start;
+      }
+      R.deferred = 1;
+      return R;
+    }
     if (p.history) {
       if (p.grid == XS_HASH) lookups_history<XS_HASH>(c, p, L, thr, nn, concs, mats, R);
       else if (p.grid == XS_UNIONIZED) lookups_history<XS_UNIONIZED>(c, p, L, thr, nn, concs, mats, R);
@@ -1114,8 +1139,7 @@ struct XsApp {
       // 2^-16 bin quantum; verified on the gathered pair, walked / searched
       // with upstream's logic otherwise
       const int pq = (int)((pe * (double)p.bins - (double)idx) * 65536.0);
-      const size_t hs = (size_t)p.bins + 1;
-      const XsHashEnt *hc = (const XsHashEnt *)ig + idx;
+        const XsHashEnt *hc = (const XsHashEnt *)ig + idx;
       const uint32_t hs32 = (uint32_t)p.bins + 1u;  // entry index < 355 * (10^7 + 1) < 2^32
       auto ent = [&](int j) { return reinterpret_cast<const uint4 *>(hc + (uint32_t)mrow[j] * hs32); };
       // #{k: pq15 > q_k} over the six 15-bit quanta by a SWAR compare: per
@@ -1272,6 +1296,98 @@ struct XsApp {
     m[4] = m4;
   }
 
+  // XS-7..XS-9 for one hash-grid lookup, one nuclide per step, each step's
+  // bracket guess and pair address computed ONCE (macro_lookup<XS_HASH>
+  // recomputes them for its prefetches: fewer live registers, more issued
+  // instructions — the trade the fused kernel's 128-register budget wants;
+  // phase 2 runs with a budget of its own and issue rate bounds it).  The
+  // software pipeline: entry j+2 loaded and entry j+4 prefetched into L1,
+  // nuclide j+1's guess and pair address computed and the pair prefetched,
+  // nuclide j's pair gathered, verified and accumulated.  The bracket logic
+  // and every FP operation are those of macro_lookup<XS_HASH> (bit-identical).
+  __device__ static __forceinline__ void macro_lookup_hash1(const XsParams &p, const double *recs, const int *ig,
+                                                            const int *nn, const double *concs,
+                                                            const uint16_t *mats, double pe, int mat, int idx,
+                                                            double *m) {
+    const int n_gp = p.n_gp, mx = xs_max_nucs(p.n_iso);
+    const int nm = nn[mat];
+    const uint16_t *mrow = mats + mat * mx;
+    const double *crow = concs + mat * mx;
+    const uint32_t hs32 = (uint32_t)p.bins + 1u;  // entry index < 355 * (10^7 + 1) < 2^32
+    const XsHashEnt *hc = (const XsHashEnt *)ig + idx;
+    auto ent = [&](int j) { return reinterpret_cast<const uint4 *>(hc + (uint32_t)mrow[j] * hs32); };
+    const int pq = (int)((pe * (double)p.bins - (double)idx) * 65536.0);
+    const uint32_t pq15 = (uint32_t)(pq < 0 ? 0 : (pq >> 1 > 32767 ? 32767 : pq >> 1));
+    const uint32_t P = (pq15 | (pq15 << 16) | 0x80008000u) - 0x00010001u;
+    // the guessed bracket lo (clamped to u_high - 1) of an entry, and its pair
+    auto guess = [&](const uint4 &h) {
+      const uint32_t mk = 0x80008000u;
+      const uint32_t x = ((P - h.y) & mk) | (((P - h.z) & mk) >> 1) | (((P - h.w) & mk) >> 2);
+      const int lo = (int)(h.x & 0xffffu) + __popc(x);
+      const int uh = (int)(h.x >> 16);
+      return lo < uh - 1 ? lo : uh - 1;
+    };
+    auto pair_at = [&](int j, int lo) {
+      return reinterpret_cast<const double2 *>(recs + ((uint32_t)mrow[j] * (uint32_t)n_gp + (uint32_t)lo) * 6u);
+    };
+    double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
+    const uint4 z = make_uint4(0, 0, 0, 0);
+    uint4 h0 = nm > 0 ? ld_(ent(0)) : z;
+    uint4 h1 = nm > 1 ? ld_(ent(1)) : z;
+    if (nm > 2) prefetch_l1(ent(2));
+    if (nm > 3) prefetch_l1(ent(3));
+    int lo0 = guess(h0);
+    const double2 *q0 = pair_at(0, lo0);
+    for (int j = 0; j < nm; j++) {
+      const uint4 h2 = j + 2 < nm ? ld_(ent(j + 2)) : z;
+      if (j + 4 < nm) prefetch_l1(ent(j + 4));
+      const double2 *q1 = q0;
+      int lo1 = lo0;
+      if (j + 1 < nm) {
+        lo1 = guess(h1);
+        q1 = pair_at(j + 1, lo1);
+        prefetch_l1(q1);
+        prefetch_l1(reinterpret_cast<const double *>(q1) + 11);
+      }
+      double2 a0 = ld_(q0 + 0), a1 = ld_(q0 + 1), a2 = ld_(q0 + 2);
+      double2 b0 = ld_(q0 + 3), b1 = ld_(q0 + 4), b2 = ld_(q0 + 5);
+      {  // verify the guessed pair; walk / upstream search otherwise (macro_lookup's gather_fix)
+        const uint4 &h = h0;
+        const double *E = reinterpret_cast<const double *>(q0) - 6 * (size_t)lo0;  // the nuclide's records
+        const int u_low = (int)(h.x & 0xffffu), uh = (int)(h.x >> 16);
+        int lo = lo0;
+        while (pe >= b0.x && a0.x < pe && lo + 2 <= uh) {
+          lo++;
+          const double2 *w2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
+          a0 = b0; a1 = b1; a2 = b2;
+          b0 = ld_(w2 + 3); b1 = ld_(w2 + 4); b2 = ld_(w2 + 5);
+        }
+        if (!(a0.x < pe && pe < b0.x && lo + 1 <= uh)) {
+          const double e_low = ld_(E + 6 * (size_t)u_low);
+          const double e_high = ld_(E + 6 * (size_t)uh);
+          int lower;
+          if (pe <= e_low) lower = 0;
+          else if (pe >= e_high) lower = n_gp - 1;
+          else lower = gs_recs(E, pe, u_low, uh);
+          const int l2 = lower == n_gp - 1 ? lower - 1 : lower;
+          const double2 *w2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)l2);
+          a0 = ld_(w2 + 0); a1 = ld_(w2 + 1); a2 = ld_(w2 + 2);
+          b0 = ld_(w2 + 3); b1 = ld_(w2 + 4); b2 = ld_(w2 + 5);
+        }
+      }
+      accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
+      h0 = h1;
+      h1 = h2;
+      q0 = q1;
+      lo0 = lo1;
+    }
+    m[0] = m0;
+    m[1] = m1;
+    m[2] = m2;
+    m[3] = m3;
+    m[4] = m4;
+  }
+
   // union position of energy pe == grid_search(u, pe, 0, n_u-1) (XS-7), via
   // the search table: ufind[floor(pe*UB)] then a short forward scan
   __device__ static __forceinline__ int union_idx(const uint32_t *uf, const uint64_t *uA, long long UB, long long n_u,
@@ -1353,6 +1469,59 @@ struct XsApp {
     R.work = (uint64_t)p.particles * (uint64_t)nL;
   }
 
+  // (A)-(C) of the event-mode lookups for the chunk of lookups [c0, c0+nc):
+  // lk_pe = their energies sorted into (material, energy) buckets, material
+  // m's slots start at mcnt[16+m] (mcnt[28] = nc); material tallies counted
+  __device__ static __forceinline__ void lookup_sort(Ctx &c, const XsParams &p, const XsLayout &L, const double *thr, long long c0,
+                                     long long nc) {
+    const int tid = threadIdx.x, T = blockDim.x;
+    double *lk_pe = (double *)(c.arena + L.lk_pe);
+    uint32_t *hist = (uint32_t *)(c.arena + L.lk_hist);
+    const XsSmem S = xs_smem(p, T);
+    uint32_t *mcnt = (uint32_t *)(ens_smem(c) + S.mcnt);
+    const long long LC = xs_lk_chunk(p);
+    const int kb = xs_lk_bits(LC);
+    const long long NB = 12LL << kb;
+    const double bscale = (double)(1LL << kb);
+    const long long g0 = (long long)c.crank * T + tid, gs = (long long)c.csize * T;
+    const Affine JG = lcg_pow(2ULL * (uint64_t)gs);
+    for (long long b = g0; b <= NB; b += gs) hist[b] = 0u;
+    team_sync(c);
+    // (A) count
+    {
+      uint64_t s = lcg_pow(2ULL * (uint64_t)(c0 + g0))(p.seed);
+      for (long long li = g0; li < nc; li += gs, s = JG(s)) {
+        uint64_t t = s;
+        const double pe = lcg_double(t);
+        const int mat = pick_mat_thr(thr, lcg_double(t));
+        long long eb = (long long)(pe * bscale);
+        eb = eb > (1LL << kb) - 1 ? (1LL << kb) - 1 : eb;
+        atomicAdd(&hist[((long long)mat << kb) + eb], 1u);
+      }
+    }
+    team_sync(c);
+    // (B) bucket offsets (one CTA), material starts to every CTA's smem
+    if (c.crank == 0) global_exclusive_scan(hist, NB + 1, ens_sh(c));
+    team_sync(c);
+    if (tid < 12) mcnt[16 + tid] = ld_(hist + ((long long)tid << kb));
+    if (tid == 12) mcnt[28] = (uint32_t)nc;
+    team_sync(c);  // every CTA has its offsets before (C) moves the cursors
+    if (c.crank == 0 && tid < 12) ens_sh(c)->tallies[5 + tid] += mcnt[17 + tid] - mcnt[16 + tid];  // per material
+    // (C) scatter energies to their buckets (hist becomes bucket ends)
+    {
+      uint64_t s = lcg_pow(2ULL * (uint64_t)(c0 + g0))(p.seed);
+      for (long long li = g0; li < nc; li += gs, s = JG(s)) {
+        uint64_t t = s;
+        const double pe = lcg_double(t);
+        const int mat = pick_mat_thr(thr, lcg_double(t));
+        long long eb = (long long)(pe * bscale);
+        eb = eb > (1LL << kb) - 1 ? (1LL << kb) - 1 : eb;
+        lk_pe[atomicAdd(&hist[((long long)mat << kb) + eb], 1u)] = pe;
+      }
+    }
+    team_sync(c);
+  }
+
   // ---- XS-6..XS-10: lookups ----------------------------------------------
   // Per chunk of at most 2^22 lookups (XsLayout.lk_*): (A) every lookup is
   // sampled (XS-6, lookup li draws 2li+1, 2li+2) and counted into its
@@ -1377,56 +1546,17 @@ struct XsApp {
     const uint64_t *uA = (const uint64_t *)(c.arena + L.uenergy);
     const uint32_t *uf = (const uint32_t *)(c.arena + L.ufind);
     double *lk_pe = (double *)(c.arena + L.lk_pe);
-    uint32_t *hist = (uint32_t *)(c.arena + L.lk_hist);
     const long long UB = xs_ubins(p);
     const XsSmem S = xs_smem(p, T);
     uint32_t *mcnt = (uint32_t *)(ens_smem(c) + S.mcnt);  // [16..28] material offsets of the chunk
     const double du = 1.0 / p.bins;
     const long long LC = xs_lk_chunk(p);
-    const int kb = xs_lk_bits(LC);
-    const long long NB = 12LL << kb;
-    const double bscale = (double)(1LL << kb);
     const long long g0 = (long long)c.crank * T + tid, gs = (long long)c.csize * T;
-    const Affine JG = lcg_pow(2ULL * (uint64_t)gs);
     unsigned long long ver = 0, bsum = 0;
     double fsum = 0.0, fabs_ = 0.0;
     for (long long c0 = 0; c0 < nL; c0 += LC) {
       const long long nc = nL - c0 < LC ? nL - c0 : LC;
-      for (long long b = g0; b <= NB; b += gs) hist[b] = 0u;
-      team_sync(c);
-      // (A) count
-      {
-        uint64_t s = lcg_pow(2ULL * (uint64_t)(c0 + g0))(p.seed);
-        for (long long li = g0; li < nc; li += gs, s = JG(s)) {
-          uint64_t t = s;
-          const double pe = lcg_double(t);
-          const int mat = pick_mat_thr(thr, lcg_double(t));
-          long long eb = (long long)(pe * bscale);
-          eb = eb > (1LL << kb) - 1 ? (1LL << kb) - 1 : eb;
-          atomicAdd(&hist[((long long)mat << kb) + eb], 1u);
-        }
-      }
-      team_sync(c);
-      // (B) bucket offsets (one CTA), material starts to every CTA's smem
-      if (c.crank == 0) global_exclusive_scan(hist, NB + 1, ens_sh(c));
-      team_sync(c);
-      if (tid < 12) mcnt[16 + tid] = ld_(hist + ((long long)tid << kb));
-      if (tid == 12) mcnt[28] = (uint32_t)nc;
-      team_sync(c);  // every CTA has its offsets before (C) moves the cursors
-      if (c.crank == 0 && tid < 12) ens_sh(c)->tallies[5 + tid] += mcnt[17 + tid] - mcnt[16 + tid];  // per material
-      // (C) scatter energies to their buckets (hist becomes bucket ends)
-      {
-        uint64_t s = lcg_pow(2ULL * (uint64_t)(c0 + g0))(p.seed);
-        for (long long li = g0; li < nc; li += gs, s = JG(s)) {
-          uint64_t t = s;
-          const double pe = lcg_double(t);
-          const int mat = pick_mat_thr(thr, lcg_double(t));
-          long long eb = (long long)(pe * bscale);
-          eb = eb > (1LL << kb) - 1 ? (1LL << kb) - 1 : eb;
-          lk_pe[atomicAdd(&hist[((long long)mat << kb) + eb], 1u)] = pe;
-        }
-      }
-      team_sync(c);
+      lookup_sort(c, p, L, thr, c0, nc);
       phase_mark_if(trc, c, 10);
       // (D) thread-per-lookup over the sorted chunk
       double *const dmp = c.dump;

@@ -178,6 +178,17 @@ struct Group {
   std::vector<double> cost;  // app_cost per kmap entry (schedule only)
   size_t kmap_off = 0;
   size_t arena_off = 0;  // this group's arena region (offset from o_arena)
+  // split phases (XS): phase 1 = the ensemble kernel with one arena slot per
+  // instance (slots = kmap.size()), phase 2 = the lookup-item kernel
+  bool split = false;
+  std::vector<uint32_t> item_count;  // per kmap entry
+  std::vector<int> item_kind;        // per kmap entry: phase-2 kernel (XS grid type)
+  std::vector<uint32_t> items;       // group-local instance of each item, by kind
+  std::vector<uint32_t> item0;       // per kmap entry: its first item
+  uint32_t kind_base[3] = {0, 0, 0}, kind_n[3] = {0, 0, 0};
+  int grid2[3] = {0, 0, 0};          // phase-2 CTAs per kind
+  size_t items_off = 0, desc_off = 0, ipart_off = 0, idone_off = 0, ctr2_off = 0;
+  size_t slots() const { return split ? kmap.size() : (size_t)grid; }
 };
 
 struct Plan {  // workspace layout (byte offsets) and groups
@@ -373,6 +384,9 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     g.smem = std::max(g.smem, sm);
     g.kmap.push_back((uint32_t)k);
     g.cost.push_back(app_cost(ap, argc, argv));
+    int kind = 0;
+    g.item_count.push_back(app_items(ap, argc, argv, &kind));
+    g.item_kind.push_back(kind);
   }
   // longest-first instance queue (LPT): teams pull the heavy instances first
   // and the light ones fill the tail (results are schedule-independent, Q5)
@@ -381,11 +395,15 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     std::vector<uint32_t> ord(g.kmap.size());
     for (size_t x = 0; x < ord.size(); x++) ord[x] = (uint32_t)x;
     std::stable_sort(ord.begin(), ord.end(), [&](uint32_t u, uint32_t v) { return g.cost[u] > g.cost[v]; });
-    std::vector<uint32_t> km(ord.size());
+    std::vector<uint32_t> km(ord.size()), ic(ord.size());
+    std::vector<int> ik(ord.size());
     std::vector<double> co(ord.size());
-    for (size_t x = 0; x < ord.size(); x++) km[x] = g.kmap[ord[x]], co[x] = g.cost[ord[x]];
+    for (size_t x = 0; x < ord.size(); x++)
+      km[x] = g.kmap[ord[x]], co[x] = g.cost[ord[x]], ic[x] = g.item_count[ord[x]], ik[x] = g.item_kind[ord[x]];
     g.kmap.swap(km);
     g.cost.swap(co);
+    g.item_count.swap(ic);
+    g.item_kind.swap(ik);
   }
   // team size: team-aware bodies get a cluster of cs CTAs when the group has
   // fewer instances than resident CTAs (the largest power of two <= 8 with
@@ -443,11 +461,44 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
       g.arena = std::max(g.arena, ar);
     }
     need_arena = std::max(need_arena, g.arena);
+    // split phases when some instance has lookup items (and arenas are host-sized:
+    // a caller's smaller arena_bytes could make an instance exit NOMEM in phase 1)
+    if (!(c->flags & ENS_F_FUSED) && !c->arena_bytes) {
+      // items grouped by kind (one phase-2 kernel each), instances in queue order within a kind
+      g.item0.assign(g.kmap.size(), 0);
+      for (int kd = 0; kd < 3; kd++) {
+        g.kind_base[kd] = (uint32_t)g.items.size();
+        for (size_t x = 0; x < g.kmap.size(); x++) {
+          if (g.item_kind[x] != kd || !g.item_count[x]) continue;
+          g.item0[x] = (uint32_t)g.items.size();
+          for (uint32_t b = 0; b < g.item_count[x]; b++) g.items.push_back((uint32_t)x);
+        }
+        g.kind_n[kd] = (uint32_t)g.items.size() - g.kind_base[kd];
+        if (g.kind_n[kd]) {
+          e = xs_items_occupancy(kd, &g.grid2[kd]);
+          if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor (phase 2)");
+        }
+      }
+      // split when it pays (measured): fewer instances than
+      // resident CTAs (phase 1 alone would leave SMs idle) and enough items to
+      // fill every phase-2 CTA.  C2 45.1 -> 38.2 ms, C2u 66.2 -> 62.9 ms;
+      // TSTAR (1024 instances) and C1 (12 items) stay fused.
+      int fill = 0;
+      for (int kd = 0; kd < 3; kd++) fill = std::max(fill, g.grid2[kd]);
+      g.split = !g.items.empty() && (((c->flags & ENS_F_SPLIT_PHASES) != 0) ||
+                                     ((int64_t)g.kmap.size() < (int64_t)ctas && (int64_t)g.items.size() >= fill));
+      if (!g.split) {
+        g.items.clear();
+        for (int kd = 0; kd < 3; kd++) g.kind_n[kd] = 0;
+      }
+    }
     P.groups.push_back(g);
   }
   P.arena_bytes = c->arena_bytes ? al(c->arena_bytes) : al(need_arena);
-  // layout: staged part
   size_t o = 0;
+  auto layout = [&]() {
+  o = 0;
+  // staged part
   P.o_blob = o; o = al(o + a->blob.size());
   P.o_tok = o; o = al(o + a->tok_off.size() * 4);
   P.o_line = o; o = al(o + a->line_tok.size() * 4);
@@ -458,9 +509,19 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     o += g.kmap.size() * 4;
   }
   o = al(o);
+  for (Group &g : P.groups) {  // split phases: item table, descriptors (item0 / n_items pre-filled)
+    if (!g.split) continue;
+    g.items_off = o; o = al(o + g.items.size() * 4);
+    g.desc_off = o; o = al(o + g.kmap.size() * sizeof(XsDesc));
+  }
   P.staged = o;
   // zeroed part
   P.o_ctr = o; o = al(o + (P.groups.size() + 1) * 8);
+  for (Group &g : P.groups) {
+    if (!g.split) continue;
+    g.ctr2_off = o; o = al(o + 3 * 8);
+    g.idone_off = o; o = al(o + g.kmap.size() * 4);
+  }
   P.o_recs = o; o = al(o + (size_t)n * sizeof(ens_record));
   P.o_pos = o; o = al(o + (size_t)n * 8);
   P.o_phase = o; o = al(o + ENS_PHASES * 8);
@@ -470,9 +531,24 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   P.o_tal = o; o = al(o + (size_t)n * ENS_TALLIES * 4);
   P.o_out = o; o = al(o + (size_t)n * P.stdout_cap);
   P.o_cmp = o; o = al(o + (size_t)n * P.stdout_cap);
+  for (Group &g : P.groups) {
+    if (!g.split) continue;
+    g.ipart_off = o; o = al(o + g.items.size() * sizeof(XsItemPart));
+  }
   P.o_arena = o;
+  };
+  layout();
+  // split groups keep one arena slot per instance: only when that fits
+  if (mem_cap) {
+    size_t need = o;
+    for (const Group &g : P.groups) need += g.slots() * (size_t)P.arena_bytes;
+    if (need > mem_cap) {
+      for (Group &g : P.groups) g.split = false;
+      layout();
+    }
+  }
   int want = 0;
-  for (const Group &g : P.groups) want = std::max(want, g.grid);
+  for (const Group &g : P.groups) want = std::max(want, (int)g.slots());
   if (P.arena_bytes && mem_cap) {
     if (mem_cap < o + P.arena_bytes) return fail(ENS_ENOMEM, "ens_launch: workspace cannot hold one arena slot");
     const uint64_t fit = (mem_cap - o) / P.arena_bytes;
@@ -480,6 +556,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
       if (c->grid_blocks) return fail(ENS_ENOMEM, "ens_launch: grid_blocks x arena does not fit the workspace");
       want = (int)fit;
       for (Group &g : P.groups) {
+        if (g.split) return fail(ENS_ENOMEM, "ens_launch: split-phase arena slots do not fit the workspace");
         g.grid = std::min(g.grid, want / g.m * g.m);  // whole CTAs of m slots
         if (g.grid <= 0)
           return fail(ENS_ENOMEM, "ens_launch: workspace cannot hold one CTA of instances_per_cta arena slots");
@@ -492,12 +569,12 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   // their kernels may run concurrently, when that fits the workspace cap
   if (P.groups.size() > 1 && !(c->flags & ENS_F_SERIAL)) {
     size_t off = 0;
-    for (const Group &g : P.groups) off += (size_t)g.grid * P.arena_bytes;
+    for (const Group &g : P.groups) off += g.slots() * P.arena_bytes;
     if (!mem_cap || o + off <= mem_cap) {
       off = 0;
       for (Group &g : P.groups) {
         g.arena_off = off;
-        off += (size_t)g.grid * P.arena_bytes;
+        off += g.slots() * P.arena_bytes;
       }
       P.concurrent = true;
       P.total = o + off;
@@ -551,6 +628,15 @@ static int enqueue(ens_run *r) {
     k.arena_base = r->ws + P.o_arena + g.arena_off;
     k.dump = P.dump_rows ? (double *)(r->ws + P.o_dump) : nullptr;
     k.dump_rows = P.dump_rows;
+    k.split = g.split ? 1u : 0u;
+    if (g.split) {
+      k.xs_desc = r->ws + g.desc_off;
+      k.items = (const uint32_t *)(r->ws + g.items_off);
+      k.n_items = (uint32_t)g.items.size();
+      k.ipart = r->ws + g.ipart_off;
+      k.idone = (uint32_t *)(r->ws + g.idone_off);
+      k.counter2 = (uint32_t *)(r->ws + g.ctr2_off);
+    }
     cudaStream_t st = r->stream;
     if (P.concurrent && gi > 0) {  // fork: group gi on an aux stream after ev0
       CU(aux_stream(gi - 1, &st));
@@ -558,6 +644,16 @@ static int enqueue(ens_run *r) {
     }
     cudaError_t e = launch_group(g.app, g.T, g.m, g.ctas(), g.cs, g.dyn(), k, st);
     if (e != cudaSuccess) return cuda_fail(e, "ens_kernel launch");
+    for (int kd = 0; g.split && kd < 3; kd++) {  // phase 2: every instance's lookup items, on every SM
+      if (!g.kind_n[kd]) continue;
+      const int ctas2 = std::max(1, std::min<int>(g.grid2[kd], (int)g.kind_n[kd]));
+      KParams k2 = k;
+      k2.item_base = g.kind_base[kd];
+      k2.n_items = g.kind_n[kd];
+      k2.counter2 = (uint32_t *)(r->ws + g.ctr2_off + 8 * kd);
+      e = launch_xs_items(kd, ctas2, k2, st);
+      if (e != cudaSuccess) return cuda_fail(e, "xs_items_kernel launch");
+    }
     if (P.concurrent && gi > 0) {  // join back into the launch stream
       CU(cudaEventRecord(r->ev_join[gi - 1], st));
       CU(cudaStreamWaitEvent(r->stream, r->ev_join[gi - 1], 0));
@@ -625,6 +721,15 @@ extern "C" int ens_launch(ens_app app, const ens_args *a, const ens_launch_cfg *
   std::memcpy(r->h_stage + P.o_line, a->line_tok.data(), a->line_tok.size() * 4);
   std::memcpy(r->h_stage + P.o_lok, P.line_of_k.data(), P.line_of_k.size() * 4);
   for (const Group &g : P.groups) std::memcpy(r->h_stage + g.kmap_off, g.kmap.data(), g.kmap.size() * 4);
+  for (const Group &g : P.groups) {
+    if (!g.split) continue;
+    std::memcpy(r->h_stage + g.items_off, g.items.data(), g.items.size() * 4);
+    for (size_t x = 0; x < g.kmap.size(); x++) {  // phase 1 fills the rest of each descriptor
+      XsDesc *d = reinterpret_cast<XsDesc *>(r->h_stage + g.desc_off) + x;
+      d->item0 = g.item0[x];
+      d->n_items = g.item_count[x];
+    }
+  }
   e = cudaMemcpyAsync(r->ws, r->h_stage, P.staged, cudaMemcpyHostToDevice, r->stream);
   if (e != cudaSuccess) {
     *out = nullptr;
@@ -793,6 +898,8 @@ extern "C" int ens_run_get_info(const ens_run *r, ens_run_info *info) {
     info->block_threads[ap] = g.T;
   }
   info->kernel_launches = (int32_t)P.groups.size();
+  for (const Group &g : P.groups)
+    for (int kd = 0; g.split && kd < 3; kd++) info->kernel_launches += g.kind_n[kd] ? 1 : 0;
   info->arena_bytes = P.arena_bytes;
   info->ws_bytes = r->ws_bytes;
   info->records_offset = P.o_recs;

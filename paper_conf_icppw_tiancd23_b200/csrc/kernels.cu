@@ -103,15 +103,22 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
 
     c.k = k;
     c.id = line;
+    c.t_start = t_start;
     c.out = p.stdout_base + (size_t)k * p.stdout_cap;
     c.phases = p.phases;
     c.flags = p.flags;
     c.dump = p.dump ? p.dump + (size_t)k * p.dump_rows * 8 : nullptr;
     c.dump_rows = p.dump_rows;
+    // split phases: one arena slot per instance (phase 2 reads the tables)
+    c.arena = p.split ? p.arena_base + (size_t)j * p.arena_bytes : arena;
+    c.desc = p.split ? p.xs_desc + (size_t)j * sizeof(XsDesc) : nullptr;
     phase_mark(c, -1);
     Result r{};
     if (App::kTeam || cr == 0) r = App::run(c, argc, s_argv);
     team_sync(c);
+    if (r.deferred) {  // split phases: phase 2 writes this instance's record
+      continue;        // (the loop head's team_sync orders the scheduler state)
+    }
     if (cs > 1 && cr != 0 && tid < ENS_TALLIES && sh.tallies[tid])  // combine tallies into rank 0
       atomicAdd(cta_shared(&sh.tallies[tid], 0), sh.tallies[tid]);
     team_sync(c);
@@ -229,6 +236,16 @@ double app_cost(uint32_t app, int argc, const char *const *argv) {
     }
   }
   return 1.0;
+}
+// split phases: phase-2 items of one instance (0 = the instance runs fused)
+// (*kind = the phase-2 kernel: the XS grid type)
+uint32_t app_items(uint32_t app, int argc, const char *const *argv, int *kind) {
+  *kind = 0;
+  if (app != APP_XSBENCH) return 0;
+  XsParams p;
+  if (xs_parse(argc, argv, p) >= 0) return 0;
+  *kind = p.grid;
+  return (uint32_t)xs_items(p);
 }
 // whether the body can run as one of M instances per CTA (NEXT 1)
 bool app_sub_aware(uint32_t app) {

@@ -1,0 +1,279 @@
+// csrc/kernels_xs2.cu — split phases, phase 2: the XSBench-style lookup
+// items of every instance of an ensemble, on every SM.
+//
+// Phase 1 (the ensemble kernel, kernels.cu: one team per instance, the
+// paper's mapping) builds each instance's tables and its (material,
+// energy)-sorted lookup chunk in a per-instance arena slot and leaves an
+// XsDesc.  This persistent kernel then pulls items — kXsItemLookups
+// consecutive sorted slots of one instance — from one atomic queue, so the
+// lookups of all instances are spread over all SMs whatever the instance
+// count (C2: 64 instances on 148 SMs), and it runs with its own register
+// budget (the lookups alone, not the init code: more resident warps to hide
+// the dependent gathers).  Each lookup is XS-7..XS-10 exactly as the fused
+// body computes it (XsApp::macro_lookup, bit-identical); an item's integer
+// sums and argmax counts and its fsum / fabs partials go to its own
+// XsItemPart, and the CTA that finishes an instance's last item sums the
+// parts in item order, writes the record, the tallies and the
+// stdout lines (XS-11), exactly what the fused body writes.
+#include <cuda_runtime.h>
+
+// phase 2's hash lookups gather one nuclide per step: with the register
+// budget of 3 CTAs/SM that beats two (measured: C2 38.8 vs 39.9 ms)
+#ifndef ENS_XS_STEP
+#define ENS_XS_STEP 1
+#endif
+#include "apps/xsbench.cuh"
+#include "kparams.h"
+
+namespace ens {
+
+#ifndef ENS_XS2_T
+#define ENS_XS2_T 256
+#endif
+// resident CTAs per SM (register budget 65536 / (T * minB)) per grid type:
+// one kernel per grid type, so each carries only its own lookup's registers
+#ifndef ENS_XS2_MINB_HASH
+#define ENS_XS2_MINB_HASH 3
+#endif
+#ifndef ENS_XS2_MINB_UNI
+#define ENS_XS2_MINB_UNI 2
+#endif
+#ifndef ENS_XS2_MINB_NUC
+#define ENS_XS2_MINB_NUC 2
+#endif
+template <int GRID>
+struct Xs2Minb {
+  static constexpr int v = GRID == XS_HASH ? ENS_XS2_MINB_HASH : GRID == XS_UNIONIZED ? ENS_XS2_MINB_UNI : ENS_XS2_MINB_NUC;
+};
+constexpr int kXs2T = ENS_XS2_T;
+constexpr uint32_t kXs2Sh = (sizeof(Shared) + 15) / 16 * 16;
+// dynamic shared memory: Shared | XsDesc | thr[12] | nn[16] | concs | mats | scratch
+constexpr uint32_t kXs2Desc = kXs2Sh;
+constexpr uint32_t kXs2Thr = kXs2Desc + (sizeof(XsDesc) + 15) / 16 * 16;
+constexpr uint32_t kXs2Nn = kXs2Thr + 12 * 8;
+constexpr uint32_t kXs2Concs = kXs2Nn + 16 * 4;
+constexpr uint32_t kXs2Mats = kXs2Concs + 12 * 321 * 8;
+constexpr uint32_t kXs2Misc = kXs2Mats + (12 * 321 * 2 + 15) / 16 * 16;  // u32: item, last, am[5], pos(2)
+constexpr uint32_t kXs2Smem = kXs2Misc + 16 * 4;
+
+template <int GRID>
+__device__ __forceinline__ void xs2_item(const XsDesc &d, const XsParams &p, long long s0, long long s1,
+                                         const int *nn, const double *concs, const uint16_t *mats, uint32_t *am,
+                                         double *dmp, uint32_t drows, unsigned long long &ver,
+                                         unsigned long long &bsum, double &fsum, double &fabs_) {
+  const double *recs = (const double *)d.recs;
+  const int *ig = (const int *)d.index;
+  const uint64_t *uA = (const uint64_t *)d.uenergy;
+  const uint32_t *uf = (const uint32_t *)d.ufind;
+  const double *lk_pe = (const double *)d.lk_pe;
+  const long long n_u = (long long)p.n_iso * p.n_gp, UB = d.ubins;
+  const double du = 1.0 / p.bins;
+  for (long long sl = s0 + threadIdx.x; sl < s1; sl += kXs2T) {
+    int mat = 0;
+#pragma unroll
+    for (int m = 1; m < 12; m++) mat += (sl >= (long long)d.mcnt[m]) ? 1 : 0;
+    const double pe = ld_(lk_pe + sl);
+    int idx = 0;
+    if (GRID == XS_UNIONIZED) idx = XsApp::union_idx(uf, uA, UB, n_u, pe);
+    else if (GRID == XS_HASH) {
+      const long long bb = (long long)(pe / du);
+      idx = bb > p.bins - 1 ? p.bins - 1 : (int)bb;  // reading Q14
+    }
+    double mv[5];
+#ifndef ENS_XS2_OLD_HASH
+    if (GRID == XS_HASH) XsApp::macro_lookup_hash1(p, recs, ig, nn, concs, mats, pe, mat, idx, mv);
+    else
+#endif
+      XsApp::macro_lookup<GRID>(p, recs, ig, nn, concs, mats, pe, mat, idx, mv);
+    const double m0 = mv[0], m1 = mv[1], m2 = mv[2], m3 = mv[3], m4 = mv[4];
+    double mxv = -1.0;  // XS-10
+    int a = 0;
+    if (m0 > mxv) { mxv = m0; a = 0; }
+    if (m1 > mxv) { mxv = m1; a = 1; }
+    if (m2 > mxv) { mxv = m2; a = 2; }
+    if (m3 > mxv) { mxv = m3; a = 3; }
+    if (m4 > mxv) { mxv = m4; a = 4; }
+    ver += (unsigned long long)(a + 1);
+    atomicAdd(&am[a], 1u);
+    if (dmp) dump_row(dmp, drows, sl, pe, mat, mv, 5, a);
+    bsum += dbits(m0) + dbits(m1) + dbits(m2) + dbits(m3) + dbits(m4);
+    fsum += m0; fsum += m1; fsum += m2; fsum += m3; fsum += m4;
+    fabs_ += fabs(m0); fabs_ += fabs(m1); fabs_ += fabs(m2); fabs_ += fabs(m3); fabs_ += fabs(m4);
+  }
+}
+
+__device__ __forceinline__ unsigned long long xs2_gtimer() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// the CTA that finished an instance's last item: XS-10's sums over its items
+// (in item order: deterministic), XS-11's stdout, the record and the tallies;
+// out of line (once per instance) so the lookup loop keeps its registers
+__device__ __noinline__ void xs2_finish(const KParams &p, Ctx &c, const XsDesc *d, uint32_t *misc) {
+  const int tid = threadIdx.x;
+  Shared *sh = ens_sh(c);
+  const uint32_t k = d->k;
+  c.out = p.stdout_base + (size_t)k * p.stdout_cap;
+  if (tid == 0) {
+    __threadfence();
+    unsigned long long tv = 0, tb = 0;
+    double tf = 0.0, ta = 0.0;
+    uint32_t tam[5] = {0, 0, 0, 0, 0};
+    const XsItemPart *ip = reinterpret_cast<const XsItemPart *>(p.ipart);
+    for (uint32_t it = d->item0; it < d->item0 + d->n_items; it++) {
+      tv += __ldcg(&ip[it].ver);
+      tb += __ldcg(&ip[it].bsum);
+      tf += __ldcg(&ip[it].fsum);
+      ta += __ldcg(&ip[it].fabs);
+      for (int a = 0; a < 5; a++) tam[a] += __ldcg(&ip[it].am[a]);
+    }
+    sh->out_len = 0;
+    sh->flags = 0;
+    const int n_iso = d->n_iso;
+    const long long lookups = (long long)d->lookups;
+    const unsigned long long vhash = tv % 999983ULL;
+    const char *grid = d->grid == XS_UNIONIZED ? "unionized" : d->grid == XS_NUCLIDE ? "nuclide" : "hash";
+    ens_printf(c, FMT_XS_HDR, n_iso == 68 ? "small" : "large", n_iso, (long long)d->n_gp, grid, lookups,
+               (unsigned long long)d->seed);
+    ens_printf(c, FMT_VERIFY, vhash);
+    uint32_t *tal = p.tallies + (size_t)k * ENS_TALLIES;
+    for (int t = 0; t < ENS_TALLIES; t++)
+      tal[t] = t < 5 ? tam[t] : (t < 17 ? d->mcnt[t - 4] - d->mcnt[t - 5] : 0u);
+    ens_record rec;
+    rec.instance = d->line;
+    rec.exit_code = 0;
+    rec.app = APP_XSBENCH;
+    rec.flags = sh->flags | ENS_RF_DONE;
+    rec.vhash = vhash;
+    rec.bitsum = tb;
+    rec.fsum = tf;
+    rec.fabs = ta;
+    rec.work = (uint64_t)lookups;
+    rec.stdout_len = sh->out_len;
+    uint32_t sm = 0;
+    if (p.flags & ENS_F_TIMESTAMPS) asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+    rec.smid = sm;
+    rec.t_start_ns = d->t_start;
+    rec.t_end_ns = (p.flags & ENS_F_TIMESTAMPS) ? xs2_gtimer() : 0ull;
+    p.recs[k] = rec;
+    const unsigned long long pos = atomicAdd(p.stdout_total, (unsigned long long)sh->out_len);
+    p.stdout_pos[k] = pos;
+    reinterpret_cast<unsigned long long *>(misc + 8)[0] = pos;
+  }
+  __syncthreads();
+  // compact the instance's stdout (whole 8-B words)
+  const unsigned long long pos = reinterpret_cast<const unsigned long long *>(misc + 8)[0];
+  const unsigned long long *src = reinterpret_cast<const unsigned long long *>(c.out);
+  unsigned long long *dst = reinterpret_cast<unsigned long long *>(p.stdout_cmp + pos);
+  for (uint32_t w = tid; w < sh->out_len / 8; w += kXs2T) dst[w] = src[w];
+}
+
+
+// items [p.item_base, p.item_base + p.n_items) of the group's queue, all of grid type GRID
+template <int GRID>
+__global__ void __launch_bounds__(kXs2T, Xs2Minb<GRID>::v) xs_items_kernel(const KParams p) {
+  const int tid = threadIdx.x;
+  Ctx c{};
+  c.sh_off = 0;
+  c.smem_off = kXs2Desc;
+  c.csize = 1;
+  c.flags = p.flags;
+  c.out_cap = p.stdout_cap;
+  Shared *sh = ens_sh(c);
+  XsDesc *d = reinterpret_cast<XsDesc *>(ens_dsmem + kXs2Desc);
+  double *thr = reinterpret_cast<double *>(ens_dsmem + kXs2Thr);
+  int *nn = reinterpret_cast<int *>(ens_dsmem + kXs2Nn);
+  double *concs = reinterpret_cast<double *>(ens_dsmem + kXs2Concs);
+  uint16_t *mats = reinterpret_cast<uint16_t *>(ens_dsmem + kXs2Mats);
+  uint32_t *misc = reinterpret_cast<uint32_t *>(ens_dsmem + kXs2Misc);
+  uint32_t *am = misc + 2;
+  int cached = 0;  // n_iso of the material tables in shared memory
+  for (;;) {
+    if (tid == 0) misc[0] = atomicAdd(p.counter2, 1u);
+    if (tid < 5) am[tid] = 0u;
+    __syncthreads();
+    if (misc[0] >= p.n_items) break;
+    const uint32_t item = p.item_base + misc[0];
+    const uint32_t j = p.items[item];
+    {  // the instance's descriptor (phase 1's stores, an earlier kernel)
+      const unsigned long long *src = reinterpret_cast<const unsigned long long *>(p.xs_desc + (size_t)j * sizeof(XsDesc));
+      unsigned long long *dst = reinterpret_cast<unsigned long long *>(d);
+      for (int w = tid; w < (int)(sizeof(XsDesc) / 8); w += kXs2T) dst[w] = src[w];
+    }
+    __syncthreads();
+    const int n_iso = d->n_iso, mx = xs_max_nucs(n_iso);
+    if (n_iso != cached) {  // XS-2 tables (constant per n_iso: CONC_SEED is fixed)
+      hm_tables(n_iso, mx, thr, nn, concs, mats);
+      __syncthreads();
+      hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
+      cached = n_iso;
+      __syncthreads();
+    }
+    XsParams xp;
+    xp.n_iso = n_iso;
+    xp.n_gp = d->n_gp;
+    xp.grid = d->grid;
+    xp.bins = d->bins;
+    xp.lookups = (long long)d->lookups;
+    const long long s0 = (long long)(item - d->item0) * kXsItemLookups;
+    const long long s1 = s0 + kXsItemLookups < xp.lookups ? s0 + kXsItemLookups : xp.lookups;
+    double *dmp = p.dump ? p.dump + (size_t)d->k * p.dump_rows * 8 : nullptr;
+    unsigned long long ver = 0, bsum = 0;
+    double fsum = 0.0, fabs_ = 0.0;
+    xs2_item<GRID>(*d, xp, s0, s1, nn, concs, mats, am, dmp, p.dump_rows, ver, bsum, fsum, fabs_);
+    ver = block_sum_u64(sh, ver);
+    bsum = block_sum_u64(sh, bsum);
+    fsum = block_sum_f64(sh, fsum);
+    fabs_ = block_sum_f64(sh, fabs_);
+    if (tid == 0) {
+      XsItemPart *ip = reinterpret_cast<XsItemPart *>(p.ipart) + item;
+      ip->ver = ver;
+      ip->bsum = bsum;
+      ip->fsum = fsum;
+      ip->fabs = fabs_;
+      for (int a = 0; a < 5; a++) ip->am[a] = am[a];
+      __threadfence();
+      misc[1] = atomicAdd(&p.idone[j], 1u) == d->n_items - 1 ? 1u : 0u;
+    }
+    __syncthreads();
+    if (misc[1]) xs2_finish(p, c, d, misc);
+    __syncthreads();  // misc, desc, am reused by the next item
+  }
+}
+
+int xs_items_threads() { return kXs2T; }
+
+static const void *xs_items_fn(int grid) {
+  switch (grid) {
+    case XS_HASH: return (const void *)xs_items_kernel<XS_HASH>;
+    case XS_UNIONIZED: return (const void *)xs_items_kernel<XS_UNIONIZED>;
+    case XS_NUCLIDE: return (const void *)xs_items_kernel<XS_NUCLIDE>;
+  }
+  return nullptr;
+}
+
+cudaError_t xs_items_occupancy(int grid, int *ctas) {
+  const void *fn = xs_items_fn(grid);
+  if (!fn) return cudaErrorInvalidValue;
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kXs2Smem);
+  if (e != cudaSuccess) return e;
+  int per_sm = 0, dev = 0, sms = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kXs2T, kXs2Smem);
+  if (e == cudaSuccess) e = cudaGetDevice(&dev);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  *ctas = per_sm * sms;
+  return e;
+}
+
+cudaError_t launch_xs_items(int grid_type, int ctas, const KParams &p, cudaStream_t st) {
+  const void *fn = xs_items_fn(grid_type);
+  if (!fn) return cudaErrorInvalidValue;
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kXs2Smem);
+  if (e != cudaSuccess) return e;
+  void *args[] = {const_cast<KParams *>(&p)};
+  return cudaLaunchKernel(fn, dim3((unsigned)ctas), dim3((unsigned)kXs2T), args, kXs2Smem, st);
+}
+
+}  // namespace ens

@@ -31,6 +31,16 @@ struct KParams {
   uint32_t sub_stride;        // dynamic smem bytes per instance slot of the CTA
   double *dump;               // [n_instances][dump_rows][8] element-wise results, or null
   uint32_t dump_rows;
+  // split phases (XS): phase 1 = this kernel with one arena slot per instance
+  // (slot = group-local queue index) and a descriptor per instance; phase 2 =
+  // the lookup kernel over the item queue
+  uint32_t split;
+  char *xs_desc;              // [n] XsDesc
+  const uint32_t *items;      // [all items] group-local instance of each item (batch = item - its item0)
+  uint32_t item_base, n_items; // phase 2: this launch's items (one grid type)
+  char *ipart;                // [n_items] XsItemPart
+  uint32_t *idone;            // [n] items finished per instance (zeroed)
+  uint32_t *counter2;         // phase-2 item counter (zeroed)
 };
 
 const void *kernel_ptr(uint32_t app, int T);
@@ -39,10 +49,15 @@ int app_max_threads(uint32_t app);
 bool app_team_aware(uint32_t app);
 double app_cost(uint32_t app, int argc, const char *const *argv);
 bool app_sub_aware(uint32_t app);
+uint32_t app_items(uint32_t app, int argc, const char *const *argv, int *kind);
 uint32_t sub_shared_bytes();
 bool app_size(uint32_t app, int argc, const char *const *argv, int T, int cs, uint64_t *arena, uint32_t *smem);
 cudaError_t launch_group(uint32_t app, int T, int m, int grid, int cs, size_t smem, const KParams &p,
                          cudaStream_t st);
 cudaError_t group_occupancy(uint32_t app, int T, int m, int cs, size_t smem, int *teams);
+// split phases, phase 2 (kernels_xs2.cu): the XS lookup-item kernel
+cudaError_t launch_xs_items(int grid_type, int ctas, const KParams &p, cudaStream_t st);
+cudaError_t xs_items_occupancy(int grid_type, int *ctas);
+int xs_items_threads();
 
 }  // namespace ens

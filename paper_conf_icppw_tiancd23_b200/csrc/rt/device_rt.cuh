@@ -141,6 +141,7 @@ struct Result {  // meaningful in thread 0 after the body returns
   uint64_t vhash, bitsum;
   double fsum, fabs;
   uint64_t work;
+  int deferred;  // set by EVERY thread: the record is written by a later phase (split phases)
 };
 
 // The team running one instance: one CTA (the paper's team = thread block,
@@ -161,6 +162,8 @@ struct Ctx {
   unsigned long long t_mark;   // tracing: last mark (team thread 0)
   double *dump;                // element-wise dump rows of this instance (testing), or null
   uint32_t dump_rows;
+  char *desc;                  // split phases: this instance's phase-2 descriptor, or null
+  unsigned long long t_start;  // ENS_F_TIMESTAMPS: %globaltimer at the instance's start (thread 0)
 };
 // element-wise dump (ens_launch_cfg.dump_rows): row `slot` = {key, mat,
 // v[0..nv), argmax}, zero-padded to 8 doubles

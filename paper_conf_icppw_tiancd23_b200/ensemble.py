@@ -23,7 +23,7 @@ class Ensemble:
 
     def __init__(self, args, app="auto", n=None, first=0, stride=1, threads=256, grid=0, arena_bytes=0,
                  stdout_bytes=0, timestamps=False, device=None, stream=None, team_ctas=0, phases=False,
-                 instances_per_cta=0, generic=False, serial=False, dump_rows=0):
+                 instances_per_cta=0, generic=False, serial=False, dump_rows=0, fused=False, split=False):
         _require_cuda()
         self.args = args
         self.app = app
@@ -33,7 +33,8 @@ class Ensemble:
         self.cfg = make_cfg(n, first=first, stride=stride, grid=grid, threads=threads, arena_bytes=arena_bytes,
                             stdout_bytes=stdout_bytes,
                             flags=(_ens.ENS_F_TIMESTAMPS if timestamps else 0) | (_ens.ENS_F_PHASES if phases else 0)
-                            | (_ens.ENS_F_GENERIC if generic else 0) | (_ens.ENS_F_SERIAL if serial else 0),
+                            | (_ens.ENS_F_GENERIC if generic else 0) | (_ens.ENS_F_SERIAL if serial else 0)
+                            | (_ens.ENS_F_FUSED if fused else 0) | (_ens.ENS_F_SPLIT_PHASES if split else 0),
                             team_ctas=team_ctas, instances_per_cta=instances_per_cta, dump_rows=dump_rows)
         self.n = n
         self.device = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
@@ -95,7 +96,10 @@ class Ensemble:
         if self.run is not None:
             self.run.close()
             self.run = None
+        big = self.workspace is not None and self.workspace.numel() > (8 << 30)
         self.workspace = None
+        if big:  # hand a large workspace back to the device (ens_workspace_bytes sizes by free memory)
+            torch.cuda.empty_cache()
 
 
 def run_text(text, app="auto", argv0=None, **kw):

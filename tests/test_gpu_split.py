@@ -1,0 +1,92 @@
+"""Split phases (ENS_F_SPLIT_PHASES): phase 1 = the ensemble kernel builds each XS instance's
+tables and sorted lookups in an arena slot of its own; phase 2 = the lookup-item kernel over
+every SM writes the records.  Results must equal the oracle's (and the fused path's) exactly:
+records, tallies, stdout, element-wise dumps."""
+import numpy as np
+import pytest
+
+pytestmark = pytest.mark.gpu
+
+from parity import assert_parity  # noqa: E402
+
+LINES = [
+    "xsbench -s small -g 1000 -l 10000 -G unionized -r 1070",
+    "xsbench -s small -g 37 -l 4096 -G unionized -r 3",          # exactly one item
+    "xsbench -s small -g 1500 -l 4097 -G hash -h 1000 -r 11",    # one item + 1 lookup
+    "xsbench -s small -g 300 -l 9000 -G nuclide -r 9",
+    "xsbench -s large -g 200 -l 12000 -G hash -h 500 -r 6",
+    "xsbench -s large -g 60 -l 5000 -G unionized -r 8",
+    "xsbench -s small -g 20000 -l 3000 -G hash -h 1000 -r 21",   # arena-scratch init
+    "xsbench -s small -g 100 -l 0 -r 5",                         # no lookups: fused in phase 1
+    "xsbench -s small -g 100 -m history -p 50 -l 4 -r 7",        # history: fused in phase 1
+    "xsbench -g 1",                                              # usage error
+    "rsbench -s small -l 500 -p 20 -w 4 -r 3",                   # other apps alongside
+    "amgmk -x 8 -y 8 -z 8 -i 5 -r 4",
+]
+
+
+def run(lines, **kw):
+    from paper_conf_icppw_tiancd23_b200.ensemble import Ensemble
+    from paper_conf_icppw_tiancd23_b200 import Args
+    e = Ensemble(Args.parse("".join(l + "\n" for l in lines)), app="auto", **kw).launch()
+    out = e.collect()
+    info = e.info()
+    e.close()
+    return out, info
+
+
+@pytest.mark.parametrize("threads,team", [(512, 0), (256, 1), (128, 2)])
+def test_split_matches_oracle(oracle, threads, team):
+    g, info = run(LINES, threads=threads, team_ctas=team, split=True)
+    assert info.kernel_launches > info.n_groups  # phase-2 kernels were launched
+    o = oracle.run_text("".join(l + "\n" for l in LINES))
+    assert_parity(g, o)
+
+
+def test_split_elementwise(oracle):
+    rows = 12000
+    g, _ = run(LINES, threads=512, split=True, dump_rows=rows)
+    o = oracle.run_text("".join(l + "\n" for l in LINES), dump=rows)
+    for k, line in enumerate(LINES):
+        if not line.startswith("xsbench") or "-l 0" in line or "history" in line or "-g 1" == line[-5:]:
+            continue
+        gd = g.dump[k]
+        gd = gd[~np.all(gd == 0, axis=1)]
+        od = o.dumps[k]
+        if len(od) == 0:
+            continue
+        gs, os_ = gd[np.lexsort((gd[:, 1], gd[:, 0]))], od[np.lexsort((od[:, 1], od[:, 0]))]
+        assert gs.shape == os_.shape, line
+        assert np.array_equal(gs.view(np.uint64), os_.view(np.uint64)), line
+
+
+def test_split_equals_fused_and_relaunch():
+    from paper_conf_icppw_tiancd23_b200.ensemble import Ensemble
+    from paper_conf_icppw_tiancd23_b200 import Args
+    lines = [f"xsbench -s large -g 300 -l 20000 -G hash -h 300 -r {i}" for i in range(6)]
+    a, _ = run(lines, threads=512, split=True)
+    b, _ = run(lines, threads=512, fused=True)
+    for f in ("instance", "exit_code", "vhash", "bitsum", "work", "stdout_len"):
+        assert np.array_equal(a.records[f], b.records[f]), f
+    assert np.allclose(a.records["fsum"], b.records["fsum"], rtol=1e-12, atol=0)
+    assert np.array_equal(a.tallies, b.tallies) and a.stdout == b.stdout
+    # relaunch on the same workspace (device-resident args): identical up to fsum / fabs, whose
+    # terms the sort's atomic bucket order permutes (as in the fused path)
+    e = Ensemble(Args.parse("".join(l + "\n" for l in lines)), app="auto", threads=512, split=True).launch()
+    r1 = e.collect()
+    e.relaunch()
+    r2 = e.collect()
+    e.close()
+    for f in ("instance", "exit_code", "vhash", "bitsum", "work", "stdout_len"):
+        assert np.array_equal(r1.records[f], r2.records[f]), f
+    assert np.allclose(r1.records["fsum"], r2.records["fsum"], rtol=1e-12, atol=0)
+    assert np.array_equal(r1.tallies, r2.tallies) and r1.stdout == r2.stdout
+
+
+def test_auto_policy():
+    # 64 large hash instances x 1M lookups: fewer instances than SMs -> split; 1024 small: fused
+    from paper_conf_icppw_tiancd23_b200 import workloads
+    _, info = run(workloads.c2(16, lookups=200000), threads=512)
+    assert info.kernel_launches == 2
+    _, info = run(workloads.tstar(300), threads=512)
+    assert info.kernel_launches == 1
