@@ -230,6 +230,19 @@ int ens_collect_dump(ens_run *r, double *out, size_t cap);
 /* CUDA-event time of the last (re)launch's kernels, in ms.                   */
 int ens_run_elapsed_ms(ens_run *r, float *ms);
 
+/* Device time of each kernel of the last (re)launch, in launch order: per
+ * app group its ensemble kernel (phase 1), then, for split XS groups, one
+ * lookup-item kernel per XS grid type present (phase 2; kind = 0 unionized,
+ * 1 nuclide, 2 hash).  Each is bracketed by CUDA events on the stream it
+ * runs on.  Returns the number of kernels (<= cap) or <0 (ENS_ERANGE if cap
+ * is too small).  Blocks until the run is done.                              */
+typedef struct {
+  int32_t app, phase, kind;  /* ens_app; 1 or 2; XS grid type of phase 2, else -1 */
+  int32_t grid_ctas, block_threads;
+  float ms;
+} ens_kernel_time;
+int ens_run_kernel_times(ens_run *r, ens_kernel_time *out, int cap);
+
 /* Tracing (launched with ENS_F_PHASES): ns[p] = sum over instances of the
  * %globaltimer time team thread 0 spent in phase p of the last (re)launch
  * (XS: 0 materials, 1 generate, 2 bucket scan, 3 scatter, 4 bucket sort,

@@ -47,6 +47,11 @@ class LaunchCfg(ctypes.Structure):
                 ("dump_rows", ctypes.c_uint32)]
 
 
+class KernelTime(ctypes.Structure):
+    _fields_ = [("app", ctypes.c_int32), ("phase", ctypes.c_int32), ("kind", ctypes.c_int32),
+                ("grid_ctas", ctypes.c_int32), ("block_threads", ctypes.c_int32), ("ms", ctypes.c_float)]
+
+
 class RunInfo(ctypes.Structure):
     _fields_ = [("n_instances", ctypes.c_int32), ("n_groups", ctypes.c_int32),
                 ("grid_blocks", ctypes.c_int32 * ENS_N_APPS), ("block_threads", ctypes.c_int32 * ENS_N_APPS),
@@ -79,6 +84,7 @@ def _load():
         "ens_collect_dump": (i, [p, p, sz]),
         "ens_run_elapsed_ms": (i, [p, ctypes.POINTER(ctypes.c_float)]),
         "ens_run_phases": (i, [p, ctypes.POINTER(ctypes.c_uint64)]),
+        "ens_run_kernel_times": (i, [p, ctypes.POINTER(KernelTime), i]),
         "ens_run_get_info": (i, [p, ctypes.POINTER(RunInfo)]),
         "ens_format_stdout": (ctypes.c_long, [u32, p, sz, p, sz]),
         "ens_run_free": (None, [p]),
@@ -97,7 +103,7 @@ lib = _load()
 EXPORTED = ["ens_load_args", "ens_parse_args", "ens_expand_args", "ens_args_count", "ens_args_get", "ens_args_free",
             "ens_workspace_bytes", "ens_launch", "ens_run_relaunch", "ens_collect", "ens_collect_dump",
             "ens_run_elapsed_ms",
-            "ens_run_phases",
+            "ens_run_phases", "ens_run_kernel_times",
             "ens_run_get_info", "ens_format_stdout", "ens_run_free", "ens_strerror", "ens_last_error",
             "ens_version"]
 
@@ -225,6 +231,14 @@ class Run:
         ms = ctypes.c_float()
         _check("ens_run_elapsed_ms", lib.ens_run_elapsed_ms(self._h, ctypes.byref(ms)))
         return ms.value
+
+    def kernel_times(self):
+        """[(app, phase, kind, grid_ctas, block_threads, ms)] of the last (re)launch's kernels."""
+        a = (KernelTime * 16)()
+        n = lib.ens_run_kernel_times(self._h, a, 16)
+        if n < 0:
+            _check("ens_run_kernel_times", n)
+        return [(a[q].app, a[q].phase, a[q].kind, a[q].grid_ctas, a[q].block_threads, a[q].ms) for q in range(n)]
 
     def phases_ns(self):
         """Per-phase device time summed over instances (launched with ENS_F_PHASES)."""

@@ -1305,6 +1305,9 @@ struct XsApp {
   // nuclide j+1's guess and pair address computed and the pair prefetched,
   // nuclide j's pair gathered, verified and accumulated.  The bracket logic
   // and every FP operation are those of macro_lookup<XS_HASH> (bit-identical).
+#ifndef ENS_XS2_PF
+#define ENS_XS2_PF 0
+#endif
   __device__ static __forceinline__ void macro_lookup_hash1(const XsParams &p, const double *recs, const int *ig,
                                                             const int *nn, const double *concs,
                                                             const uint16_t *mats, double pe, int mat, int idx,
@@ -1331,6 +1334,29 @@ struct XsApp {
       return reinterpret_cast<const double2 *>(recs + ((uint32_t)mrow[j] * (uint32_t)n_gp + (uint32_t)lo) * 6u);
     };
     double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
+#if ENS_XS2_PF > 0
+    // deep software pipeline: entry j+PF+3 prefetched into L1, entry j+PF
+    // loaded (prefetched 3 steps ago) and its pair prefetched into L1 (PF
+    // steps ahead of its use: about one L2 round trip at 6 warps per
+    // scheduler), entry j re-loaded (an L1 hit) for this step's bracket
+    constexpr int PF = ENS_XS2_PF;
+    for (int j = 0; j < PF + 3 && j < nm; j++) prefetch_l1(ent(j));
+    for (int j = 0; j < PF && j < nm; j++) {
+      const double2 *q = pair_at(j, guess(ld_(ent(j))));
+      prefetch_l1(q);
+      prefetch_l1(reinterpret_cast<const double *>(q) + 11);
+    }
+    for (int j = 0; j < nm; j++) {
+      const uint4 h0 = ld_(ent(j));
+      if (j + PF + 3 < nm) prefetch_l1(ent(j + PF + 3));
+      if (j + PF < nm) {
+        const double2 *q = pair_at(j + PF, guess(ld_(ent(j + PF))));
+        prefetch_l1(q);
+        prefetch_l1(reinterpret_cast<const double *>(q) + 11);
+      }
+      const int lo0 = guess(h0);
+      const double2 *q0 = pair_at(j, lo0);
+#else
     const uint4 z = make_uint4(0, 0, 0, 0);
     uint4 h0 = nm > 0 ? ld_(ent(0)) : z;
     uint4 h1 = nm > 1 ? ld_(ent(1)) : z;
@@ -1349,6 +1375,7 @@ struct XsApp {
         prefetch_l1(q1);
         prefetch_l1(reinterpret_cast<const double *>(q1) + 11);
       }
+#endif
       double2 a0 = ld_(q0 + 0), a1 = ld_(q0 + 1), a2 = ld_(q0 + 2);
       double2 b0 = ld_(q0 + 3), b1 = ld_(q0 + 4), b2 = ld_(q0 + 5);
       {  // verify the guessed pair; walk / upstream search otherwise (macro_lookup's gather_fix)
@@ -1376,10 +1403,12 @@ struct XsApp {
         }
       }
       accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
+#if ENS_XS2_PF == 0
       h0 = h1;
       h1 = h2;
       q0 = q1;
       lo0 = lo1;
+#endif
     }
     m[0] = m0;
     m[1] = m1;

@@ -226,6 +226,11 @@ struct ens_run {
   std::string c_text;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   std::vector<cudaEvent_t> ev_join;  // concurrent groups: one per forked group
+  struct KTime {                     // one kernel of a launch, bracketed by two events on its stream
+    ens_kernel_time info;
+    cudaEvent_t a = nullptr, b = nullptr;
+  };
+  std::vector<KTime> kt;
   uint32_t flags = 0;
   bool launched = false;
   uint64_t d2h = 0;
@@ -642,8 +647,28 @@ static int enqueue(ens_run *r) {
       CU(aux_stream(gi - 1, &st));
       CU(cudaStreamWaitEvent(st, r->ev0, 0));
     }
+    size_t nk = 0;  // kernels of this launch so far (r->kt grows on the first enqueue)
+    for (size_t q = 0; q < gi; q++) nk += 1 + (P.groups[q].split ? (P.groups[q].kind_n[0] > 0) + (P.groups[q].kind_n[1] > 0) + (P.groups[q].kind_n[2] > 0) : 0);
+    auto kt_begin = [&](int phase, int kind, int grid, int block) -> int {
+      if (r->kt.size() <= nk) {
+        ens_run::KTime t;
+        if (cudaEventCreate(&t.a) != cudaSuccess || cudaEventCreate(&t.b) != cudaSuccess) return -1;
+        r->kt.push_back(t);
+      }
+      ens_kernel_time &i = r->kt[nk].info;
+      i.app = (int32_t)(g.app == APP_NOTFOUND ? 0u : g.app);
+      i.phase = phase;
+      i.kind = kind;
+      i.grid_ctas = grid;
+      i.block_threads = block;
+      i.ms = 0.f;
+      return cudaEventRecord(r->kt[nk].a, st) == cudaSuccess ? 0 : -1;
+    };
+    auto kt_end = [&]() -> int { return cudaEventRecord(r->kt[nk++].b, st) == cudaSuccess ? 0 : -1; };
+    if (kt_begin(1, -1, g.ctas(), g.T)) return fail(ENS_ECUDA, "ens_launch: kernel timing events");
     cudaError_t e = launch_group(g.app, g.T, g.m, g.ctas(), g.cs, g.dyn(), k, st);
     if (e != cudaSuccess) return cuda_fail(e, "ens_kernel launch");
+    if (kt_end()) return fail(ENS_ECUDA, "ens_launch: kernel timing events");
     for (int kd = 0; g.split && kd < 3; kd++) {  // phase 2: every instance's lookup items, on every SM
       if (!g.kind_n[kd]) continue;
       const int ctas2 = std::max(1, std::min<int>(g.grid2[kd], (int)g.kind_n[kd]));
@@ -651,8 +676,10 @@ static int enqueue(ens_run *r) {
       k2.item_base = g.kind_base[kd];
       k2.n_items = g.kind_n[kd];
       k2.counter2 = (uint32_t *)(r->ws + g.ctr2_off + 8 * kd);
+      if (kt_begin(2, kd, ctas2, xs_items_threads())) return fail(ENS_ECUDA, "ens_launch: kernel timing events");
       e = launch_xs_items(kd, ctas2, k2, st);
       if (e != cudaSuccess) return cuda_fail(e, "xs_items_kernel launch");
+      if (kt_end()) return fail(ENS_ECUDA, "ens_launch: kernel timing events");
     }
     if (P.concurrent && gi > 0) {  // join back into the launch stream
       CU(cudaEventRecord(r->ev_join[gi - 1], st));
@@ -884,6 +911,24 @@ extern "C" int ens_run_elapsed_ms(ens_run *r, float *ms) {
   return ENS_OK;
 }
 
+extern "C" int ens_run_kernel_times(ens_run *r, ens_kernel_time *out, int cap) {
+  if (!r || (!out && cap)) return fail(ENS_EINVAL, "ens_run_kernel_times: NULL");
+  if (!r->launched || r->P.n == 0) return 0;
+  CU(cudaEventSynchronize(r->ev1));
+  int n = 0;
+  for (int q = 0; q < (int)r->P.groups.size(); q++) {
+    const Group &g = r->P.groups[q];
+    n += 1 + (g.split ? (g.kind_n[0] > 0) + (g.kind_n[1] > 0) + (g.kind_n[2] > 0) : 0);
+  }
+  if (cap < n) return fail(ENS_ERANGE, "ens_run_kernel_times: cap smaller than the kernel count");
+  for (int q = 0; q < n; q++) {
+    ens_kernel_time t = r->kt[(size_t)q].info;
+    CU(cudaEventElapsedTime(&t.ms, r->kt[(size_t)q].a, r->kt[(size_t)q].b));
+    out[q] = t;
+  }
+  return n;
+}
+
 extern "C" int ens_run_get_info(const ens_run *r, ens_run_info *info) {
   if (!r || !info) return fail(ENS_EINVAL, "ens_run_get_info: NULL");
   std::memset(info, 0, sizeof *info);
@@ -931,6 +976,10 @@ extern "C" void ens_run_free(ens_run *r) {
   if (r->ev0) cudaEventDestroy(r->ev0);
   if (r->ev1) cudaEventDestroy(r->ev1);
   for (cudaEvent_t ej : r->ev_join) cudaEventDestroy(ej);
+  for (auto &t : r->kt) {
+    cudaEventDestroy(t.a);
+    cudaEventDestroy(t.b);
+  }
   delete r;
 }
 

@@ -3,6 +3,10 @@
     python tools/ncu_summary.py launches <ncu --csv log> <out.json> "<command>"
         per-launch device times of `ncu --metrics gpu__time_duration.sum
         --clock-control none --csv ...` (cold-cache, serialised)
+    python tools/ncu_summary.py counters <report.ncu-rep> <workload>
+        per kernel of the capture: dram__bytes_read.sum + dram__bytes_write.sum and
+        smsp__inst_executed.sum into profiles/ncu_counters.json[workload] (read by
+        bench.py's roofline: the dram and issue candidates)
     python tools/ncu_summary.py full <report.ncu-rep> <out.txt> [workload]
         key counters of one `ncu --set full` capture + warp-stall samples by
         source line; with a workload name, also writes profiles/traffic.json
@@ -112,7 +116,54 @@ def full(rep, out, workload=None):
         print(f"traffic[{workload}] = {tb:.4g} B -> {tp}")
 
 
+APP_OF = {"EchoApp": 1, "XsApp": 2, "RsApp": 3, "AmgApp": 4, "PrApp": 5}
+
+
+def kernel_key(name):
+    """bench.py's key of a kernel: phase1_app<id> for ens_kernel<App,T>, phase2_kind<grid> for
+    xs_items_kernel<grid>."""
+    m = re.search(r"xs_items_kernel<\(?i?n?t?\)?(\d)>", name)
+    if m:
+        return f"phase2_kind{m.group(1)}"
+    for k, v in APP_OF.items():
+        if k in name:
+            return f"phase1_app{v}"
+    return None
+
+
+def counters(rep, workload):
+    raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv", "--metrics",
+                          "dram__bytes_read.sum,dram__bytes_write.sum,smsp__inst_executed.sum,gpu__time_duration.sum"],
+                         capture_output=True, text=True).stdout
+    rows = list(csv.reader(raw.splitlines()))
+    hdr, units = rows[0], rows[1]
+    out = {}
+    for r in rows[2:]:
+        d = {hdr[i]: (r[i], units[i]) for i in range(len(hdr))}
+        key = kernel_key(d["Kernel Name"][0])
+        if not key:
+            continue
+        tb = 0.0
+        for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
+            v, u = d[k]
+            tb += float(v.replace(",", "")) * UNIT.get(u, 1)
+        ms = float(d["gpu__time_duration.sum"][0].replace(",", ""))
+        if d["gpu__time_duration.sum"][1] == "us":
+            ms /= 1e3
+        out[key] = {"dram_bytes": tb, "inst_executed": float(d["smsp__inst_executed.sum"][0].replace(",", "")),
+                    "ncu_ms": ms, "kernel": d["Kernel Name"][0], "source": os.path.relpath(rep, ROOT)}
+    p = os.path.join(ROOT, "profiles", "ncu_counters.json")
+    allc = json.load(open(p)) if os.path.exists(p) else {}
+    allc[workload] = {"kernels": out, "note": "one ncu --set full capture of a warm launch (--clock-control none); "
+                                              "per-launch counters, cold-cache serialised times"}
+    json.dump(allc, open(p, "w"), indent=1)
+    print(f"{workload}: {list(out)} -> {p}")
+
+
 if __name__ == "__main__":
+    if sys.argv[1] == "counters":
+        counters(sys.argv[2], sys.argv[3])
+        sys.exit(0)
     if sys.argv[1] == "launches":
         launches(sys.argv[2], sys.argv[3], sys.argv[4] if len(sys.argv) > 4 else "")
     else:
