@@ -389,6 +389,37 @@ ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   return S;
 }
 
+// split phases, phase 1b (the init-item kernel): a compact layout without the
+// material tables — pick_mat thresholds, the lookup sort's material offsets,
+// the LCG jump tables, then the per-nuclide sort's counters and keys exactly
+// as xs_smem places them (so init_nuc_t's hash-column reuse test is the same)
+ENS_HD XsSmem xs_init_smem(const XsParams &p) {
+  XsSmem S{};
+  uint32_t o = 0;
+  S.thr = o; o += 12 * 8;
+  S.nn = o; o += 16 * 4;
+  S.concs = o;
+  S.mats = o;
+  S.mcnt = o; o += 32 * 4;
+  S.jmp = o; o += 5 * 64 * 16;
+  S.nbkt = o;
+  if (p.grid != XS_UNIONIZED && xs_nuc_smem(p)) {
+    o += (uint32_t)align_up((uint64_t)xs_nbn(p.n_gp) * 4, 16);
+    S.ubkt = o;
+    S.nkey = o;
+    o += (uint32_t)align_up((uint64_t)p.n_gp * 6, 16);
+    if (p.grid == XS_HASH) {
+      const uint64_t need = align_up((uint64_t)(p.bins + 1) * 4, 16) + (uint64_t)p.n_gp * 4, have = o - S.nbkt;
+      if (need > have && need - have <= 16384) o = S.nbkt + (uint32_t)align_up(need, 16);
+    }
+  } else {
+    S.ubkt = o;
+    S.nkey = o;
+  }
+  S.total = o;
+  return S;
+}
+
 // ============================ RSBench-style ================================
 struct RsParams {
   int n_nuc = 355;

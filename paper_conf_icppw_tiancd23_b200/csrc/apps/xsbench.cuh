@@ -190,7 +190,11 @@ struct XsApp {
     __syncthreads();
     hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
     phase_mark(c, 0);
-    if (p.grid == XS_UNIONIZED) {
+    // split phases: a hash / nuclide instance's per-nuclide tables are built
+    // by the init-item kernel (kernels_xs2.cu) running beside this kernel
+    const bool init_items = c.desc && xs_split_ok(p) && p.grid != XS_UNIONIZED;
+    if (init_items) {
+    } else if (p.grid == XS_UNIONIZED) {
       const bool warp_path = xs_warp_union(p) && !(c.flags & ENS_F_GENERIC);
       if (!warp_path && !xs_smem_nb(p)) init(c, p, L, S, c.csize > 1);  // block-wide, striped over the team
       else if (c.crank == 0 && !(warp_path && init_warp(c, p, L, S)))
@@ -200,27 +204,13 @@ struct XsApp {
     }
     team_sync(c);
     if (c.desc && xs_split_ok(p)) {  // split phases: sort the lookups, hand them to phase 2
-      uint32_t *mcnt = (uint32_t *)(ens_smem(c) + S.mcnt);
-      lookup_sort(c, p, L, thr, 0, p.lookups);
-      if (c.crank == 0 && threadIdx.x == 0) {
-        XsDesc *d = reinterpret_cast<XsDesc *>(c.desc);
-        d->recs = (uint64_t)(c.arena + L.recs);
-        d->index = (uint64_t)(c.arena + L.index);
-        d->uenergy = (uint64_t)(c.arena + L.uenergy);
-        d->ufind = (uint64_t)(c.arena + L.ufind);
-        d->lk_pe = (uint64_t)(c.arena + L.lk_pe);
-        d->lookups = (uint64_t)p.lookups;
-        d->seed = p.seed;
-        d->ubins = xs_ubins(p);
-        for (int m = 0; m < 13; m++) d->mcnt[m] = mcnt[16 + m];
-        d->n_iso = p.n_iso;
-        d->n_gp = p.n_gp;
-        d->grid = p.grid;
-        d->bins = p.bins;
-        d->k = c.k;
-        d->line = c.id;
-        d->t_start = c.t_start;
+      if (init_items) {  // the init-item kernel builds the tables, sorts and writes the descriptor
+        R.deferred = 1;
+        return R;
       }
+      uint32_t *mcnt = (uint32_t *)(ens_smem(c) + S.mcnt);
+      lookup_sort(c, p, L, thr, mcnt, 0, p.lookups);
+      if (c.crank == 0 && threadIdx.x == 0) write_desc(c, p, L, mcnt);
       R.deferred = 1;
       return R;
     }
@@ -243,6 +233,27 @@ struct XsApp {
     ens_printf(c, FMT_VERIFY, (unsigned long long)R.vhash);
     R.exit_code = 0;
     return R;
+  }
+
+  // split phases: the instance's phase-2 descriptor (one thread)
+  __device__ static void write_desc(const Ctx &c, const XsParams &p, const XsLayout &L, const uint32_t *mcnt) {
+    XsDesc *d = reinterpret_cast<XsDesc *>(c.desc);
+    d->recs = (uint64_t)(c.arena + L.recs);
+    d->index = (uint64_t)(c.arena + L.index);
+    d->uenergy = (uint64_t)(c.arena + L.uenergy);
+    d->ufind = (uint64_t)(c.arena + L.ufind);
+    d->lk_pe = (uint64_t)(c.arena + L.lk_pe);
+    d->lookups = (uint64_t)p.lookups;
+    d->seed = p.seed;
+    d->ubins = xs_ubins(p);
+    for (int m = 0; m < 13; m++) d->mcnt[m] = mcnt[16 + m];
+    d->n_iso = p.n_iso;
+    d->n_gp = p.n_gp;
+    d->grid = p.grid;
+    d->bins = p.bins;
+    d->k = c.k;
+    d->line = c.id;
+    d->t_start = c.t_start;
   }
 
   // the LCG state s advanced by 6r draws (record r's draws are 6r+1..6r+6,
@@ -371,21 +382,36 @@ struct XsApp {
   // walk over the sorted energies, each bin written once (XS-5: ig[i][b] = grid_search(E_i, b*du) = min(#{k>=1: E_k <= b*du}, n_gp-2)).
   // SMK: the sort's keys and counters in shared memory (n_gp <= kXsSmemGp),
   // else in this CTA's arena scratch (L2 atomics; the same algorithm)
+  // The team's CTAs take nuclides crank, crank + csize, ... with per-CTA
+  // scratch in the arena; init_nuc_range runs nuclides [i0, i1) with the
+  // caller's scratch (split phases: one nuclide per work item, kernels_xs2.cu)
   __device__ static void init_nuc(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
-    if (xs_nuc_smem(p)) init_nuc_t<true>(c, p, L, S);
-    else init_nuc_t<false>(c, p, L, S);
+    char *ekey = c.arena + L.keys + (size_t)c.crank * p.n_gp * 8;
+    char *col = c.arena + L.hcol + (size_t)c.crank * (p.bins + 1) * 4;
+    char *gscr = c.arena + L.nscr + (size_t)c.crank * xs_nscr_bytes(p);
+    init_nuc_range(c, p, L, S, (int)c.crank, p.n_iso, (int)c.csize, ekey, col, gscr);
+  }
+  __device__ static void init_nuc_range(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S, int i0,
+                                        int i1, int istep, char *ekey, char *col, char *gscr) {
+    if (xs_nuc_smem(p)) init_nuc_t<true>(c, p, L, S, i0, i1, istep, ekey, col, gscr);
+    else init_nuc_t<false>(c, p, L, S, i0, i1, istep, ekey, col, gscr);
+  }
+  // per-CTA scratch bytes of init_nuc_range: sorted energies, hash column, sort scratch
+  ENS_HD static uint64_t nuc_scratch_bytes(const XsParams &p) {
+    return align_up((uint64_t)p.n_gp * 8, 256) + align_up((uint64_t)(p.bins + 1) * 4, 256) + xs_nscr_bytes(p);
   }
   template <bool SMK>
-  __device__ static __noinline__ void init_nuc_t(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
+  __device__ static __noinline__ void init_nuc_t(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S,
+                                                 int i0, int i1, int istep, char *ekey_scr, char *col_scr,
+                                                 char *gscr) {
     const bool trc = tracing(c);  // tracing (ENS_F_PHASES) thread, cached
     const int tid = threadIdx.x, T = blockDim.x;
-    const int n_iso = p.n_iso, n_gp = p.n_gp;
+    const int n_gp = p.n_gp;
     const int nbn = xs_nbn(n_gp);
-    char *gscr = c.arena + L.nscr + (size_t)c.crank * xs_nscr_bytes(p);
     uint32_t *nb = SMK ? (uint32_t *)(ens_smem(c) + S.nbkt) : (uint32_t *)gscr;
     const Affine *jt = (const Affine *)(ens_smem(c) + S.jmp);
     double *recs = (double *)(c.arena + L.recs);
-    unsigned long long *ekey = (unsigned long long *)(c.arena + L.keys);  // sorted energies (this CTA's)
+    unsigned long long *ekey = (unsigned long long *)ekey_scr;  // sorted energies (this CTA's)
     const size_t kofs = SMK ? 0 : align_up((uint64_t)nbn * 4, 256);
     uint32_t *K = SMK ? (uint32_t *)(ens_smem(c) + S.nkey) : (uint32_t *)(gscr + kofs);  // sort keys, then
     uint16_t *J = SMK ? (uint16_t *)(ens_smem(c) + S.nkey + (size_t)n_gp * 4)            // record indices j
@@ -397,10 +423,8 @@ struct XsApp {
     auto nkey_bkt = [&](uint32_t key) { return kbits ? (int)(key >> (32 - kbits)) : 0; };
     const double du = 1.0 / p.bins;
     const Affine J6T = lcg_pow(6ULL * T), J24T = lcg_pow(24ULL * T);
-    // this CTA takes nuclides crank, crank + csize, ... with its own scratch
-    ekey += (size_t)c.crank * n_gp;
-    for (int i = (int)c.crank; i < n_iso; i += (int)c.csize) {
-      int *col = (int *)(c.arena + L.hcol) + (size_t)c.crank * (p.bins + 1);  // this CTA's column
+    for (int i = i0; i < i1; i += istep) {
+      int *col = (int *)col_scr;  // this CTA's column
       XsHashEnt *ent = (XsHashEnt *)ig + (size_t)i * (p.bins + 1);
       const uint32_t r0 = (uint32_t)i * (uint32_t)n_gp;  // record i*n_gp + j
       for (int b = tid; b < nbn; b += T) nb[b] = 0;
@@ -1305,9 +1329,6 @@ struct XsApp {
   // nuclide j+1's guess and pair address computed and the pair prefetched,
   // nuclide j's pair gathered, verified and accumulated.  The bracket logic
   // and every FP operation are those of macro_lookup<XS_HASH> (bit-identical).
-#ifndef ENS_XS2_PF
-#define ENS_XS2_PF 0
-#endif
   __device__ static __forceinline__ void macro_lookup_hash1(const XsParams &p, const double *recs, const int *ig,
                                                             const int *nn, const double *concs,
                                                             const uint16_t *mats, double pe, int mat, int idx,
@@ -1334,29 +1355,6 @@ struct XsApp {
       return reinterpret_cast<const double2 *>(recs + ((uint32_t)mrow[j] * (uint32_t)n_gp + (uint32_t)lo) * 6u);
     };
     double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
-#if ENS_XS2_PF > 0
-    // deep software pipeline: entry j+PF+3 prefetched into L1, entry j+PF
-    // loaded (prefetched 3 steps ago) and its pair prefetched into L1 (PF
-    // steps ahead of its use: about one L2 round trip at 6 warps per
-    // scheduler), entry j re-loaded (an L1 hit) for this step's bracket
-    constexpr int PF = ENS_XS2_PF;
-    for (int j = 0; j < PF + 3 && j < nm; j++) prefetch_l1(ent(j));
-    for (int j = 0; j < PF && j < nm; j++) {
-      const double2 *q = pair_at(j, guess(ld_(ent(j))));
-      prefetch_l1(q);
-      prefetch_l1(reinterpret_cast<const double *>(q) + 11);
-    }
-    for (int j = 0; j < nm; j++) {
-      const uint4 h0 = ld_(ent(j));
-      if (j + PF + 3 < nm) prefetch_l1(ent(j + PF + 3));
-      if (j + PF < nm) {
-        const double2 *q = pair_at(j + PF, guess(ld_(ent(j + PF))));
-        prefetch_l1(q);
-        prefetch_l1(reinterpret_cast<const double *>(q) + 11);
-      }
-      const int lo0 = guess(h0);
-      const double2 *q0 = pair_at(j, lo0);
-#else
     const uint4 z = make_uint4(0, 0, 0, 0);
     uint4 h0 = nm > 0 ? ld_(ent(0)) : z;
     uint4 h1 = nm > 1 ? ld_(ent(1)) : z;
@@ -1375,7 +1373,6 @@ struct XsApp {
         prefetch_l1(q1);
         prefetch_l1(reinterpret_cast<const double *>(q1) + 11);
       }
-#endif
       double2 a0 = ld_(q0 + 0), a1 = ld_(q0 + 1), a2 = ld_(q0 + 2);
       double2 b0 = ld_(q0 + 3), b1 = ld_(q0 + 4), b2 = ld_(q0 + 5);
       {  // verify the guessed pair; walk / upstream search otherwise (macro_lookup's gather_fix)
@@ -1403,12 +1400,10 @@ struct XsApp {
         }
       }
       accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
-#if ENS_XS2_PF == 0
       h0 = h1;
       h1 = h2;
       q0 = q1;
       lo0 = lo1;
-#endif
     }
     m[0] = m0;
     m[1] = m1;
@@ -1501,13 +1496,11 @@ struct XsApp {
   // (A)-(C) of the event-mode lookups for the chunk of lookups [c0, c0+nc):
   // lk_pe = their energies sorted into (material, energy) buckets, material
   // m's slots start at mcnt[16+m] (mcnt[28] = nc); material tallies counted
-  __device__ static __forceinline__ void lookup_sort(Ctx &c, const XsParams &p, const XsLayout &L, const double *thr, long long c0,
-                                     long long nc) {
+  __device__ static __forceinline__ void lookup_sort(Ctx &c, const XsParams &p, const XsLayout &L, const double *thr,
+                                                     uint32_t *mcnt, long long c0, long long nc) {
     const int tid = threadIdx.x, T = blockDim.x;
     double *lk_pe = (double *)(c.arena + L.lk_pe);
     uint32_t *hist = (uint32_t *)(c.arena + L.lk_hist);
-    const XsSmem S = xs_smem(p, T);
-    uint32_t *mcnt = (uint32_t *)(ens_smem(c) + S.mcnt);
     const long long LC = xs_lk_chunk(p);
     const int kb = xs_lk_bits(LC);
     const long long NB = 12LL << kb;
@@ -1585,7 +1578,7 @@ struct XsApp {
     double fsum = 0.0, fabs_ = 0.0;
     for (long long c0 = 0; c0 < nL; c0 += LC) {
       const long long nc = nL - c0 < LC ? nL - c0 : LC;
-      lookup_sort(c, p, L, thr, c0, nc);
+      lookup_sort(c, p, L, thr, mcnt, c0, nc);
       phase_mark_if(trc, c, 10);
       // (D) thread-per-lookup over the sorted chunk
       double *const dmp = c.dump;

@@ -187,9 +187,22 @@ struct Group {
   std::vector<uint32_t> item0;       // per kmap entry: its first item
   uint32_t kind_base[3] = {0, 0, 0}, kind_n[3] = {0, 0, 0};
   int grid2[3] = {0, 0, 0};          // phase-2 CTAs per kind
+  // phase 1b (hash / nuclide split instances): (instance, nuclide) init items
+  std::vector<uint32_t> init_items;  // pairs
+  uint64_t init_scr_bytes = 0;       // per init CTA
+  int grid3 = 0;
+  size_t smem3 = 0;
+  size_t init_off = 0, ctr3_off = 0, init_scr_off = 0;
   size_t items_off = 0, desc_off = 0, ipart_off = 0, idone_off = 0, ctr2_off = 0;
   size_t slots() const { return split ? kmap.size() : (size_t)grid; }
 };
+
+// kernels one launch of group g enqueues: the ensemble kernel, the init items,
+// one lookup-item kernel per XS grid type present
+static int kernels_of(const Group &g) {
+  if (!g.split) return 1;
+  return 1 + (g.init_items.empty() ? 0 : 1) + (g.kind_n[0] > 0) + (g.kind_n[1] > 0) + (g.kind_n[2] > 0);
+}
 
 struct Plan {  // workspace layout (byte offsets) and groups
   int n = 0;
@@ -226,6 +239,7 @@ struct ens_run {
   std::string c_text;
   cudaEvent_t ev0 = nullptr, ev1 = nullptr;
   std::vector<cudaEvent_t> ev_join;  // concurrent groups: one per forked group
+  std::vector<cudaEvent_t> ev_fork, ev_fork_join;  // per group: phase 1b fork / join
   struct KTime {                     // one kernel of a launch, bracketed by two events on its stream
     ens_kernel_time info;
     cudaEvent_t a = nullptr, b = nullptr;
@@ -297,11 +311,11 @@ cudaError_t d2h_copy(void *dst, const void *src, size_t bytes) {
 // non-blocking stream, created once per process.
 cudaError_t aux_stream(size_t i, cudaStream_t *out) {
   static std::mutex mu;
-  static cudaStream_t streams[64][ENS_N_APPS] = {};
+  static cudaStream_t streams[64][ENS_N_APPS + 1] = {};  // [ENS_N_APPS]: phase 1b
   int dev = 0;
   cudaError_t e = cudaGetDevice(&dev);
   if (e != cudaSuccess) return e;
-  if (dev < 0 || dev >= 64 || i >= (size_t)ENS_N_APPS) return cudaErrorInvalidValue;
+  if (dev < 0 || dev >= 64 || i > (size_t)ENS_N_APPS) return cudaErrorInvalidValue;
   std::lock_guard<std::mutex> lk(mu);
   if (!streams[dev][i]) {
     e = cudaStreamCreateWithFlags(&streams[dev][i], cudaStreamNonBlocking);
@@ -496,6 +510,35 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
         g.items.clear();
         for (int kd = 0; kd < 3; kd++) g.kind_n[kd] = 0;
       }
+      if (g.split) {  // phase 1b: sort items (first: the longest), then (instance, nuclide) table items
+        std::vector<uint32_t> nuc_items;
+        uint32_t smem_need = 0;
+        for (size_t x = 0; x < g.kmap.size(); x++) {
+          int argc;
+          const char *const *argv;
+          ens_args_get(a, (int)P.line_of_k[g.kmap[x]], &argc, &argv);
+          int ni = 0;
+          uint32_t sm3 = 0;
+          const uint64_t scr = app_init_scratch(ap, argc, argv, &ni, &sm3);
+          if (!g.item_count[x] || !ni) continue;
+          g.init_scr_bytes = std::max<uint64_t>(g.init_scr_bytes, al(scr));
+          smem_need = std::max(smem_need, sm3);
+          g.init_items.push_back((uint32_t)x);
+          g.init_items.push_back(0xffffffffu);  // its sort item
+          for (int i = 0; i < ni; i++) {
+            nuc_items.push_back((uint32_t)x);
+            nuc_items.push_back((uint32_t)i);
+          }
+        }
+        g.init_items.insert(g.init_items.end(), nuc_items.begin(), nuc_items.end());
+        if (!g.init_items.empty()) {
+          g.smem3 = xs_init_smem_off() + (smem_need + 15u) / 16u * 16u;
+          e = xs_init_items_occupancy(kXsInitThreads, g.smem3, &g.grid3);
+          if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveBlocksPerMultiprocessor (phase 1b)");
+          if (g.grid3 <= 0) return fail(ENS_EINVAL, "ens_launch: init items need more shared memory than an SM has");
+          g.grid3 = std::max(1, std::min<int>(g.grid3, (int)(g.init_items.size() / 2)));
+        }
+      }
     }
     P.groups.push_back(g);
   }
@@ -518,6 +561,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     if (!g.split) continue;
     g.items_off = o; o = al(o + g.items.size() * 4);
     g.desc_off = o; o = al(o + g.kmap.size() * sizeof(XsDesc));
+    g.init_off = o; o = al(o + g.init_items.size() * 4);
   }
   P.staged = o;
   // zeroed part
@@ -525,6 +569,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   for (Group &g : P.groups) {
     if (!g.split) continue;
     g.ctr2_off = o; o = al(o + 3 * 8);
+    g.ctr3_off = o; o = al(o + 8);
     g.idone_off = o; o = al(o + g.kmap.size() * 4);
   }
   P.o_recs = o; o = al(o + (size_t)n * sizeof(ens_record));
@@ -539,6 +584,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   for (Group &g : P.groups) {
     if (!g.split) continue;
     g.ipart_off = o; o = al(o + g.items.size() * sizeof(XsItemPart));
+    g.init_scr_off = o; o = al(o + (size_t)g.grid3 * g.init_scr_bytes);
   }
   P.o_arena = o;
   };
@@ -641,6 +687,12 @@ static int enqueue(ens_run *r) {
       k.ipart = r->ws + g.ipart_off;
       k.idone = (uint32_t *)(r->ws + g.idone_off);
       k.counter2 = (uint32_t *)(r->ws + g.ctr2_off);
+      k.init_items = (const uint32_t *)(r->ws + g.init_off);
+      k.n_init_items = (uint32_t)(g.init_items.size() / 2);
+      k.counter3 = (uint32_t *)(r->ws + g.ctr3_off);
+      k.init_scr = r->ws + g.init_scr_off;
+      k.init_scr_bytes = g.init_scr_bytes;
+      k.init_smem_off = xs_init_smem_off();
     }
     cudaStream_t st = r->stream;
     if (P.concurrent && gi > 0) {  // fork: group gi on an aux stream after ev0
@@ -648,7 +700,7 @@ static int enqueue(ens_run *r) {
       CU(cudaStreamWaitEvent(st, r->ev0, 0));
     }
     size_t nk = 0;  // kernels of this launch so far (r->kt grows on the first enqueue)
-    for (size_t q = 0; q < gi; q++) nk += 1 + (P.groups[q].split ? (P.groups[q].kind_n[0] > 0) + (P.groups[q].kind_n[1] > 0) + (P.groups[q].kind_n[2] > 0) : 0);
+    for (size_t q = 0; q < gi; q++) nk += kernels_of(P.groups[q]);
     auto kt_begin = [&](int phase, int kind, int grid, int block) -> int {
       if (r->kt.size() <= nk) {
         ens_run::KTime t;
@@ -665,10 +717,24 @@ static int enqueue(ens_run *r) {
       return cudaEventRecord(r->kt[nk].a, st) == cudaSuccess ? 0 : -1;
     };
     auto kt_end = [&]() -> int { return cudaEventRecord(r->kt[nk++].b, st) == cudaSuccess ? 0 : -1; };
+    cudaStream_t st3 = nullptr;
+    if (g.split && !g.init_items.empty()) {  // phase 1b beside phase 1: fork after this group's start
+      CU(aux_stream(ENS_N_APPS, &st3));
+      CU(cudaEventRecord(r->ev_fork[gi], st));
+      CU(cudaStreamWaitEvent(st3, r->ev_fork[gi], 0));
+      std::swap(st, st3);
+      if (kt_begin(3, -1, g.grid3, kXsInitThreads)) return fail(ENS_ECUDA, "ens_launch: kernel timing events");
+      cudaError_t e3 = launch_xs_init_items(g.grid3, kXsInitThreads, g.smem3, k, st);
+      if (e3 != cudaSuccess) return cuda_fail(e3, "xs_init_items_kernel launch");
+      if (kt_end()) return fail(ENS_ECUDA, "ens_launch: kernel timing events");
+      CU(cudaEventRecord(r->ev_fork_join[gi], st));
+      std::swap(st, st3);
+    }
     if (kt_begin(1, -1, g.ctas(), g.T)) return fail(ENS_ECUDA, "ens_launch: kernel timing events");
     cudaError_t e = launch_group(g.app, g.T, g.m, g.ctas(), g.cs, g.dyn(), k, st);
     if (e != cudaSuccess) return cuda_fail(e, "ens_kernel launch");
     if (kt_end()) return fail(ENS_ECUDA, "ens_launch: kernel timing events");
+    if (st3) CU(cudaStreamWaitEvent(st, r->ev_fork_join[gi], 0));  // phase 2 after both
     for (int kd = 0; g.split && kd < 3; kd++) {  // phase 2: every instance's lookup items, on every SM
       if (!g.kind_n[kd]) continue;
       const int ctas2 = std::max(1, std::min<int>(g.grid2[kd], (int)g.kind_n[kd]));
@@ -729,6 +795,13 @@ extern "C" int ens_launch(ens_app app, const ens_args *a, const ens_launch_cfg *
       e = cudaEventCreateWithFlags(&ej, cudaEventDisableTiming);
       if (e == cudaSuccess) r->ev_join.push_back(ej);
     }
+  for (size_t gi = 0; gi < P.groups.size() && e == cudaSuccess; gi++) {
+    cudaEvent_t a = nullptr, b = nullptr;
+    e = cudaEventCreateWithFlags(&a, cudaEventDisableTiming);
+    if (e == cudaSuccess) e = cudaEventCreateWithFlags(&b, cudaEventDisableTiming);
+    r->ev_fork.push_back(a);
+    r->ev_fork_join.push_back(b);
+  }
   if (e != cudaSuccess) {
     ens_run_free(r);
     return cuda_fail(e, "cudaEventCreate");
@@ -751,6 +824,7 @@ extern "C" int ens_launch(ens_app app, const ens_args *a, const ens_launch_cfg *
   for (const Group &g : P.groups) {
     if (!g.split) continue;
     std::memcpy(r->h_stage + g.items_off, g.items.data(), g.items.size() * 4);
+    if (!g.init_items.empty()) std::memcpy(r->h_stage + g.init_off, g.init_items.data(), g.init_items.size() * 4);
     for (size_t x = 0; x < g.kmap.size(); x++) {  // phase 1 fills the rest of each descriptor
       XsDesc *d = reinterpret_cast<XsDesc *>(r->h_stage + g.desc_off) + x;
       d->item0 = g.item0[x];
@@ -918,7 +992,7 @@ extern "C" int ens_run_kernel_times(ens_run *r, ens_kernel_time *out, int cap) {
   int n = 0;
   for (int q = 0; q < (int)r->P.groups.size(); q++) {
     const Group &g = r->P.groups[q];
-    n += 1 + (g.split ? (g.kind_n[0] > 0) + (g.kind_n[1] > 0) + (g.kind_n[2] > 0) : 0);
+    n += kernels_of(g);
   }
   if (cap < n) return fail(ENS_ERANGE, "ens_run_kernel_times: cap smaller than the kernel count");
   for (int q = 0; q < n; q++) {
@@ -943,8 +1017,8 @@ extern "C" int ens_run_get_info(const ens_run *r, ens_run_info *info) {
     info->block_threads[ap] = g.T;
   }
   info->kernel_launches = (int32_t)P.groups.size();
-  for (const Group &g : P.groups)
-    for (int kd = 0; g.split && kd < 3; kd++) info->kernel_launches += g.kind_n[kd] ? 1 : 0;
+  info->kernel_launches = 0;
+  for (const Group &g : P.groups) info->kernel_launches += kernels_of(g);
   info->arena_bytes = P.arena_bytes;
   info->ws_bytes = r->ws_bytes;
   info->records_offset = P.o_recs;
@@ -976,6 +1050,8 @@ extern "C" void ens_run_free(ens_run *r) {
   if (r->ev0) cudaEventDestroy(r->ev0);
   if (r->ev1) cudaEventDestroy(r->ev1);
   for (cudaEvent_t ej : r->ev_join) cudaEventDestroy(ej);
+  for (cudaEvent_t ej : r->ev_fork) if (ej) cudaEventDestroy(ej);
+  for (cudaEvent_t ej : r->ev_fork_join) if (ej) cudaEventDestroy(ej);
   for (auto &t : r->kt) {
     cudaEventDestroy(t.a);
     cudaEventDestroy(t.b);

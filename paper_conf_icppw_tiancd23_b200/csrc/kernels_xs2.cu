@@ -243,6 +243,101 @@ __global__ void __launch_bounds__(kXs2T, Xs2Minb<GRID>::v) xs_items_kernel(const
   }
 }
 
+// ---- split phases, phase 1b: the per-nuclide tables of hash / nuclide
+// instances (XS-3..XS-5: sort, records, hash column), one (instance,
+// nuclide) item at a time, on every SM, beside the ensemble kernel (which
+// meanwhile samples and sorts each instance's lookups).  Each item re-reads
+// its instance's command line (the same XsParams the instance parses) and
+// runs XsApp::init_nuc_range for that one nuclide with this CTA's scratch.
+constexpr uint32_t kXsInitArgv = kXs2Sh;                                  // char *argv[ENS_MAX_ARGC + 1]
+constexpr uint32_t kXsInitMisc = kXsInitArgv + (ENS_MAX_ARGC + 2) * 8;    // u32 item
+constexpr uint32_t kXsInitApp = kXsInitMisc + 64;                          // the app's shared memory
+
+// Items 2j' (sort items, one per instance, first in the queue: the longest)
+// and (instance, nuclide) table items.  A sort item samples and sorts the
+// instance's lookups (XsApp::lookup_sort on this CTA alone) and writes its
+// descriptor; a nuclide item builds one nuclide's sorted records and hash /
+// nuclide grid column.  Two CTAs of 256 threads per SM (compact shared
+// memory: no material tables), so one CTA's barrier-separated phases overlap
+// the other's.
+constexpr uint32_t kXsSortItem = 0xffffffffu;
+
+__global__ void __launch_bounds__(256, 2) xs_init_items_kernel(const KParams p) {
+  const int tid = threadIdx.x, T = blockDim.x;
+  Ctx c{};
+  c.sh_off = 0;
+  c.smem_off = kXsInitApp;
+  c.csize = 1;
+  c.flags = p.flags;
+  char **argv = reinterpret_cast<char **>(ens_dsmem + kXsInitArgv);
+  uint32_t *misc = reinterpret_cast<uint32_t *>(ens_dsmem + kXsInitMisc);
+  char *scr = p.init_scr + (size_t)blockIdx.x * p.init_scr_bytes;
+  bool jt_ok = false;  // the LCG jump tables (seed- and layout-independent: S.jmp is fixed)
+  for (;;) {
+    if (tid == 0) misc[0] = atomicAdd(p.counter3, 1u);
+    __syncthreads();
+    const uint32_t it = misc[0];
+    if (it >= p.n_init_items) break;
+    const uint32_t j = p.init_items[2 * it], i = p.init_items[2 * it + 1];
+    const uint32_t k = p.kmap[j], line = p.line_of_k[k], t0 = p.line_tok[line];
+    const int argc = (int)(p.line_tok[line + 1] - t0);
+    for (int a = tid; a < argc; a += T) argv[a] = const_cast<char *>(p.blob) + p.tok_off[t0 + a];
+    if (tid == 0) argv[argc] = nullptr;
+    __syncthreads();
+    XsParams xp;
+    xs_parse(argc, argv, xp);  // a valid line: the host made items only for those
+    const XsSmem S = xs_init_smem(xp);
+    const XsLayout L = xs_layout(xp, (int)p.team_ctas);  // the instance's arena, as phase 1 lays it out
+    c.arena = p.arena_base + (size_t)j * p.arena_bytes;
+    if (i == kXsSortItem) {  // XS-6 for every lookup, sorted by (material, energy); the descriptor
+      double *thr = reinterpret_cast<double *>(ens_smem(c) + S.thr);
+      uint32_t *mcnt = reinterpret_cast<uint32_t *>(ens_smem(c) + S.mcnt);
+      if (tid < 12) thr[tid] = hm_threshold(tid);
+      __syncthreads();
+      XsApp::lookup_sort(c, xp, L, thr, mcnt, 0, xp.lookups);
+      if (tid == 0) {
+        c.desc = p.xs_desc + (size_t)j * sizeof(XsDesc);
+        c.k = k;
+        c.id = line;
+        c.t_start = 0;
+        XsApp::write_desc(c, xp, L, mcnt);
+      }
+    } else {
+      if (!jt_ok) {
+        Affine *jt = reinterpret_cast<Affine *>(ens_smem(c) + S.jmp);
+        for (int x = tid; x < 320; x += T) jt[x] = lcg_pow((6ULL * (uint64_t)(x & 63)) << (6 * (x >> 6)));
+        jt_ok = true;
+        __syncthreads();
+      }
+      const uint64_t e8 = align_up((uint64_t)xp.n_gp * 8, 256), c4 = align_up((uint64_t)(xp.bins + 1) * 4, 256);
+      XsApp::init_nuc_range(c, xp, L, S, (int)i, (int)i + 1, 1, scr, scr + e8, scr + e8 + c4);
+    }
+    __syncthreads();  // argv, misc, scratch reused by the next item
+  }
+}
+
+uint32_t xs_init_smem_off() { return kXsInitApp; }
+
+cudaError_t xs_init_items_occupancy(int threads, size_t smem, int *ctas) {
+  const void *fn = (const void *)xs_init_items_kernel;
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  int per_sm = 0, dev = 0, sms = 0;
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, threads, smem);
+  if (e == cudaSuccess) e = cudaGetDevice(&dev);
+  if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+  *ctas = per_sm * sms;
+  return e;
+}
+
+cudaError_t launch_xs_init_items(int ctas, int threads, size_t smem, const KParams &p, cudaStream_t st) {
+  const void *fn = (const void *)xs_init_items_kernel;
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+  if (e != cudaSuccess) return e;
+  void *args[] = {const_cast<KParams *>(&p)};
+  return cudaLaunchKernel(fn, dim3((unsigned)ctas), dim3((unsigned)threads), args, smem, st);
+}
+
 int xs_items_threads() { return kXs2T; }
 
 static const void *xs_items_fn(int grid) {

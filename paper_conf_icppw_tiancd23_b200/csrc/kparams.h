@@ -41,6 +41,14 @@ struct KParams {
   char *ipart;                // [n_items] XsItemPart
   uint32_t *idone;            // [n] items finished per instance (zeroed)
   uint32_t *counter2;         // phase-2 item counter (zeroed)
+  // split phases, hash / nuclide tables: (group-local instance, nuclide) init
+  // items, run by the init-item kernel beside the ensemble kernel
+  const uint32_t *init_items; // [n_init_items][2]
+  uint32_t n_init_items;
+  uint32_t *counter3;         // init-item counter (zeroed)
+  char *init_scr;             // [grid][init_scr_bytes] per-CTA scratch
+  uint64_t init_scr_bytes;
+  uint32_t init_smem_off;     // dynamic smem offset of the app's shared memory
 };
 
 const void *kernel_ptr(uint32_t app, int T);
@@ -59,5 +67,10 @@ cudaError_t group_occupancy(uint32_t app, int T, int m, int cs, size_t smem, int
 cudaError_t launch_xs_items(int grid_type, int ctas, const KParams &p, cudaStream_t st);
 cudaError_t xs_items_occupancy(int grid_type, int *ctas);
 int xs_items_threads();
+cudaError_t launch_xs_init_items(int ctas, int threads, size_t smem, const KParams &p, cudaStream_t st);
+cudaError_t xs_init_items_occupancy(int threads, size_t smem, int *ctas);
+uint32_t xs_init_smem_off();
+uint64_t app_init_scratch(uint32_t app, int argc, const char *const *argv, int *n_items, uint32_t *smem);
+constexpr int kXsInitThreads = 256;  // init-item kernel block (launch bounds 256 x 2 CTAs/SM)
 
 }  // namespace ens

