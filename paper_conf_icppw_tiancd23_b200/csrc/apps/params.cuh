@@ -468,6 +468,8 @@ ENS_HD int rs_parse(int argc, const char *const *argv, RsParams &p) {
 }
 
 struct RsLayout {
+  uint64_t poff_g, woff_g, concs_g;  // split phases: global copies of the shared-memory pole /
+                                     // window offsets and concentrations, for phase 2
   uint64_t pole_off;   // [n_nuc+1] int32 prefix of n_poles
   uint64_t win_off;    // [n_nuc+1] int32 prefix of n_windows
   uint64_t poles;      // [total_poles] x 64 B {EA, RT, RA, RF} complex
@@ -491,6 +493,9 @@ ENS_HD RsLayout rs_layout(const RsParams &p) {
   RsLayout L{};
   const uint64_t tp = (uint64_t)p.avg_poles * p.n_nuc, tw = (uint64_t)p.avg_windows * p.n_nuc;
   uint64_t o = 0;
+  L.poff_g = o; o = align_up(o + (p.n_nuc + 1) * 4ULL, 256);
+  L.woff_g = o; o = align_up(o + (p.n_nuc + 1) * 4ULL, 256);
+  L.concs_g = o; o = align_up(o + 12ULL * xs_max_nucs(p.n_nuc) * 8, 256);
   L.pole_off = o; o = align_up(o + (p.n_nuc + 1) * 4ULL, 256);
   L.win_off = o; o = align_up(o + (p.n_nuc + 1) * 4ULL, 256);
   L.poles = o; o = align_up(o + tp * 64, 256);
@@ -503,6 +508,30 @@ ENS_HD RsLayout rs_layout(const RsParams &p) {
   L.total = o;
   return L;
 }
+// split phases (see XsDesc): RS instances whose lookups fit one sorted chunk
+constexpr long long kRsItemLookups = 2048;
+ENS_HD bool rs_split_ok(const RsParams &p) { return p.lookups > 0 && p.lookups <= kRsLkChunk; }
+ENS_HD long long rs_items(const RsParams &p) {
+  return rs_split_ok(p) ? (p.lookups + kRsItemLookups - 1) / kRsItemLookups : 0;
+}
+struct RsDesc {            // written by phase 1, read by phase 2
+  uint64_t poles, pole_l, windows, k0rs, lk_e, poff, woff, concs;  // device addresses in the arena
+  uint64_t lookups, seed, t_start;
+  uint32_t mcnt[13];
+  int32_t n_nuc, doppler, avg_poles, avg_windows;
+  uint32_t k, line;
+  uint32_t item0, n_items; // this instance's items in the phase-2 queue (host-staged)
+};
+struct RsItemPart {
+  unsigned long long ver, bsum, terms, near;
+  double fsum, fabs;
+  uint32_t am[4];
+};
+// one descriptor / item-part stride for every split app
+constexpr uint32_t kDescBytes = ((sizeof(XsDesc) > sizeof(RsDesc) ? sizeof(XsDesc) : sizeof(RsDesc)) + 15) / 16 * 16;
+constexpr uint32_t kPartBytes =
+    ((sizeof(XsItemPart) > sizeof(RsItemPart) ? sizeof(XsItemPart) : sizeof(RsItemPart)) + 15) / 16 * 16;
+
 struct RsSmem {
   uint32_t thr, nn, concs, mats, npol, nwin, mcnt, total;
 };

@@ -185,8 +185,8 @@ struct Group {
   std::vector<int> item_kind;        // per kmap entry: phase-2 kernel (XS grid type)
   std::vector<uint32_t> items;       // group-local instance of each item, by kind
   std::vector<uint32_t> item0;       // per kmap entry: its first item
-  uint32_t kind_base[3] = {0, 0, 0}, kind_n[3] = {0, 0, 0};
-  int grid2[3] = {0, 0, 0};          // phase-2 CTAs per kind
+  uint32_t kind_base[4] = {0, 0, 0, 0}, kind_n[4] = {0, 0, 0, 0};  // kinds: XS grid types 0..2, RS 3
+  int grid2[4] = {0, 0, 0, 0};       // phase-2 CTAs per kind
   // phase 1b (hash / nuclide split instances): (instance, nuclide) init items
   std::vector<uint32_t> init_items;  // pairs
   uint64_t init_scr_bytes = 0;       // per init CTA
@@ -201,7 +201,8 @@ struct Group {
 // one lookup-item kernel per XS grid type present
 static int kernels_of(const Group &g) {
   if (!g.split) return 1;
-  return 1 + (g.init_items.empty() ? 0 : 1) + (g.kind_n[0] > 0) + (g.kind_n[1] > 0) + (g.kind_n[2] > 0);
+  return 1 + (g.init_items.empty() ? 0 : 1) + (g.kind_n[0] > 0) + (g.kind_n[1] > 0) + (g.kind_n[2] > 0) +
+         (g.kind_n[3] > 0);
 }
 
 struct Plan {  // workspace layout (byte offsets) and groups
@@ -485,7 +486,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     if (!(c->flags & ENS_F_FUSED) && !c->arena_bytes) {
       // items grouped by kind (one phase-2 kernel each), instances in queue order within a kind
       g.item0.assign(g.kmap.size(), 0);
-      for (int kd = 0; kd < 3; kd++) {
+      for (int kd = 0; kd < 4; kd++) {
         g.kind_base[kd] = (uint32_t)g.items.size();
         for (size_t x = 0; x < g.kmap.size(); x++) {
           if (g.item_kind[x] != kd || !g.item_count[x]) continue;
@@ -503,12 +504,12 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
       // fill every phase-2 CTA.  C2 45.1 -> 38.2 ms, C2u 66.2 -> 62.9 ms;
       // TSTAR (1024 instances) and C1 (12 items) stay fused.
       int fill = 0;
-      for (int kd = 0; kd < 3; kd++) fill = std::max(fill, g.grid2[kd]);
+      for (int kd = 0; kd < 4; kd++) fill = std::max(fill, g.grid2[kd]);
       g.split = !g.items.empty() && (((c->flags & ENS_F_SPLIT_PHASES) != 0) ||
                                      ((int64_t)g.kmap.size() < (int64_t)ctas && (int64_t)g.items.size() >= fill));
       if (!g.split) {
         g.items.clear();
-        for (int kd = 0; kd < 3; kd++) g.kind_n[kd] = 0;
+        for (int kd = 0; kd < 4; kd++) g.kind_n[kd] = 0;
       }
       if (g.split) {  // phase 1b: sort items (first: the longest), then (instance, nuclide) table items
         std::vector<uint32_t> nuc_items;
@@ -560,7 +561,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   for (Group &g : P.groups) {  // split phases: item table, descriptors (item0 / n_items pre-filled)
     if (!g.split) continue;
     g.items_off = o; o = al(o + g.items.size() * 4);
-    g.desc_off = o; o = al(o + g.kmap.size() * sizeof(XsDesc));
+    g.desc_off = o; o = al(o + g.kmap.size() * kDescBytes);
     g.init_off = o; o = al(o + g.init_items.size() * 4);
   }
   P.staged = o;
@@ -568,7 +569,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   P.o_ctr = o; o = al(o + (P.groups.size() + 1) * 8);
   for (Group &g : P.groups) {
     if (!g.split) continue;
-    g.ctr2_off = o; o = al(o + 3 * 8);
+    g.ctr2_off = o; o = al(o + 4 * 8);
     g.ctr3_off = o; o = al(o + 8);
     g.idone_off = o; o = al(o + g.kmap.size() * 4);
   }
@@ -583,7 +584,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   P.o_cmp = o; o = al(o + (size_t)n * P.stdout_cap);
   for (Group &g : P.groups) {
     if (!g.split) continue;
-    g.ipart_off = o; o = al(o + g.items.size() * sizeof(XsItemPart));
+    g.ipart_off = o; o = al(o + g.items.size() * kPartBytes);
     g.init_scr_off = o; o = al(o + (size_t)g.grid3 * g.init_scr_bytes);
   }
   P.o_arena = o;
@@ -735,7 +736,7 @@ static int enqueue(ens_run *r) {
     if (e != cudaSuccess) return cuda_fail(e, "ens_kernel launch");
     if (kt_end()) return fail(ENS_ECUDA, "ens_launch: kernel timing events");
     if (st3) CU(cudaStreamWaitEvent(st, r->ev_fork_join[gi], 0));  // phase 2 after both
-    for (int kd = 0; g.split && kd < 3; kd++) {  // phase 2: every instance's lookup items, on every SM
+    for (int kd = 0; g.split && kd < 4; kd++) {  // phase 2: every instance's lookup items, on every SM
       if (!g.kind_n[kd]) continue;
       const int ctas2 = std::max(1, std::min<int>(g.grid2[kd], (int)g.kind_n[kd]));
       KParams k2 = k;
@@ -826,9 +827,14 @@ extern "C" int ens_launch(ens_app app, const ens_args *a, const ens_launch_cfg *
     std::memcpy(r->h_stage + g.items_off, g.items.data(), g.items.size() * 4);
     if (!g.init_items.empty()) std::memcpy(r->h_stage + g.init_off, g.init_items.data(), g.init_items.size() * 4);
     for (size_t x = 0; x < g.kmap.size(); x++) {  // phase 1 fills the rest of each descriptor
-      XsDesc *d = reinterpret_cast<XsDesc *>(r->h_stage + g.desc_off) + x;
-      d->item0 = g.item0[x];
-      d->n_items = g.item_count[x];
+      char *dp = r->h_stage + g.desc_off + x * kDescBytes;
+      if (g.app == APP_RSBENCH) {
+        reinterpret_cast<RsDesc *>(dp)->item0 = g.item0[x];
+        reinterpret_cast<RsDesc *>(dp)->n_items = g.item_count[x];
+      } else {
+        reinterpret_cast<XsDesc *>(dp)->item0 = g.item0[x];
+        reinterpret_cast<XsDesc *>(dp)->n_items = g.item_count[x];
+      }
     }
   }
   e = cudaMemcpyAsync(r->ws, r->h_stage, P.staged, cudaMemcpyHostToDevice, r->stream);

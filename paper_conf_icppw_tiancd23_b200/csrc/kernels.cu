@@ -111,7 +111,7 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
     c.dump_rows = p.dump_rows;
     // split phases: one arena slot per instance (phase 2 reads the tables)
     c.arena = p.split ? p.arena_base + (size_t)j * p.arena_bytes : arena;
-    c.desc = p.split ? p.xs_desc + (size_t)j * sizeof(XsDesc) : nullptr;
+    c.desc = p.split ? p.xs_desc + (size_t)j * kDescBytes : nullptr;
     phase_mark(c, -1);
     Result r{};
     if (App::kTeam || cr == 0) r = App::run(c, argc, s_argv);
@@ -241,6 +241,12 @@ double app_cost(uint32_t app, int argc, const char *const *argv) {
 // (*kind = the phase-2 kernel: the XS grid type)
 uint32_t app_items(uint32_t app, int argc, const char *const *argv, int *kind) {
   *kind = 0;
+  if (app == APP_RSBENCH) {  // kind 3: the RS lookup-item kernel
+    RsParams q;
+    if (rs_parse(argc, argv, q) >= 0) return 0;
+    *kind = 3;
+    return (uint32_t)rs_items(q);
+  }
   if (app != APP_XSBENCH) return 0;
   XsParams p;
   if (xs_parse(argc, argv, p) >= 0) return 0;

@@ -22,6 +22,7 @@
 #ifndef ENS_XS_STEP
 #define ENS_XS_STEP 1
 #endif
+#include "apps/rsbench.cuh"
 #include "apps/xsbench.cuh"
 #include "kparams.h"
 
@@ -121,13 +122,13 @@ __device__ __noinline__ void xs2_finish(const KParams &p, Ctx &c, const XsDesc *
     unsigned long long tv = 0, tb = 0;
     double tf = 0.0, ta = 0.0;
     uint32_t tam[5] = {0, 0, 0, 0, 0};
-    const XsItemPart *ip = reinterpret_cast<const XsItemPart *>(p.ipart);
     for (uint32_t it = d->item0; it < d->item0 + d->n_items; it++) {
-      tv += __ldcg(&ip[it].ver);
-      tb += __ldcg(&ip[it].bsum);
-      tf += __ldcg(&ip[it].fsum);
-      ta += __ldcg(&ip[it].fabs);
-      for (int a = 0; a < 5; a++) tam[a] += __ldcg(&ip[it].am[a]);
+      const XsItemPart *ip = reinterpret_cast<const XsItemPart *>(p.ipart + (size_t)it * kPartBytes);
+      tv += __ldcg(&ip->ver);
+      tb += __ldcg(&ip->bsum);
+      tf += __ldcg(&ip->fsum);
+      ta += __ldcg(&ip->fabs);
+      for (int a = 0; a < 5; a++) tam[a] += __ldcg(&ip->am[a]);
     }
     sh->out_len = 0;
     sh->flags = 0;
@@ -198,7 +199,7 @@ __global__ void __launch_bounds__(kXs2T, Xs2Minb<GRID>::v) xs_items_kernel(const
     const uint32_t item = p.item_base + misc[0];
     const uint32_t j = p.items[item];
     {  // the instance's descriptor (phase 1's stores, an earlier kernel)
-      const unsigned long long *src = reinterpret_cast<const unsigned long long *>(p.xs_desc + (size_t)j * sizeof(XsDesc));
+      const unsigned long long *src = reinterpret_cast<const unsigned long long *>(p.xs_desc + (size_t)j * kDescBytes);
       unsigned long long *dst = reinterpret_cast<unsigned long long *>(d);
       for (int w = tid; w < (int)(sizeof(XsDesc) / 8); w += kXs2T) dst[w] = src[w];
     }
@@ -228,7 +229,7 @@ __global__ void __launch_bounds__(kXs2T, Xs2Minb<GRID>::v) xs_items_kernel(const
     fsum = block_sum_f64(sh, fsum);
     fabs_ = block_sum_f64(sh, fabs_);
     if (tid == 0) {
-      XsItemPart *ip = reinterpret_cast<XsItemPart *>(p.ipart) + item;
+      XsItemPart *ip = reinterpret_cast<XsItemPart *>(p.ipart + (size_t)item * kPartBytes);
       ip->ver = ver;
       ip->bsum = bsum;
       ip->fsum = fsum;
@@ -296,7 +297,7 @@ __global__ void __launch_bounds__(256, 2) xs_init_items_kernel(const KParams p) 
       __syncthreads();
       XsApp::lookup_sort(c, xp, L, thr, mcnt, 0, xp.lookups);
       if (tid == 0) {
-        c.desc = p.xs_desc + (size_t)j * sizeof(XsDesc);
+        c.desc = p.xs_desc + (size_t)j * kDescBytes;
         c.k = k;
         c.id = line;
         c.t_start = 0;
@@ -338,24 +339,220 @@ cudaError_t launch_xs_init_items(int ctas, int threads, size_t smem, const KPara
   return cudaLaunchKernel(fn, dim3((unsigned)ctas), dim3((unsigned)threads), args, smem, st);
 }
 
+
+// ---- split phases, phase 2 of RSBench-style instances (kind 3) ----------
+// Items of kRsItemLookups sorted lookups of one instance; per item the
+// instance's pole / window offsets and concentrations (phase 1 copied them
+// to its arena) are staged in shared memory and every lookup is RsApp::lookup
+// (RS-3, bit-identical to the fused body).  The last item's CTA writes the
+// record, tallies (argmax, materials, pole-term counters) and stdout.
+constexpr uint32_t kRsDesc = kXs2Sh;
+constexpr uint32_t kRsThr = kRsDesc + (kDescBytes + 15) / 16 * 16;
+constexpr uint32_t kRsNn = kRsThr + 12 * 8;
+constexpr uint32_t kRsConcs = kRsNn + 16 * 4;
+constexpr uint32_t kRsMats = kRsConcs + 12 * 321 * 8;
+constexpr uint32_t kRsOff = kRsMats + (12 * 321 * 2 + 15) / 16 * 16;  // poff, woff: 2 x [356] int
+constexpr uint32_t kRsMisc = kRsOff + 2 * 356 * 4;
+constexpr uint32_t kRsSmem = kRsMisc + 16 * 4;
+#ifndef ENS_RS2_MINB
+#define ENS_RS2_MINB 2
+#endif
+
+__device__ __noinline__ void rs2_finish(const KParams &p, Ctx &c, const RsDesc *d, uint32_t *misc) {
+  const int tid = threadIdx.x;
+  Shared *sh = ens_sh(c);
+  const uint32_t k = d->k;
+  c.out = p.stdout_base + (size_t)k * p.stdout_cap;
+  if (tid == 0) {
+    __threadfence();
+    unsigned long long tv = 0, tb = 0, tt = 0, tn = 0;
+    double tf = 0.0, ta = 0.0;
+    uint32_t tam[4] = {0, 0, 0, 0};
+    for (uint32_t it = d->item0; it < d->item0 + d->n_items; it++) {
+      const RsItemPart *ip = reinterpret_cast<const RsItemPart *>(p.ipart + (size_t)it * kPartBytes);
+      tv += __ldcg(&ip->ver);
+      tb += __ldcg(&ip->bsum);
+      tt += __ldcg(&ip->terms);
+      tn += __ldcg(&ip->near);
+      tf += __ldcg(&ip->fsum);
+      ta += __ldcg(&ip->fabs);
+      for (int a = 0; a < 4; a++) tam[a] += __ldcg(&ip->am[a]);
+    }
+    sh->out_len = 0;
+    sh->flags = 0;
+    const unsigned long long vhash = tv % 999983ULL;
+    const long long lookups = (long long)d->lookups;
+    ens_printf(c, FMT_RS_HDR, d->n_nuc == 68 ? "small" : "large", d->n_nuc, d->avg_poles, d->avg_windows, d->doppler,
+               lookups, (unsigned long long)d->seed);
+    ens_printf(c, FMT_VERIFY, vhash);
+    uint32_t *tal = p.tallies + (size_t)k * ENS_TALLIES;
+    for (int t = 0; t < ENS_TALLIES; t++) {
+      uint32_t v = 0;
+      if (t < 4) v = tam[t];
+      else if (t >= 5 && t < 17) v = d->mcnt[t - 4] - d->mcnt[t - 5];
+      else if (t == 24) v = (uint32_t)tt;
+      else if (t == 25) v = (uint32_t)(tt >> 32);
+      else if (t == 26) v = (uint32_t)tn;
+      tal[t] = v;
+    }
+    ens_record rec;
+    rec.instance = d->line;
+    rec.exit_code = 0;
+    rec.app = APP_RSBENCH;
+    rec.flags = sh->flags | ENS_RF_DONE;
+    rec.vhash = vhash;
+    rec.bitsum = tb;
+    rec.fsum = tf;
+    rec.fabs = ta;
+    rec.work = (uint64_t)lookups;
+    rec.stdout_len = sh->out_len;
+    uint32_t sm = 0;
+    if (p.flags & ENS_F_TIMESTAMPS) asm volatile("mov.u32 %0, %%smid;" : "=r"(sm));
+    rec.smid = sm;
+    rec.t_start_ns = d->t_start;
+    rec.t_end_ns = (p.flags & ENS_F_TIMESTAMPS) ? xs2_gtimer() : 0ull;
+    p.recs[k] = rec;
+    const unsigned long long pos = atomicAdd(p.stdout_total, (unsigned long long)sh->out_len);
+    p.stdout_pos[k] = pos;
+    reinterpret_cast<unsigned long long *>(misc + 8)[0] = pos;
+  }
+  __syncthreads();
+  const unsigned long long pos = reinterpret_cast<const unsigned long long *>(misc + 8)[0];
+  const unsigned long long *src = reinterpret_cast<const unsigned long long *>(c.out);
+  unsigned long long *dst = reinterpret_cast<unsigned long long *>(p.stdout_cmp + pos);
+  for (uint32_t w = tid; w < sh->out_len / 8; w += kXs2T) dst[w] = src[w];
+}
+
+__global__ void __launch_bounds__(kXs2T, ENS_RS2_MINB) rs_items_kernel(const KParams p) {
+  const int tid = threadIdx.x;
+  Ctx c{};
+  c.sh_off = 0;
+  c.smem_off = kRsDesc;
+  c.csize = 1;
+  c.flags = p.flags;
+  c.out_cap = p.stdout_cap;
+  Shared *sh = ens_sh(c);
+  RsDesc *d = reinterpret_cast<RsDesc *>(ens_dsmem + kRsDesc);
+  double *thr = reinterpret_cast<double *>(ens_dsmem + kRsThr);
+  int *nn = reinterpret_cast<int *>(ens_dsmem + kRsNn);
+  double *concs = reinterpret_cast<double *>(ens_dsmem + kRsConcs);
+  uint16_t *mats = reinterpret_cast<uint16_t *>(ens_dsmem + kRsMats);
+  int *poff = reinterpret_cast<int *>(ens_dsmem + kRsOff);
+  int *woff = poff + 356;
+  uint32_t *misc = reinterpret_cast<uint32_t *>(ens_dsmem + kRsMisc);
+  uint32_t *am = misc + 2;
+  int cached = 0;  // n_nuc of the material lists in shared memory
+  uint32_t cached_j = 0xffffffffu;
+  for (;;) {
+    if (tid == 0) misc[0] = atomicAdd(p.counter2, 1u);
+    if (tid < 4) am[tid] = 0u;
+    __syncthreads();
+    if (misc[0] >= p.n_items) break;
+    const uint32_t item = p.item_base + misc[0];
+    const uint32_t j = p.items[item];
+    if (j != cached_j) {  // a new instance: its descriptor and shared tables
+      const unsigned long long *src = reinterpret_cast<const unsigned long long *>(p.xs_desc + (size_t)j * kDescBytes);
+      unsigned long long *dst = reinterpret_cast<unsigned long long *>(d);
+      for (int w = tid; w < (int)(sizeof(RsDesc) / 8); w += kXs2T) dst[w] = src[w];
+      __syncthreads();
+      const int n_nuc = d->n_nuc, mx = xs_max_nucs(n_nuc);
+      if (n_nuc != cached) {
+        hm_tables(n_nuc, mx, thr, nn, concs, mats);
+        cached = n_nuc;
+      }
+      __syncthreads();
+      const int *pg = reinterpret_cast<const int *>(d->poff), *wg = reinterpret_cast<const int *>(d->woff);
+      const double *cg = reinterpret_cast<const double *>(d->concs);
+      for (int i = tid; i <= n_nuc; i += kXs2T) {
+        poff[i] = pg[i];
+        woff[i] = wg[i];
+      }
+      for (int x = tid; x < 12 * mx; x += kXs2T) concs[x] = cg[x];
+      cached_j = j;
+      __syncthreads();
+    }
+    const int n_nuc = d->n_nuc, mx = xs_max_nucs(n_nuc);
+    const long long L = (long long)d->lookups;
+    const long long s0 = (long long)(item - d->item0) * kRsItemLookups;
+    const long long s1 = s0 + kRsItemLookups < L ? s0 + kRsItemLookups : L;
+    const double *poles = reinterpret_cast<const double *>(d->poles);
+    const uint8_t *pl = reinterpret_cast<const uint8_t *>(d->pole_l);
+    const double *wins = reinterpret_cast<const double *>(d->windows);
+    const double *k0 = reinterpret_cast<const double *>(d->k0rs);
+    const double *lk_e = reinterpret_cast<const double *>(d->lk_e);
+    double *dmp = p.dump ? p.dump + (size_t)d->k * p.dump_rows * 8 : nullptr;
+    unsigned long long ver = 0, bsum = 0, terms = 0, near = 0;
+    double fsum = 0.0, fabs_ = 0.0;
+    for (long long sl = s0 + tid; sl < s1; sl += kXs2T) {
+      int mat = 0;
+#pragma unroll
+      for (int m = 1; m < 12; m++) mat += (sl >= (long long)d->mcnt[m]) ? 1 : 0;
+      const double E = ld_(lk_e + sl);
+      double macro[4];
+      RsApp::lookup(d->doppler, E, mat, nn, mats, mx, concs, poff, woff, poles, pl, wins, k0, macro, terms, near);
+      double mxv = -DBL_MAX;
+      int a = 0;
+#pragma unroll
+      for (int q = 0; q < 4; q++)
+        if (macro[q] > mxv) {
+          mxv = macro[q];
+          a = q;
+        }
+      ver += (unsigned long long)(a + 1);
+      atomicAdd(&am[a], 1u);
+      if (dmp) dump_row(dmp, p.dump_rows, sl, E, mat, macro, 4, a);
+#pragma unroll
+      for (int q = 0; q < 4; q++) {
+        bsum += dbits(macro[q]);
+        fsum += macro[q];
+        fabs_ += fabs(macro[q]);
+      }
+    }
+    ver = block_sum_u64(sh, ver);
+    bsum = block_sum_u64(sh, bsum);
+    terms = block_sum_u64(sh, terms);
+    near = block_sum_u64(sh, near);
+    fsum = block_sum_f64(sh, fsum);
+    fabs_ = block_sum_f64(sh, fabs_);
+    if (tid == 0) {
+      RsItemPart *ip = reinterpret_cast<RsItemPart *>(p.ipart + (size_t)item * kPartBytes);
+      ip->ver = ver;
+      ip->bsum = bsum;
+      ip->terms = terms;
+      ip->near = near;
+      ip->fsum = fsum;
+      ip->fabs = fabs_;
+      for (int a = 0; a < 4; a++) ip->am[a] = am[a];
+      __threadfence();
+      misc[1] = atomicAdd(&p.idone[j], 1u) == d->n_items - 1 ? 1u : 0u;
+    }
+    __syncthreads();
+    if (misc[1]) rs2_finish(p, c, d, misc);
+    __syncthreads();  // misc, am reused by the next item
+  }
+}
+
 int xs_items_threads() { return kXs2T; }
 
+// phase-2 kernel of an item kind: XS grid types 0..2, RS 3
 static const void *xs_items_fn(int grid) {
   switch (grid) {
     case XS_HASH: return (const void *)xs_items_kernel<XS_HASH>;
     case XS_UNIONIZED: return (const void *)xs_items_kernel<XS_UNIONIZED>;
     case XS_NUCLIDE: return (const void *)xs_items_kernel<XS_NUCLIDE>;
+    case 3: return (const void *)rs_items_kernel;
   }
   return nullptr;
 }
+static uint32_t items_smem(int kind) { return kind == 3 ? kRsSmem : kXs2Smem; }
 
 cudaError_t xs_items_occupancy(int grid, int *ctas) {
   const void *fn = xs_items_fn(grid);
   if (!fn) return cudaErrorInvalidValue;
-  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kXs2Smem);
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)items_smem(grid));
   if (e != cudaSuccess) return e;
   int per_sm = 0, dev = 0, sms = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kXs2T, kXs2Smem);
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kXs2T, items_smem(grid));
   if (e == cudaSuccess) e = cudaGetDevice(&dev);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   *ctas = per_sm * sms;
@@ -365,10 +562,10 @@ cudaError_t xs_items_occupancy(int grid, int *ctas) {
 cudaError_t launch_xs_items(int grid_type, int ctas, const KParams &p, cudaStream_t st) {
   const void *fn = xs_items_fn(grid_type);
   if (!fn) return cudaErrorInvalidValue;
-  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)kXs2Smem);
+  cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)items_smem(grid_type));
   if (e != cudaSuccess) return e;
   void *args[] = {const_cast<KParams *>(&p)};
-  return cudaLaunchKernel(fn, dim3((unsigned)ctas), dim3((unsigned)kXs2T), args, kXs2Smem, st);
+  return cudaLaunchKernel(fn, dim3((unsigned)ctas), dim3((unsigned)kXs2T), args, items_smem(grid_type), st);
 }
 
 }  // namespace ens
