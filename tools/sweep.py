@@ -8,7 +8,8 @@ of `reps` relaunches, arguments resident).  The paper's metric is the relative
 speedup T1*N/TN, T1 = the same launch at N = 1 with the same T
 (one T1 per thread-limit panel, reading Q7); "linear" = N is its upper bound
 (P:549-554).  Teams are one CTA (the paper's team = one thread block,
-P:313-318), M = 1.  Also reported: instances/s and busy SMs (from the
+P:313-318), M = 1, every instance start to finish in the one ensemble kernel
+(ENS_F_FUSED: the paper's mapping).  Also reported: instances/s and busy SMs (from the
 per-instance smid of the records).
 """
 import argparse
@@ -33,7 +34,7 @@ APPS = {
 
 def time_launch(lines, threads, reps):
     text = "".join(l + "\n" for l in lines)
-    e = Ensemble(Args.parse(text), app="auto", threads=threads, team_ctas=1, timestamps=True).launch()
+    e = Ensemble(Args.parse(text), app="auto", threads=threads, team_ctas=1, timestamps=True, fused=True).launch()
     torch.cuda.synchronize()
     ts = []
     for _ in range(reps):
@@ -53,10 +54,10 @@ def time_launch(lines, threads, reps):
 
 def main():
     ap = argparse.ArgumentParser()
-    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "sweep_r1.json"))
-    ap.add_argument("--max-n", type=int, default=1024)
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "sweep_r2.json"))
+    ap.add_argument("--max-n", type=int, default=4096)
     ap.add_argument("--reps", type=int, default=3)
-    ap.add_argument("--threads", default="32,1024")
+    ap.add_argument("--threads", default="32,256,1024")
     ap.add_argument("--apps", default=",".join(APPS))
     a = ap.parse_args()
     torch.cuda.set_device(0)
@@ -80,7 +81,8 @@ def main():
                 rows.append(row)
                 print(f"{app:10s} T={Treal:5d} N={n:5d} grid={grid:5d} {ms:9.3f} ms  speedup {row['speedup']:8.2f}"
                       f"  sms {sms:3d}  ok={ok}", flush=True)
-    out = {"what": "T1*N/TN on one B200 (paper Fig. 6 metric, P:540-554); team = 1 CTA; median of reps",
+    out = {"what": "T1*N/TN on one B200 (paper Fig. 6 metric, P:540-554); team = 1 CTA, fused; median of reps",
+           "paper_context": "up to 51x at 64 instances on an A100 40GB (P:44-45, P:639-640)",
            "device": torch.cuda.get_device_name(0), "apps": APPS, "rows": rows}
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
     with open(a.out, "w") as f:
