@@ -122,6 +122,10 @@ APP_OF = {"EchoApp": 1, "XsApp": 2, "RsApp": 3, "AmgApp": 4, "PrApp": 5}
 def kernel_key(name):
     """bench.py's key of a kernel: phase1_app<id> for ens_kernel<App,T>, phase2_kind<grid> for
     xs_items_kernel<grid>."""
+    if "xs_init_items_kernel" in name:
+        return "phase3_app2"
+    if "rs_items_kernel" in name:
+        return "phase2_kind3"
     m = re.search(r"xs_items_kernel<\(?i?n?t?\)?(\d)>", name)
     if m:
         return f"phase2_kind{m.group(1)}"
@@ -152,7 +156,7 @@ def counters(rep, workload):
             ms /= 1e3
         out[key] = {"dram_bytes": tb, "inst_executed": float(d["smsp__inst_executed.sum"][0].replace(",", "")),
                     "ncu_ms": ms, "kernel": d["Kernel Name"][0], "source": os.path.relpath(rep, ROOT)}
-    p = os.path.join(ROOT, "profiles", "ncu_counters.json")
+    p = os.environ.get("NCU_COUNTERS", os.path.join(ROOT, "profiles", "ncu_counters.json"))
     allc = json.load(open(p)) if os.path.exists(p) else {}
     allc[workload] = {"kernels": out, "note": "one ncu --set full capture of a warm launch (--clock-control none); "
                                               "per-launch counters, cold-cache serialised times"}
