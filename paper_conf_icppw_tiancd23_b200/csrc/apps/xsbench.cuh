@@ -208,9 +208,7 @@ struct XsApp {
         R.deferred = 1;
         return R;
       }
-      uint32_t *mcnt = (uint32_t *)(ens_smem(c) + S.mcnt);
-      lookup_sort(c, p, L, thr, mcnt, 0, p.lookups);
-      if (c.crank == 0 && threadIdx.x == 0) write_desc(c, p, L, mcnt);
+      split_sort(c, p, L, S, thr);
       R.deferred = 1;
       return R;
     }
@@ -233,6 +231,15 @@ struct XsApp {
     ens_printf(c, FMT_VERIFY, (unsigned long long)R.vhash);
     R.exit_code = 0;
     return R;
+  }
+
+  // split phases, phase 1 (unionized): sort the lookups and leave the
+  // descriptor; out of line, so the fused path's registers are its own
+  __device__ static __noinline__ void split_sort(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S,
+                                                 const double *thr) {
+    uint32_t *mcnt = (uint32_t *)(ens_smem(c) + S.mcnt);
+    lookup_sort(c, p, L, thr, mcnt, 0, p.lookups);
+    if (c.crank == 0 && threadIdx.x == 0) write_desc(c, p, L, mcnt);
   }
 
   // split phases: the instance's phase-2 descriptor (one thread)

@@ -274,19 +274,25 @@ __global__ void __launch_bounds__(256, 2) xs_init_items_kernel(const KParams p) 
   uint32_t *misc = reinterpret_cast<uint32_t *>(ens_dsmem + kXsInitMisc);
   char *scr = p.init_scr + (size_t)blockIdx.x * p.init_scr_bytes;
   bool jt_ok = false;  // the LCG jump tables (seed- and layout-independent: S.jmp is fixed)
+  uint32_t cached_j = 0xffffffffu;  // the instance whose command line xp holds (items are instance-major)
+  XsParams xp;
   for (;;) {
     if (tid == 0) misc[0] = atomicAdd(p.counter3, 1u);
     __syncthreads();
     const uint32_t it = misc[0];
     if (it >= p.n_init_items) break;
     const uint32_t j = p.init_items[2 * it], i = p.init_items[2 * it + 1];
-    const uint32_t k = p.kmap[j], line = p.line_of_k[k], t0 = p.line_tok[line];
-    const int argc = (int)(p.line_tok[line + 1] - t0);
-    for (int a = tid; a < argc; a += T) argv[a] = const_cast<char *>(p.blob) + p.tok_off[t0 + a];
-    if (tid == 0) argv[argc] = nullptr;
-    __syncthreads();
-    XsParams xp;
-    xs_parse(argc, argv, xp);  // a valid line: the host made items only for those
+    const uint32_t k = p.kmap[j], line = p.line_of_k[k];
+    if (j != cached_j) {
+      const uint32_t t0 = p.line_tok[line];
+      const int argc = (int)(p.line_tok[line + 1] - t0);
+      for (int a = tid; a < argc; a += T) argv[a] = const_cast<char *>(p.blob) + p.tok_off[t0 + a];
+      if (tid == 0) argv[argc] = nullptr;
+      __syncthreads();
+      xp = XsParams();
+      xs_parse(argc, argv, xp);  // a valid line: the host made items only for those
+      cached_j = j;
+    }
     const XsSmem S = xs_init_smem(xp);
     const XsLayout L = xs_layout(xp, (int)p.team_ctas);  // the instance's arena, as phase 1 lays it out
     c.arena = p.arena_base + (size_t)j * p.arena_bytes;

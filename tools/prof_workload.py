@@ -1,6 +1,6 @@
 """One warm launch of a bench workload, for profilers (not the bench).
 
-    python tools/prof_workload.py <C1|C2|C2U|C3|C4|C5|TSTAR> [relaunches] [--threads T] [--team K] [--fused]
+    python tools/prof_workload.py <C1|C2|C2U|C3|C4|C5|TSTAR> [relaunches] [--threads T] [--team K] [--fused | --split]
 
 Launches the workload's ensemble once (cold) and relaunches it `relaunches` times (default 1):
 `ncu --launch-skip <kernels per launch> --launch-count 1 -k regex:ens_kernel` then captures a
@@ -23,6 +23,9 @@ def main():
     fused = "--fused" in argv
     if fused:
         argv.remove("--fused")
+    split = "--split" in argv
+    if split:
+        argv.remove("--split")
     opt = {}
     for k in ("--threads", "--team"):
         if k in argv:
@@ -34,7 +37,7 @@ def main():
     lines, desc = bench.workload_lines(name, 1)
     threads = opt.get("--threads", bench.THREADS.get(name, 256))
     e = Ensemble(Args.parse(workloads.text(lines)), app="auto", threads=threads,
-                 team_ctas=opt.get("--team", 0), fused=fused).launch()
+                 team_ctas=opt.get("--team", 0), fused=fused, split=split).launch()
     torch.cuda.synchronize()
     for _ in range(reps):
         a, b = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -42,7 +45,7 @@ def main():
         e.relaunch()
         b.record()
         torch.cuda.synchronize()
-        print(f"{name}{' fused' if fused else ''}: {a.elapsed_time(b):.3f} ms", flush=True)
+        print(f"{name}{' fused' if fused else ''}{' split' if split else ''}: {a.elapsed_time(b):.3f} ms", flush=True)
     r = e.collect(stdout=False)
     i = e.info()
     print(f"exit ok={bool((r.records['exit_code'] == 0).all())} kernels/launch={i.kernel_launches} "
