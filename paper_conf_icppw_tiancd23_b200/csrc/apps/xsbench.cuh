@@ -1336,6 +1336,8 @@ struct XsApp {
   // nuclide j+1's guess and pair address computed and the pair prefetched,
   // nuclide j's pair gathered, verified and accumulated.  The bracket logic
   // and every FP operation are those of macro_lookup<XS_HASH> (bit-identical).
+  // Split phases' phase 2 only: the tables were written by an earlier kernel
+  // and nothing writes them now, so the loads take the read-only path (ldro).
   __device__ static __forceinline__ void macro_lookup_hash1(const XsParams &p, const double *recs, const int *ig,
                                                             const int *nn, const double *concs,
                                                             const uint16_t *mats, double pe, int mat, int idx,
@@ -1363,14 +1365,14 @@ struct XsApp {
     };
     double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
     const uint4 z = make_uint4(0, 0, 0, 0);
-    uint4 h0 = nm > 0 ? ld_(ent(0)) : z;
-    uint4 h1 = nm > 1 ? ld_(ent(1)) : z;
+    uint4 h0 = nm > 0 ? ldro(ent(0)) : z;
+    uint4 h1 = nm > 1 ? ldro(ent(1)) : z;
     if (nm > 2) prefetch_l1(ent(2));
     if (nm > 3) prefetch_l1(ent(3));
     int lo0 = guess(h0);
     const double2 *q0 = pair_at(0, lo0);
     for (int j = 0; j < nm; j++) {
-      const uint4 h2 = j + 2 < nm ? ld_(ent(j + 2)) : z;
+      const uint4 h2 = j + 2 < nm ? ldro(ent(j + 2)) : z;
       if (j + 4 < nm) prefetch_l1(ent(j + 4));
       const double2 *q1 = q0;
       int lo1 = lo0;
@@ -1380,8 +1382,8 @@ struct XsApp {
         prefetch_l1(q1);
         prefetch_l1(reinterpret_cast<const double *>(q1) + 11);
       }
-      double2 a0 = ld_(q0 + 0), a1 = ld_(q0 + 1), a2 = ld_(q0 + 2);
-      double2 b0 = ld_(q0 + 3), b1 = ld_(q0 + 4), b2 = ld_(q0 + 5);
+      double2 a0 = ldro(q0 + 0), a1 = ldro(q0 + 1), a2 = ldro(q0 + 2);
+      double2 b0 = ldro(q0 + 3), b1 = ldro(q0 + 4), b2 = ldro(q0 + 5);
       {  // verify the guessed pair; walk / upstream search otherwise (macro_lookup's gather_fix)
         const uint4 &h = h0;
         const double *E = reinterpret_cast<const double *>(q0) - 6 * (size_t)lo0;  // the nuclide's records
@@ -1391,19 +1393,19 @@ struct XsApp {
           lo++;
           const double2 *w2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
           a0 = b0; a1 = b1; a2 = b2;
-          b0 = ld_(w2 + 3); b1 = ld_(w2 + 4); b2 = ld_(w2 + 5);
+          b0 = ldro(w2 + 3); b1 = ldro(w2 + 4); b2 = ldro(w2 + 5);
         }
         if (!(a0.x < pe && pe < b0.x && lo + 1 <= uh)) {
-          const double e_low = ld_(E + 6 * (size_t)u_low);
-          const double e_high = ld_(E + 6 * (size_t)uh);
+          const double e_low = ldro(E + 6 * (size_t)u_low);
+          const double e_high = ldro(E + 6 * (size_t)uh);
           int lower;
           if (pe <= e_low) lower = 0;
           else if (pe >= e_high) lower = n_gp - 1;
           else lower = gs_recs(E, pe, u_low, uh);
           const int l2 = lower == n_gp - 1 ? lower - 1 : lower;
           const double2 *w2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)l2);
-          a0 = ld_(w2 + 0); a1 = ld_(w2 + 1); a2 = ld_(w2 + 2);
-          b0 = ld_(w2 + 3); b1 = ld_(w2 + 4); b2 = ld_(w2 + 5);
+          a0 = ldro(w2 + 0); a1 = ldro(w2 + 1); a2 = ldro(w2 + 2);
+          b0 = ldro(w2 + 3); b1 = ldro(w2 + 4); b2 = ldro(w2 + 5);
         }
       }
       accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);

@@ -73,7 +73,7 @@ __device__ __forceinline__ void xs2_item(const XsDesc &d, const XsParams &p, lon
     int mat = 0;
 #pragma unroll
     for (int m = 1; m < 12; m++) mat += (sl >= (long long)d.mcnt[m]) ? 1 : 0;
-    const double pe = ld_(lk_pe + sl);
+    const double pe = ldro(lk_pe + sl);  // read-only here: phase 1 wrote it
     int idx = 0;
     if (GRID == XS_UNIONIZED) idx = XsApp::union_idx(uf, uA, UB, n_u, pe);
     else if (GRID == XS_HASH) {

@@ -321,6 +321,11 @@ __device__ inline double block_max_f64(Shared *sh, double v) {
 template <class T>
 __device__ __forceinline__ T ld_(const T *p) { return *p; }
 
+// Read-only global load (ld.global.nc): only for data no thread writes during
+// the kernel — split phases' phase 2 reads tables an earlier kernel wrote.
+template <class T>
+__device__ __forceinline__ T ldro(const T *p) { return __ldg(p); }
+
 // bring the line holding p into L1 without holding registers
 __device__ __forceinline__ void prefetch_l1(const void *p) { asm volatile("prefetch.global.L1 [%0];" ::"l"(p)); }
 
