@@ -493,9 +493,9 @@ __global__ void __launch_bounds__(kXs2T, ENS_RS2_MINB) rs_items_kernel(const KPa
       int mat = 0;
 #pragma unroll
       for (int m = 1; m < 12; m++) mat += (sl >= (long long)d->mcnt[m]) ? 1 : 0;
-      const double E = ld_(lk_e + sl);
+      const double E = ldro(lk_e + sl);
       double macro[4];
-      RsApp::lookup(d->doppler, E, mat, nn, mats, mx, concs, poff, woff, poles, pl, wins, k0, macro, terms, near);
+      RsApp::lookup<true>(d->doppler, E, mat, nn, mats, mx, concs, poff, woff, poles, pl, wins, k0, macro, terms, near);
       double mxv = -DBL_MAX;
       int a = 0;
 #pragma unroll
