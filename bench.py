@@ -504,6 +504,7 @@ def main():
     dist_on = world > 1
     if dist_on:
         os.environ.setdefault("NCCL_DEBUG", "INFO")  # comm_nranks visible in the driver's log
+        os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
         torch.cuda.set_device(local)
         torch.distributed.init_process_group("nccl", device_id=torch.device("cuda", local))
     else:
