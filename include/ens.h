@@ -67,6 +67,16 @@ enum {
                                  streams so one's tail overlaps the next)      */
   ENS_F_FUSED = 1u << 4,      /* run every instance start to finish inside the
                                  one ensemble kernel (the paper's mapping)     */
+  ENS_F_CLC = 1u << 6,        /* scheduler ablation (Blackwell cluster launch
+                                 control): the ensemble kernel is launched with
+                                 one CTA per instance (the paper's N teams); a
+                                 CTA that finished its instance cancels a CTA
+                                 the hardware has not launched yet
+                                 (clusterlaunchcontrol.try_cancel) and runs its
+                                 instance, instead of persistent CTAs pulling ids
+                                 from an atomic counter.  Arena slots come from
+                                 a pool as large as the resident CTAs.  Teams of
+                                 one CTA, M = 1.  Results are identical.       */
   ENS_F_SPLIT_PHASES = 1u << 5 /* run XSBench-style event-mode instances whose
                                  lookups fit one sorted chunk (<= 2^22) in
                                  SPLIT PHASES: the ensemble kernel builds every

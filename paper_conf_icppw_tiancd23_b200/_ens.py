@@ -16,7 +16,8 @@ LIB_PATH = os.environ.get("ENS_LIB_PATH") or os.path.join(PKG_DIR, "libens.so") 
 ENS_OK, ENS_EINVAL, ENS_ENOENT, ENS_ENOMEM, ENS_ECUDA, ENS_ERANGE, ENS_EBUSY, ENS_EPARSE = 0, -1, -2, -3, -4, -5, -6, -7
 ENS_EXIT_USAGE, ENS_EXIT_NOMEM, ENS_EXIT_NOTFOUND = 1, 12, 127
 ENS_RF_STDOUT_TRUNC, ENS_RF_NOMEM, ENS_RF_NOT_RUN, ENS_RF_DONE = 1, 2, 4, 8
-ENS_F_TIMESTAMPS, ENS_F_PHASES, ENS_F_GENERIC, ENS_F_SERIAL, ENS_F_FUSED, ENS_F_SPLIT_PHASES = 1, 2, 4, 8, 16, 32
+ENS_F_TIMESTAMPS, ENS_F_PHASES, ENS_F_GENERIC, ENS_F_SERIAL, ENS_F_FUSED, ENS_F_SPLIT_PHASES, ENS_F_CLC = \
+    1, 2, 4, 8, 16, 32, 64
 ENS_PHASES = 16
 ENS_APP_BY_ARGV0, ENS_APP_ECHO, ENS_APP_XSBENCH, ENS_APP_RSBENCH, ENS_APP_AMGMK, ENS_APP_PAGERANK = 0, 1, 2, 3, 4, 5
 ENS_N_APPS = 6

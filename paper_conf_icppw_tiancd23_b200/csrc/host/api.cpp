@@ -172,7 +172,9 @@ struct Group {
   uint32_t smem = 0;    // app shared memory of one instance
   uint32_t sub = 0;     // dynamic smem per instance row: scheduler state + app smem
   size_t dyn() const { return (size_t)m * sub; }
-  int ctas() const { return grid * cs / m; }
+  bool clc = false;     // ENS_F_CLC: one CTA per instance launched; grid = arena slots
+  size_t slot_bm_off = 0;
+  int ctas() const { return clc ? (int)kmap.size() : grid * cs / m; }
   uint64_t arena = 0;
   std::vector<uint32_t> kmap;
   std::vector<double> cost;  // app_cost per kmap entry (schedule only)
@@ -446,7 +448,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
       const int64_t nn = (int64_t)g.kmap.size();
       if (grid > nn) grid = (int)((nn + g.m - 1) / g.m * g.m);
       g.grid = std::max(grid, g.m);
-    } else if (app_team_aware(ap)) {
+    } else if (app_team_aware(ap) && !(c->flags & ENS_F_CLC)) {
       if (c->team_ctas > 0) {
         while (cs * 2 <= c->team_ctas && cs < kMaxTeamCtas) cs *= 2;
       } else if (!c->grid_blocks) {
@@ -471,6 +473,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
       g.grid = std::max(grid, 1);
     }
     g.cs = cs;
+    g.clc = (c->flags & ENS_F_CLC) && g.m == 1 && cs == 1;
     for (uint32_t k : g.kmap) {  // arena of this team size
       int argc;
       const char *const *argv;
@@ -567,6 +570,10 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
   P.staged = o;
   // zeroed part
   P.o_ctr = o; o = al(o + (P.groups.size() + 1) * 8);
+  for (Group &g : P.groups) {  // ENS_F_CLC: arena-slot pool bitmaps
+    if (!g.clc) continue;
+    g.slot_bm_off = o; o = al(o + ((size_t)g.grid + 31) / 32 * 4);
+  }
   for (Group &g : P.groups) {
     if (!g.split) continue;
     g.ctr2_off = o; o = al(o + 4 * 8);
@@ -681,6 +688,9 @@ static int enqueue(ens_run *r) {
     k.dump = P.dump_rows ? (double *)(r->ws + P.o_dump) : nullptr;
     k.dump_rows = P.dump_rows;
     k.split = g.split ? 1u : 0u;
+    k.clc = g.clc ? 1u : 0u;
+    k.slot_bm = g.clc ? (uint32_t *)(r->ws + g.slot_bm_off) : nullptr;
+    k.n_slots = (uint32_t)g.grid;
     if (g.split) {
       k.xs_desc = r->ws + g.desc_off;
       k.items = (const uint32_t *)(r->ws + g.items_off);

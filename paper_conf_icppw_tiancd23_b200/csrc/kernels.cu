@@ -57,7 +57,54 @@ struct SubShared {
   char *argv[ENS_MAX_ARGC + 1];
   unsigned long long pos;
   uint32_t j;
+  uint32_t clc_phase;          // ENS_F_CLC: the mbarrier's phase parity
+  alignas(16) uint4 clc_res;   // ENS_F_CLC: the try_cancel response
+  unsigned long long clc_mbar;
 };
+
+#if !ENS_SUB
+// ENS_F_CLC (SURVEY.md §8(a) S3 ablation): cluster launch control.  The grid
+// has one CTA per instance (the paper's N teams); a CTA that finished its
+// instance cancels a CTA of the grid the hardware has not launched yet and
+// runs that one's instance instead (clusterlaunchcontrol.try_cancel: the
+// response arrives in shared memory through an mbarrier transaction).
+// Returns false when every CTA has been launched.  One thread.
+__device__ __forceinline__ bool clc_steal(SubShared *ss, uint32_t *x) {
+  const uint32_t mbar = (uint32_t)__cvta_generic_to_shared(&ss->clc_mbar);
+  const uint32_t res = (uint32_t)__cvta_generic_to_shared(&ss->clc_res);
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], 16;" ::"r"(mbar) : "memory");
+  asm volatile("clusterlaunchcontrol.try_cancel.async.shared::cta.mbarrier::complete_tx::bytes.b128 [%0], [%1];" ::"r"(res),
+               "r"(mbar)
+               : "memory");
+  uint32_t done = 0;
+  while (!done)
+    asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                 : "=r"(done)
+                 : "r"(mbar), "r"(ss->clc_phase)
+                 : "memory");
+  ss->clc_phase ^= 1u;
+  uint32_t ok = 0, v = 0;
+  asm volatile("{ .reg .pred p; .reg .b128 r; ld.shared.b128 r, [%2];\n\t"
+               "clusterlaunchcontrol.query_cancel.is_canceled.pred.b128 p, r;\n\t"
+               "selp.u32 %0, 1, 0, p;\n\t"
+               "@p clusterlaunchcontrol.query_cancel.get_first_ctaid::x.b32.b128 %1, r; }"
+               : "=r"(ok), "=r"(v)
+               : "r"(res)
+               : "memory");
+  *x = v;
+  return ok != 0;
+}
+// ENS_F_CLC: arena slots are not CTA ids (the grid has N CTAs) but a pool as
+// large as the resident CTAs: a CTA claims a free bit of the pool bitmap on
+// arrival and returns it on exit (memory = resident CTAs x arena, as with the
+// persistent grid)
+__device__ __forceinline__ uint32_t slot_claim(uint32_t *bm, uint32_t n_slots) {
+  for (uint32_t i = blockIdx.x % n_slots;; i = i + 1 == n_slots ? 0 : i + 1) {
+    const uint32_t bit = 1u << (i & 31);
+    if (!(atomicOr(&bm[i >> 5], bit) & bit)) return i;
+  }
+}
+#endif
 constexpr uint32_t kSubSharedBytes = (sizeof(SubShared) + 15) / 16 * 16;
 
 // T = threads per CTA (the launch bound); the instance runs on the CTA's row
@@ -71,7 +118,25 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
   char **s_argv = ss->argv;
   const uint32_t cs = p.team_ctas;  // cluster dims (cs, 1, 1); M > 1 only with cs == 1
   const uint32_t cr = cs > 1 ? cooperative_groups::this_cluster().block_rank() : 0u;
-  char *const arena = p.arena_base + ((size_t)(blockIdx.x / cs) * M + y) * p.arena_bytes;
+#if ENS_SUB
+  const bool clc = false;
+#else
+  const bool clc = p.clc != 0;  // M == 1 and cs == 1 (host-enforced)
+#endif
+  uint32_t slot = (blockIdx.x / cs) * M + y;
+#if !ENS_SUB
+  if (clc && !p.split) {
+    if (tid == 0) ss->j = slot_claim(p.slot_bm, p.n_slots);
+    __syncthreads();
+    slot = ss->j;
+  }
+  if (clc && tid == 0) {
+    ss->clc_phase = 0;
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"((uint32_t)__cvta_generic_to_shared(&ss->clc_mbar)));
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+#endif
+  char *const arena = p.arena_base + (size_t)slot * p.arena_bytes;
   Ctx c;
   c.arena = arena;
   c.arena_cap = p.arena_bytes;
@@ -80,8 +145,21 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
   c.smem_off = c.sh_off + kSubSharedBytes;
   c.crank = cr;
   c.csize = cs;
+  bool first = true;
   for (;;) {
+#if ENS_SUB
     if (tid == 0 && cr == 0) ss->j = atomicAdd(p.counter, 1u);
+#else
+    if (tid == 0 && cr == 0) {
+      if (!clc) ss->j = atomicAdd(p.counter, 1u);
+      else if (first) ss->j = blockIdx.x;  // this CTA's own instance
+      else {
+        uint32_t x = 0;
+        ss->j = clc_steal(ss, &x) ? x : 0xffffffffu;  // an unlaunched CTA's instance, or done
+      }
+    }
+    first = false;
+#endif
     team_sync(c);
     const uint32_t j = cr == 0 ? ss->j : *cta_shared(&ss->j, 0);
     if (cs > 1) team_sync(c);  // every rank has read s_j before rank 0 may exit
@@ -153,6 +231,13 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
     }
     team_sync(c);  // j, pos, argv, sh reused by the next instance
   }
+#if !ENS_SUB
+  if (clc && !p.split && tid == 0) {  // the arena slot back to the pool (its writes first)
+    __threadfence();
+    atomicAnd(&p.slot_bm[slot >> 5], ~(1u << (slot & 31)));
+  }
+#endif
+  (void)first;
 }
 
 template <class App, int T>

@@ -49,6 +49,11 @@ struct KParams {
   char *init_scr;             // [grid][init_scr_bytes] per-CTA scratch
   uint64_t init_scr_bytes;
   uint32_t init_smem_off;     // dynamic smem offset of the app's shared memory
+  // ENS_F_CLC: one CTA per instance, cluster launch control for the rest,
+  // arena slots from a bitmap pool of n_slots
+  uint32_t clc;
+  uint32_t *slot_bm;          // [ceil(n_slots / 32)] (zeroed)
+  uint32_t n_slots;
 };
 
 const void *kernel_ptr(uint32_t app, int T);

@@ -23,7 +23,7 @@ class Ensemble:
 
     def __init__(self, args, app="auto", n=None, first=0, stride=1, threads=256, grid=0, arena_bytes=0,
                  stdout_bytes=0, timestamps=False, device=None, stream=None, team_ctas=0, phases=False,
-                 instances_per_cta=0, generic=False, serial=False, dump_rows=0, fused=False, split=False):
+                 instances_per_cta=0, generic=False, serial=False, dump_rows=0, fused=False, split=False, clc=False):
         _require_cuda()
         self.args = args
         self.app = app
@@ -34,7 +34,8 @@ class Ensemble:
                             stdout_bytes=stdout_bytes,
                             flags=(_ens.ENS_F_TIMESTAMPS if timestamps else 0) | (_ens.ENS_F_PHASES if phases else 0)
                             | (_ens.ENS_F_GENERIC if generic else 0) | (_ens.ENS_F_SERIAL if serial else 0)
-                            | (_ens.ENS_F_FUSED if fused else 0) | (_ens.ENS_F_SPLIT_PHASES if split else 0),
+                            | (_ens.ENS_F_FUSED if fused else 0) | (_ens.ENS_F_SPLIT_PHASES if split else 0)
+                            | (_ens.ENS_F_CLC if clc else 0),
                             team_ctas=team_ctas, instances_per_cta=instances_per_cta, dump_rows=dump_rows)
         self.n = n
         self.device = torch.device("cuda", torch.cuda.current_device()) if device is None else torch.device(device)
