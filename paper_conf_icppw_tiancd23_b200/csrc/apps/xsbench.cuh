@@ -191,7 +191,7 @@ struct XsApp {
     hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
     phase_mark(c, 0);
     // split phases: a hash / nuclide instance's per-nuclide tables are built
-    // by the init-item kernel (kernels_xs2.cu) running beside this kernel
+    // by the init-item kernel (kernels_items.cu) running beside this kernel
     const bool init_items = c.desc && xs_split_ok(p) && p.grid != XS_UNIONIZED;
     if (init_items) {
     } else if (p.grid == XS_UNIONIZED) {
@@ -391,7 +391,7 @@ struct XsApp {
   // else in this CTA's arena scratch (L2 atomics; the same algorithm)
   // The team's CTAs take nuclides crank, crank + csize, ... with per-CTA
   // scratch in the arena; init_nuc_range runs nuclides [i0, i1) with the
-  // caller's scratch (split phases: one nuclide per work item, kernels_xs2.cu)
+  // caller's scratch (split phases: one nuclide per work item, kernels_items.cu)
   __device__ static void init_nuc(Ctx &c, const XsParams &p, const XsLayout &L, const XsSmem &S) {
     char *ekey = c.arena + L.keys + (size_t)c.crank * p.n_gp * 8;
     char *col = c.arena + L.hcol + (size_t)c.crank * (p.bins + 1) * 4;

@@ -1,5 +1,6 @@
-// csrc/kernels_xs2.cu — split phases, phase 2: the XSBench-style lookup
-// items of every instance of an ensemble, on every SM.
+// csrc/kernels_items.cu — the split-phase item kernels: phase 1b (XS
+// per-nuclide tables and lookup sorts) and phase 2 (XS and RS lookup items of
+// every instance of an ensemble, on every SM).
 //
 // Phase 1 (the ensemble kernel, kernels.cu: one team per instance, the
 // paper's mapping) builds each instance's tables and its (material,

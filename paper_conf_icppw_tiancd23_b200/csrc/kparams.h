@@ -68,7 +68,7 @@ bool app_size(uint32_t app, int argc, const char *const *argv, int T, int cs, ui
 cudaError_t launch_group(uint32_t app, int T, int m, int grid, int cs, size_t smem, const KParams &p,
                          cudaStream_t st);
 cudaError_t group_occupancy(uint32_t app, int T, int m, int cs, size_t smem, int *teams);
-// split phases, phase 2 (kernels_xs2.cu): the XS lookup-item kernel
+// split phases, phase 2 (kernels_items.cu): the XS lookup-item kernel
 cudaError_t launch_xs_items(int grid_type, int ctas, const KParams &p, cudaStream_t st);
 cudaError_t xs_items_occupancy(int grid_type, int *ctas);
 int xs_items_threads();
