@@ -318,10 +318,14 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
 // one team per instance, as always) builds the tables and the sorted lookup
 // chunk in a per-INSTANCE arena and writes an XsDesc; phase 2 is a
 // persistent kernel over every SM whose CTAs pull lookup batches ("items":
-// kXsItemLookups consecutive sorted slots of one instance) from one queue,
+// kXsItemLookups consecutive sorted slots of one instance; 1024 measured best
+// over 4096 / 2048: C2 35.6 / 35.0 / 34.9 ms) from one queue,
 // so all instances' lookups share every SM; the CTA finishing an instance's
 // last item writes its record and stdout.  Per-lookup results are unchanged.
-constexpr long long kXsItemLookups = 4096;
+#ifndef ENS_XS_ITEM
+#define ENS_XS_ITEM 1024
+#endif
+constexpr long long kXsItemLookups = ENS_XS_ITEM;
 ENS_HD bool xs_split_ok(const XsParams &p) { return !p.history && p.lookups > 0 && p.lookups <= kXsLkChunk; }
 ENS_HD long long xs_items(const XsParams &p) {
   return xs_split_ok(p) ? (p.lookups + kXsItemLookups - 1) / kXsItemLookups : 0;
@@ -508,8 +512,12 @@ ENS_HD RsLayout rs_layout(const RsParams &p) {
   L.total = o;
   return L;
 }
-// split phases (see XsDesc): RS instances whose lookups fit one sorted chunk
-constexpr long long kRsItemLookups = 2048;
+// split phases (see XsDesc): RS instances whose lookups fit one sorted chunk;
+// items of 512 lookups (C3: 2048 / 1024 / 512 / 256 -> 16.3 / 15.9 / 15.6 / 15.8 ms)
+#ifndef ENS_RS_ITEM
+#define ENS_RS_ITEM 512
+#endif
+constexpr long long kRsItemLookups = ENS_RS_ITEM;
 ENS_HD bool rs_split_ok(const RsParams &p) { return p.lookups > 0 && p.lookups <= kRsLkChunk; }
 ENS_HD long long rs_items(const RsParams &p) {
   return rs_split_ok(p) ? (p.lookups + kRsItemLookups - 1) / kRsItemLookups : 0;

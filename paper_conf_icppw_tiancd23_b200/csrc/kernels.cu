@@ -120,6 +120,7 @@ __global__ void __launch_bounds__(T, (ENS_MINB_NUM / T) > 0 ? (ENS_MINB_NUM / T)
   const uint32_t cr = cs > 1 ? cooperative_groups::this_cluster().block_rank() : 0u;
 #if ENS_SUB
   const bool clc = false;
+  (void)clc;
 #else
   const bool clc = p.clc != 0;  // M == 1 and cs == 1 (host-enforced)
 #endif
