@@ -264,9 +264,15 @@ struct XsLayout {
 // (~8 lookups per bucket).
 constexpr long long kXsLkChunk = 1LL << 22;
 ENS_HD long long xs_lk_chunk(const XsParams &p) { return p.lookups < kXsLkChunk ? p.lookups : kXsLkChunk; }
+#ifndef ENS_XS_LK_KB_MAX
+#define ENS_XS_LK_KB_MAX 18
+#endif
+#ifndef ENS_XS_LK_PER_BKT
+#define ENS_XS_LK_PER_BKT 8
+#endif
 ENS_HD int xs_lk_bits(long long n_c) {
   int kb = 0;
-  while (kb < 18 && (12LL << kb) * 8 < n_c) kb++;
+  while (kb < ENS_XS_LK_KB_MAX && (12LL << kb) * ENS_XS_LK_PER_BKT < n_c) kb++;
   return kb;
 }
 // hash index entry (a private accelerator; results are unchanged): the
@@ -326,6 +332,12 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
 #define ENS_XS_ITEM 1024
 #endif
 constexpr long long kXsItemLookups = ENS_XS_ITEM;
+// split phases, phase 1b: lookups per count / scatter item of the lookup sort
+#ifndef ENS_XS_SORT_ITEM
+#define ENS_XS_SORT_ITEM 65536
+#endif
+constexpr long long kXsSortChunk = ENS_XS_SORT_ITEM;
+ENS_HD int xs_sort_items(const XsParams &p) { return (int)((xs_lk_chunk(p) + kXsSortChunk - 1) / kXsSortChunk); }
 ENS_HD bool xs_split_ok(const XsParams &p) { return !p.history && p.lookups > 0 && p.lookups <= kXsLkChunk; }
 ENS_HD long long xs_items(const XsParams &p) {
   return xs_split_ok(p) ? (p.lookups + kXsItemLookups - 1) / kXsItemLookups : 0;
@@ -355,8 +367,23 @@ constexpr int kXsStep = ENS_XS_STEP;
 // dynamic shared memory layout: material tables + the sort's bucket counters
 constexpr int kXsMaxT = 512;  // XsApp::kMaxT
 struct XsSmem {
-  uint32_t thr, nn, mats, concs, mcnt, jmp, nbkt, ubkt, nkey, total;
+  uint32_t thr, nn, mats, concs, mcnt, jmp, nbkt, ubkt, nkey, njdx, total;
 };
+// hash / nuclide grids, per-nuclide sort in shared memory: [nkey] u32 sort
+// keys (after the sort: the hash column's per-record codes, init_nuc_t) |
+// [nbkt] u32 bucket counters | [njdx] u16 record indices; the hash column
+// (bins+1 u32) reuses [nbkt, end) once the records are written, the region
+// grown by up to 16 KB so that it fits (else it goes to arena scratch)
+ENS_HD uint32_t xs_nuc_smem_block(const XsParams &p, uint32_t o, XsSmem &S) {
+  S.nkey = o; o += (uint32_t)align_up((uint64_t)p.n_gp * 4, 16);
+  S.nbkt = o; o += (uint32_t)align_up((uint64_t)xs_nbn(p.n_gp) * 4, 16);
+  S.njdx = o; o += (uint32_t)align_up((uint64_t)p.n_gp * 2, 16);
+  if (p.grid == XS_HASH) {
+    const uint64_t need = align_up((uint64_t)(p.bins + 1) * 4, 16), have = o - S.nbkt;
+    if (need > have && need - have <= 16384) o = S.nbkt + (uint32_t)need;
+  }
+  return o;
+}
 // T = the block size the instance runs with
 ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   XsSmem S{};
@@ -368,21 +395,16 @@ ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   S.mats = o; o += (uint32_t)align_up(12 * mx * 2, 16);  // nuclide ids (u16)
   S.mcnt = o; o += 32 * 4;                // material counts / offsets of a lookup chunk
   S.jmp = o; o += 5 * 64 * 16;            // LCG jump tables: A^(6 d 64^l), l < 5, d < 64
-  S.nbkt = o;  // per-nuclide sort buckets (hash / nuclide grids); unionized: per-warp sweep rows
-  if (p.grid != XS_UNIONIZED) o += xs_nuc_smem(p) ? (uint32_t)align_up((uint64_t)xs_nbn(p.n_gp) * 4, 16) : 0u;
-  else o += (uint32_t)(T / 32) * 2u * (uint32_t)xs_iso_pad(p.n_iso) * 4u;
-  S.ubkt = o;  // unionized, small: bucket counters, then chunk owner counts
-  if (xs_smem_nb(p)) o += (uint32_t)kXsSmemBkt * 4u;
-  // hash / nuclide grids: one nuclide's u32 sort keys and u16 record indices
-  S.nkey = o;
-  if (p.grid != XS_UNIONIZED && xs_nuc_smem(p)) {
-    o += (uint32_t)align_up((uint64_t)p.n_gp * 6, 16);
-    // the hash column + quantization keys reuse [nbkt, total) after the sort;
-    // grow the region by up to 16 KB so that they fit (else arena scratch)
-    if (p.grid == XS_HASH) {
-      const uint64_t need = align_up((uint64_t)(p.bins + 1) * 4, 16) + (uint64_t)p.n_gp * 4, have = o - S.nbkt;
-      if (need > have && need - have <= 16384) o = S.nbkt + (uint32_t)align_up(need, 16);
-    }
+  if (p.grid != XS_UNIONIZED) {  // hash / nuclide grids: one nuclide's sort (xs_nuc_smem_block)
+    if (xs_nuc_smem(p)) o = xs_nuc_smem_block(p, o, S);
+    else S.nkey = S.nbkt = S.njdx = o;
+    S.ubkt = o;
+  } else {
+    S.nbkt = o;  // unionized: per-warp sweep rows
+    o += (uint32_t)(T / 32) * 2u * (uint32_t)xs_iso_pad(p.n_iso) * 4u;
+    S.ubkt = o;  // unionized, small: bucket counters, then chunk owner counts
+    if (xs_smem_nb(p)) o += (uint32_t)kXsSmemBkt * 4u;
+    S.nkey = S.njdx = o;
   }
   // unionized warp path: kXsWarpScr per warp, overlaying nbkt / ubkt
   if (xs_warp_union(p)) {
@@ -406,20 +428,9 @@ ENS_HD XsSmem xs_init_smem(const XsParams &p) {
   S.mats = o;
   S.mcnt = o; o += 32 * 4;
   S.jmp = o; o += 5 * 64 * 16;
-  S.nbkt = o;
-  if (p.grid != XS_UNIONIZED && xs_nuc_smem(p)) {
-    o += (uint32_t)align_up((uint64_t)xs_nbn(p.n_gp) * 4, 16);
-    S.ubkt = o;
-    S.nkey = o;
-    o += (uint32_t)align_up((uint64_t)p.n_gp * 6, 16);
-    if (p.grid == XS_HASH) {
-      const uint64_t need = align_up((uint64_t)(p.bins + 1) * 4, 16) + (uint64_t)p.n_gp * 4, have = o - S.nbkt;
-      if (need > have && need - have <= 16384) o = S.nbkt + (uint32_t)align_up(need, 16);
-    }
-  } else {
-    S.ubkt = o;
-    S.nkey = o;
-  }
+  if (p.grid != XS_UNIONIZED && xs_nuc_smem(p)) o = xs_nuc_smem_block(p, o, S);
+  else S.nkey = S.nbkt = S.njdx = o;
+  S.ubkt = o;
   S.total = o;
   return S;
 }

@@ -421,7 +421,7 @@ struct XsApp {
     unsigned long long *ekey = (unsigned long long *)ekey_scr;  // sorted energies (this CTA's)
     const size_t kofs = SMK ? 0 : align_up((uint64_t)nbn * 4, 256);
     uint32_t *K = SMK ? (uint32_t *)(ens_smem(c) + S.nkey) : (uint32_t *)(gscr + kofs);  // sort keys, then
-    uint16_t *J = SMK ? (uint16_t *)(ens_smem(c) + S.nkey + (size_t)n_gp * 4)            // record indices j
+    uint16_t *J = SMK ? (uint16_t *)(ens_smem(c) + S.njdx)                               // record indices j
                       : (uint16_t *)(gscr + kofs + align_up((uint64_t)n_gp * 4, 256));
     int *ig = (int *)(c.arena + L.index);
     const bool hash = p.grid == XS_HASH;
@@ -468,8 +468,26 @@ struct XsApp {
       __syncthreads();
       phase_mark_if(trc, c, 4);
       // records written in sorted order (coalesced, evict-first), their draws
-      // re-generated from the jump tables; the sorted energies to `ekey`
+      // re-generated from the jump tables.  Hash grid: bin b's column entry
+      // is #{k >= 1: E_k <= b*du} (XS-5), i.e. k on [bfirst(E_k),
+      // bfirst(E_k+1)); with the column in shared memory (sm_col) each
+      // record's bfirst and its quantization key are computed here, while its
+      // energy is in a register, into the dead sort keys: W[k] = bin(E_k) << 16
+      // | q15(E_k) << 1 | (bfirst(E_k) - bin(E_k)) (that difference is 0 or 1
+      // unless E_k sits within a few ulps of a bin edge; any other value sends
+      // the nuclide's column pass back to the exact energies in the records);
+      // otherwise the sorted energies go to `ekey` (arena scratch)
+      auto bfirst = [&](double e) {  // first bin b with e <= b*du (bins if none; bins <= 10^7: int)
+        int bb = (int)(e * p.bins);
+        while (bb > 0 && (double)(bb - 1) * du >= e) bb--;
+        while (bb < p.bins && (double)bb * du < e) bb++;
+        return bb;
+      };
+      const uint32_t col_b = (uint32_t)align_up((uint64_t)(p.bins + 1) * 4, 16);
+      const bool sm_col = SMK && hash && p.bins < 65536 && col_b <= S.total - S.nbkt;
+      uint32_t *W = K;
       double *rec_i = recs + (size_t)i * n_gp * 6;
+      int anom = 0;
 #pragma unroll 2
       for (int k = tid; k < n_gp; k += T) {
         uint64_t t = jump6(jt, r0 + J[k], p.gseed);
@@ -479,53 +497,53 @@ struct XsApp {
         __stcs(d, make_double2(e, x1));
         __stcs(d + 1, make_double2(x2, x3));
         __stcs(d + 2, make_double2(x4, x5));
-        ekey[k] = dbits(e);
+        if (sm_col) {  // the entry pass's (e * bins - b) * 2^16 at b = bin(e), as integers
+          const double y = e * (double)p.bins;
+          int be = (int)y;
+          be = be < p.bins ? be : p.bins;
+          const double x = (y - (double)be) * 65536.0;
+          const int q = x < 0.0 ? 0 : (x >= 65535.0 ? 65535 : (int)x);
+          const int db = bfirst(e) - be;
+          anom |= db < 0 || db > 1;
+          W[k] = ((uint32_t)be << 16) | ((uint32_t)(q >> 1) << 1) | (uint32_t)(db & 1);
+        } else {
+          ekey[k] = dbits(e);
+        }
       }
-      __syncthreads();
+      const bool anomaly = __syncthreads_or(anom) != 0;
       phase_mark_if(trc, c, 8);
       if (hash) {
-        // column by a merge walk over the sorted energies: bin b's count
-        // #{k >= 1: E_k <= b*du} is k on [bfirst(E_k), bfirst(E_k+1)) (0
-        // before bfirst(E_1)); each bin is written once, clamped to n_gp-2.
-        // When it fits, the column and each energy's quantization key fk =
-        // bin(E) << 16 | q(E within its bin) live in the shared memory the
-        // sort no longer needs (the 16-B entries then take no global loads);
-        // otherwise the column goes to this CTA's arena scratch.
-        auto bfirst = [&](double e) {  // first bin b with e <= b*du (bins if none; bins <= 10^7: int)
-          int bb = (int)(e * p.bins);
-          while (bb > 0 && (double)(bb - 1) * du >= e) bb--;
-          while (bb < p.bins && (double)bb * du < e) bb++;
-          return bb;
-        };
-        const uint32_t col_b = (uint32_t)align_up((uint64_t)(p.bins + 1) * 4, 16);
-        const bool sm_col = col_b + (uint32_t)n_gp * 4u <= S.total - S.nbkt && p.bins < 65536;
-        int *colp = sm_col ? (int *)(ens_smem(c) + S.nbkt) : col;
-        uint32_t *fk = (uint32_t *)(ens_smem(c) + S.nbkt + col_b);
+        int *colp = sm_col ? (int *)(ens_smem(c) + S.nbkt) : col;  // overlays the dead counters and J
         constexpr int U = 4;  // independent iterations per thread (loads first)
-        for (int k0 = tid; k0 < n_gp; k0 += U * T) {
-          unsigned long long ek[U], ek1[U];
-#pragma unroll
-          for (int u = 0; u < U; u++) {
-            const int k = k0 + u * T;
-            ek[u] = k < n_gp ? ld_(ekey + k) : 0ull;
-            ek1[u] = k + 1 < n_gp ? ld_(ekey + k + 1) : 0ull;
+        if (sm_col) {
+          auto bf_at = [&](int k) {
+            if (anomaly) return bfirst(ld_(rec_i + 6 * (size_t)k));  // this CTA's records (bar.sync-ordered)
+            const uint32_t w = W[k];
+            return (int)(w >> 16) + (int)(w & 1u);
+          };
+          for (int k = tid; k < n_gp; k += T) {
+            const int lo = k == 0 ? 0 : bf_at(k);
+            const int hi = k + 1 < n_gp ? bf_at(k + 1) : p.bins;
+            const int v = k < n_gp - 2 ? k : n_gp - 2;
+            for (int b = lo; b < hi; b++) colp[b] = v;
           }
+        } else {
+          for (int k0 = tid; k0 < n_gp; k0 += U * T) {
+            unsigned long long ek[U], ek1[U];
 #pragma unroll
-          for (int u = 0; u < U; u++) {
-            const int k = k0 + u * T;
-            if (k < n_gp) {
-              const double e = __longlong_as_double((long long)ek[u]);
-              const int lo = k == 0 ? 0 : bfirst(e);
-              const int hi = k + 1 < n_gp ? bfirst(__longlong_as_double((long long)ek1[u])) : p.bins;
-              const int v = k < n_gp - 2 ? k : n_gp - 2;
-              for (int b = lo; b < hi; b++) colp[b] = v;
-              if (sm_col) {  // the entry pass's (e * bins - b) * 2^16 at b = bin(e), as integers
-                const double y = e * (double)p.bins;
-                int be = (int)y;
-                be = be < p.bins ? be : p.bins;
-                const double x = (y - (double)be) * 65536.0;
-                const int q = x < 0.0 ? 0 : (x >= 65535.0 ? 65535 : (int)x);
-                fk[k] = ((uint32_t)be << 16) | (uint32_t)q;
+            for (int u = 0; u < U; u++) {
+              const int k = k0 + u * T;
+              ek[u] = k < n_gp ? ld_(ekey + k) : 0ull;
+              ek1[u] = k + 1 < n_gp ? ld_(ekey + k + 1) : 0ull;
+            }
+#pragma unroll
+            for (int u = 0; u < U; u++) {
+              const int k = k0 + u * T;
+              if (k < n_gp) {
+                const int lo = k == 0 ? 0 : bfirst(__longlong_as_double((long long)ek[u]));
+                const int hi = k + 1 < n_gp ? bfirst(__longlong_as_double((long long)ek1[u])) : p.bins;
+                const int v = k < n_gp - 2 ? k : n_gp - 2;
+                for (int b = lo; b < hi; b++) colp[b] = v;
               }
             }
           }
@@ -542,13 +560,13 @@ struct XsApp {
             h.u_high = (uint16_t)(uh + 1);
 #pragma unroll
             for (int k = 0; k < 6; k++) {
-              int q = 65535;
+              uint32_t q15 = 32767u;
               if (ul + 1 + k <= n_gp - 1) {
-                const uint32_t f = fk[ul + 1 + k];
-                const int fb = (int)(f >> 16);
-                q = fb == b ? (int)(f & 0xffffu) : (fb > b ? 65535 : 0);
+                const uint32_t w = W[ul + 1 + k];
+                const int fb = (int)(w >> 16);
+                q15 = fb == b ? (w >> 1) & 0x7fffu : (fb > b ? 32767u : 0u);
               }
-              h.q[k] = (uint16_t)(q >> 1);  // 15-bit quanta (SWAR compare in guess)
+              h.q[k] = (uint16_t)q15;  // 15-bit quanta (SWAR compare in guess)
             }
             __stcs(reinterpret_cast<uint4 *>(ent + b), *reinterpret_cast<const uint4 *>(&h));
           }
@@ -1327,100 +1345,6 @@ struct XsApp {
     m[4] = m4;
   }
 
-  // XS-7..XS-9 for one hash-grid lookup, one nuclide per step, each step's
-  // bracket guess and pair address computed ONCE (macro_lookup<XS_HASH>
-  // recomputes them for its prefetches: fewer live registers, more issued
-  // instructions — the trade the fused kernel's 128-register budget wants;
-  // phase 2 runs with a budget of its own and issue rate bounds it).  The
-  // software pipeline: entry j+2 loaded and entry j+4 prefetched into L1,
-  // nuclide j+1's guess and pair address computed and the pair prefetched,
-  // nuclide j's pair gathered, verified and accumulated.  The bracket logic
-  // and every FP operation are those of macro_lookup<XS_HASH> (bit-identical).
-  // Split phases' phase 2 only: the tables were written by an earlier kernel
-  // and nothing writes them now, so the loads take the read-only path (ldro).
-  __device__ static __forceinline__ void macro_lookup_hash1(const XsParams &p, const double *recs, const int *ig,
-                                                            const int *nn, const double *concs,
-                                                            const uint16_t *mats, double pe, int mat, int idx,
-                                                            double *m) {
-    const int n_gp = p.n_gp, mx = xs_max_nucs(p.n_iso);
-    const int nm = nn[mat];
-    const uint16_t *mrow = mats + mat * mx;
-    const double *crow = concs + mat * mx;
-    const uint32_t hs32 = (uint32_t)p.bins + 1u;  // entry index < 355 * (10^7 + 1) < 2^32
-    const XsHashEnt *hc = (const XsHashEnt *)ig + idx;
-    auto ent = [&](int j) { return reinterpret_cast<const uint4 *>(hc + (uint32_t)mrow[j] * hs32); };
-    const int pq = (int)((pe * (double)p.bins - (double)idx) * 65536.0);
-    const uint32_t pq15 = (uint32_t)(pq < 0 ? 0 : (pq >> 1 > 32767 ? 32767 : pq >> 1));
-    const uint32_t P = (pq15 | (pq15 << 16) | 0x80008000u) - 0x00010001u;
-    // the guessed bracket lo (clamped to u_high - 1) of an entry, and its pair
-    auto guess = [&](const uint4 &h) {
-      const uint32_t mk = 0x80008000u;
-      const uint32_t x = ((P - h.y) & mk) | (((P - h.z) & mk) >> 1) | (((P - h.w) & mk) >> 2);
-      const int lo = (int)(h.x & 0xffffu) + __popc(x);
-      const int uh = (int)(h.x >> 16);
-      return lo < uh - 1 ? lo : uh - 1;
-    };
-    auto pair_at = [&](int j, int lo) {
-      return reinterpret_cast<const double2 *>(recs + ((uint32_t)mrow[j] * (uint32_t)n_gp + (uint32_t)lo) * 6u);
-    };
-    double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
-    const uint4 z = make_uint4(0, 0, 0, 0);
-    uint4 h0 = nm > 0 ? ldro(ent(0)) : z;
-    uint4 h1 = nm > 1 ? ldro(ent(1)) : z;
-    if (nm > 2) prefetch_l1(ent(2));
-    if (nm > 3) prefetch_l1(ent(3));
-    int lo0 = guess(h0);
-    const double2 *q0 = pair_at(0, lo0);
-    for (int j = 0; j < nm; j++) {
-      const uint4 h2 = j + 2 < nm ? ldro(ent(j + 2)) : z;
-      if (j + 4 < nm) prefetch_l1(ent(j + 4));
-      const double2 *q1 = q0;
-      int lo1 = lo0;
-      if (j + 1 < nm) {
-        lo1 = guess(h1);
-        q1 = pair_at(j + 1, lo1);
-        prefetch_l1(q1);
-        prefetch_l1(reinterpret_cast<const double *>(q1) + 11);
-      }
-      double2 a0 = ldro(q0 + 0), a1 = ldro(q0 + 1), a2 = ldro(q0 + 2);
-      double2 b0 = ldro(q0 + 3), b1 = ldro(q0 + 4), b2 = ldro(q0 + 5);
-      {  // verify the guessed pair; walk / upstream search otherwise (macro_lookup's gather_fix)
-        const uint4 &h = h0;
-        const double *E = reinterpret_cast<const double *>(q0) - 6 * (size_t)lo0;  // the nuclide's records
-        const int u_low = (int)(h.x & 0xffffu), uh = (int)(h.x >> 16);
-        int lo = lo0;
-        while (pe >= b0.x && a0.x < pe && lo + 2 <= uh) {
-          lo++;
-          const double2 *w2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
-          a0 = b0; a1 = b1; a2 = b2;
-          b0 = ldro(w2 + 3); b1 = ldro(w2 + 4); b2 = ldro(w2 + 5);
-        }
-        if (!(a0.x < pe && pe < b0.x && lo + 1 <= uh)) {
-          const double e_low = ldro(E + 6 * (size_t)u_low);
-          const double e_high = ldro(E + 6 * (size_t)uh);
-          int lower;
-          if (pe <= e_low) lower = 0;
-          else if (pe >= e_high) lower = n_gp - 1;
-          else lower = gs_recs(E, pe, u_low, uh);
-          const int l2 = lower == n_gp - 1 ? lower - 1 : lower;
-          const double2 *w2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)l2);
-          a0 = ldro(w2 + 0); a1 = ldro(w2 + 1); a2 = ldro(w2 + 2);
-          b0 = ldro(w2 + 3); b1 = ldro(w2 + 4); b2 = ldro(w2 + 5);
-        }
-      }
-      accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
-      h0 = h1;
-      h1 = h2;
-      q0 = q1;
-      lo0 = lo1;
-    }
-    m[0] = m0;
-    m[1] = m1;
-    m[2] = m2;
-    m[3] = m3;
-    m[4] = m4;
-  }
-
   // union position of energy pe == grid_search(u, pe, 0, n_u-1) (XS-7), via
   // the search table: ufind[floor(pe*UB)] then a short forward scan
   __device__ static __forceinline__ int union_idx(const uint32_t *uf, const uint64_t *uA, long long UB, long long n_u,
@@ -1551,6 +1475,79 @@ struct XsApp {
       }
     }
     team_sync(c);
+  }
+
+  // ---- split phases, phase 1b: lookup_sort in items on any CTAs ----------
+  // The instance's one chunk (xs_split_ok: lookups <= kXsLkChunk) is sorted
+  // exactly as lookup_sort sorts it, its passes cut into items of
+  // kXsSortChunk lookups: (A) count items add into the arena histogram
+  // (RED), the CTA finishing the last one scans it (B, lk_scan), then (C)
+  // scatter items move each lookup's energy to its bucket.  Lookup li draws
+  // 2li+1 (energy) and 2li+2 (material: the first i >= 1 with roll < thr[i],
+  // i.e. 1 + #{i >= 1: thr[i] <= roll} (thr increasing), 0 past thr[11]).
+  // U lookups per thread are sampled before their atomics issue, so U
+  // atomics (and, scattering, U returned cursors) are in flight per thread.
+  __device__ static void lk_pass(const XsParams &p, char *arena, const XsLayout &L, const double *thr,
+                                 long long l0, long long l1, bool scatter, const Affine &JT) {
+    const int tid = threadIdx.x, T = blockDim.x;
+    uint32_t *hist = (uint32_t *)(arena + L.lk_hist);
+    double *lk_pe = (double *)(arena + L.lk_pe);
+    const int kb = xs_lk_bits(xs_lk_chunk(p));
+    const double bscale = (double)(1LL << kb);
+    const long long emax = (1LL << kb) - 1;
+    double th[11];
+#pragma unroll
+    for (int m = 0; m < 11; m++) th[m] = thr[m + 1];
+    constexpr int U = 8;
+    uint64_t s = lcg_pow(2ULL * (uint64_t)(l0 + tid))(p.seed);
+    for (long long li0 = l0 + tid; li0 < l1; li0 += (long long)U * T) {
+      double pe[U];
+      uint32_t bk[U];
+#pragma unroll
+      for (int u = 0; u < U; u++) {
+        uint64_t t = s;
+        pe[u] = lcg_double(t);
+        const double roll = lcg_double(t);
+        int n = 0;
+#pragma unroll
+        for (int m = 0; m < 11; m++) n += roll >= th[m] ? 1 : 0;
+        const int mat = n == 11 ? 0 : n + 1;
+        long long eb = (long long)(pe[u] * bscale);
+        eb = eb > emax ? emax : eb;
+        bk[u] = (uint32_t)(((long long)mat << kb) + eb);
+        s = JT(s);
+      }
+      if (!scatter) {
+#pragma unroll
+        for (int u = 0; u < U; u++)
+          if (li0 + (long long)u * T < l1) atomicAdd(&hist[bk[u]], 1u);
+      } else {
+        uint32_t pos[U];
+#pragma unroll
+        for (int u = 0; u < U; u++)
+          if (li0 + (long long)u * T < l1) pos[u] = atomicAdd(&hist[bk[u]], 1u);
+#pragma unroll
+        for (int u = 0; u < U; u++)
+          if (li0 + (long long)u * T < l1) lk_pe[pos[u]] = pe[u];
+      }
+    }
+  }
+  // (B): bucket offsets and the material starts mcnt[16..28] (one CTA)
+  __device__ static void lk_scan(const Ctx &c, const XsParams &p, const XsLayout &L, uint32_t *mcnt) {
+    const int tid = threadIdx.x;
+    uint32_t *hist = (uint32_t *)(c.arena + L.lk_hist);
+    const long long nc = xs_lk_chunk(p);
+    const int kb = xs_lk_bits(nc);
+    global_exclusive_scan(hist, (12LL << kb) + 1, ens_sh(c));
+    __syncthreads();
+    if (tid < 12) mcnt[16 + tid] = ld_(hist + ((long long)tid << kb));
+    if (tid == 12) mcnt[28] = (uint32_t)nc;
+    __syncthreads();
+  }
+  __device__ static void lk_zero(const Ctx &c, const XsParams &p, const XsLayout &L) {
+    uint32_t *hist = (uint32_t *)(c.arena + L.lk_hist);
+    const long long n = (12LL << xs_lk_bits(xs_lk_chunk(p))) + 1;
+    for (long long b = threadIdx.x; b < n; b += blockDim.x) hist[b] = 0u;
   }
 
   // ---- XS-6..XS-10: lookups ----------------------------------------------

@@ -194,7 +194,7 @@ struct Group {
   uint64_t init_scr_bytes = 0;       // per init CTA
   int grid3 = 0;
   size_t smem3 = 0;
-  size_t init_off = 0, ctr3_off = 0, init_scr_off = 0;
+  size_t init_off = 0, ctr3_off = 0, init_scr_off = 0, isync_off = 0;
   size_t items_off = 0, desc_off = 0, ipart_off = 0, idone_off = 0, ctr2_off = 0;
   size_t slots() const { return split ? kmap.size() : (size_t)grid; }
 };
@@ -514,27 +514,36 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
         g.items.clear();
         for (int kd = 0; kd < 4; kd++) g.kind_n[kd] = 0;
       }
-      if (g.split) {  // phase 1b: sort items (first: the longest), then (instance, nuclide) table items
-        std::vector<uint32_t> nuc_items;
+      if (g.split) {  // phase 1b: the lookup sorts' items and the (instance, nuclide) table items
+        // queue: zero items, count items, a first share of the nuclide items
+        // (the scans finish meanwhile), scatter items, the other nuclide items
+        std::vector<uint32_t> zero_items, count_items, scatter_items, nuc_items;
         uint32_t smem_need = 0;
+        auto pair = [](std::vector<uint32_t> &v, size_t x, uint32_t i) {
+          v.push_back((uint32_t)x);
+          v.push_back(i);
+        };
         for (size_t x = 0; x < g.kmap.size(); x++) {
           int argc;
           const char *const *argv;
           ens_args_get(a, (int)P.line_of_k[g.kmap[x]], &argc, &argv);
-          int ni = 0;
+          int ni = 0, ns = 0;
           uint32_t sm3 = 0;
-          const uint64_t scr = app_init_scratch(ap, argc, argv, &ni, &sm3);
+          const uint64_t scr = app_init_scratch(ap, argc, argv, &ni, &ns, &sm3);
           if (!g.item_count[x] || !ni) continue;
           g.init_scr_bytes = std::max<uint64_t>(g.init_scr_bytes, al(scr));
           smem_need = std::max(smem_need, sm3);
-          g.init_items.push_back((uint32_t)x);
-          g.init_items.push_back(0xffffffffu);  // its sort item
-          for (int i = 0; i < ni; i++) {
-            nuc_items.push_back((uint32_t)x);
-            nuc_items.push_back((uint32_t)i);
-          }
+          pair(zero_items, x, kXsZeroItem);
+          for (int q = 0; q < ns; q++) pair(count_items, x, kXsCountItem | (uint32_t)q);
+          for (int q = 0; q < ns; q++) pair(scatter_items, x, kXsScatterItem | (uint32_t)q);
+          for (int i = 0; i < ni; i++) pair(nuc_items, x, (uint32_t)i);
         }
-        g.init_items.insert(g.init_items.end(), nuc_items.begin(), nuc_items.end());
+        const size_t first = std::min(nuc_items.size(), (size_t)2 * 4 * (size_t)std::max(1, (int)ctas));  // pairs: 4 x ctas items
+        g.init_items = zero_items;
+        g.init_items.insert(g.init_items.end(), count_items.begin(), count_items.end());
+        g.init_items.insert(g.init_items.end(), nuc_items.begin(), nuc_items.begin() + first);
+        g.init_items.insert(g.init_items.end(), scatter_items.begin(), scatter_items.end());
+        g.init_items.insert(g.init_items.end(), nuc_items.begin() + first, nuc_items.end());
         if (!g.init_items.empty()) {
           g.smem3 = xs_init_smem_off() + (smem_need + 15u) / 16u * 16u;
           e = xs_init_items_occupancy(kXsInitThreads, g.smem3, &g.grid3);
@@ -579,6 +588,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
     g.ctr2_off = o; o = al(o + 4 * 8);
     g.ctr3_off = o; o = al(o + 8);
     g.idone_off = o; o = al(o + g.kmap.size() * 4);
+    if (!g.init_items.empty()) g.isync_off = o, o = al(o + g.kmap.size() * kInitSyncBytes);
   }
   P.o_recs = o; o = al(o + (size_t)n * sizeof(ens_record));
   P.o_pos = o; o = al(o + (size_t)n * 8);
@@ -704,6 +714,7 @@ static int enqueue(ens_run *r) {
       k.init_scr = r->ws + g.init_scr_off;
       k.init_scr_bytes = g.init_scr_bytes;
       k.init_smem_off = xs_init_smem_off();
+      k.init_sync = g.init_items.empty() ? nullptr : r->ws + g.isync_off;
     }
     cudaStream_t st = r->stream;
     if (P.concurrent && gi > 0) {  // fork: group gi on an aux stream after ev0

@@ -53,10 +53,96 @@ constexpr uint32_t kXs2Sh = (sizeof(Shared) + 15) / 16 * 16;
 constexpr uint32_t kXs2Desc = kXs2Sh;
 constexpr uint32_t kXs2Thr = kXs2Desc + (sizeof(XsDesc) + 15) / 16 * 16;
 constexpr uint32_t kXs2Nn = kXs2Thr + 12 * 8;
+// hash grids: material rows padded by kXs2RowPad copies of their first
+// nuclide, so the lookup's look-ahead loads need no bounds tests
+constexpr int kXs2RowPad = 4;
 constexpr uint32_t kXs2Concs = kXs2Nn + 16 * 4;
-constexpr uint32_t kXs2Mats = kXs2Concs + 12 * 321 * 8;
-constexpr uint32_t kXs2Misc = kXs2Mats + (12 * 321 * 2 + 15) / 16 * 16;  // u32: item, last, am[5], pos(2)
+constexpr uint32_t kXs2Mats = kXs2Concs + 12 * (321 + kXs2RowPad) * 8;
+constexpr uint32_t kXs2Misc = kXs2Mats + (12 * (321 + kXs2RowPad) * 2 + 15) / 16 * 16;  // u32: item, last, am[5], pos(2)
 constexpr uint32_t kXs2Smem = kXs2Misc + 16 * 4;
+
+// Phase 2's hash-grid lookup: XS-7..XS-9 for one lookup, bit-identical to
+// XsApp::macro_lookup<XS_HASH> (the same bracket guess, verification, walk /
+// upstream fallback and accumulate(), nuclides summed in list order), one
+// nuclide per step: entry j+2 loaded and entry j+4 prefetched into L1,
+// nuclide j+1's guess and pair address computed and its pair prefetched,
+// nuclide j's pair gathered, verified and accumulated.  The material row
+// mrow / crow has kXs2RowPad padding entries (valid nuclides), so the
+// look-ahead needs no bounds tests; entry and record indices are 32-bit
+// sums (n_iso * (bins + 1) and n_iso * n_gp * 6 stay below 2^32).  The
+// tables were written by an earlier kernel: read-only loads (ldro).
+__device__ __forceinline__ void xs2_hash_lookup(const uint16_t *mrow, const double *crow, int nm, const double *recs,
+                                                const XsHashEnt *ig, int bins, int n_gp, double pe, int idx,
+                                                double *m) {
+  const uint32_t hs32 = (uint32_t)bins + 1u;
+  auto ent = [&](int j) { return reinterpret_cast<const uint4 *>(ig + ((uint32_t)idx + (uint32_t)mrow[j] * hs32)); };
+  auto base = [&](int j) { return (uint32_t)mrow[j] * (uint32_t)n_gp; };  // the nuclide's first record
+  auto pair_at = [&](uint32_t rb, int lo) {
+    return reinterpret_cast<const double2 *>(recs + (rb + (uint32_t)lo) * 6u);
+  };
+  const int pq = (int)((pe * (double)bins - (double)idx) * 65536.0);
+  const uint32_t pq15 = (uint32_t)(pq < 0 ? 0 : (pq >> 1 > 32767 ? 32767 : pq >> 1));
+  const uint32_t P = (pq15 | (pq15 << 16) | 0x80008000u) - 0x00010001u;
+  auto guess = [&](const uint4 &h) {  // #{k: pq15 > q_k} over the six 15-bit quanta (XsApp::macro_lookup)
+    const uint32_t mk = 0x80008000u;
+    const uint32_t x = ((P - h.y) & mk) | (((P - h.z) & mk) >> 1) | (((P - h.w) & mk) >> 2);
+    const int lo = (int)(h.x & 0xffffu) + __popc(x);
+    const int uh = (int)(h.x >> 16);
+    return lo < uh - 1 ? lo : uh - 1;
+  };
+  double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
+  uint4 h0 = ldro(ent(0)), h1 = ldro(ent(1));
+  prefetch_l1(ent(2));
+  prefetch_l1(ent(3));
+  uint32_t rb0 = base(0);
+  int lo0 = guess(h0);
+  const double2 *q0 = pair_at(rb0, lo0);
+  for (int j = 0; j < nm; j++) {
+    const uint4 h2 = ldro(ent(j + 2));
+    prefetch_l1(ent(j + 4));
+    const int lo1 = guess(h1);
+    const uint32_t rb1 = base(j + 1);
+    const double2 *q1 = pair_at(rb1, lo1);
+    prefetch_l1(q1);
+    prefetch_l1(reinterpret_cast<const double *>(q1) + 11);
+    double2 a0 = ldro(q0 + 0), a1 = ldro(q0 + 1), a2 = ldro(q0 + 2);
+    double2 b0 = ldro(q0 + 3), b1 = ldro(q0 + 4), b2 = ldro(q0 + 5);
+    {  // verify the guessed pair; walk / upstream search otherwise (macro_lookup's gather_fix)
+      const double *E = recs + rb0 * 6u;  // the nuclide's records
+      const int u_low = (int)(h0.x & 0xffffu), uh = (int)(h0.x >> 16);
+      int lo = lo0;
+      while (pe >= b0.x && a0.x < pe && lo + 2 <= uh) {
+        lo++;
+        const double2 *w2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
+        a0 = b0; a1 = b1; a2 = b2;
+        b0 = ldro(w2 + 3); b1 = ldro(w2 + 4); b2 = ldro(w2 + 5);
+      }
+      if (!(a0.x < pe && pe < b0.x && lo + 1 <= uh)) {
+        const double e_low = ldro(E + 6 * (size_t)u_low);
+        const double e_high = ldro(E + 6 * (size_t)uh);
+        int lower;
+        if (pe <= e_low) lower = 0;
+        else if (pe >= e_high) lower = n_gp - 1;
+        else lower = gs_recs(E, pe, u_low, uh);
+        const int l2 = lower == n_gp - 1 ? lower - 1 : lower;
+        const double2 *w2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)l2);
+        a0 = ldro(w2 + 0); a1 = ldro(w2 + 1); a2 = ldro(w2 + 2);
+        b0 = ldro(w2 + 3); b1 = ldro(w2 + 4); b2 = ldro(w2 + 5);
+      }
+    }
+    XsApp::accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
+    h0 = h1;
+    h1 = h2;
+    q0 = q1;
+    lo0 = lo1;
+    rb0 = rb1;
+  }
+  m[0] = m0;
+  m[1] = m1;
+  m[2] = m2;
+  m[3] = m3;
+  m[4] = m4;
+}
 
 template <int GRID>
 __device__ __forceinline__ void xs2_item(const XsDesc &d, const XsParams &p, long long s0, long long s1,
@@ -82,11 +168,13 @@ __device__ __forceinline__ void xs2_item(const XsDesc &d, const XsParams &p, lon
       idx = bb > p.bins - 1 ? p.bins - 1 : (int)bb;  // reading Q14
     }
     double mv[5];
-#ifndef ENS_XS2_OLD_HASH
-    if (GRID == XS_HASH) XsApp::macro_lookup_hash1(p, recs, ig, nn, concs, mats, pe, mat, idx, mv);
-    else
-#endif
+    if (GRID == XS_HASH) {
+      const int rw = xs_max_nucs(p.n_iso) + kXs2RowPad;
+      xs2_hash_lookup(mats + mat * rw, concs + mat * rw, nn[mat], recs, reinterpret_cast<const XsHashEnt *>(ig),
+                      p.bins, p.n_gp, pe, idx, mv);
+    } else {
       XsApp::macro_lookup<GRID>(p, recs, ig, nn, concs, mats, pe, mat, idx, mv);
+    }
     const double m0 = mv[0], m1 = mv[1], m2 = mv[2], m3 = mv[3], m4 = mv[4];
     double mxv = -1.0;  // XS-10
     int a = 0;
@@ -207,9 +295,24 @@ __global__ void __launch_bounds__(kXs2T, Xs2Minb<GRID>::v) xs_items_kernel(const
     __syncthreads();
     const int n_iso = d->n_iso, mx = xs_max_nucs(n_iso);
     if (n_iso != cached) {  // XS-2 tables (constant per n_iso: CONC_SEED is fixed)
-      hm_tables(n_iso, mx, thr, nn, concs, mats);
-      __syncthreads();
-      hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
+      if (GRID == XS_HASH) {  // rows of mx + kXs2RowPad, the padding = the row's first nuclide
+        const int rw = mx + kXs2RowPad;
+        if (tid < 12) {
+          nn[tid] = hm_num_nucs(n_iso, tid);
+          thr[tid] = hm_threshold(tid);
+        }
+        for (int x = tid; x < 12 * rw; x += kXs2T) {
+          const int m = x / rw, jj = x % rw, nm = hm_num_nucs(n_iso, m);
+          const int jn = jj < nm ? jj : 0;
+          mats[x] = (uint16_t)hm_nuc(m, jn);
+          uint64_t s = lcg_pow((uint64_t)hm_draw(n_iso, m, jn))(1070ULL * 1070ULL);  // hm_concs' draw
+          concs[x] = lcg_double(s);
+        }
+      } else {
+        hm_tables(n_iso, mx, thr, nn, concs, mats);
+        __syncthreads();
+        hm_concs(n_iso, mx, concs, 1070ULL * 1070ULL);
+      }
       cached = n_iso;
       __syncthreads();
     }
@@ -255,14 +358,46 @@ constexpr uint32_t kXsInitArgv = kXs2Sh;                                  // cha
 constexpr uint32_t kXsInitMisc = kXsInitArgv + (ENS_MAX_ARGC + 2) * 8;    // u32 item
 constexpr uint32_t kXsInitApp = kXsInitMisc + 64;                          // the app's shared memory
 
-// Items 2j' (sort items, one per instance, first in the queue: the longest)
-// and (instance, nuclide) table items.  A sort item samples and sorts the
-// instance's lookups (XsApp::lookup_sort on this CTA alone) and writes its
-// descriptor; a nuclide item builds one nuclide's sorted records and hash /
-// nuclide grid column.  Two CTAs of 256 threads per SM (compact shared
-// memory: no material tables), so one CTA's barrier-separated phases overlap
-// the other's.
-constexpr uint32_t kXsSortItem = 0xffffffffu;
+// Per (instance, item kind): a zero item clears the instance's lookup
+// histogram; count items (kXsSortChunk lookups each) add into it, the CTA
+// finishing the last count item scans it and writes the descriptor; scatter
+// items then move the lookups to their buckets (XsApp::lk_pass, lk_scan:
+// lookup_sort cut into items); a nuclide item builds one nuclide's sorted
+// records and hash / nuclide grid column.  The host orders the queue zero
+// items, count items, a first share of the nuclide items, scatter items, the
+// rest: an item that waits (count on zero, scatter on the scan) only waits
+// for items pulled before it, by running CTAs (no deadlock), and in practice
+// finds them done.  Two CTAs of 256 threads per SM (compact shared memory:
+// no material tables), so one CTA's barrier-separated phases overlap the
+// other's.
+struct XsInitSync {            // per instance, zeroed before the launch
+  uint32_t zdone;              // histogram zeroed
+  uint32_t cdone;              // count items finished
+  uint32_t sdone;              // histogram scanned, descriptor written
+  uint32_t pstate;             // parsed command line: 0 none, 1 being written, 2 ready
+  uint32_t pad[4];
+  XsParams p;                  // the instance's parsed command line (pstate == 2)
+};
+static_assert(sizeof(XsInitSync) <= kInitSyncBytes, "XsInitSync");
+
+__device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t *f) {
+  uint32_t v;
+  asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
+  return v;
+}
+// the whole CTA waits until *f != 0 (thread 0 acquires, the barrier orders the rest)
+__device__ __forceinline__ void cta_wait_flag(const uint32_t *f) {
+  if (threadIdx.x == 0)
+    while (!ld_acquire_u32(f)) __nanosleep(256);
+  __syncthreads();
+}
+// after a __syncthreads(): publish the CTA's global writes and set *f = v
+__device__ __forceinline__ void cta_set_flag(uint32_t *f, uint32_t v) {
+  if (threadIdx.x == 0) {
+    __threadfence();
+    asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(f), "r"(v) : "memory");
+  }
+}
 
 __global__ void __launch_bounds__(256, 2) xs_init_items_kernel(const KParams p) {
   const int tid = threadIdx.x, T = blockDim.x;
@@ -271,11 +406,15 @@ __global__ void __launch_bounds__(256, 2) xs_init_items_kernel(const KParams p) 
   c.smem_off = kXsInitApp;
   c.csize = 1;
   c.flags = p.flags;
+  c.phases = p.phases;  // tracing (ENS_F_PHASES): 1..9 init_nuc_t's phases; sort items: 11 zero, 12 count,
+                        // 13 scan, 14 scatter, 15 waiting
   char **argv = reinterpret_cast<char **>(ens_dsmem + kXsInitArgv);
   uint32_t *misc = reinterpret_cast<uint32_t *>(ens_dsmem + kXsInitMisc);
   char *scr = p.init_scr + (size_t)blockIdx.x * p.init_scr_bytes;
-  bool jt_ok = false;  // the LCG jump tables (seed- and layout-independent: S.jmp is fixed)
-  uint32_t cached_j = 0xffffffffu;  // the instance whose command line xp holds (items are instance-major)
+  bool jt_ok = false;   // the LCG jump tables (seed- and layout-independent: S.jmp is fixed)
+  bool thr_ok = false;  // pick_mat thresholds (constant)
+  const Affine JT = lcg_pow(2ULL * (uint64_t)T);  // T lookups' draws
+  uint32_t cached_j = 0xffffffffu;  // the instance whose command line xp holds
   XsParams xp;
   for (;;) {
     if (tid == 0) misc[0] = atomicAdd(p.counter3, 1u);
@@ -283,32 +422,77 @@ __global__ void __launch_bounds__(256, 2) xs_init_items_kernel(const KParams p) 
     const uint32_t it = misc[0];
     if (it >= p.n_init_items) break;
     const uint32_t j = p.init_items[2 * it], i = p.init_items[2 * it + 1];
+    phase_mark(c, -1);
     const uint32_t k = p.kmap[j], line = p.line_of_k[k];
-    if (j != cached_j) {
-      const uint32_t t0 = p.line_tok[line];
-      const int argc = (int)(p.line_tok[line + 1] - t0);
-      for (int a = tid; a < argc; a += T) argv[a] = const_cast<char *>(p.blob) + p.tok_off[t0 + a];
-      if (tid == 0) argv[argc] = nullptr;
+    XsInitSync *sy = reinterpret_cast<XsInitSync *>(p.init_sync + (size_t)j * kInitSyncBytes);
+    if (j != cached_j) {  // the command line: parsed once per instance, by whichever CTA comes first
+      if (tid == 0) misc[1] = ld_acquire_u32(&sy->pstate);
       __syncthreads();
-      xp = XsParams();
-      xs_parse(argc, argv, xp);  // a valid line: the host made items only for those
+      if (misc[1] == 2u) {
+        xp = sy->p;
+      } else {
+        const uint32_t t0 = p.line_tok[line];
+        const int argc = (int)(p.line_tok[line + 1] - t0);
+        for (int a = tid; a < argc; a += T) argv[a] = const_cast<char *>(p.blob) + p.tok_off[t0 + a];
+        if (tid == 0) argv[argc] = nullptr;
+        __syncthreads();
+        xp = XsParams();
+        xs_parse(argc, argv, xp);  // a valid line: the host made items only for those
+        if (tid == 0 && atomicCAS(&sy->pstate, 0u, 1u) == 0u) {
+          sy->p = xp;
+          __threadfence();
+          asm volatile("st.release.gpu.global.u32 [%0], %1;" ::"l"(&sy->pstate), "r"(2u) : "memory");
+        }
+      }
       cached_j = j;
     }
+    phase_mark(c, 0);
     const XsSmem S = xs_init_smem(xp);
     const XsLayout L = xs_layout(xp, (int)p.team_ctas);  // the instance's arena, as phase 1 lays it out
     c.arena = p.arena_base + (size_t)j * p.arena_bytes;
-    if (i == kXsSortItem) {  // XS-6 for every lookup, sorted by (material, energy); the descriptor
+    if (i >= kXsScatterItem) {  // the lookup sort's items
       double *thr = reinterpret_cast<double *>(ens_smem(c) + S.thr);
-      uint32_t *mcnt = reinterpret_cast<uint32_t *>(ens_smem(c) + S.mcnt);
-      if (tid < 12) thr[tid] = hm_threshold(tid);
-      __syncthreads();
-      XsApp::lookup_sort(c, xp, L, thr, mcnt, 0, xp.lookups);
-      if (tid == 0) {
-        c.desc = p.xs_desc + (size_t)j * kDescBytes;
-        c.k = k;
-        c.id = line;
-        c.t_start = 0;
-        XsApp::write_desc(c, xp, L, mcnt);
+      if (!thr_ok) {
+        if (tid < 12) thr[tid] = hm_threshold(tid);
+        thr_ok = true;
+        __syncthreads();
+      }
+      if (i == kXsZeroItem) {
+        XsApp::lk_zero(c, xp, L);
+        __syncthreads();
+        cta_set_flag(&sy->zdone, 1u);
+        phase_mark(c, 11);
+      } else {
+        const bool scatter = !(i & kXsCountItem);
+        const long long ch = (long long)(i & 0x3fffffffu), nc = xs_lk_chunk(xp);
+        const long long l0 = ch * kXsSortChunk, l1 = l0 + kXsSortChunk < nc ? l0 + kXsSortChunk : nc;
+        cta_wait_flag(scatter ? &sy->sdone : &sy->zdone);
+        phase_mark(c, 15);
+        XsApp::lk_pass(xp, c.arena, L, thr, l0, l1, scatter, JT);
+        __syncthreads();
+        phase_mark(c, scatter ? 14 : 12);
+        if (!scatter) {
+          if (tid == 0) {
+            __threadfence();
+            misc[1] = atomicAdd(&sy->cdone, 1u) == (uint32_t)xs_sort_items(xp) - 1u ? 1u : 0u;
+            __threadfence();
+          }
+          __syncthreads();
+          if (misc[1]) {  // the last count item: (B) and the descriptor
+            uint32_t *mcnt = reinterpret_cast<uint32_t *>(ens_smem(c) + S.mcnt);
+            XsApp::lk_scan(c, xp, L, mcnt);
+            if (tid == 0) {
+              c.desc = p.xs_desc + (size_t)j * kDescBytes;
+              c.k = k;
+              c.id = line;
+              c.t_start = 0;
+              XsApp::write_desc(c, xp, L, mcnt);
+            }
+            __syncthreads();
+            cta_set_flag(&sy->sdone, 1u);
+            phase_mark(c, 13);
+          }
+        }
       }
     } else {
       if (!jt_ok) {

@@ -49,6 +49,7 @@ struct KParams {
   char *init_scr;             // [grid][init_scr_bytes] per-CTA scratch
   uint64_t init_scr_bytes;
   uint32_t init_smem_off;     // dynamic smem offset of the app's shared memory
+  char *init_sync;            // [n] x kInitSyncBytes per-instance phase-1b state (zeroed)
   // ENS_F_CLC: one CTA per instance, cluster launch control for the rest,
   // arena slots from a bitmap pool of n_slots
   uint32_t clc;
@@ -75,7 +76,12 @@ int xs_items_threads();
 cudaError_t launch_xs_init_items(int ctas, int threads, size_t smem, const KParams &p, cudaStream_t st);
 cudaError_t xs_init_items_occupancy(int threads, size_t smem, int *ctas);
 uint32_t xs_init_smem_off();
-uint64_t app_init_scratch(uint32_t app, int argc, const char *const *argv, int *n_items, uint32_t *smem);
+uint64_t app_init_scratch(uint32_t app, int argc, const char *const *argv, int *n_items, int *n_sort, uint32_t *smem);
+constexpr uint32_t kInitSyncBytes = 128;  // XsInitSync (kernels_items.cu)
+// phase-1b item codes (the second word of an init item; nuclide items are < 2^16)
+constexpr uint32_t kXsZeroItem = 0xffffffffu;     // zero the lookup histogram
+constexpr uint32_t kXsCountItem = 0x80000000u;    // | chunk: count lookups
+constexpr uint32_t kXsScatterItem = 0x40000000u;  // | chunk: scatter lookups
 constexpr int kXsInitThreads = 256;  // init-item kernel block (launch bounds 256 x 2 CTAs/SM)
 
 }  // namespace ens
