@@ -61,24 +61,52 @@ constexpr uint32_t kXs2Mats = kXs2Concs + 12 * (321 + kXs2RowPad) * 8;
 constexpr uint32_t kXs2Misc = kXs2Mats + (12 * (321 + kXs2RowPad) * 2 + 15) / 16 * 16;  // u32: item, last, am[5], pos(2)
 constexpr uint32_t kXs2Smem = kXs2Misc + 16 * 4;
 
+// 32-bit shared-window loads (the material row's address is computed once
+// per lookup; each step's loads then take immediate offsets)
+__device__ __forceinline__ uint32_t lds_u16(uint32_t a) {
+  unsigned short v;
+  asm("ld.shared.u16 %0, [%1];" : "=h"(v) : "r"(a));
+  return v;
+}
+__device__ __forceinline__ double lds_f64(uint32_t a) {
+  double v;
+  asm("ld.shared.f64 %0, [%1];" : "=d"(v) : "r"(a));
+  return v;
+}
+
 // Phase 2's hash-grid lookup: XS-7..XS-9 for one lookup, bit-identical to
 // XsApp::macro_lookup<XS_HASH> (the same bracket guess, verification, walk /
 // upstream fallback and accumulate(), nuclides summed in list order), one
 // nuclide per step: entry j+2 loaded and entry j+4 prefetched into L1,
 // nuclide j+1's guess and pair address computed and its pair prefetched,
 // nuclide j's pair gathered, verified and accumulated.  The material row
-// mrow / crow has kXs2RowPad padding entries (valid nuclides), so the
-// look-ahead needs no bounds tests; entry and record indices are 32-bit
-// sums (n_iso * (bins + 1) and n_iso * n_gp * 6 stay below 2^32).  The
-// tables were written by an earlier kernel: read-only loads (ldro).
-__device__ __forceinline__ void xs2_hash_lookup(const uint16_t *mrow, const double *crow, int nm, const double *recs,
+// (mrow_s / crow_s: shared-window addresses) has kXs2RowPad padding entries
+// (valid nuclides), so the look-ahead needs no bounds tests; entry and
+// record indices are 32-bit sums (n_iso * (bins + 1) and n_iso * n_gp * 6
+// stay below 2^32).  A nuclide's entry is consumed when its guess is made
+// (its u_low / u_high travel with the pair).  The tables were written by an
+// earlier kernel: read-only loads (ldro).
+// L1 prefetches (measured on C2's phase 2: all on 19.5 ms; no entry
+// prefetch 21.9, one pair line 20.5, no pair prefetch 22.1; pairs prefetched
+// two steps ahead instead of one 19.9)
+#ifndef ENS_XS2_PF_ENT
+#define ENS_XS2_PF_ENT 1
+#endif
+#ifndef ENS_XS2_PF_PAIR
+#define ENS_XS2_PF_PAIR 2
+#endif
+struct Xs2Pair {
+  const double2 *q;  // the guessed pair
+  int lo;            // its lower index
+  uint32_t rb;       // the nuclide's first record
+  uint32_t hx;       // its entry's u_low | u_high << 16
+};
+__device__ __forceinline__ void xs2_hash_lookup(uint32_t mrow_s, uint32_t crow_s, int nm, const double *recs,
                                                 const XsHashEnt *ig, int bins, int n_gp, double pe, int idx,
                                                 double *m) {
   const uint32_t hs32 = (uint32_t)bins + 1u;
-  auto ent = [&](int j) { return reinterpret_cast<const uint4 *>(ig + ((uint32_t)idx + (uint32_t)mrow[j] * hs32)); };
-  auto base = [&](int j) { return (uint32_t)mrow[j] * (uint32_t)n_gp; };  // the nuclide's first record
-  auto pair_at = [&](uint32_t rb, int lo) {
-    return reinterpret_cast<const double2 *>(recs + (rb + (uint32_t)lo) * 6u);
+  auto ent = [&](int j) {
+    return reinterpret_cast<const uint4 *>(ig + ((uint32_t)idx + lds_u16(mrow_s + 2u * (uint32_t)j) * hs32));
   };
   const int pq = (int)((pe * (double)bins - (double)idx) * 65536.0);
   const uint32_t pq15 = (uint32_t)(pq < 0 ? 0 : (pq >> 1 > 32767 ? 32767 : pq >> 1));
@@ -90,27 +118,27 @@ __device__ __forceinline__ void xs2_hash_lookup(const uint16_t *mrow, const doub
     const int uh = (int)(h.x >> 16);
     return lo < uh - 1 ? lo : uh - 1;
   };
+  auto pair_of = [&](int j, const uint4 &h, Xs2Pair &o) {
+    o.rb = lds_u16(mrow_s + 2u * (uint32_t)j) * (uint32_t)n_gp;
+    o.lo = guess(h);
+    o.hx = h.x;
+    o.q = reinterpret_cast<const double2 *>(recs + (o.rb + (uint32_t)o.lo) * 6u);
+  };
   double m0 = 0.0, m1 = 0.0, m2 = 0.0, m3 = 0.0, m4 = 0.0;
-  uint4 h0 = ldro(ent(0)), h1 = ldro(ent(1));
-  prefetch_l1(ent(2));
-  prefetch_l1(ent(3));
-  uint32_t rb0 = base(0);
-  int lo0 = guess(h0);
-  const double2 *q0 = pair_at(rb0, lo0);
-  for (int j = 0; j < nm; j++) {
-    const uint4 h2 = ldro(ent(j + 2));
-    prefetch_l1(ent(j + 4));
-    const int lo1 = guess(h1);
-    const uint32_t rb1 = base(j + 1);
-    const double2 *q1 = pair_at(rb1, lo1);
-    prefetch_l1(q1);
-    prefetch_l1(reinterpret_cast<const double *>(q1) + 11);
-    double2 a0 = ldro(q0 + 0), a1 = ldro(q0 + 1), a2 = ldro(q0 + 2);
-    double2 b0 = ldro(q0 + 3), b1 = ldro(q0 + 4), b2 = ldro(q0 + 5);
-    {  // verify the guessed pair; walk / upstream search otherwise (macro_lookup's gather_fix)
-      const double *E = recs + rb0 * 6u;  // the nuclide's records
-      const int u_low = (int)(h0.x & 0xffffu), uh = (int)(h0.x >> 16);
-      int lo = lo0;
+  // nuclide j: gather its guessed pair pA, verify it (walk / search
+  // otherwise) and accumulate
+  auto gather_acc = [&](int j, const Xs2Pair &pA) {
+    double2 a0 = ldro(pA.q + 0), a1 = ldro(pA.q + 1), a2 = ldro(pA.q + 2);
+    double2 b0 = ldro(pA.q + 3), b1 = ldro(pA.q + 4), b2 = ldro(pA.q + 5);
+    const int uh = (int)(pA.hx >> 16);
+    // the guessed pair is upstream's bracket iff E[lo] < pe < E[lo+1] and
+    // lo+1 <= u_high; else walk / search (macro_lookup's gather_fix; the
+    // walk's own test fails at once on a valid bracket, so skipping both is
+    // the same logic)
+    if (!(a0.x < pe && pe < b0.x && pA.lo + 1 <= uh)) {
+      const double *E = recs + pA.rb * 6u;  // the nuclide's records
+      const int u_low = (int)(pA.hx & 0xffffu);
+      int lo = pA.lo;
       while (pe >= b0.x && a0.x < pe && lo + 2 <= uh) {
         lo++;
         const double2 *w2 = reinterpret_cast<const double2 *>(E + 6 * (size_t)lo);
@@ -130,12 +158,27 @@ __device__ __forceinline__ void xs2_hash_lookup(const uint16_t *mrow, const doub
         b0 = ldro(w2 + 3); b1 = ldro(w2 + 4); b2 = ldro(w2 + 5);
       }
     }
-    XsApp::accumulate(pe, crow[j], a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
-    h0 = h1;
-    h1 = h2;
-    q0 = q1;
-    lo0 = lo1;
-    rb0 = rb1;
+    XsApp::accumulate(pe, lds_f64(crow_s + 8u * (uint32_t)j), a0, a1, a2, b0, b1, b2, m0, m1, m2, m3, m4);
+  };
+  // step j: hB = entry j+1, hC <- entry j+2; pA = nuclide j's pair, pB <- nuclide j+1's
+  auto step = [&](int j, const uint4 &hB, uint4 &hC, const Xs2Pair &pA, Xs2Pair &pB) {
+    hC = ldro(ent(j + 2));
+    if (ENS_XS2_PF_ENT) prefetch_l1(ent(j + 4));
+    pair_of(j + 1, hB, pB);
+    if (ENS_XS2_PF_PAIR >= 1) prefetch_l1(pB.q);
+    if (ENS_XS2_PF_PAIR >= 2) prefetch_l1(reinterpret_cast<const double *>(pB.q) + 11);
+    gather_acc(j, pA);
+  };
+  uint4 h0 = ldro(ent(0)), h1 = ldro(ent(1));
+  prefetch_l1(ent(2));
+  prefetch_l1(ent(3));
+  Xs2Pair p0, p1;
+  pair_of(0, h0, p0);  // entry 0 consumed: h0 is free
+  int j = 0;
+  for (; j < nm; j++) {  // (unrolled by two without copies: spills at 80 registers, 21.8 vs 19.5 ms)
+    step(j, h1, h0, p0, p1);
+    h1 = h0;
+    p0 = p1;
   }
   m[0] = m0;
   m[1] = m1;
@@ -170,8 +213,9 @@ __device__ __forceinline__ void xs2_item(const XsDesc &d, const XsParams &p, lon
     double mv[5];
     if (GRID == XS_HASH) {
       const int rw = xs_max_nucs(p.n_iso) + kXs2RowPad;
-      xs2_hash_lookup(mats + mat * rw, concs + mat * rw, nn[mat], recs, reinterpret_cast<const XsHashEnt *>(ig),
-                      p.bins, p.n_gp, pe, idx, mv);
+      xs2_hash_lookup((uint32_t)__cvta_generic_to_shared(mats + mat * rw),
+                      (uint32_t)__cvta_generic_to_shared(concs + mat * rw), nn[mat], recs,
+                      reinterpret_cast<const XsHashEnt *>(ig), p.bins, p.n_gp, pe, idx, mv);
     } else {
       XsApp::macro_lookup<GRID>(p, recs, ig, nn, concs, mats, pe, mat, idx, mv);
     }
