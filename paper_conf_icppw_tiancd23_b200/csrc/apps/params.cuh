@@ -254,6 +254,8 @@ struct XsLayout {
   uint64_t nscr;      // hash / nuclide, n_gp > kXsSmemGp: [cs] x xs_nscr_bytes per-nuclide sort scratch
   uint64_t lk_pe;     // event mode: [chunk] lookup energies sorted by (material, energy)
   uint64_t lk_hist;   // event mode: [(12 << kb) + 1] u32 (material, energy) bucket counts -> cursors
+                      // (split phases, phase 1b: [12 << cb][chunks] coarse counts -> offsets)
+  uint64_t lk_tmp;    // split phases, phase 1b: [chunk] energies in coarse-bucket order
   uint64_t total;
 };
 // Event-mode lookups are sampled, then bucket-sorted by (material, energy)
@@ -288,6 +290,9 @@ struct XsHashEnt {
 };
 // cs = CTAs in the team: hash / nuclide grids give each CTA its own
 // per-nuclide scratch
+ENS_HD int xs_lk_cbits(int kb);
+ENS_HD int xs_sort_items(const XsParams &p);
+ENS_HD bool xs_split_ok(const XsParams &p);
 ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
   XsLayout L{};
   const uint64_t n_u = (uint64_t)p.n_iso * p.n_gp;
@@ -312,8 +317,12 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
   if (p.grid != XS_UNIONIZED) { L.nscr = o; o = align_up(o + (uint64_t)cs * xs_nscr_bytes(p), 256); }
   if (!p.history) {
     const long long n_c = xs_lk_chunk(p);
+    const int kb = xs_lk_bits(n_c);
+    const uint64_t coarse = (12ULL << xs_lk_cbits(kb)) * (uint64_t)xs_sort_items(p) + 1;
     L.lk_pe = o; o = align_up(o + (uint64_t)n_c * 8, 256);
-    L.lk_hist = o; o = align_up(o + ((12ULL << xs_lk_bits(n_c)) + 1) * 4, 256);
+    L.lk_hist = o; o = align_up(o + (((12ULL << kb) + 1) > coarse ? ((12ULL << kb) + 1) : coarse) * 4, 256);
+    L.lk_tmp = o;
+    if (xs_split_ok(p) && p.grid != XS_UNIONIZED) o = align_up(o + (uint64_t)n_c * 8, 256);
   }
   L.total = o;
   return L;
@@ -338,6 +347,19 @@ constexpr long long kXsItemLookups = ENS_XS_ITEM;
 #endif
 constexpr long long kXsSortChunk = ENS_XS_SORT_ITEM;
 ENS_HD int xs_sort_items(const XsParams &p) { return (int)((xs_lk_chunk(p) + kXsSortChunk - 1) / kXsSortChunk); }
+// ... the sort's (material, energy) bucket key (kb energy bits) splits into a
+// coarse bucket (material, top cb bits: counted and scattered in shared
+// memory per chunk) and a fine sub-bucket (the other kb - cb bits: sorted per
+// coarse bucket by a warp); fine items take kXsFineGroup coarse buckets
+ENS_HD int xs_lk_cbits(int kb) { return kb < 8 ? kb : 8; }
+constexpr int kXsFineGroup = 64;
+ENS_HD int xs_sort_fine_items(const XsParams &p) {
+  const int kb = xs_lk_bits(xs_lk_chunk(p));
+  return ((12 << xs_lk_cbits(kb)) + kXsFineGroup - 1) / kXsFineGroup;
+}
+// shared memory of the sort items: the coarse counters (12 << 8 u32) or 8
+// warps' fine counters (1 << (18 - 8) u32 each)
+constexpr uint32_t kXsLkSortSmem = 8u * 1024u * 4u;
 ENS_HD bool xs_split_ok(const XsParams &p) { return !p.history && p.lookups > 0 && p.lookups <= kXsLkChunk; }
 ENS_HD long long xs_items(const XsParams &p) {
   return xs_split_ok(p) ? (p.lookups + kXsItemLookups - 1) / kXsItemLookups : 0;
@@ -367,17 +389,27 @@ constexpr int kXsStep = ENS_XS_STEP;
 // dynamic shared memory layout: material tables + the sort's bucket counters
 constexpr int kXsMaxT = 512;  // XsApp::kMaxT
 struct XsSmem {
-  uint32_t thr, nn, mats, concs, mcnt, jmp, nbkt, ubkt, nkey, njdx, total;
+  uint32_t thr, nn, mats, concs, mcnt, jmp, nbkt, ubkt, nkey, njdx, njdx2, total;
 };
+// per-nuclide sort buckets when the sort runs in shared memory (~4 keys each:
+// the rank pass, init_nuc_t, wants few buckets and two index arrays)
+#ifndef ENS_XS_NBN_SMEM_DIV
+#define ENS_XS_NBN_SMEM_DIV 4
+#endif
+ENS_HD int xs_nbn_smem(int n_gp) {
+  return pow2_ceil(n_gp) / ENS_XS_NBN_SMEM_DIV > 0 ? pow2_ceil(n_gp) / ENS_XS_NBN_SMEM_DIV : 1;
+}
 // hash / nuclide grids, per-nuclide sort in shared memory: [nkey] u32 sort
 // keys (after the sort: the hash column's per-record codes, init_nuc_t) |
-// [nbkt] u32 bucket counters | [njdx] u16 record indices; the hash column
-// (bins+1 u32) reuses [nbkt, end) once the records are written, the region
-// grown by up to 16 KB so that it fits (else it goes to arena scratch)
+// [nbkt] u32 bucket counters | [njdx] u16 record indices in bucket order |
+// [njdx2] u16 record indices sorted; the hash column (bins+1 u32) reuses
+// [nbkt, end) once the records are written, the region grown by up to 16 KB
+// so that it fits (else it goes to arena scratch)
 ENS_HD uint32_t xs_nuc_smem_block(const XsParams &p, uint32_t o, XsSmem &S) {
   S.nkey = o; o += (uint32_t)align_up((uint64_t)p.n_gp * 4, 16);
-  S.nbkt = o; o += (uint32_t)align_up((uint64_t)xs_nbn(p.n_gp) * 4, 16);
+  S.nbkt = o; o += (uint32_t)align_up((uint64_t)xs_nbn_smem(p.n_gp) * 4, 16);
   S.njdx = o; o += (uint32_t)align_up((uint64_t)p.n_gp * 2, 16);
+  S.njdx2 = o; o += (uint32_t)align_up((uint64_t)p.n_gp * 2, 16);
   if (p.grid == XS_HASH) {
     const uint64_t need = align_up((uint64_t)(p.bins + 1) * 4, 16), have = o - S.nbkt;
     if (need > have && need - have <= 16384) o = S.nbkt + (uint32_t)need;
@@ -397,14 +429,14 @@ ENS_HD XsSmem xs_smem(const XsParams &p, int T) {
   S.jmp = o; o += 5 * 64 * 16;            // LCG jump tables: A^(6 d 64^l), l < 5, d < 64
   if (p.grid != XS_UNIONIZED) {  // hash / nuclide grids: one nuclide's sort (xs_nuc_smem_block)
     if (xs_nuc_smem(p)) o = xs_nuc_smem_block(p, o, S);
-    else S.nkey = S.nbkt = S.njdx = o;
+    else S.nkey = S.nbkt = S.njdx = S.njdx2 = o;
     S.ubkt = o;
   } else {
     S.nbkt = o;  // unionized: per-warp sweep rows
     o += (uint32_t)(T / 32) * 2u * (uint32_t)xs_iso_pad(p.n_iso) * 4u;
     S.ubkt = o;  // unionized, small: bucket counters, then chunk owner counts
     if (xs_smem_nb(p)) o += (uint32_t)kXsSmemBkt * 4u;
-    S.nkey = S.njdx = o;
+    S.nkey = S.njdx = S.njdx2 = o;
   }
   // unionized warp path: kXsWarpScr per warp, overlaying nbkt / ubkt
   if (xs_warp_union(p)) {
@@ -429,8 +461,9 @@ ENS_HD XsSmem xs_init_smem(const XsParams &p) {
   S.mcnt = o; o += 32 * 4;
   S.jmp = o; o += 5 * 64 * 16;
   if (p.grid != XS_UNIONIZED && xs_nuc_smem(p)) o = xs_nuc_smem_block(p, o, S);
-  else S.nkey = S.nbkt = S.njdx = o;
+  else S.nkey = S.nbkt = S.njdx = S.njdx2 = o;
   S.ubkt = o;
+  if (o < S.nkey + kXsLkSortSmem) o = S.nkey + kXsLkSortSmem;  // the lookup sort's items use [nkey, ...)
   S.total = o;
   return S;
 }

@@ -414,7 +414,7 @@ struct XsApp {
     const bool trc = tracing(c);  // tracing (ENS_F_PHASES) thread, cached
     const int tid = threadIdx.x, T = blockDim.x;
     const int n_gp = p.n_gp;
-    const int nbn = xs_nbn(n_gp);
+    const int nbn = SMK ? xs_nbn_smem(n_gp) : xs_nbn(n_gp);
     uint32_t *nb = SMK ? (uint32_t *)(ens_smem(c) + S.nbkt) : (uint32_t *)gscr;
     const Affine *jt = (const Affine *)(ens_smem(c) + S.jmp);
     double *recs = (double *)(c.arena + L.recs);
@@ -464,7 +464,50 @@ struct XsApp {
       }
       __syncthreads();
       phase_mark_if(trc, c, 3);
-      for (int b = tid; b < nbn; b += T) isort_keys(K, J, b ? (int)nb[b - 1] : 0, (int)nb[b], jt, r0, p.gseed);
+      // sort within buckets: in shared memory, a thread per key counts the
+      // keys of its bucket that sort before it — (energy, j) order: equal
+      // 32-bit keys (rare) compare the re-drawn energies, then j — and
+      // places its record index there (J2: sorted order); in arena scratch,
+      // an insertion sort per bucket in place
+      uint16_t *Js = J;
+      if (SMK) {
+        Js = (uint16_t *)(ens_smem(c) + S.njdx2);
+        for (int x = tid; x < n_gp; x += T) {
+          const uint32_t vk = K[x];
+          const uint16_t vj = J[x];
+          const int b = nkey_bkt(vk);
+          const int lo = b ? (int)nb[b - 1] : 0, hi = (int)nb[b];
+          // buckets of <= 8 keys (~4 on average): eight independent predicated
+          // loads (the key at x counts itself as "not before"); equal keys or
+          // a larger bucket take the exact loop
+          int rank = 0;
+          bool slow = hi - lo > 8;
+#pragma unroll
+          for (int q = 0; q < 8; q++) {
+            const int y = lo + q;
+            const uint32_t yk = K[y < n_gp ? y : n_gp - 1];
+            const bool in = y < hi;
+            rank += (in && yk < vk) ? 1 : 0;
+            slow |= in && yk == vk && y != x;
+          }
+          if (slow) {
+            rank = 0;
+            for (int y = lo; y < hi; y++) {
+              const uint32_t yk = K[y];
+              if (yk < vk) {
+                rank++;
+              } else if (yk == vk && y != x) {
+                const uint16_t yj = J[y];
+                const double ey = rec_energy(jt, r0 + yj, p.gseed), ev = rec_energy(jt, r0 + vj, p.gseed);
+                rank += (ey < ev || (ey == ev && yj < vj)) ? 1 : 0;
+              }
+            }
+          }
+          Js[lo + rank] = vj;
+        }
+      } else {
+        for (int b = tid; b < nbn; b += T) isort_keys(K, J, b ? (int)nb[b - 1] : 0, (int)nb[b], jt, r0, p.gseed);
+      }
       __syncthreads();
       phase_mark_if(trc, c, 4);
       // records written in sorted order (coalesced, evict-first), their draws
@@ -490,7 +533,7 @@ struct XsApp {
       int anom = 0;
 #pragma unroll 2
       for (int k = tid; k < n_gp; k += T) {
-        uint64_t t = jump6(jt, r0 + J[k], p.gseed);
+        uint64_t t = jump6(jt, r0 + Js[k], p.gseed);
         const double e = lcg_double(t), x1 = lcg_double(t), x2 = lcg_double(t), x3 = lcg_double(t),
                      x4 = lcg_double(t), x5 = lcg_double(t);
         double2 *d = reinterpret_cast<double2 *>(rec_i + 6 * (size_t)k);
@@ -1477,32 +1520,48 @@ struct XsApp {
     team_sync(c);
   }
 
-  // ---- split phases, phase 1b: lookup_sort in items on any CTAs ----------
+  // ---- split phases, phase 1b: the lookup sort in items on any CTAs -------
   // The instance's one chunk (xs_split_ok: lookups <= kXsLkChunk) is sorted
-  // exactly as lookup_sort sorts it, its passes cut into items of
-  // kXsSortChunk lookups: (A) count items add into the arena histogram
-  // (RED), the CTA finishing the last one scans it (B, lk_scan), then (C)
-  // scatter items move each lookup's energy to its bucket.  Lookup li draws
-  // 2li+1 (energy) and 2li+2 (material: the first i >= 1 with roll < thr[i],
-  // i.e. 1 + #{i >= 1: thr[i] <= roll} (thr increasing), 0 past thr[11]).
-  // U lookups per thread are sampled before their atomics issue, so U
-  // atomics (and, scattering, U returned cursors) are in flight per thread.
-  __device__ static void lk_pass(const XsParams &p, char *arena, const XsLayout &L, const double *thr,
-                                 long long l0, long long l1, bool scatter, const Affine &JT) {
-    const int tid = threadIdx.x, T = blockDim.x;
-    uint32_t *hist = (uint32_t *)(arena + L.lk_hist);
-    double *lk_pe = (double *)(arena + L.lk_pe);
-    const int kb = xs_lk_bits(xs_lk_chunk(p));
-    const double bscale = (double)(1LL << kb);
-    const long long emax = (1LL << kb) - 1;
+  // into lookup_sort's (material, energy-bucket) order — the same buckets
+  // (kb energy bits per material); only the order within a bucket (atomic
+  // in either) may differ — in three kinds of items, all counting in shared
+  // memory: (A) count item ch samples lookups [ch*kXsSortChunk, ...) (XS-6:
+  // lookup li draws 2li+1, 2li+2) and writes its coarse histogram — coarse
+  // bucket ck = (material, top cb energy bits) — as column ch of CH[ck][NC];
+  // the CTA finishing the last count item scans CH (B: in (ck, ch) order
+  // that gives each chunk's cursor into each coarse bucket) and writes the
+  // descriptor; (C) scatter item ch re-samples its lookups and moves each
+  // energy to its coarse bucket in lk_tmp; (D) fine item g sorts coarse
+  // buckets [g*G, (g+1)*G) by the remaining kb - cb energy bits into lk_pe,
+  // a warp per coarse bucket.  pick_mat: the first i >= 1 with roll <
+  // thr[i] is 1 + #{i >= 1: thr[i] <= roll} (thr increasing), 0 past thr[11].
+  struct LkKey {
+    int kb, cb, fb, nck, nc;  // energy bits, coarse bits, fine bits, coarse buckets, chunks
+  };
+  __device__ static LkKey lk_key(const XsParams &p) {
+    LkKey k;
+    k.kb = xs_lk_bits(xs_lk_chunk(p));
+    k.cb = xs_lk_cbits(k.kb);
+    k.fb = k.kb - k.cb;
+    k.nck = 12 << k.cb;
+    k.nc = xs_sort_items(p);
+    return k;
+  }
+  // lookups [l0, l1) of the chunk: fn(energy, coarse bucket) for each
+  template <class F>
+  __device__ static __forceinline__ void lk_sample(const XsParams &p, const LkKey &K, const double *thr, long long l0,
+                                                   long long l1, const Affine &JT, F fn) {
+    const int T = blockDim.x;
+    const double bscale = (double)(1LL << K.kb);
+    const long long emax = (1LL << K.kb) - 1;
     double th[11];
 #pragma unroll
     for (int m = 0; m < 11; m++) th[m] = thr[m + 1];
-    constexpr int U = 8;
-    uint64_t s = lcg_pow(2ULL * (uint64_t)(l0 + tid))(p.seed);
-    for (long long li0 = l0 + tid; li0 < l1; li0 += (long long)U * T) {
+    constexpr int U = 4;
+    uint64_t s = lcg_pow(2ULL * (uint64_t)(l0 + threadIdx.x))(p.seed);
+    for (long long li0 = l0 + threadIdx.x; li0 < l1; li0 += (long long)U * T) {
       double pe[U];
-      uint32_t bk[U];
+      uint32_t ck[U];
 #pragma unroll
       for (int u = 0; u < U; u++) {
         uint64_t t = s;
@@ -1514,40 +1573,126 @@ struct XsApp {
         const int mat = n == 11 ? 0 : n + 1;
         long long eb = (long long)(pe[u] * bscale);
         eb = eb > emax ? emax : eb;
-        bk[u] = (uint32_t)(((long long)mat << kb) + eb);
+        ck[u] = ((uint32_t)mat << K.cb) + (uint32_t)(eb >> K.fb);
         s = JT(s);
       }
-      if (!scatter) {
 #pragma unroll
-        for (int u = 0; u < U; u++)
-          if (li0 + (long long)u * T < l1) atomicAdd(&hist[bk[u]], 1u);
-      } else {
-        uint32_t pos[U];
-#pragma unroll
-        for (int u = 0; u < U; u++)
-          if (li0 + (long long)u * T < l1) pos[u] = atomicAdd(&hist[bk[u]], 1u);
-#pragma unroll
-        for (int u = 0; u < U; u++)
-          if (li0 + (long long)u * T < l1) lk_pe[pos[u]] = pe[u];
-      }
+      for (int u = 0; u < U; u++)
+        if (li0 + (long long)u * T < l1) fn(pe[u], ck[u]);
     }
   }
-  // (B): bucket offsets and the material starts mcnt[16..28] (one CTA)
+  // (A)
+  __device__ static void lk_count(const Ctx &c, const XsParams &p, const XsLayout &L, const double *thr, int ch,
+                                  const Affine &JT, uint32_t *sc) {
+    const LkKey K = lk_key(p);
+    const long long nc = xs_lk_chunk(p), l0 = (long long)ch * kXsSortChunk;
+    const long long l1 = l0 + kXsSortChunk < nc ? l0 + kXsSortChunk : nc;
+    for (int x = threadIdx.x; x < K.nck; x += blockDim.x) sc[x] = 0u;
+    __syncthreads();
+    lk_sample(p, K, thr, l0, l1, JT, [&](double, uint32_t ck) { atomicAdd(&sc[ck], 1u); });
+    __syncthreads();
+    uint32_t *CH = (uint32_t *)(c.arena + L.lk_hist);
+    for (int x = threadIdx.x; x < K.nck; x += blockDim.x) CH[(size_t)x * K.nc + ch] = sc[x];
+  }
+  // (B): coarse-bucket cursors and the material starts mcnt[16..28] (one CTA)
   __device__ static void lk_scan(const Ctx &c, const XsParams &p, const XsLayout &L, uint32_t *mcnt) {
     const int tid = threadIdx.x;
-    uint32_t *hist = (uint32_t *)(c.arena + L.lk_hist);
-    const long long nc = xs_lk_chunk(p);
-    const int kb = xs_lk_bits(nc);
-    global_exclusive_scan(hist, (12LL << kb) + 1, ens_sh(c));
+    const LkKey K = lk_key(p);
+    uint32_t *CH = (uint32_t *)(c.arena + L.lk_hist);
+    global_exclusive_scan(CH, (long long)K.nck * K.nc, ens_sh(c));
     __syncthreads();
-    if (tid < 12) mcnt[16 + tid] = ld_(hist + ((long long)tid << kb));
-    if (tid == 12) mcnt[28] = (uint32_t)nc;
+    if (tid < 12) mcnt[16 + tid] = ld_(CH + ((size_t)tid << K.cb) * K.nc);
+    if (tid == 12) mcnt[28] = (uint32_t)xs_lk_chunk(p);
     __syncthreads();
   }
-  __device__ static void lk_zero(const Ctx &c, const XsParams &p, const XsLayout &L) {
-    uint32_t *hist = (uint32_t *)(c.arena + L.lk_hist);
-    const long long n = (12LL << xs_lk_bits(xs_lk_chunk(p))) + 1;
-    for (long long b = threadIdx.x; b < n; b += blockDim.x) hist[b] = 0u;
+  // (C)
+  __device__ static void lk_scatter(const Ctx &c, const XsParams &p, const XsLayout &L, const double *thr, int ch,
+                                    const Affine &JT, uint32_t *sc) {
+    const LkKey K = lk_key(p);
+    const long long nc = xs_lk_chunk(p), l0 = (long long)ch * kXsSortChunk;
+    const long long l1 = l0 + kXsSortChunk < nc ? l0 + kXsSortChunk : nc;
+    const uint32_t *CH = (const uint32_t *)(c.arena + L.lk_hist);
+    for (int x = threadIdx.x; x < K.nck; x += blockDim.x) sc[x] = __ldcg(CH + (size_t)x * K.nc + ch);
+    __syncthreads();
+    double *tmp = (double *)(c.arena + L.lk_tmp);
+    lk_sample(p, K, thr, l0, l1, JT, [&](double pe, uint32_t ck) { tmp[atomicAdd(&sc[ck], 1u)] = pe; });
+  }
+  // (D)
+  __device__ static void lk_fine(const Ctx &c, const XsParams &p, const XsLayout &L, int g, uint32_t *sc) {
+    const LkKey K = lk_key(p);
+    const int lane = threadIdx.x & 31, w = threadIdx.x >> 5, nw = blockDim.x >> 5;
+    const int nf = 1 << K.fb;
+    uint32_t *cnt = sc + (size_t)w * nf;
+    const uint32_t *CH = (const uint32_t *)(c.arena + L.lk_hist);
+    const double *tmp = (const double *)(c.arena + L.lk_tmp);
+    double *lk_pe = (double *)(c.arena + L.lk_pe);
+    const long long n = xs_lk_chunk(p);
+    const double bscale = (double)(1LL << K.kb);
+    const long long emax = (1LL << K.kb) - 1;
+    auto fine = [&](double pe) {
+      long long eb = (long long)(pe * bscale);
+      eb = eb > emax ? emax : eb;
+      return (int)(eb & (nf - 1));
+    };
+    const int ck1 = (g + 1) * kXsFineGroup < K.nck ? (g + 1) * kXsFineGroup : K.nck;
+    for (int ck = g * kXsFineGroup + w; ck < ck1; ck += nw) {
+      const long long s0 = __ldcg(CH + (size_t)ck * K.nc);  // other CTAs' stores: L2
+      const long long s1 = ck + 1 < K.nck ? (long long)__ldcg(CH + (size_t)(ck + 1) * K.nc) : n;
+      for (int f = lane; f < nf; f += 32) cnt[f] = 0u;
+      __syncwarp();
+      // buckets of <= 32 * kR energies (~325 at C2's size) are loaded once,
+      // all loads in flight, and kept in registers; larger ones re-read
+      constexpr int kR = 16;
+      const bool inreg = s1 - s0 <= 32 * kR;
+      double v[kR];
+#pragma unroll
+      for (int r = 0; r < kR; r++) {
+        const long long i = s0 + lane + 32 * r;
+        v[r] = inreg && i < s1 ? __ldcg(tmp + i) : 0.0;
+      }
+      if (inreg) {
+#pragma unroll
+        for (int r = 0; r < kR; r++)
+          if (s0 + lane + 32 * r < s1) atomicAdd(&cnt[fine(v[r])], 1u);
+      } else {
+        for (long long i = s0 + lane; i < s1; i += 32) atomicAdd(&cnt[fine(__ldcg(tmp + i))], 1u);
+      }
+      __syncwarp();
+      {  // exclusive scan of cnt[0, nf): lane l owns entries [l*per, (l+1)*per)
+        const int per = nf >= 32 ? nf / 32 : 1;
+        uint32_t loc = 0;
+        for (int q = 0; q < per; q++) {
+          const int f = lane * per + q;
+          if (f < nf) loc += cnt[f];
+        }
+        uint32_t inc = loc;
+        for (int o = 1; o < 32; o <<= 1) {
+          const uint32_t t = __shfl_up_sync(0xffffffffu, inc, o);
+          if (lane >= o) inc += t;
+        }
+        uint32_t run = inc - loc;
+        for (int q = 0; q < per; q++) {
+          const int f = lane * per + q;
+          if (f < nf) {
+            const uint32_t v = cnt[f];
+            cnt[f] = run;
+            run += v;
+          }
+        }
+      }
+      __syncwarp();
+      if (inreg) {
+#pragma unroll
+        for (int r = 0; r < kR; r++)
+          if (s0 + lane + 32 * r < s1) lk_pe[s0 + atomicAdd(&cnt[fine(v[r])], 1u)] = v[r];
+      } else {
+        for (long long i = s0 + lane; i < s1; i += 32) {
+          const double pe = __ldcg(tmp + i);
+          lk_pe[s0 + atomicAdd(&cnt[fine(pe)], 1u)] = pe;
+        }
+      }
+      __syncwarp();
+    }
   }
 
   // ---- XS-6..XS-10: lookups ----------------------------------------------

@@ -515,9 +515,9 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
         for (int kd = 0; kd < 4; kd++) g.kind_n[kd] = 0;
       }
       if (g.split) {  // phase 1b: the lookup sorts' items and the (instance, nuclide) table items
-        // queue: zero items, count items, a first share of the nuclide items
-        // (the scans finish meanwhile), scatter items, the other nuclide items
-        std::vector<uint32_t> zero_items, count_items, scatter_items, nuc_items;
+        // queue: count items, a share of the nuclide items (the scans finish
+        // meanwhile), scatter items, another share, fine items, the rest
+        std::vector<uint32_t> count_items, scatter_items, fine_items, nuc_items;
         uint32_t smem_need = 0;
         auto pair = [](std::vector<uint32_t> &v, size_t x, uint32_t i) {
           v.push_back((uint32_t)x);
@@ -527,23 +527,25 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
           int argc;
           const char *const *argv;
           ens_args_get(a, (int)P.line_of_k[g.kmap[x]], &argc, &argv);
-          int ni = 0, ns = 0;
+          int ni = 0, ns = 0, nf = 0;
           uint32_t sm3 = 0;
-          const uint64_t scr = app_init_scratch(ap, argc, argv, &ni, &ns, &sm3);
+          const uint64_t scr = app_init_scratch(ap, argc, argv, &ni, &ns, &nf, &sm3);
           if (!g.item_count[x] || !ni) continue;
           g.init_scr_bytes = std::max<uint64_t>(g.init_scr_bytes, al(scr));
           smem_need = std::max(smem_need, sm3);
-          pair(zero_items, x, kXsZeroItem);
           for (int q = 0; q < ns; q++) pair(count_items, x, kXsCountItem | (uint32_t)q);
           for (int q = 0; q < ns; q++) pair(scatter_items, x, kXsScatterItem | (uint32_t)q);
+          for (int q = 0; q < nf; q++) pair(fine_items, x, kXsFineItem | (uint32_t)q);
           for (int i = 0; i < ni; i++) pair(nuc_items, x, (uint32_t)i);
         }
-        const size_t first = std::min(nuc_items.size(), (size_t)2 * 4 * (size_t)std::max(1, (int)ctas));  // pairs: 4 x ctas items
-        g.init_items = zero_items;
-        g.init_items.insert(g.init_items.end(), count_items.begin(), count_items.end());
-        g.init_items.insert(g.init_items.end(), nuc_items.begin(), nuc_items.begin() + first);
+        const size_t share = (size_t)2 * 2 * (size_t)std::max(1, (int)ctas);  // pairs: 2 x ctas items
+        const size_t f1 = std::min(nuc_items.size(), share), f2 = std::min(nuc_items.size(), 2 * share);
+        g.init_items = count_items;
+        g.init_items.insert(g.init_items.end(), nuc_items.begin(), nuc_items.begin() + f1);
         g.init_items.insert(g.init_items.end(), scatter_items.begin(), scatter_items.end());
-        g.init_items.insert(g.init_items.end(), nuc_items.begin() + first, nuc_items.end());
+        g.init_items.insert(g.init_items.end(), nuc_items.begin() + f1, nuc_items.begin() + f2);
+        g.init_items.insert(g.init_items.end(), fine_items.begin(), fine_items.end());
+        g.init_items.insert(g.init_items.end(), nuc_items.begin() + f2, nuc_items.end());
         if (!g.init_items.empty()) {
           g.smem3 = xs_init_smem_off() + (smem_need + 15u) / 16u * 16u;
           e = xs_init_items_occupancy(kXsInitThreads, g.smem3, &g.grid3);

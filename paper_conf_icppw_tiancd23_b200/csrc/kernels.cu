@@ -341,15 +341,18 @@ uint32_t app_items(uint32_t app, int argc, const char *const *argv, int *kind) {
 }
 // split phases: per-CTA scratch of the init-item kernel for one instance and
 // its number of init items (hash / nuclide grids: one per nuclide; 0 = none)
-uint64_t app_init_scratch(uint32_t app, int argc, const char *const *argv, int *n_items, int *n_sort, uint32_t *smem) {
+uint64_t app_init_scratch(uint32_t app, int argc, const char *const *argv, int *n_items, int *n_sort, int *n_fine,
+                          uint32_t *smem) {
   *n_items = 0;
   *n_sort = 0;
+  *n_fine = 0;
   *smem = 0;
   if (app != APP_XSBENCH) return 0;
   XsParams p;
   if (xs_parse(argc, argv, p) >= 0 || !xs_split_ok(p) || p.grid == XS_UNIONIZED) return 0;
   *n_items = p.n_iso;
   *n_sort = xs_sort_items(p);
+  *n_fine = xs_sort_fine_items(p);
   *smem = xs_init_smem(p).total;
   return XsApp::nuc_scratch_bytes(p);
 }

@@ -402,22 +402,21 @@ constexpr uint32_t kXsInitArgv = kXs2Sh;                                  // cha
 constexpr uint32_t kXsInitMisc = kXsInitArgv + (ENS_MAX_ARGC + 2) * 8;    // u32 item
 constexpr uint32_t kXsInitApp = kXsInitMisc + 64;                          // the app's shared memory
 
-// Per (instance, item kind): a zero item clears the instance's lookup
-// histogram; count items (kXsSortChunk lookups each) add into it, the CTA
-// finishing the last count item scans it and writes the descriptor; scatter
-// items then move the lookups to their buckets (XsApp::lk_pass, lk_scan:
-// lookup_sort cut into items); a nuclide item builds one nuclide's sorted
-// records and hash / nuclide grid column.  The host orders the queue zero
-// items, count items, a first share of the nuclide items, scatter items, the
-// rest: an item that waits (count on zero, scatter on the scan) only waits
-// for items pulled before it, by running CTAs (no deadlock), and in practice
-// finds them done.  Two CTAs of 256 threads per SM (compact shared memory:
-// no material tables), so one CTA's barrier-separated phases overlap the
-// other's.
+// Per instance: count items, the scan (by the CTA finishing the last count
+// item, which also writes the descriptor), scatter items, fine items
+// (XsApp::lk_count / lk_scan / lk_scatter / lk_fine: the lookup sort in
+// items); per (instance, nuclide) a nuclide item building that nuclide's
+// sorted records and hash / nuclide grid column.  The host orders the queue
+// count items, a share of the nuclide items, scatter items, another share,
+// fine items, the rest: an item that waits (scatter on the scan, fine on
+// every scatter item of its instance) only waits for items pulled before
+// it, by running CTAs (no deadlock), and in practice finds them done.  Two
+// CTAs of 256 threads per SM (compact shared memory: no material tables), so
+// one CTA's barrier-separated phases overlap the other's.
 struct XsInitSync {            // per instance, zeroed before the launch
-  uint32_t zdone;              // histogram zeroed
+  uint32_t fdone;              // scatter items finished
   uint32_t cdone;              // count items finished
-  uint32_t sdone;              // histogram scanned, descriptor written
+  uint32_t sdone;              // coarse histogram scanned, descriptor written
   uint32_t pstate;             // parsed command line: 0 none, 1 being written, 2 ready
   uint32_t pad[4];
   XsParams p;                  // the instance's parsed command line (pstate == 2)
@@ -429,10 +428,10 @@ __device__ __forceinline__ uint32_t ld_acquire_u32(const uint32_t *f) {
   asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(f) : "memory");
   return v;
 }
-// the whole CTA waits until *f != 0 (thread 0 acquires, the barrier orders the rest)
-__device__ __forceinline__ void cta_wait_flag(const uint32_t *f) {
+// the whole CTA waits until *f >= v (thread 0 acquires, the barrier orders the rest)
+__device__ __forceinline__ void cta_wait_flag(const uint32_t *f, uint32_t v = 1u) {
   if (threadIdx.x == 0)
-    while (!ld_acquire_u32(f)) __nanosleep(256);
+    while (ld_acquire_u32(f) < v) __nanosleep(256);
   __syncthreads();
 }
 // after a __syncthreads(): publish the CTA's global writes and set *f = v
@@ -450,8 +449,8 @@ __global__ void __launch_bounds__(256, 2) xs_init_items_kernel(const KParams p) 
   c.smem_off = kXsInitApp;
   c.csize = 1;
   c.flags = p.flags;
-  c.phases = p.phases;  // tracing (ENS_F_PHASES): 1..9 init_nuc_t's phases; sort items: 11 zero, 12 count,
-                        // 13 scan, 14 scatter, 15 waiting
+  c.phases = p.phases;  // tracing (ENS_F_PHASES): 1..9 init_nuc_t's phases; sort items: 12 count, 13 scan,
+                        // 14 scatter, 11 fine, 15 waiting
   char **argv = reinterpret_cast<char **>(ens_dsmem + kXsInitArgv);
   uint32_t *misc = reinterpret_cast<uint32_t *>(ens_dsmem + kXsInitMisc);
   char *scr = p.init_scr + (size_t)blockIdx.x * p.init_scr_bytes;
@@ -494,49 +493,54 @@ __global__ void __launch_bounds__(256, 2) xs_init_items_kernel(const KParams p) 
     const XsSmem S = xs_init_smem(xp);
     const XsLayout L = xs_layout(xp, (int)p.team_ctas);  // the instance's arena, as phase 1 lays it out
     c.arena = p.arena_base + (size_t)j * p.arena_bytes;
-    if (i >= kXsScatterItem) {  // the lookup sort's items
+    if (i >= kXsFineItem) {  // the lookup sort's items
       double *thr = reinterpret_cast<double *>(ens_smem(c) + S.thr);
+      uint32_t *sc = reinterpret_cast<uint32_t *>(ens_smem(c) + S.nkey);  // kXsLkSortSmem bytes
       if (!thr_ok) {
         if (tid < 12) thr[tid] = hm_threshold(tid);
         thr_ok = true;
         __syncthreads();
       }
-      if (i == kXsZeroItem) {
-        XsApp::lk_zero(c, xp, L);
+      const int q = (int)(i & 0x1fffffffu);
+      if (i & kXsCountItem) {
+        XsApp::lk_count(c, xp, L, thr, q, JT, sc);
         __syncthreads();
-        cta_set_flag(&sy->zdone, 1u);
-        phase_mark(c, 11);
-      } else {
-        const bool scatter = !(i & kXsCountItem);
-        const long long ch = (long long)(i & 0x3fffffffu), nc = xs_lk_chunk(xp);
-        const long long l0 = ch * kXsSortChunk, l1 = l0 + kXsSortChunk < nc ? l0 + kXsSortChunk : nc;
-        cta_wait_flag(scatter ? &sy->sdone : &sy->zdone);
-        phase_mark(c, 15);
-        XsApp::lk_pass(xp, c.arena, L, thr, l0, l1, scatter, JT);
+        phase_mark(c, 12);
+        if (tid == 0) {
+          __threadfence();
+          misc[1] = atomicAdd(&sy->cdone, 1u) == (uint32_t)xs_sort_items(xp) - 1u ? 1u : 0u;
+          __threadfence();
+        }
         __syncthreads();
-        phase_mark(c, scatter ? 14 : 12);
-        if (!scatter) {
+        if (misc[1]) {  // the last count item: (B) and the descriptor
+          uint32_t *mcnt = reinterpret_cast<uint32_t *>(ens_smem(c) + S.mcnt);
+          XsApp::lk_scan(c, xp, L, mcnt);
           if (tid == 0) {
-            __threadfence();
-            misc[1] = atomicAdd(&sy->cdone, 1u) == (uint32_t)xs_sort_items(xp) - 1u ? 1u : 0u;
-            __threadfence();
+            c.desc = p.xs_desc + (size_t)j * kDescBytes;
+            c.k = k;
+            c.id = line;
+            c.t_start = 0;
+            XsApp::write_desc(c, xp, L, mcnt);
           }
           __syncthreads();
-          if (misc[1]) {  // the last count item: (B) and the descriptor
-            uint32_t *mcnt = reinterpret_cast<uint32_t *>(ens_smem(c) + S.mcnt);
-            XsApp::lk_scan(c, xp, L, mcnt);
-            if (tid == 0) {
-              c.desc = p.xs_desc + (size_t)j * kDescBytes;
-              c.k = k;
-              c.id = line;
-              c.t_start = 0;
-              XsApp::write_desc(c, xp, L, mcnt);
-            }
-            __syncthreads();
-            cta_set_flag(&sy->sdone, 1u);
-            phase_mark(c, 13);
-          }
+          cta_set_flag(&sy->sdone, 1u);
+          phase_mark(c, 13);
         }
+      } else if (i & kXsScatterItem) {
+        cta_wait_flag(&sy->sdone);
+        phase_mark(c, 15);
+        XsApp::lk_scatter(c, xp, L, thr, q, JT, sc);
+        __syncthreads();
+        if (tid == 0) {
+          __threadfence();
+          atomicAdd(&sy->fdone, 1u);
+        }
+        phase_mark(c, 14);
+      } else {
+        cta_wait_flag(&sy->fdone, (uint32_t)xs_sort_items(xp));
+        phase_mark(c, 15);
+        XsApp::lk_fine(c, xp, L, q, sc);
+        phase_mark(c, 11);
       }
     } else {
       if (!jt_ok) {

@@ -76,12 +76,13 @@ int xs_items_threads();
 cudaError_t launch_xs_init_items(int ctas, int threads, size_t smem, const KParams &p, cudaStream_t st);
 cudaError_t xs_init_items_occupancy(int threads, size_t smem, int *ctas);
 uint32_t xs_init_smem_off();
-uint64_t app_init_scratch(uint32_t app, int argc, const char *const *argv, int *n_items, int *n_sort, uint32_t *smem);
+uint64_t app_init_scratch(uint32_t app, int argc, const char *const *argv, int *n_items, int *n_sort, int *n_fine,
+                          uint32_t *smem);
 constexpr uint32_t kInitSyncBytes = 128;  // XsInitSync (kernels_items.cu)
 // phase-1b item codes (the second word of an init item; nuclide items are < 2^16)
-constexpr uint32_t kXsZeroItem = 0xffffffffu;     // zero the lookup histogram
 constexpr uint32_t kXsCountItem = 0x80000000u;    // | chunk: count lookups
 constexpr uint32_t kXsScatterItem = 0x40000000u;  // | chunk: scatter lookups
+constexpr uint32_t kXsFineItem = 0x20000000u;     // | group: sort coarse buckets
 constexpr int kXsInitThreads = 256;  // init-item kernel block (launch bounds 256 x 2 CTAs/SM)
 
 }  // namespace ens
