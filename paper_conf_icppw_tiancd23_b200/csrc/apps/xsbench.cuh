@@ -564,12 +564,17 @@ struct XsApp {
             const uint32_t w = W[k];
             return (int)(w >> 16) + (int)(w & 1u);
           };
-          for (int k = tid; k < n_gp; k += T) {
-            const int lo = k == 0 ? 0 : bf_at(k);
-            const int hi = k + 1 < n_gp ? bf_at(k + 1) : p.bins;
-            const int v = k < n_gp - 2 ? k : n_gp - 2;
-            for (int b = lo; b < hi; b++) colp[b] = v;
+          // bin b's column entry min(#{k >= 1: bfirst(E_k) <= b}, n_gp-2): a
+          // histogram of bfirst (shared atomics), then an inclusive scan
+          // (the clamp is applied where the entries read it)
+          for (int b = tid; b <= p.bins; b += T) colp[b] = 0;
+          __syncthreads();
+          for (int k = 1 + tid; k < n_gp; k += T) {
+            const int bf = bf_at(k);
+            if (bf < p.bins) atomicAdd(&colp[bf], 1);
           }
+          __syncthreads();
+          global_exclusive_scan<true>(reinterpret_cast<uint32_t *>(colp), p.bins, ens_sh(c));
         } else {
           for (int k0 = tid; k0 < n_gp; k0 += U * T) {
             unsigned long long ek[U], ek1[U];
@@ -597,7 +602,8 @@ struct XsApp {
           // entries {u_low, u_high, q(E[u_low+1..u_low+6])} from shared memory:
           // q = 0 below bin b, 65535 above it or past the grid
           for (int b = tid; b <= p.bins; b += T) {
-            const int ul = colp[b], uh = b < p.bins ? colp[b + 1] : n_gp - 2;
+            const int c0 = colp[b], c1 = b < p.bins ? colp[b + 1] : n_gp - 2;
+            const int ul = c0 < n_gp - 2 ? c0 : n_gp - 2, uh = c1 < n_gp - 2 ? c1 : n_gp - 2;
             XsHashEnt h;
             h.u_low = (uint16_t)ul;
             h.u_high = (uint16_t)(uh + 1);

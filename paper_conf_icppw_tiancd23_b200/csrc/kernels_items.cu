@@ -457,8 +457,10 @@ __global__ void __launch_bounds__(256, 2) xs_init_items_kernel(const KParams p) 
   bool jt_ok = false;   // the LCG jump tables (seed- and layout-independent: S.jmp is fixed)
   bool thr_ok = false;  // pick_mat thresholds (constant)
   const Affine JT = lcg_pow(2ULL * (uint64_t)T);  // T lookups' draws
-  uint32_t cached_j = 0xffffffffu;  // the instance whose command line xp holds
+  uint32_t cached_j = 0xffffffffu;  // the instance whose command line xp holds (and its layouts)
   XsParams xp;
+  XsSmem xS{};
+  XsLayout xL{};
   for (;;) {
     if (tid == 0) misc[0] = atomicAdd(p.counter3, 1u);
     __syncthreads();
@@ -488,10 +490,12 @@ __global__ void __launch_bounds__(256, 2) xs_init_items_kernel(const KParams p) 
         }
       }
       cached_j = j;
+      xS = xs_init_smem(xp);
+      xL = xs_layout(xp, (int)p.team_ctas);  // the instance's arena, as phase 1 lays it out
     }
     phase_mark(c, 0);
-    const XsSmem S = xs_init_smem(xp);
-    const XsLayout L = xs_layout(xp, (int)p.team_ctas);  // the instance's arena, as phase 1 lays it out
+    const XsSmem &S = xS;
+    const XsLayout &L = xL;
     c.arena = p.arena_base + (size_t)j * p.arena_bytes;
     if (i >= kXsFineItem) {  // the lookup sort's items
       double *thr = reinterpret_cast<double *>(ens_smem(c) + S.thr);
