@@ -30,6 +30,10 @@ CASES = {
     "split": ([XS.format(g=g, s=i) for i, g in enumerate(["hash", "unionized", "nuclide", "hash"])] +
               ["rsbench -s small -l 2500 -p 20 -w 4 -r 5", "rsbench -s small -l 300 -p 12 -w 3 -d -r 6"],
               dict(threads=128, split=True)),
+    # phase 1b's lookup sort over several chunks (count / scan / scatter / fine items
+    # and their cross-CTA flags), two hash instances
+    "split2": (["xsbench -s small -g 200 -l 140000 -G hash -h 150 -r %d" % (7 + i) for i in range(2)],
+               dict(threads=128, split=True)),
 }
 
 
