@@ -35,10 +35,10 @@ def test_ens_run_cli_matches_oracle(tmp_path, gpus):
     f.write_text(TEXT)
     out = tmp_path / "run.json"
     p = subprocess.run([ENS_RUN, "-f", str(f), "-t", "128", "--gpus", str(gpus), "--json", str(out)],
-                       capture_output=True, text=True, timeout=300)
+                       capture_output=True, timeout=300)
     assert p.returncode == 0, p.stderr
     o = oracle_lib.run_text(TEXT)
-    assert p.stdout == "".join(o.stdout)
+    assert p.stdout == b"".join(o.stdout)
     d = json.loads(out.read_text())
     assert d["instances"] == len(o.records) and d["gpus"] == gpus
     for k, r in enumerate(d["records"]):
@@ -48,5 +48,5 @@ def test_ens_run_cli_matches_oracle(tmp_path, gpus):
             assert r[key] == int(b[key]), (k, key, r[key], b[key])
         tol = 1e-12 * max(abs(float(b["fabs"])), 1e-300)
         assert abs(r["fsum"] - float(b["fsum"])) <= tol and abs(r["fabs"] - float(b["fabs"])) <= tol
-        assert r["stdout"] == o.stdout[k]
+        assert r["stdout"].encode() == o.stdout[k]
     assert np.count_nonzero([r["exit_code"] for r in d["records"]]) == d["nonzero_exit"]

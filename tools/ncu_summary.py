@@ -67,53 +67,81 @@ def launches(log, out, command):
     print(f"{len(res)} launches -> {out}")
 
 
+def summary_of(rep):
+    """profiles/<report name>.txt: the committed summary of a capture (the .ncu-rep stays in gpurun_out/)."""
+    return os.path.join("profiles", os.path.basename(rep).replace(".ncu-rep", ".txt"))
+
+
+def _rx(name):
+    """ncu --kernel-name regex for a kernel name of the raw page (short demangled form,
+    e.g. `void ens_kernel<XsApp, 512>(KParams)`; the source page knows it as
+    `ens::ens_kernel<ens::XsApp, (int)512>`): the identifier, then each template argument."""
+    base = name.split("(")[0]
+    if base.startswith("void "):
+        base = base[5:]
+    ident, _, targs = base.partition("<")
+    rx = ident
+    if targs:
+        rx += "<" + "".join(".*" + re.escape(t.strip()) for t in targs.rstrip(">").split(",")) + ">"
+    return "regex:" + rx
+
+
 def full(rep, out, workload=None):
+    """Every kernel of the capture: key counters, then warp-stall samples by source line."""
     raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv"], capture_output=True, text=True).stdout
     rows = list(csv.reader(raw.splitlines()))
-    hdr, units, vals = rows[0], rows[1], rows[2]
-    d = {hdr[i]: (vals[i], units[i]) for i in range(len(hdr))}
-    lines = [f"kernel: {d.get('Kernel Name', ('?',))[0]}  grid {d.get('Grid Size', ('?',))[0]} "
-             f"block {d.get('Block Size', ('?',))[0]}", "", "key counters (one launch):"]
-    for k in KEYS:
-        if k in d:
-            lines.append(f"  {k:58s} {d[k][0]:>22s} {d[k][1]}")
-    src = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass"],
-                         capture_output=True, text=True).stdout
-    agg, tot, text, cur, hdr2 = collections.Counter(), 0, {}, None, None
-    for r in csv.reader(src.splitlines()):
-        if len(r) == 2 and r[0] == "File Path":
-            cur = r[1].split("/")[-1]
-            continue
-        if r and r[0] == "Line No":
-            hdr2 = r
-            continue
-        if hdr2 and len(r) >= 5 and r[0].isdigit():
-            try:
-                x = int(r[4] or 0)
-            except ValueError:
+    hdr, units = rows[0], rows[1]
+    lines, dom = [], None
+    for vals in rows[2:]:
+        d = {hdr[i]: (vals[i], units[i]) for i in range(len(hdr))}
+        name = d.get("Kernel Name", ("?",))[0]
+        lines += [f"kernel: {name}  grid {d.get('Grid Size', ('?',))[0]} block {d.get('Block Size', ('?',))[0]}",
+                  "", "key counters (one launch):"]
+        for k in KEYS:
+            if k in d:
+                lines.append(f"  {k:58s} {d[k][0]:>22s} {d[k][1]}")
+        ms = float(d["gpu__time_duration.sum"][0].replace(",", "")) * {"ms": 1.0, "us": 1e-3, "usecond": 1e-3,
+                                                                         "msecond": 1.0, "ns": 1e-6,
+                                                                         "nsecond": 1e-6}.get(d["gpu__time_duration.sum"][1], 1.0)
+        tb = sum(float(d[k][0].replace(",", "")) * UNIT.get(d[k][1], 1)
+                 for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"))
+        if dom is None or ms > dom[0]:
+            dom = (ms, tb, name)
+        src = subprocess.run(["ncu", "-i", rep, "--page", "source", "--csv", "--print-source", "cuda,sass",
+                              "--kernel-name-base", "demangled", "--kernel-name", _rx(name)],
+                             capture_output=True, text=True).stdout
+        agg, tot, text, cur, hdr2 = collections.Counter(), 0, {}, None, None
+        for r in csv.reader(src.splitlines()):
+            if len(r) == 2 and r[0] == "File Path":
+                cur = r[1].split("/")[-1]
                 continue
-            key = (cur, int(r[0]))
-            agg[key] += x
-            tot += x
-            text[key] = r[1].strip()[:90]
-    lines += ["", f"warp-stall samples by source line (top 30 of {tot}):"]
-    for key, x in agg.most_common(30):
-        lines.append(f"  {100.0 * x / max(tot, 1):5.1f}%  {key[0]}:{key[1]}  {text[key]}")
-    open(out, "w").write("\n".join(lines) + "\n")
+            if r and r[0] == "Line No":
+                hdr2 = r
+                continue
+            if hdr2 and len(r) >= 5 and r[0].isdigit():
+                try:
+                    x = int(r[4] or 0)
+                except ValueError:
+                    continue
+                key = (cur, int(r[0]))
+                agg[key] += x
+                tot += x
+                text[key] = r[1].strip()[:90]
+        lines += ["", f"warp-stall samples by source line (top 20 of {tot}):"]
+        for key, x in agg.most_common(20):
+            lines.append(f"  {100.0 * x / max(tot, 1):5.1f}%  {key[0]}:{key[1]}  {text[key]}")
+        lines += ["", ""]
+    open(out, "w").write("\n".join(lines))
     print(f"-> {out}")
-    if workload:
-        tb = 0.0
-        for k in ("dram__bytes_read.sum", "dram__bytes_write.sum"):
-            v, u = d[k]
-            tb += float(v.replace(",", "")) * UNIT.get(u, 1)
+    if workload and dom:
         tp = os.path.join(ROOT, "profiles", "traffic.json")
         t = json.load(open(tp)) if os.path.exists(tp) else {}
-        t[workload] = tb
+        t[workload] = dom[1]
         t[f"_source_{workload}"] = (f"ncu --set full, {os.path.relpath(out, ROOT)}: dram__bytes_read.sum + "
-                                    f"dram__bytes_write.sum of one launch")
+                                    f"dram__bytes_write.sum of one launch of the longest kernel ({dom[2]})")
         t.pop("_source", None)
         json.dump(t, open(tp, "w"), indent=1)
-        print(f"traffic[{workload}] = {tb:.4g} B -> {tp}")
+        print(f"traffic[{workload}] = {dom[1]:.4g} B ({dom[2]}) -> {tp}")
 
 
 APP_OF = {"EchoApp": 1, "XsApp": 2, "RsApp": 3, "AmgApp": 4, "PrApp": 5}
@@ -155,7 +183,7 @@ def counters(rep, workload):
         if d["gpu__time_duration.sum"][1] == "us":
             ms /= 1e3
         out[key] = {"dram_bytes": tb, "inst_executed": float(d["smsp__inst_executed.sum"][0].replace(",", "")),
-                    "ncu_ms": ms, "kernel": d["Kernel Name"][0], "source": os.path.relpath(rep, ROOT)}
+                    "ncu_ms": ms, "kernel": d["Kernel Name"][0], "source": summary_of(rep)}
     p = os.environ.get("NCU_COUNTERS", os.path.join(ROOT, "profiles", "ncu_counters.json"))
     allc = json.load(open(p)) if os.path.exists(p) else {}
     allc[workload] = {"kernels": out, "note": "one ncu --set full capture of a warm launch (--clock-control none); "
