@@ -453,6 +453,11 @@ def roofline(name, lines, res, kt, clocks, peak_hbm, peak_kind):
     out = {"kernel": f"{kname} x {dom[3]} CTAs", "kernel_ms": dom_ms,
            "kernels": [{"app": k[0], "phase": k[1], "kind": k[2], "ctas": k[3], "threads": k[4], "ms": k[5]} for k in kt],
            "traffic": traffic, "candidates": cand}
+    if c and "l1tex_busy" in c:
+        # measured utilisations of the same kernel under ncu (not live): for a latency-bound
+        # kernel no roofline binds; these say how close the L1/TEX pipe and the schedulers are
+        out["ncu_utilization"] = {"l1tex_busy": c["l1tex_busy"], "issue_active": c.get("issue_active"),
+                                  "source": c.get("source")}
     if bk:
         b = valid[bk]
         out.update({"bound": {"hbm": "hbm", "dram": "hbm", "issue": "alu", "fp64": "alu"}[bk], "binding": bk,

@@ -165,7 +165,9 @@ def kernel_key(name):
 
 def counters(rep, workload):
     raw = subprocess.run(["ncu", "-i", rep, "--page", "raw", "--csv", "--metrics",
-                          "dram__bytes_read.sum,dram__bytes_write.sum,smsp__inst_executed.sum,gpu__time_duration.sum"],
+                          "dram__bytes_read.sum,dram__bytes_write.sum,smsp__inst_executed.sum,gpu__time_duration.sum,"
+                          "l1tex__throughput.avg.pct_of_peak_sustained_active,"
+                          "smsp__issue_active.avg.pct_of_peak_sustained_active"],
                          capture_output=True, text=True).stdout
     rows = list(csv.reader(raw.splitlines()))
     hdr, units = rows[0], rows[1]
@@ -184,6 +186,10 @@ def counters(rep, workload):
             ms /= 1e3
         out[key] = {"dram_bytes": tb, "inst_executed": float(d["smsp__inst_executed.sum"][0].replace(",", "")),
                     "ncu_ms": ms, "kernel": d["Kernel Name"][0], "source": summary_of(rep)}
+        for m, k in (("l1tex__throughput.avg.pct_of_peak_sustained_active", "l1tex_busy"),
+                     ("smsp__issue_active.avg.pct_of_peak_sustained_active", "issue_active")):
+            if m in d:
+                out[key][k] = float(d[m][0].replace(",", "")) / 100.0
     p = os.environ.get("NCU_COUNTERS", os.path.join(ROOT, "profiles", "ncu_counters.json"))
     allc = json.load(open(p)) if os.path.exists(p) else {}
     allc[workload] = {"kernels": out, "note": "one ncu --set full capture of a warm launch (--clock-control none); "
