@@ -1,6 +1,6 @@
 """Per-kernel CUDA-event times of a bench workload (a probe, not the bench).
 
-    python tools/ktimes.py <C1|C2|C2U|C3|C4|C5|TSTAR> [reps] [--phases] [--env K=V ...]
+    python tools/ktimes.py <C1|C2|C2U|C3|C4|C5|TSTAR> [reps] [--phases] [--split | --fused]
 
 Launches the workload once (cold), relaunches it `reps` times (default 5) and
 prints the best launch time and, for that launch, every kernel's time
@@ -24,11 +24,16 @@ def main():
     phases = "--phases" in argv
     if phases:
         argv.remove("--phases")
+    mode = {}
+    for flag in ("--split", "--fused"):
+        if flag in argv:
+            argv.remove(flag)
+            mode[flag[2:]] = True
     name = argv[0]
     reps = int(argv[1]) if len(argv) > 1 else 5
     lines, _ = bench.workload_lines(name, 1)
     threads = bench.THREADS.get(name, 256)
-    e = Ensemble(Args.parse(workloads.text(lines)), app="auto", threads=threads, phases=phases).launch()
+    e = Ensemble(Args.parse(workloads.text(lines)), app="auto", threads=threads, phases=phases, **mode).launch()
     torch.cuda.synchronize()
     best, kt, ph = None, None, None
     for _ in range(reps):
