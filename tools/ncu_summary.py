@@ -134,7 +134,7 @@ def full(rep, out, workload=None):
     open(out, "w").write("\n".join(lines))
     print(f"-> {out}")
     if workload and dom:
-        tp = os.path.join(ROOT, "profiles", "traffic.json")
+        tp = os.environ.get("NCU_TRAFFIC", os.path.join(ROOT, "profiles", "traffic.json"))
         t = json.load(open(tp)) if os.path.exists(tp) else {}
         t[workload] = dom[1]
         t[f"_source_{workload}"] = (f"ncu --set full, {os.path.relpath(out, ROOT)}: dram__bytes_read.sum + "

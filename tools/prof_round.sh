@@ -15,3 +15,15 @@ for W in "$@"; do
     python tools/prof_workload.py "$W" 1 > "gpurun_out/ncu_${W}_${TAG}.log" 2>&1
   tail -1 "gpurun_out/ncu_${W}_${TAG}.log"
 done
+# summaries on the box (the reports exceed gpurun's 64 MiB copy-back): with
+# SUMMARISE=1, gpurun_out/ gets the per-workload .txt, ncu_counters.json and
+# traffic.json (copies of profiles/ updated), and the reports are removed
+if [ "${SUMMARISE:-0}" = 1 ]; then
+  cp profiles/ncu_counters.json gpurun_out/ncu_counters.json
+  cp profiles/traffic.json gpurun_out/traffic.json
+  for W in "$@"; do
+    NCU_TRAFFIC=gpurun_out/traffic.json python tools/ncu_summary.py full "gpurun_out/ncu_${W}_${TAG}.ncu-rep" "gpurun_out/ncu_${W}_${TAG}.txt" "$W"
+    NCU_COUNTERS=gpurun_out/ncu_counters.json python tools/ncu_summary.py counters "gpurun_out/ncu_${W}_${TAG}.ncu-rep" "$W"
+    rm -f "gpurun_out/ncu_${W}_${TAG}.ncu-rep"
+  done
+fi
