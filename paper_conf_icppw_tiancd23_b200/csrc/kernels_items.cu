@@ -199,6 +199,7 @@ __device__ __forceinline__ void xs2_item(const XsDesc &d, const XsParams &p, lon
   const double *lk_pe = (const double *)d.lk_pe;
   const long long n_u = (long long)p.n_iso * p.n_gp, UB = d.ubins;
   const double du = 1.0 / p.bins;
+  const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(ens_dsmem);  // the shared window base, once
   for (long long sl = s0 + threadIdx.x; sl < s1; sl += kXs2T) {
     int mat = 0;
 #pragma unroll
@@ -213,8 +214,8 @@ __device__ __forceinline__ void xs2_item(const XsDesc &d, const XsParams &p, lon
     double mv[5];
     if (GRID == XS_HASH) {
       const int rw = xs_max_nucs(p.n_iso) + kXs2RowPad;
-      xs2_hash_lookup((uint32_t)__cvta_generic_to_shared(mats + mat * rw),
-                      (uint32_t)__cvta_generic_to_shared(concs + mat * rw), nn[mat], recs,
+      xs2_hash_lookup(sbase + kXs2Mats + 2u * (uint32_t)(mat * rw), sbase + kXs2Concs + 8u * (uint32_t)(mat * rw),
+                      nn[mat], recs,
                       reinterpret_cast<const XsHashEnt *>(ig), p.bins, p.n_gp, pe, idx, mv);
     } else {
       XsApp::macro_lookup<GRID>(p, recs, ig, nn, concs, mats, pe, mat, idx, mv);
@@ -589,6 +590,10 @@ cudaError_t launch_xs_init_items(int ctas, int threads, size_t smem, const KPara
 // to its arena) are staged in shared memory and every lookup is RsApp::lookup
 // (RS-3, bit-identical to the fused body).  The last item's CTA writes the
 // record, tallies (argmax, materials, pole-term counters) and stdout.
+// (Measured and reverted: warp-granular items — each warp pulling its own
+// 64 / 256 / 1024 lookups, no CTA barrier per item, offsets and
+// concentrations read from the arena — C3 phase 2 14.1 / 17.3 / 36.6 ms
+// against 14.0 ms with CTA items of 512.)
 constexpr uint32_t kRsDesc = kXs2Sh;
 constexpr uint32_t kRsThr = kRsDesc + (kDescBytes + 15) / 16 * 16;
 constexpr uint32_t kRsNn = kRsThr + 12 * 8;
