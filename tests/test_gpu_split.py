@@ -90,3 +90,32 @@ def test_auto_policy():
     assert info.kernel_launches >= 2
     _, info = run(workloads.tstar(300), threads=512)
     assert info.kernel_launches == 1
+
+
+# phase 1b's lookup sort in items: chunk boundaries (kXsSortChunk = 65536 lookups per count /
+# scatter item), several chunks, coarse buckets with and without fine bits, both table kinds
+SORT_LINES = [
+    "xsbench -s small -g 300 -l 65536 -G hash -h 200 -r 31",    # exactly one chunk
+    "xsbench -s small -g 300 -l 65537 -G hash -h 200 -r 32",    # one chunk + 1 lookup
+    "xsbench -s large -g 120 -l 140000 -G hash -h 300 -r 33",   # three chunks
+    "xsbench -s small -g 250 -l 200003 -G nuclide -r 34",       # four chunks, nuclide grid
+    "xsbench -s small -g 90 -l 700 -G hash -h 50 -r 35",        # coarse buckets only (kb <= 8)
+]
+
+
+def test_split_lookup_sort_items(oracle):
+    text = "".join(l + "\n" for l in SORT_LINES)
+    g, info = run(SORT_LINES, threads=256, split=True, dump_rows=2000)
+    assert info.kernel_launches > info.n_groups
+    o = oracle.run_text(text, dump=2000)
+    assert_parity(g, o)
+    for k in range(len(SORT_LINES)):  # the first 2000 sorted slots, element by element (as a set)
+        gd = g.dump[k]
+        gd = gd[~np.all(gd == 0, axis=1)]
+        n_l = int(SORT_LINES[k].split("-l ")[1].split()[0])
+        assert len(gd) == min(2000, n_l)
+        # every dumped (energy, material) row is one of the oracle's lookups with its exact results
+        od = oracle.run_text(SORT_LINES[k] + "\n", dump=n_l).dumps[0]
+        keys = {(r[0], r[1]): r for r in od}
+        for r in gd:
+            assert np.array_equal(np.asarray(keys[(r[0], r[1])]).view(np.uint64), r.view(np.uint64))
