@@ -449,7 +449,8 @@ def roofline(name, lines, res, kt, clocks, peak_hbm, peak_kind):
                                      "RS body is built --fmad=false: 1 FLOP per DP instruction, half of this at most"}
     valid = {k: v for k, v in cand.items() if v["frac"] <= 1.05}
     bk = max(valid, key=lambda k: valid[k]["frac"]) if valid else None
-    kname = ("xs_items_kernel<%d>" % dom[2]) if phase == 2 else f"ens_kernel<app {dom[0]},{dom[4]}>"
+    kname = (("rs_items_kernel" if dom[2] == 3 else "xs_items_kernel<%d>" % dom[2]) if phase == 2
+             else "xs_init_items_kernel" if phase == 3 else f"ens_kernel<app {dom[0]},{dom[4]}>")
     out = {"kernel": f"{kname} x {dom[3]} CTAs", "kernel_ms": dom_ms,
            "kernels": [{"app": k[0], "phase": k[1], "kind": k[2], "ctas": k[3], "threads": k[4], "ms": k[5]} for k in kt],
            "traffic": traffic, "candidates": cand}
@@ -598,7 +599,8 @@ def main():
                 "mapping": "one CTA per instance, fused (the paper's team = thread block), both runs",
                 "product_default": {"T1_ms": t1a, "TN_ms": head["ms_per_step"],
                                     "value": t1a * len(lines) / head["ms_per_step"],
-                                    "mapping": "auto: solo on an 8-CTA cluster team; 64 instances in split phases"},
+                                    "mapping": "auto (the library's choice): split phases in both runs; a lone "
+                                               "instance's table builds and lookups already spread over every SM"},
                 "paper_context": "51x at 64 instances on A100 40GB (P:44-45, P:639-640)"}
     if rank == 0:
         out = {"metric": METRIC, "value": head["value"], "unit": "instances/s", "n_gpus": world, "steps": a.steps,
