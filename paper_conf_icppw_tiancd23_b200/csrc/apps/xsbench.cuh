@@ -503,6 +503,7 @@ struct XsApp {
               }
             }
           }
+          ENS_CHECK(lo + rank < hi);
           Js[lo + rank] = vj;
         }
       } else {
@@ -1595,7 +1596,10 @@ struct XsApp {
     const long long l1 = l0 + kXsSortChunk < nc ? l0 + kXsSortChunk : nc;
     for (int x = threadIdx.x; x < K.nck; x += blockDim.x) sc[x] = 0u;
     __syncthreads();
-    lk_sample(p, K, thr, l0, l1, JT, [&](double, uint32_t ck) { atomicAdd(&sc[ck], 1u); });
+    lk_sample(p, K, thr, l0, l1, JT, [&](double, uint32_t ck) {
+      ENS_CHECK(ck < (uint32_t)K.nck);
+      atomicAdd(&sc[ck], 1u);
+    });
     __syncthreads();
     uint32_t *CH = (uint32_t *)(c.arena + L.lk_hist);
     for (int x = threadIdx.x; x < K.nck; x += blockDim.x) CH[(size_t)x * K.nc + ch] = sc[x];
@@ -1607,6 +1611,8 @@ struct XsApp {
     uint32_t *CH = (uint32_t *)(c.arena + L.lk_hist);
     global_exclusive_scan(CH, (long long)K.nck * K.nc, ens_sh(c));
     __syncthreads();
+    // the last cursor plus the last chunk's last count is the chunk size (every lookup counted once)
+    ENS_CHECK(ld_(CH + (size_t)K.nck * K.nc - 1) <= (uint32_t)xs_lk_chunk(p));
     if (tid < 12) mcnt[16 + tid] = ld_(CH + ((size_t)tid << K.cb) * K.nc);
     if (tid == 12) mcnt[28] = (uint32_t)xs_lk_chunk(p);
     __syncthreads();
@@ -1621,7 +1627,11 @@ struct XsApp {
     for (int x = threadIdx.x; x < K.nck; x += blockDim.x) sc[x] = __ldcg(CH + (size_t)x * K.nc + ch);
     __syncthreads();
     double *tmp = (double *)(c.arena + L.lk_tmp);
-    lk_sample(p, K, thr, l0, l1, JT, [&](double pe, uint32_t ck) { tmp[atomicAdd(&sc[ck], 1u)] = pe; });
+    lk_sample(p, K, thr, l0, l1, JT, [&](double pe, uint32_t ck) {
+      const uint32_t pos = atomicAdd(&sc[ck], 1u);
+      ENS_CHECK(ck < (uint32_t)K.nck && pos < (uint32_t)nc);
+      tmp[pos] = pe;
+    });
   }
   // (D)
   __device__ static void lk_fine(const Ctx &c, const XsParams &p, const XsLayout &L, int g, uint32_t *sc) {
@@ -1644,6 +1654,7 @@ struct XsApp {
     for (int ck = g * kXsFineGroup + w; ck < ck1; ck += nw) {
       const long long s0 = __ldcg(CH + (size_t)ck * K.nc);  // other CTAs' stores: L2
       const long long s1 = ck + 1 < K.nck ? (long long)__ldcg(CH + (size_t)(ck + 1) * K.nc) : n;
+      ENS_CHECK(s0 <= s1 && s1 <= n);
       for (int f = lane; f < nf; f += 32) cnt[f] = 0u;
       __syncwarp();
       // buckets of <= 32 * kR energies (~325 at C2's size) are loaded once,
@@ -1690,7 +1701,11 @@ struct XsApp {
       if (inreg) {
 #pragma unroll
         for (int r = 0; r < kR; r++)
-          if (s0 + lane + 32 * r < s1) lk_pe[s0 + atomicAdd(&cnt[fine(v[r])], 1u)] = v[r];
+          if (s0 + lane + 32 * r < s1) {
+            const long long pos = s0 + atomicAdd(&cnt[fine(v[r])], 1u);
+            ENS_CHECK(pos < s1);
+            lk_pe[pos] = v[r];
+          }
       } else {
         for (long long i = s0 + lane; i < s1; i += 32) {
           const double pe = __ldcg(tmp + i);

@@ -121,6 +121,7 @@ __device__ __forceinline__ void xs2_hash_lookup(uint32_t mrow_s, uint32_t crow_s
   auto pair_of = [&](int j, const uint4 &h, Xs2Pair &o) {
     o.rb = lds_u16(mrow_s + 2u * (uint32_t)j) * (uint32_t)n_gp;
     o.lo = guess(h);
+    ENS_CHECK(o.lo >= 0 && o.lo + 1 < n_gp);
     o.hx = h.x;
     o.q = reinterpret_cast<const double2 *>(recs + (o.rb + (uint32_t)o.lo) * 6u);
   };

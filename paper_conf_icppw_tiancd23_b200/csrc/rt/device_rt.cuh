@@ -190,6 +190,17 @@ __device__ __forceinline__ unsigned long long gtimer() {
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
   return t;
 }
+// bounds / invariant checks of the cross-CTA paths (compute-sanitizer is not
+// available on the GPU pool): built with -DENS_CHECKS=1 a failed check traps
+// (the launch fails with an illegal-instruction error); off in the product
+#ifndef ENS_CHECKS
+#define ENS_CHECKS 0
+#endif
+#define ENS_CHECK(cond)                  \
+  do {                                   \
+    if (ENS_CHECKS && !(cond)) __trap(); \
+  } while (0)
+
 // tracing: is this the thread that marks phases?  Hot loops test a cached
 // copy (phase_mark_if): the Ctx lives in local memory across calls
 __device__ __forceinline__ bool tracing(const Ctx &c) { return c.phases && threadIdx.x == 0 && c.crank == 0; }
