@@ -766,7 +766,7 @@ static int enqueue(ens_run *r) {
       k2.item_base = g.kind_base[kd];
       k2.n_items = g.kind_n[kd];
       k2.counter2 = (uint32_t *)(r->ws + g.ctr2_off + 8 * kd);
-      if (kt_begin(2, kd, ctas2, xs_items_threads())) return fail(ENS_ECUDA, "ens_launch: kernel timing events");
+      if (kt_begin(2, kd, ctas2, xs_items_threads(kd))) return fail(ENS_ECUDA, "ens_launch: kernel timing events");
       e = launch_xs_items(kd, ctas2, k2, st);
       if (e != cudaSuccess) return cuda_fail(e, "xs_items_kernel launch");
       if (kt_end()) return fail(ENS_ECUDA, "ens_launch: kernel timing events");

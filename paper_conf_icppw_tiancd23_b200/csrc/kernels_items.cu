@@ -43,6 +43,14 @@ namespace ens {
 #ifndef ENS_XS2_MINB_NUC
 #define ENS_XS2_MINB_NUC 2
 #endif
+// threads per CTA of the XS lookup-item kernel per grid type (ENS_XS2_T_HASH: hash grids)
+#ifndef ENS_XS2_T_HASH
+#define ENS_XS2_T_HASH 256
+#endif
+template <int GRID>
+struct Xs2T {
+  static constexpr int v = GRID == XS_HASH ? ENS_XS2_T_HASH : ENS_XS2_T;
+};
 template <int GRID>
 struct Xs2Minb {
   static constexpr int v = GRID == XS_HASH ? ENS_XS2_MINB_HASH : GRID == XS_UNIONIZED ? ENS_XS2_MINB_UNI : ENS_XS2_MINB_NUC;
@@ -86,6 +94,11 @@ __device__ __forceinline__ double lds_f64(uint32_t a) {
 // stay below 2^32).  A nuclide's entry is consumed when its guess is made
 // (its u_low / u_high travel with the pair).  The tables were written by an
 // earlier kernel: read-only loads (ldro).
+// Block shape and register budget (C2's phase 2, measured): 256 threads x 3
+// CTAs at 80 registers (24 warps) 19.5 ms; 352 x 2 at 88 (22 warps, no
+// spills) 21.4; 320 x 2 (20 warps) 24.2; 192 x 4 21.1; 256 x 4 at 64
+// (spills) 21.8; 128 x 6 22.2; the pair's last 64 bytes loaded only when
+// needed (fewer registers) 22.1 (x3) / 21.5 (x4): latency exposed.
 // L1 prefetches (measured on C2's phase 2: all on 19.5 ms; no entry
 // prefetch 21.9, one pair line 20.5, no pair prefetch 22.1; pairs prefetched
 // two steps ahead instead of one 19.9)
@@ -201,7 +214,7 @@ __device__ __forceinline__ void xs2_item(const XsDesc &d, const XsParams &p, lon
   const long long n_u = (long long)p.n_iso * p.n_gp, UB = d.ubins;
   const double du = 1.0 / p.bins;
   const uint32_t sbase = (uint32_t)__cvta_generic_to_shared(ens_dsmem);  // the shared window base, once
-  for (long long sl = s0 + threadIdx.x; sl < s1; sl += kXs2T) {
+  for (long long sl = s0 + threadIdx.x; sl < s1; sl += Xs2T<GRID>::v) {
     int mat = 0;
 #pragma unroll
     for (int m = 1; m < 12; m++) mat += (sl >= (long long)d.mcnt[m]) ? 1 : 0;
@@ -303,13 +316,14 @@ __device__ __noinline__ void xs2_finish(const KParams &p, Ctx &c, const XsDesc *
   const unsigned long long pos = reinterpret_cast<const unsigned long long *>(misc + 8)[0];
   const unsigned long long *src = reinterpret_cast<const unsigned long long *>(c.out);
   unsigned long long *dst = reinterpret_cast<unsigned long long *>(p.stdout_cmp + pos);
-  for (uint32_t w = tid; w < sh->out_len / 8; w += kXs2T) dst[w] = src[w];
+  for (uint32_t w = tid; w < sh->out_len / 8; w += blockDim.x) dst[w] = src[w];
 }
 
 
 // items [p.item_base, p.item_base + p.n_items) of the group's queue, all of grid type GRID
 template <int GRID>
-__global__ void __launch_bounds__(kXs2T, Xs2Minb<GRID>::v) xs_items_kernel(const KParams p) {
+__global__ void __launch_bounds__(Xs2T<GRID>::v, Xs2Minb<GRID>::v) xs_items_kernel(const KParams p) {
+  constexpr int T = Xs2T<GRID>::v;
   const int tid = threadIdx.x;
   Ctx c{};
   c.sh_off = 0;
@@ -336,7 +350,7 @@ __global__ void __launch_bounds__(kXs2T, Xs2Minb<GRID>::v) xs_items_kernel(const
     {  // the instance's descriptor (phase 1's stores, an earlier kernel)
       const unsigned long long *src = reinterpret_cast<const unsigned long long *>(p.xs_desc + (size_t)j * kDescBytes);
       unsigned long long *dst = reinterpret_cast<unsigned long long *>(d);
-      for (int w = tid; w < (int)(sizeof(XsDesc) / 8); w += kXs2T) dst[w] = src[w];
+      for (int w = tid; w < (int)(sizeof(XsDesc) / 8); w += T) dst[w] = src[w];
     }
     __syncthreads();
     const int n_iso = d->n_iso, mx = xs_max_nucs(n_iso);
@@ -347,7 +361,7 @@ __global__ void __launch_bounds__(kXs2T, Xs2Minb<GRID>::v) xs_items_kernel(const
           nn[tid] = hm_num_nucs(n_iso, tid);
           thr[tid] = hm_threshold(tid);
         }
-        for (int x = tid; x < 12 * rw; x += kXs2T) {
+        for (int x = tid; x < 12 * rw; x += T) {
           const int m = x / rw, jj = x % rw, nm = hm_num_nucs(n_iso, m);
           const int jn = jj < nm ? jj : 0;
           mats[x] = (uint16_t)hm_nuc(m, jn);
@@ -586,6 +600,7 @@ cudaError_t launch_xs_init_items(int ctas, int threads, size_t smem, const KPara
 
 
 // ---- split phases, phase 2 of RSBench-style instances (kind 3) ----------
+constexpr int kRs2T = 256;  // threads per CTA
 // Items of kRsItemLookups sorted lookups of one instance; per item the
 // instance's pole / window offsets and concentrations (phase 1 copied them
 // to its arena) are staged in shared memory and every lookup is RsApp::lookup
@@ -669,10 +684,10 @@ __device__ __noinline__ void rs2_finish(const KParams &p, Ctx &c, const RsDesc *
   const unsigned long long pos = reinterpret_cast<const unsigned long long *>(misc + 8)[0];
   const unsigned long long *src = reinterpret_cast<const unsigned long long *>(c.out);
   unsigned long long *dst = reinterpret_cast<unsigned long long *>(p.stdout_cmp + pos);
-  for (uint32_t w = tid; w < sh->out_len / 8; w += kXs2T) dst[w] = src[w];
+  for (uint32_t w = tid; w < sh->out_len / 8; w += kRs2T) dst[w] = src[w];
 }
 
-__global__ void __launch_bounds__(kXs2T, ENS_RS2_MINB) rs_items_kernel(const KParams p) {
+__global__ void __launch_bounds__(kRs2T, ENS_RS2_MINB) rs_items_kernel(const KParams p) {
   const int tid = threadIdx.x;
   Ctx c{};
   c.sh_off = 0;
@@ -702,7 +717,7 @@ __global__ void __launch_bounds__(kXs2T, ENS_RS2_MINB) rs_items_kernel(const KPa
     if (j != cached_j) {  // a new instance: its descriptor and shared tables
       const unsigned long long *src = reinterpret_cast<const unsigned long long *>(p.xs_desc + (size_t)j * kDescBytes);
       unsigned long long *dst = reinterpret_cast<unsigned long long *>(d);
-      for (int w = tid; w < (int)(sizeof(RsDesc) / 8); w += kXs2T) dst[w] = src[w];
+      for (int w = tid; w < (int)(sizeof(RsDesc) / 8); w += kRs2T) dst[w] = src[w];
       __syncthreads();
       const int n_nuc = d->n_nuc, mx = xs_max_nucs(n_nuc);
       if (n_nuc != cached) {
@@ -712,11 +727,11 @@ __global__ void __launch_bounds__(kXs2T, ENS_RS2_MINB) rs_items_kernel(const KPa
       __syncthreads();
       const int *pg = reinterpret_cast<const int *>(d->poff), *wg = reinterpret_cast<const int *>(d->woff);
       const double *cg = reinterpret_cast<const double *>(d->concs);
-      for (int i = tid; i <= n_nuc; i += kXs2T) {
+      for (int i = tid; i <= n_nuc; i += kRs2T) {
         poff[i] = pg[i];
         woff[i] = wg[i];
       }
-      for (int x = tid; x < 12 * mx; x += kXs2T) concs[x] = cg[x];
+      for (int x = tid; x < 12 * mx; x += kRs2T) concs[x] = cg[x];
       cached_j = j;
       __syncthreads();
     }
@@ -732,7 +747,7 @@ __global__ void __launch_bounds__(kXs2T, ENS_RS2_MINB) rs_items_kernel(const KPa
     double *dmp = p.dump ? p.dump + (size_t)d->k * p.dump_rows * 8 : nullptr;
     unsigned long long ver = 0, bsum = 0, terms = 0, near = 0;
     double fsum = 0.0, fabs_ = 0.0;
-    for (long long sl = s0 + tid; sl < s1; sl += kXs2T) {
+    for (long long sl = s0 + tid; sl < s1; sl += kRs2T) {
       int mat = 0;
 #pragma unroll
       for (int m = 1; m < 12; m++) mat += (sl >= (long long)d->mcnt[m]) ? 1 : 0;
@@ -781,7 +796,15 @@ __global__ void __launch_bounds__(kXs2T, ENS_RS2_MINB) rs_items_kernel(const KPa
   }
 }
 
-int xs_items_threads() { return kXs2T; }
+// threads per CTA of the phase-2 kernel of an item kind: XS grid types 0..2, RS 3
+int xs_items_threads(int kind) {
+  switch (kind) {
+    case XS_HASH: return Xs2T<XS_HASH>::v;
+    case XS_UNIONIZED: return Xs2T<XS_UNIONIZED>::v;
+    case XS_NUCLIDE: return Xs2T<XS_NUCLIDE>::v;
+  }
+  return kRs2T;
+}
 
 // phase-2 kernel of an item kind: XS grid types 0..2, RS 3
 static const void *xs_items_fn(int grid) {
@@ -801,7 +824,7 @@ cudaError_t xs_items_occupancy(int grid, int *ctas) {
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)items_smem(grid));
   if (e != cudaSuccess) return e;
   int per_sm = 0, dev = 0, sms = 0;
-  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kXs2T, items_smem(grid));
+  e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, xs_items_threads(grid), items_smem(grid));
   if (e == cudaSuccess) e = cudaGetDevice(&dev);
   if (e == cudaSuccess) e = cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
   *ctas = per_sm * sms;
@@ -814,7 +837,8 @@ cudaError_t launch_xs_items(int grid_type, int ctas, const KParams &p, cudaStrea
   cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)items_smem(grid_type));
   if (e != cudaSuccess) return e;
   void *args[] = {const_cast<KParams *>(&p)};
-  return cudaLaunchKernel(fn, dim3((unsigned)ctas), dim3((unsigned)kXs2T), args, items_smem(grid_type), st);
+  return cudaLaunchKernel(fn, dim3((unsigned)ctas), dim3((unsigned)xs_items_threads(grid_type)), args,
+                          items_smem(grid_type), st);
 }
 
 }  // namespace ens

@@ -72,7 +72,7 @@ cudaError_t group_occupancy(uint32_t app, int T, int m, int cs, size_t smem, int
 // split phases, phase 2 (kernels_items.cu): the XS lookup-item kernel
 cudaError_t launch_xs_items(int grid_type, int ctas, const KParams &p, cudaStream_t st);
 cudaError_t xs_items_occupancy(int grid_type, int *ctas);
-int xs_items_threads();
+int xs_items_threads(int kind);
 cudaError_t launch_xs_init_items(int ctas, int threads, size_t smem, const KParams &p, cudaStream_t st);
 cudaError_t xs_init_items_occupancy(int threads, size_t smem, int *ctas);
 uint32_t xs_init_smem_off();
