@@ -357,9 +357,9 @@ ENS_HD int xs_sort_fine_items(const XsParams &p) {
   const int kb = xs_lk_bits(xs_lk_chunk(p));
   return ((12 << xs_lk_cbits(kb)) + kXsFineGroup - 1) / kXsFineGroup;
 }
-// shared memory of the sort items: the coarse counters (12 << 8 u32) or 8
-// warps' fine counters (1 << (18 - 8) u32 each)
-constexpr uint32_t kXsLkSortSmem = 8u * 1024u * 4u;
+// shared memory of the sort items: the coarse counters (12 << 8 u32) or up to
+// 16 warps' fine counters (1 << (18 - 8) u32 each)
+constexpr uint32_t kXsLkSortSmem = 16u * 1024u * 4u;
 ENS_HD bool xs_split_ok(const XsParams &p) { return !p.history && p.lookups > 0 && p.lookups <= kXsLkChunk; }
 ENS_HD long long xs_items(const XsParams &p) {
   return xs_split_ok(p) ? (p.lookups + kXsItemLookups - 1) / kXsItemLookups : 0;

@@ -458,7 +458,7 @@ __device__ __forceinline__ void cta_set_flag(uint32_t *f, uint32_t v) {
   }
 }
 
-__global__ void __launch_bounds__(256, 2) xs_init_items_kernel(const KParams p) {
+__global__ void __launch_bounds__(kXsInitThreads, 2) xs_init_items_kernel(const KParams p) {
   const int tid = threadIdx.x, T = blockDim.x;
   Ctx c{};
   c.sh_off = 0;

@@ -83,6 +83,10 @@ constexpr uint32_t kInitSyncBytes = 128;  // XsInitSync (kernels_items.cu)
 constexpr uint32_t kXsCountItem = 0x80000000u;    // | chunk: count lookups
 constexpr uint32_t kXsScatterItem = 0x40000000u;  // | chunk: scatter lookups
 constexpr uint32_t kXsFineItem = 0x20000000u;     // | group: sort coarse buckets
-constexpr int kXsInitThreads = 256;  // init-item kernel block (launch bounds 256 x 2 CTAs/SM)
+#ifndef ENS_XS_INIT_T
+#define ENS_XS_INIT_T 256
+#endif
+constexpr int kXsInitThreads = ENS_XS_INIT_T;  // init-item kernel block (launch bounds: 2 CTAs/SM; C2's 1b:
+                                               // 256 8.07 ms, 320 8.27, 384 8.45 at 80 registers)
 
 }  // namespace ens
