@@ -119,3 +119,14 @@ def test_split_lookup_sort_items(oracle):
         keys = {(r[0], r[1]): r for r in od}
         for r in gd:
             assert np.array_equal(np.asarray(keys[(r[0], r[1])]).view(np.uint64), r.view(np.uint64))
+
+
+def test_split_largest_chunk(oracle):
+    # xs_split_ok's limit: 2^22 lookups (64 count / scatter items, kb = 18: coarse 8 + fine 10
+    # energy bits) is split; one more lookup runs fused over two sorted chunks
+    lines = ["xsbench -s small -g 200 -l 4194304 -G hash -h 100 -r 41",
+             "xsbench -s small -g 200 -l 4194305 -G hash -h 100 -r 42"]
+    g, info = run(lines, threads=512)
+    assert info.kernel_launches > info.n_groups  # the first instance's phase-2 kernel ran
+    o = oracle.run_text("".join(l + "\n" for l in lines))
+    assert_parity(g, o)
