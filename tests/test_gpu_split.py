@@ -130,3 +130,23 @@ def test_split_largest_chunk(oracle):
     assert info.kernel_launches > info.n_groups  # the first instance's phase-2 kernel ran
     o = oracle.run_text("".join(l + "\n" for l in lines))
     assert_parity(g, o)
+
+
+def test_split_column_paths(oracle):
+    # phase 1b's hash column: shared-memory histogram (bins < 65536 and it fits), the global-column
+    # path (bins >= 65536), and the arena-scratch sort (n_gp > 16384) with each
+    lines = ["xsbench -s small -g 3000 -l 20000 -G hash -h 70000 -r 51",
+             "xsbench -s small -g 18000 -l 20000 -G hash -h 70000 -r 52",
+             "xsbench -s small -g 18000 -l 20000 -G hash -h 5000 -r 53",
+             "xsbench -s small -g 4000 -l 20000 -G hash -h 3 -r 54",
+             "xsbench -s small -g 2 -l 5000 -G hash -h 1000 -r 55"]
+    text = "".join(l + "\n" for l in lines)
+    g, info = run(lines, threads=256, split=True, dump_rows=20000)
+    assert info.kernel_launches > info.n_groups
+    o = oracle.run_text(text, dump=20000)
+    assert_parity(g, o)
+    for k in range(len(lines)):
+        gd = g.dump[k]
+        gd = gd[~np.all(gd == 0, axis=1)]
+        gs, os_ = gd[np.lexsort((gd[:, 1], gd[:, 0]))], o.dumps[k][np.lexsort((o.dumps[k][:, 1], o.dumps[k][:, 0]))]
+        assert gs.shape == os_.shape and np.array_equal(gs.view(np.uint64), os_.view(np.uint64)), lines[k]
