@@ -196,9 +196,14 @@ struct XsApp {
     if (init_items) {
     } else if (p.grid == XS_UNIONIZED) {
       const bool warp_path = xs_warp_union(p) && !(c.flags & ENS_F_GENERIC);
-      if (!warp_path && !xs_smem_nb(p)) init(c, p, L, S, c.csize > 1);  // block-wide, striped over the team
-      else if (c.crank == 0 && !(warp_path && init_warp(c, p, L, S)))
-        init(c, p, L, S, false);  // one CTA builds the union (shared-memory counters / warp-path overflow)
+      if (!warp_path && !xs_smem_nb(p)) {
+        init(c, p, L, S, c.csize > 1);  // block-wide, striped over the team
+      } else {
+        // the warp path striped over the team's CTAs (team-uniform result); on a
+        // chunk overflow, or with shared-memory counters, one CTA builds the union
+        const bool ok = warp_path && init_warp(c, p, L, S);
+        if (!ok && c.crank == 0) init(c, p, L, S, false);
+      }
     } else {
       init_nuc(c, p, L, S);  // nuclides striped over the team's CTAs
     }
@@ -1049,19 +1054,20 @@ struct XsApp {
       asm volatile("cp.async.commit_group;" ::: "memory");
     };
     int buf = 0;
-    if (warp < NC) {
-      load(warp);
+    const int gw = warp + (int)c.crank * nw, gn = nw * (int)c.csize;  // chunks striped over the team's warps
+    if (gw < NC) {
+      load(gw);
       stage(0);
     }
-    for (int ch = warp; ch < NC; ch += nw, buf ^= 1) {
+    for (int ch = gw; ch < NC; ch += gn, buf ^= 1) {
       const int m = m_n;
       const long long e0 = e0_n;
-      if (ch + nw < NC) load(ch + nw);
+      if (ch + gn < NC) load(ch + gn);
       asm volatile("cp.async.wait_all;" ::: "memory");
       __syncwarp();
       if (m > kXsChunkCap) {
         ovf = 1;
-        if (ch + nw < NC) stage(buf ^ 1);
+        if (ch + gn < NC) stage(buf ^ 1);
         continue;
       }
       const unsigned long long *Eg = Eg0 + buf * kXsChunkCap;
@@ -1101,7 +1107,7 @@ struct XsApp {
         uf[b] = (uint32_t)(v > 0 ? v : 0);
       }
       phase_mark_if(trc, c, 15);
-      if (ch + nw < NC) stage(buf ^ 1);  // the next chunk's gather overlaps this chunk's rows
+      if (ch + gn < NC) stage(buf ^ 1);  // the next chunk's gather overlaps this chunk's rows
       chunk_sweep<Q>(Ou, m, ig, e0, ip, n_gp, lane, vq, wq);
       __syncwarp();
       phase_mark_if(trc, c, 9);
@@ -1122,15 +1128,15 @@ struct XsApp {
     const Affine J32 = lcg_pow(6ULL * 32ULL);
     const uint64_t gseed = p.gseed;
 
-    // (N) nuclides, a warp each
-    for (int x = tid; x < (NC + 1) * (ip - n_iso); x += T)
+    // (N) nuclides, a warp each (striped over the team's CTAs)
+    for (int x = tid + (int)c.crank * T; x < (NC + 1) * (ip - n_iso); x += T * (int)c.csize)
       ust[(x / (ip - n_iso)) * ip + n_iso + x % (ip - n_iso)] = 0;  // pad columns
     {
       char *scr = ens_smem(c) + S.nbkt + (size_t)warp * kXsNucScr;
       uint32_t *K = (uint32_t *)scr;
       uint16_t *J = (uint16_t *)(scr + kXsWarpGp * 4);
       uint32_t *cnt = (uint32_t *)(scr + kXsWarpGp * 6);
-      for (int i = warp; i < n_iso && warp < nw; i += nw) {
+      for (int i = warp + (int)c.crank * nw; i < n_iso && warp < nw; i += nw * (int)c.csize) {
         const uint32_t r0 = (uint32_t)i * (uint32_t)n_gp;
         for (int b = lane; b < kXsNucBkt; b += 32) cnt[b] = 0;
         __syncwarp();
@@ -1187,12 +1193,12 @@ struct XsApp {
         phase_mark_if(trc, c, 5);
       }
     }
-    __syncthreads();
+    team_sync(c);  // every nuclide's sorted run and ustart column, team-wide
     phase_mark_if(trc, c, 6);
 
-    // (U) union chunks, a warp each
+    // (U) union chunks, a warp each (striped over the team's CTAs)
     const unsigned ovf = ip <= 128 ? union_chunks<3, 1>(c, p, L, S) : union_chunks<12, 3>(c, p, L, S);
-    const int bad = __syncthreads_or((int)ovf);
+    const bool bad = team_any(c, (int)ovf);
     phase_mark_if(trc, c, 8);
     return !bad;
   }

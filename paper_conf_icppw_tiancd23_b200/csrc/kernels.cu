@@ -396,6 +396,10 @@ bool app_size(uint32_t app, int argc, const char *const *argv, int T, int cs, ui
 }
 
 static cudaError_t set_smem(const void *fn, size_t smem) {
+  if (kMaxTeamCtas > 8) {  // clusters of up to 16 CTAs (non-portable size)
+    const cudaError_t e = cudaFuncSetAttribute(fn, cudaFuncAttributeNonPortableClusterSizeAllowed, 1);
+    if (e != cudaSuccess) return e;
+  }
   if (smem == 0) return cudaSuccess;
   return cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
 }

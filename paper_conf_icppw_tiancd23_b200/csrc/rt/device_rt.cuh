@@ -94,7 +94,10 @@ ENS_HD uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 // ---------------------------------------------------------------------------
 // per-instance context (identical copy in every thread of the block)
 // ---------------------------------------------------------------------------
-constexpr int kMaxTeamCtas = 8;  // portable thread-block-cluster size
+#ifndef ENS_MAX_TEAM
+#define ENS_MAX_TEAM 8
+#endif
+constexpr int kMaxTeamCtas = ENS_MAX_TEAM;  // thread-block-cluster size (8 portable; 16 non-portable)
 constexpr int kMaxSubTeams = 8;  // M instances per CTA (named barriers 1..8)
 
 // Barrier of the threads running this instance.  With M instances per CTA
@@ -355,6 +358,17 @@ __device__ inline unsigned long long team_sum_u64(Ctx &c, unsigned long long v) 
     for (uint32_t r = 0; r < c.csize; r++) t += ens_sh(c)->team_u[r];
   team_sync(c);
   return t;
+}
+// whether any thread of the team has v != 0 (valid in every thread of every CTA)
+__device__ inline bool team_any(Ctx &c, int v) {
+  v = __syncthreads_or(v);
+  if (c.csize == 1) return v != 0;
+  if (threadIdx.x == 0) *cta_shared(&ens_sh(c)->team_u[c.crank], 0) = (unsigned long long)(v != 0);
+  team_sync(c);
+  unsigned long long t = 0;
+  for (uint32_t r = 0; r < c.csize; r++) t |= *cta_shared(&ens_sh(c)->team_u[r], 0);
+  team_sync(c);  // team_u is reused
+  return t != 0;
 }
 __device__ inline double team_sum_f64(Ctx &c, double v) {
   v = block_sum_f64(ens_sh(c), v);
