@@ -95,7 +95,7 @@ ENS_HD uint64_t align_up(uint64_t x, uint64_t a) { return (x + a - 1) / a * a; }
 // per-instance context (identical copy in every thread of the block)
 // ---------------------------------------------------------------------------
 #ifndef ENS_MAX_TEAM
-#define ENS_MAX_TEAM 8
+#define ENS_MAX_TEAM 16
 #endif
 constexpr int kMaxTeamCtas = ENS_MAX_TEAM;  // thread-block-cluster size (8 portable; 16 non-portable)
 constexpr int kMaxSubTeams = 8;  // M instances per CTA (named barriers 1..8)
