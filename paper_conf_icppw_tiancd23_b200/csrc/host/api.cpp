@@ -508,8 +508,11 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
       // TSTAR (1024 instances) and C1 (12 items) stay fused.
       int fill = 0;
       for (int kd = 0; kd < 4; kd++) fill = std::max(fill, g.grid2[kd]);
+      // RS groups split at any instance count: the item kernel's read-only loads and its own
+      // register budget beat the fused body (C5's 1024 RS lines: 26.1 -> 23.7 ms)
       g.split = !g.items.empty() && (((c->flags & ENS_F_SPLIT_PHASES) != 0) ||
-                                     ((int64_t)g.kmap.size() < (int64_t)ctas && (int64_t)g.items.size() >= fill));
+                                     (((int64_t)g.kmap.size() < (int64_t)ctas || ap == APP_RSBENCH) &&
+                                      (int64_t)g.items.size() >= fill));
       if (!g.split) {
         g.items.clear();
         for (int kd = 0; kd < 4; kd++) g.kind_n[kd] = 0;
