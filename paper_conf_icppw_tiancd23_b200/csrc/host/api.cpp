@@ -508,10 +508,23 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
       // TSTAR (1024 instances) and C1 (12 items) stay fused.
       int fill = 0;
       for (int kd = 0; kd < 4; kd++) fill = std::max(fill, g.grid2[kd]);
-      // RS groups split at any instance count: the item kernel's read-only loads and its own
-      // register budget beat the fused body (C5's 1024 RS lines: 26.1 -> 23.7 ms)
+      // RS groups, and XS groups with per-nuclide table items (hash / nuclide grids), split at
+      // any instance count: the item kernels' read-only loads, register budgets and all-SM table
+      // builds beat the fused body (C5's 1024 RS lines: 26.1 -> 23.7 ms; 300 C2 lines: 240 -> 128 ms);
+      // unionized XS groups only below the resident CTAs (T*: 8.94 split vs 8.92 ms fused)
+      bool any_init = false;
+      if (ap == APP_XSBENCH)
+        for (size_t x = 0; x < g.kmap.size() && !any_init; x++) {
+          int argc;
+          const char *const *argv;
+          ens_args_get(a, (int)P.line_of_k[g.kmap[x]], &argc, &argv);
+          int ni = 0, ns = 0, nf = 0;
+          uint32_t sm3 = 0;
+          app_init_scratch(ap, argc, argv, &ni, &ns, &nf, &sm3);
+          any_init = ni > 0;
+        }
       g.split = !g.items.empty() && (((c->flags & ENS_F_SPLIT_PHASES) != 0) ||
-                                     (((int64_t)g.kmap.size() < (int64_t)ctas || ap == APP_RSBENCH) &&
+                                     (((int64_t)g.kmap.size() < (int64_t)ctas || ap == APP_RSBENCH || any_init) &&
                                       (int64_t)g.items.size() >= fill));
       if (!g.split) {
         g.items.clear();
