@@ -599,6 +599,25 @@ cudaError_t launch_xs_init_items(int ctas, int threads, size_t smem, const KPara
 }
 
 
+// TMA bulk copy global -> this CTA's shared memory, completing on mbarrier
+// `mbar` (16-B aligned addresses, size a multiple of 16; one thread)
+__device__ __forceinline__ void bulk_g2s(void *sdst, const void *gsrc, uint32_t bytes, uint32_t mbar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          (uint32_t)__cvta_generic_to_shared(sdst)),
+      "l"(gsrc), "r"(bytes), "r"(mbar)
+      : "memory");
+}
+// every thread waits for the mbarrier's phase `parity` to complete
+__device__ __forceinline__ void mbar_wait(uint32_t mbar, uint32_t parity) {
+  uint32_t done = 0;
+  while (!done)
+    asm volatile("{ .reg .pred p; mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2; selp.u32 %0, 1, 0, p; }"
+                 : "=r"(done)
+                 : "r"(mbar), "r"(parity)
+                 : "memory");
+}
+
 // ---- split phases, phase 2 of RSBench-style instances (kind 3) ----------
 constexpr int kRs2T = 256;  // threads per CTA
 // Items of kRsItemLookups sorted lookups of one instance; per item the
@@ -707,6 +726,14 @@ __global__ void __launch_bounds__(kRs2T, ENS_RS2_MINB) rs_items_kernel(const KPa
   uint32_t *am = misc + 2;
   int cached = 0;  // n_nuc of the material lists in shared memory
   uint32_t cached_j = 0xffffffffu;
+  // the staging mbarrier (misc[12..13]) and its phase parity
+  const uint32_t mbar = (uint32_t)__cvta_generic_to_shared(misc + 12);
+  uint32_t mphase = 0;
+  if (tid == 0) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], 1;" ::"r"(mbar) : "memory");
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  __syncthreads();
   for (;;) {
     if (tid == 0) misc[0] = atomicAdd(p.counter2, 1u);
     if (tid < 4) am[tid] = 0u;
@@ -725,13 +752,20 @@ __global__ void __launch_bounds__(kRs2T, ENS_RS2_MINB) rs_items_kernel(const KPa
         cached = n_nuc;
       }
       __syncthreads();
-      const int *pg = reinterpret_cast<const int *>(d->poff), *wg = reinterpret_cast<const int *>(d->woff);
-      const double *cg = reinterpret_cast<const double *>(d->concs);
-      for (int i = tid; i <= n_nuc; i += kRs2T) {
-        poff[i] = pg[i];
-        woff[i] = wg[i];
+      // the instance's pole / window offsets and concentrations (phase 1's arena copies,
+      // 256-B aligned regions) staged by the TMA engine: three bulk global->shared copies
+      // completing on one mbarrier, while the threads wait on its phase
+      if (tid == 0) {
+        const uint32_t bo = ((uint32_t)(n_nuc + 1) * 4u + 15u) & ~15u, bc = 12u * (uint32_t)mx * 8u;
+        asm volatile("fence.proxy.async.shared::cta;" ::: "memory");  // earlier generic reads of the buffers
+        asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(mbar), "r"(2u * bo + bc)
+                     : "memory");
+        bulk_g2s(poff, reinterpret_cast<const void *>(d->poff), bo, mbar);
+        bulk_g2s(woff, reinterpret_cast<const void *>(d->woff), bo, mbar);
+        bulk_g2s(concs, reinterpret_cast<const void *>(d->concs), bc, mbar);
       }
-      for (int x = tid; x < 12 * mx; x += kRs2T) concs[x] = cg[x];
+      mbar_wait(mbar, mphase);
+      mphase ^= 1u;
       cached_j = j;
       __syncthreads();
     }
