@@ -508,12 +508,18 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
       // TSTAR (1024 instances) and C1 (12 items) stay fused.
       int fill = 0;
       for (int kd = 0; kd < 4; kd++) fill = std::max(fill, g.grid2[kd]);
-      // RS groups, and XS groups with per-nuclide table items (hash / nuclide grids), split at
-      // any instance count: the item kernels' read-only loads, register budgets and all-SM table
-      // builds beat the fused body (C5's 1024 RS lines: 26.1 -> 23.7 ms; 300 C2 lines: 240 -> 128 ms);
-      // unionized XS groups only below the resident CTAs (T*: 8.94 split vs 8.92 ms fused)
+      // RS groups, and XS groups with per-nuclide table items (hash / nuclide grids) whose
+      // instances are not small, split at any instance count: the item kernels' read-only
+      // loads, register budgets and all-SM table builds beat the fused body (C5's 1024 RS lines:
+      // 26.1 -> 23.7 ms; 300 C2 lines: 240 -> 128 ms; 600 small 11303-point lines with 200k
+      // lookups: 42.6 -> 29.9 ms) — but 1024 small 1000-point lines with 10k lookups run fused
+      // faster (6.8 vs 7.3 ms): XS groups below an average app_cost of 2^20 stay fused;
+      // unionized XS groups split only below the resident CTAs (T*: 8.94 split vs 8.92 fused)
+      double mean_cost = 0.0;
+      for (double w : g.cost) mean_cost += w;
+      mean_cost /= std::max<size_t>(1, g.cost.size());
       bool any_init = false;
-      if (ap == APP_XSBENCH)
+      if (ap == APP_XSBENCH && mean_cost >= 1048576.0)
         for (size_t x = 0; x < g.kmap.size() && !any_init; x++) {
           int argc;
           const char *const *argv;
