@@ -90,6 +90,13 @@ def test_auto_policy():
     assert info.kernel_launches >= 2
     _, info = run(workloads.tstar(300), threads=512)
     assert info.kernel_launches == 1
+    # above the resident CTAs: large hash instances split, small ones stay fused; RS splits
+    _, info = run(workloads.c2(200, lookups=100000), threads=512)
+    assert info.kernel_launches >= 3
+    _, info = run([f"xsbench -s small -g 1000 -l 10000 -G hash -h 1000 -r {i}" for i in range(300)], threads=512)
+    assert info.kernel_launches == 1
+    _, info = run([f"rsbench -s small -l 2000 -p 100 -w 10 -r {i}" for i in range(400)], threads=512)
+    assert info.kernel_launches == 2
 
 
 # phase 1b's lookup sort in items: chunk boundaries (kXsSortChunk = 65536 lookups per count /
