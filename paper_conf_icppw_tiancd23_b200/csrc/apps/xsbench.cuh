@@ -447,7 +447,8 @@ struct XsApp {
       }
       __syncthreads();
       phase_mark_if(trc, c, 1);
-      global_exclusive_scan(nb, nbn, ens_sh(c));
+      if (SMK) smem_scan(nb, nbn, ens_sh(c));
+      else global_exclusive_scan(nb, nbn, ens_sh(c));
       phase_mark_if(trc, c, 2);
       {  // scatter {key, j} in shared memory, four atomics in flight
         uint64_t s = jump6(jt, r0 + (uint32_t)tid, p.gseed);
@@ -580,7 +581,7 @@ struct XsApp {
             if (bf < p.bins) atomicAdd(&colp[bf], 1);
           }
           __syncthreads();
-          global_exclusive_scan<true>(reinterpret_cast<uint32_t *>(colp), p.bins, ens_sh(c));
+          smem_scan<true>(reinterpret_cast<uint32_t *>(colp), p.bins, ens_sh(c));
         } else {
           for (int k0 = tid; k0 < n_gp; k0 += U * T) {
             unsigned long long ek[U], ek1[U];

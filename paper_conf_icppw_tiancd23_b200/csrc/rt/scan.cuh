@@ -67,4 +67,50 @@ __device__ inline void global_exclusive_scan(uint32_t *a, long long n, Shared *s
   }
 }
 
+// the same prefix sum of a shared-memory array in one pass: thread t owns the
+// contiguous segment [tK, tK + K), K = ceil(n / T) rounded up to odd (the
+// lanes' segments then start in distinct banks: no conflicts), so the whole
+// array costs three barriers instead of three per 8T-element tile.  The
+// caller has synchronised the array's producers; returns after a barrier.
+template <bool INCL = false>
+__device__ inline void smem_scan(uint32_t *a, int n, Shared *sh) {
+  const int tid = threadIdx.x, T = blockDim.x, lane = tid & 31, w = tid >> 5, nw = T >> 5;
+  const int K = ((n + T - 1) / T) | 1;
+  const int b0 = tid * K;
+  uint32_t sum = 0;
+#pragma unroll 4
+  for (int i = 0; i < K; i++) {
+    const int x = b0 + i;
+    if (x < n) sum += a[x];
+  }
+  uint32_t inc = sum;
+  for (int o = 1; o < 32; o <<= 1) {
+    const uint32_t t = __shfl_up_sync(0xffffffffu, inc, o);
+    if (lane >= o) inc += t;
+  }
+  if (lane == 31) sh->red_u[w] = inc;
+  __syncthreads();
+  if (w == 0) {
+    const unsigned long long t = lane < nw ? sh->red_u[lane] : 0ULL;
+    unsigned long long ti = t;
+    for (int o = 1; o < 32; o <<= 1) {
+      const unsigned long long u = __shfl_up_sync(0xffffffffu, ti, o);
+      if (lane >= o) ti += u;
+    }
+    if (lane < nw) sh->red_u[lane] = ti - t;  // exclusive warp offsets
+  }
+  __syncthreads();
+  uint32_t run = (uint32_t)sh->red_u[w] + inc - sum;
+#pragma unroll 4
+  for (int i = 0; i < K; i++) {
+    const int x = b0 + i;
+    if (x < n) {
+      const uint32_t t = a[x];
+      a[x] = INCL ? run + t : run;
+      run += t;
+    }
+  }
+  __syncthreads();
+}
+
 }  // namespace ens
