@@ -157,3 +157,15 @@ def test_split_column_paths(oracle):
         gd = gd[~np.all(gd == 0, axis=1)]
         gs, os_ = gd[np.lexsort((gd[:, 1], gd[:, 0]))], o.dumps[k][np.lexsort((o.dumps[k][:, 1], o.dumps[k][:, 0]))]
         assert gs.shape == os_.shape and np.array_equal(gs.view(np.uint64), os_.view(np.uint64)), lines[k]
+
+
+def test_split_above_resident_ctas_parity(oracle):
+    # the policy's any-N splits (RS groups; XS hash groups of non-small instances) against the
+    # oracle, with more instances than resident CTAs, next to a small-hash group that stays fused
+    lines = ([f"xsbench -s large -g 2000 -l 20000 -G hash -h 1500 -r {200 + i}" for i in range(160)] +
+             [f"rsbench -s small -l 600 -p 40 -w 8 {'-d ' if i % 4 == 0 else ''}-r {300 + i}" for i in range(300)] +
+             [f"xsbench -s small -g 300 -l 2000 -G hash -h 100 -r {700 + i}" for i in range(200)])
+    g, info = run(lines, threads=512)
+    assert info.kernel_launches >= 5  # XS: ensemble + init items + hash items; RS: ensemble + items
+    o = oracle.run_text("".join(l + "\n" for l in lines))
+    assert_parity(g, o)
