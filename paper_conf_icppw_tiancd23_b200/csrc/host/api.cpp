@@ -467,6 +467,18 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
         e = group_occupancy(ap, g.T, 1, cs, g.dyn(), &teams);
         if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters");
         if (teams <= 0) cs = 1, teams = ctas;
+        // an automatic team size whose clusters cannot all be resident at once (a GPC holds only
+        // so many 16- or 8-CTA clusters) would run the ensemble in two waves: halve it until
+        // every instance has a resident team (XS at N = 8: 0.47 ms on 7 16-CTA teams)
+        while (!c->team_ctas && !c->grid_blocks && cs > 1 && (int64_t)teams < (int64_t)g.kmap.size()) {
+          cs >>= 1;
+          teams = ctas;
+          if (cs > 1) {
+            e = group_occupancy(ap, g.T, 1, cs, g.dyn(), &teams);
+            if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters");
+            if (teams <= 0) cs = 1, teams = ctas;
+          }
+        }
       }
       int grid = c->grid_blocks ? std::max(1, c->grid_blocks / cs) : teams;
       grid = (int)std::min<int64_t>(grid, (int64_t)g.kmap.size());

@@ -1,6 +1,6 @@
 """SWEEP: the paper's Fig. 6 measurement on B200.
 
-    python tools/sweep.py [--out profiles/sweep_r1.json] [--max-n 1024] [--reps 3]
+    python tools/sweep.py [--out profiles/sweep_r1.json] [--max-n 1024] [--reps 3] [--auto]
 
 For each app and thread limit T, the ensemble of N instances (distinct seeds)
 is launched N = 1, 2, 4, ... and timed with CUDA events on its stream (median
@@ -10,7 +10,9 @@ speedup T1*N/TN, T1 = the same launch at N = 1 with the same T
 (P:549-554).  Teams are one CTA (the paper's team = one thread block,
 P:313-318), M = 1, every instance start to finish in the one ensemble kernel
 (ENS_F_FUSED: the paper's mapping).  Also reported: instances/s and busy SMs (from the
-per-instance smid of the records).
+per-instance smid of the records).  With --auto the launches use the product's own mapping
+instead (cluster teams, split phases, longest-first queue: the library's defaults), so the
+curve shows what the framework delivers at each N next to the paper's mapping.
 """
 import argparse
 import json
@@ -32,9 +34,10 @@ APPS = {
 }
 
 
-def time_launch(lines, threads, reps):
+def time_launch(lines, threads, reps, auto=False):
     text = "".join(l + "\n" for l in lines)
-    e = Ensemble(Args.parse(text), app="auto", threads=threads, team_ctas=1, timestamps=True, fused=True).launch()
+    kw = {} if auto else dict(team_ctas=1, fused=True)
+    e = Ensemble(Args.parse(text), app="auto", threads=threads, timestamps=True, **kw).launch()
     torch.cuda.synchronize()
     ts = []
     for _ in range(reps):
@@ -59,6 +62,7 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--threads", default="32,256,1024")
     ap.add_argument("--apps", default=",".join(APPS))
+    ap.add_argument("--auto", action="store_true", help="the library's default mapping (not the paper's)")
     a = ap.parse_args()
     torch.cuda.set_device(0)
     ns = []
@@ -73,7 +77,7 @@ def main():
             t1 = None
             for n in ns:
                 lines = [tmpl.format(s=1 + i) for i in range(n)]
-                ms, ok, sms, Treal, grid = time_launch(lines, T, a.reps)
+                ms, ok, sms, Treal, grid = time_launch(lines, T, a.reps, a.auto)
                 if n == 1:
                     t1 = ms
                 row = {"app": app, "T_limit": T, "T": Treal, "N": n, "grid": grid, "ms": ms, "ok": ok,
@@ -81,7 +85,10 @@ def main():
                 rows.append(row)
                 print(f"{app:10s} T={Treal:5d} N={n:5d} grid={grid:5d} {ms:9.3f} ms  speedup {row['speedup']:8.2f}"
                       f"  sms {sms:3d}  ok={ok}", flush=True)
-    out = {"what": "T1*N/TN on one B200 (paper Fig. 6 metric, P:540-554); team = 1 CTA, fused; median of reps",
+    what = ("T1*N/TN on one B200 (paper Fig. 6 metric, P:540-554); the library's default mapping (cluster teams, "
+            "split phases); median of reps" if a.auto else
+            "T1*N/TN on one B200 (paper Fig. 6 metric, P:540-554); team = 1 CTA, fused; median of reps")
+    out = {"what": what,
            "paper_context": "up to 51x at 64 instances on an A100 40GB (P:44-45, P:639-640)",
            "device": torch.cuda.get_device_name(0), "apps": APPS, "rows": rows}
     os.makedirs(os.path.dirname(a.out), exist_ok=True)
