@@ -154,10 +154,14 @@ typedef struct {
   uint64_t arena_bytes;
   uint32_t stdout_bytes;
   uint32_t flags;
-  int32_t team_ctas;  /* CTAs per team for team-aware bodies (XSBench): 1, 2,
-                         4 or 8 (a thread-block cluster with distributed shared
-                         memory); 0 = auto (largest power of two <= 8 with
-                         n x team_ctas <= resident CTAs), ignored by other apps */
+  int32_t team_ctas;  /* CTAs per team for team-aware bodies (XSBench, RSBench):
+                         1..16 (a thread-block cluster with distributed shared
+                         memory; above 8 a non-portable cluster size; larger
+                         values are capped at 16); 0 = auto (the largest power
+                         of two <= 16 with n x team_ctas <= resident CTAs, then
+                         shrunk until every instance's cluster is resident, or
+                         sized for the heaviest instance of an uneven ensemble),
+                         ignored by other apps */
   int32_t instances_per_cta; /* M, the paper's (N/M, M, 1) block mapping
                          (P:393-404): M instances share one CTA, each on the
                          row threadIdx.y of block_threads/M threads with its

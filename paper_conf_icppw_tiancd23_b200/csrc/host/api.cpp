@@ -450,7 +450,7 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
       g.grid = std::max(grid, g.m);
     } else if (app_team_aware(ap) && !(c->flags & ENS_F_CLC)) {
       if (c->team_ctas > 0) {
-        while (cs * 2 <= c->team_ctas && cs < kMaxTeamCtas) cs *= 2;
+        cs = (int)std::min<uint32_t>(c->team_ctas, (uint32_t)kMaxTeamCtas);  // any cluster size up to the cap
       } else if (!c->grid_blocks) {
         while (cs < kMaxTeamCtas && (int64_t)g.kmap.size() * cs * 2 <= ctas) cs *= 2;
         // uneven ensembles: a team large enough that the heaviest instance
@@ -468,10 +468,11 @@ static int make_plan(ens_app app, const ens_args *a, const ens_launch_cfg *c, si
         if (e != cudaSuccess) return cuda_fail(e, "cudaOccupancyMaxActiveClusters");
         if (teams <= 0) cs = 1, teams = ctas;
         // an automatic team size whose clusters cannot all be resident at once (a GPC holds only
-        // so many 16- or 8-CTA clusters) would run the ensemble in two waves: halve it until
-        // every instance has a resident team (XS at N = 8: 0.47 ms on 7 16-CTA teams)
+        // so many 16- or 8-CTA clusters) would run the ensemble in two waves: shrink it (any
+        // size, not only powers of two) until every instance has a resident team (XS at N = 8:
+        // 0.47 ms on 7 16-CTA teams)
         while (!c->team_ctas && !c->grid_blocks && cs > 1 && (int64_t)teams < (int64_t)g.kmap.size()) {
-          cs >>= 1;
+          cs -= 1;
           teams = ctas;
           if (cs > 1) {
             e = group_occupancy(ap, g.T, 1, cs, g.dyn(), &teams);

@@ -118,7 +118,7 @@ def test_more_instances_than_blocks(oracle, grid):
     assert_parity(g, o)
 
 
-@pytest.mark.parametrize("team", [2, 4, 8, 16])
+@pytest.mark.parametrize("team", [2, 3, 4, 6, 8, 13, 16])
 def test_cluster_team_parity(oracle, team):
     """A team = a thread-block cluster of `team` CTAs (XS is team-aware): same results."""
     lines = [XS_CASES[0], XS_CASES[1], XS_CASES[2], XS_CASES[4], XS_CASES[10], "xsbench -s small -g 77 -l 999 -G hash -h 5 -r 2",
@@ -159,7 +159,7 @@ RS_UNEVEN = [f"rsbench -s small -l {L} -p {P} -w {W}{d} -r {i + 1}"
                                                (1500, 100, 50, " -d"), (50, 10, 5, ""), (700, 300, 30, "")])]
 
 
-@pytest.mark.parametrize("team", [0, 1, 2, 8, 16])
+@pytest.mark.parametrize("team", [0, 1, 2, 5, 8, 16])
 def test_rs_team_parity(oracle, team):
     """RS is team-aware: a cluster of CTAs stripes the pole/window draws and the sorted lookup
     batches; the auto team (0) sizes it for the heaviest instance of an uneven ensemble and the
@@ -174,7 +174,7 @@ def test_rs_chunk_boundary(oracle):
     assert_parity(g, o)
 
 
-@pytest.mark.parametrize("team", [1, 2, 8, 16])
+@pytest.mark.parametrize("team", [1, 2, 3, 8, 16])
 def test_xs_blockwide_union_team(oracle, team):
     """The block-wide unionized init (n_gp > 1024, counters in the arena) is striped over the
     team's CTAs (cluster barriers between passes): same union, index grid and records."""
@@ -185,7 +185,7 @@ def test_xs_blockwide_union_team(oracle, team):
     assert_parity(g, o)
 
 
-@pytest.mark.parametrize("team", [2, 8, 16])
+@pytest.mark.parametrize("team", [2, 5, 8, 16])
 def test_xs_warp_union_team(oracle, team):
     """The unionized warp-path init (n_gp <= 1024) striped over a team's CTAs: nuclides and
     union chunks on every CTA, a cluster barrier between, the chunk-overflow fallback decided
