@@ -249,6 +249,7 @@ struct XsLayout {
   uint64_t ufind;     // unionized: [xs_ubins] u32 union search table (private accelerator)
   uint64_t chist;     // unionized: [n_chunks][n_iso] u32 owner counts per sweep chunk
   uint64_t ustart;    // unionized, warp path: [NC+1][iso_pad] i32 #{k: E_i[k] < ch/NC}
+  uint64_t inv;       // unionized: [n_u] u32 record id at each sorted position (block path)
   uint64_t index;     // unionized [n_u][xs_iso_pad] int32 / hash [n_iso][bins+1] XsHashEnt
   uint64_t hcol;      // hash: [cs][bins+1] int32 column being built
   uint64_t nscr;      // hash / nuclide, n_gp > kXsSmemGp: [cs] x xs_nscr_bytes per-nuclide sort scratch
@@ -309,6 +310,7 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
     L.ufind = o; o = align_up(o + (uint64_t)xs_ubins(p) * 4, 256);
     L.chist = o; o = align_up(o + nch * (uint64_t)p.n_iso * 4, 256);
     if (xs_warp_union(p)) { L.ustart = o; o = align_up(o + (uint64_t)xs_iso_pad(p.n_iso) * (xs_uchunks(p) + 1) * 4, 256); }
+    L.inv = o; o = align_up(o + n_u * 4, 256);  // the block path (also under ENS_F_GENERIC)
     L.index = o; o = align_up(o + n_u * (uint64_t)xs_iso_pad(p.n_iso) * 4, 256);
   } else if (p.grid == XS_HASH) {
     L.index = o; o = align_up(o + (uint64_t)p.n_iso * (p.bins + 1) * 16, 256);

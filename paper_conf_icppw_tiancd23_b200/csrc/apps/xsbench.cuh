@@ -280,18 +280,6 @@ struct XsApp {
     if (r >> 24) s = jt[256 + ((r >> 24) & 63u)](s);
     return s;
   }
-  // record r at dst: E (the key's energy, draw 6r+1) and draws 6r+2..6r+6
-  __device__ static __forceinline__ void put_record(const Affine *jt, uint32_t r, unsigned long long ebits,
-                                                    uint64_t gseed, double *dst) {
-    uint64_t t = lcg_next(jump6(jt, r, gseed));  // past the energy draw
-    const double x1 = lcg_double(t), x2 = lcg_double(t), x3 = lcg_double(t), x4 = lcg_double(t),
-                 x5 = lcg_double(t);
-    double2 *d = reinterpret_cast<double2 *>(dst);  // evict-first: the tables stream past L2
-    __stcs(d, make_double2(__longlong_as_double((long long)ebits), x1));
-    __stcs(d + 1, make_double2(x2, x3));
-    __stcs(d + 2, make_double2(x4, x5));
-  }
-
   // sort keys[lo, hi) by (energy, record id): <= 8 in registers, else in place
   __device__ static __forceinline__ void sort_bucket(XsKey *keys, long long lo, long long hi) {
     const int cnt = (int)(hi - lo);
@@ -347,9 +335,11 @@ struct XsApp {
   // <= u_e} and row values clip(cnt_i(e) - 1, 0, n_gp-2).  Each union row
   // changes exactly one count (its owner's): the owner's lane updates it,
   // then the warp copies the row out as 16-B vectors.  The owner's count
-  // before its increment is the sorted position of that record (stored in
-  // keys[e].pad).
-  __device__ static __forceinline__ void sweep(XsKey *keys, const uint32_t *chist, int *ig, int *sw, long long n_u,
+  // before its increment is the sorted position s of that record: the
+  // record id goes to inv[s] (each owner's positions are written in order),
+  // so that (R) writes the records in sorted order.
+  __device__ static __forceinline__ void sweep(const XsKey *keys, uint32_t *inv, const uint32_t *chist, int *ig,
+                                               int *sw, long long n_u,
                                                int n_iso, int n_gp, long long nch, int crank, int csize) {
     const int tid = threadIdx.x, T = blockDim.x, lane = tid & 31, warp = tid >> 5, nw = T >> 5;
     const int ip = xs_iso_pad(n_iso), ng4 = ip >> 2;
@@ -375,7 +365,7 @@ struct XsApp {
             const int c = cnt[own_cur];
             cnt[own_cur] = c + 1;
             val[own_cur] = clip(c + 1);
-            keys[g + sl].pad = (unsigned)(own_cur * n_gp + c);
+            inv[(size_t)own_cur * n_gp + c] = keys[g + sl].idx;
           }
           __syncwarp();
           for (int q = lane; q < ng4; q += 32) row[q] = reinterpret_cast<const int4 *>(val)[q];
@@ -782,9 +772,21 @@ struct XsApp {
       for (long long b = lo; b < hi; b++) uf[b] = (uint32_t)e;
     }
     sync();
-    for (long long i = g0; i < n_iso; i += GS) {  // exclusive scan over chunks per owner
+    for (long long i = g0; i < n_iso; i += GS) {  // exclusive scan over chunks per owner, kU loads in
+      constexpr int kU = 16;                      // flight (one at a time: an L2 round trip per chunk)
       uint32_t run = 0;
-      for (long long ch = 0; ch < nch; ch++) {
+      long long ch = 0;
+      for (; ch + kU <= nch; ch += kU) {
+        uint32_t v[kU];
+#pragma unroll
+        for (int u = 0; u < kU; u++) v[u] = chist[(ch + u) * n_iso + i];
+#pragma unroll
+        for (int u = 0; u < kU; u++) {
+          chist[(ch + u) * n_iso + i] = run;
+          run += v[u];
+        }
+      }
+      for (; ch < nch; ch++) {
         const uint32_t v = chist[ch * n_iso + i];
         chist[ch * n_iso + i] = run;
         run += v;
@@ -795,19 +797,29 @@ struct XsApp {
     // (W) sweep: a warp per chunk, lanes own nuclides; row e of the index grid
     // is clip(#{k>=1: E_i[k] <= u_e}, 0, n_gp-2) = clip(cnt_i(e) - 1, ...),
     // and the owner's new count is the sorted position of that record (XS-4).
-    sweep(keys, chist, ig, (int *)(ens_smem(c) + S.nbkt), n_u, n_iso, n_gp, nch, team ? (int)c.crank : 0,
+    uint32_t *inv = (uint32_t *)(c.arena + L.inv);
+    sweep(keys, inv, chist, ig, (int *)(ens_smem(c) + S.nbkt), n_u, n_iso, n_gp, nch, team ? (int)c.crank : 0,
           team ? (int)c.csize : 1);
     sync();
     XS_STOP(7);
-    // (R) records to their sorted positions, keys read coalesced
-    for (long long e0 = g0; e0 < n_u; e0 += 2LL * GS) {
-      XsKey k[2];
+    // (R) records in sorted order (coalesced 48-B writes): sorted position s
+    // holds record inv[s], its energy re-drawn with the other five
+    for (long long s0 = g0; s0 < n_u; s0 += 2LL * GS) {
+      unsigned r[2];
 #pragma unroll
       for (int q = 0; q < 2; q++)
-        if (e0 + q * GS < n_u) k[q] = keys[e0 + q * GS];
+        if (s0 + q * GS < n_u) r[q] = inv[s0 + q * GS];
 #pragma unroll
       for (int q = 0; q < 2; q++)
-        if (e0 + q * GS < n_u) put_record(jt, k[q].idx, k[q].key, p.gseed, recs + 6 * (size_t)k[q].pad);
+        if (s0 + q * GS < n_u) {
+          uint64_t t = jump6(jt, r[q], p.gseed);
+          const double e = lcg_double(t), x1 = lcg_double(t), x2 = lcg_double(t), x3 = lcg_double(t),
+                       x4 = lcg_double(t), x5 = lcg_double(t);
+          double2 *d = reinterpret_cast<double2 *>(recs + 6 * (size_t)(s0 + q * GS));
+          __stcs(d, make_double2(e, x1));  // evict-first: the tables stream past L2
+          __stcs(d + 1, make_double2(x2, x3));
+          __stcs(d + 2, make_double2(x4, x5));
+        }
     }
     sync();
     phase_mark_if(trc, c, 8);

@@ -1,6 +1,6 @@
 """Per-kernel CUDA-event times of a bench workload (a probe, not the bench).
 
-    python tools/ktimes.py <C1|C2|C2U|C3|C4|C5|TSTAR> [reps] [--phases] [--split | --fused]
+    python tools/ktimes.py <C1|C2|C2U|C3|C4|C5|TSTAR> [reps] [--phases] [--split | --fused] [--team CS]
 
 Launches the workload once (cold), relaunches it `reps` times (default 5) and
 prints the best launch time and, for that launch, every kernel's time
@@ -29,6 +29,10 @@ def main():
         if flag in argv:
             argv.remove(flag)
             mode[flag[2:]] = True
+    if "--team" in argv:
+        i = argv.index("--team")
+        mode["team_ctas"] = int(argv[i + 1])
+        del argv[i:i + 2]
     name = argv[0]
     reps = int(argv[1]) if len(argv) > 1 else 5
     lines, _ = bench.workload_lines(name, 1)
