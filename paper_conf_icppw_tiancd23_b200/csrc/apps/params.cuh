@@ -173,10 +173,13 @@ ENS_HD long long xs_smem_nb(const XsParams &p) {
   while (nb * 2 <= n_u / 2 && nb < kXsSmemBkt) nb *= 2;
   return nb;
 }
+#ifndef ENS_XS_UBKT_DIV
+#define ENS_XS_UBKT_DIV 4
+#endif
 ENS_HD long long xs_buckets(const XsParams &p) {
   const long long n_u = (long long)p.n_iso * p.n_gp;
   if (xs_smem_nb(p)) return xs_smem_nb(p);
-  if (p.grid == XS_UNIONIZED) return pow2_ceil((int)((n_u + 1) / 2));
+  if (p.grid == XS_UNIONIZED) return pow2_ceil((int)((n_u + ENS_XS_UBKT_DIV - 1) / ENS_XS_UBKT_DIV));
   return (long long)p.n_iso * (pow2_ceil(p.n_gp) / 2 > 0 ? pow2_ceil(p.n_gp) / 2 : 1);
 }
 // per-nuclide sort buckets of the hash / nuclide init (~ENS_XS_NBN_DIV / 2 keys each)

@@ -368,7 +368,7 @@ struct XsApp {
             inv[(size_t)own_cur * n_gp + c] = keys[g + sl].idx;
           }
           __syncwarp();
-          for (int q = lane; q < ng4; q += 32) row[q] = reinterpret_cast<const int4 *>(val)[q];
+          for (int q = lane; q < ng4; q += 32) __stcs(row + q, reinterpret_cast<const int4 *>(val)[q]);  // evict-first
         }
         __syncwarp();
       }
