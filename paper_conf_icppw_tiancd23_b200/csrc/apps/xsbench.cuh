@@ -530,9 +530,9 @@ struct XsApp {
       int anom = 0;
 #pragma unroll 2
       for (int k = tid; k < n_gp; k += T) {
-        uint64_t t = jump6(jt, r0 + Js[k], p.gseed);
-        const double e = lcg_double(t), x1 = lcg_double(t), x2 = lcg_double(t), x3 = lcg_double(t),
-                     x4 = lcg_double(t), x5 = lcg_double(t);
+        double x[6];  // draws 6r+1..6r+6: energy, five cross sections
+        lcg_doubles6(jump6(jt, r0 + Js[k], p.gseed), x);
+        const double e = x[0], x1 = x[1], x2 = x[2], x3 = x[3], x4 = x[4], x5 = x[5];
         double2 *d = reinterpret_cast<double2 *>(rec_i + 6 * (size_t)k);
         __stcs(d, make_double2(e, x1));
         __stcs(d + 1, make_double2(x2, x3));
@@ -812,9 +812,9 @@ struct XsApp {
 #pragma unroll
       for (int q = 0; q < 2; q++)
         if (s0 + q * GS < n_u) {
-          uint64_t t = jump6(jt, r[q], p.gseed);
-          const double e = lcg_double(t), x1 = lcg_double(t), x2 = lcg_double(t), x3 = lcg_double(t),
-                       x4 = lcg_double(t), x5 = lcg_double(t);
+          double x[6];  // draws 6r+1..6r+6: energy, five cross sections
+          lcg_doubles6(jump6(jt, r[q], p.gseed), x);
+          const double e = x[0], x1 = x[1], x2 = x[2], x3 = x[3], x4 = x[4], x5 = x[5];
           double2 *d = reinterpret_cast<double2 *>(recs + 6 * (size_t)(s0 + q * GS));
           __stcs(d, make_double2(e, x1));  // evict-first: the tables stream past L2
           __stcs(d + 1, make_double2(x2, x3));
@@ -1184,9 +1184,9 @@ struct XsApp {
           const int k = k0 + lane;
           int chk = NC;
           if (k < n_gp) {
-            uint64_t t = jump6(jt, r0 + J[k], gseed);
-            const double e = lcg_double(t), x1 = lcg_double(t), x2 = lcg_double(t), x3 = lcg_double(t),
-                         x4 = lcg_double(t), x5 = lcg_double(t);
+            double x[6];  // draws 6r+1..6r+6: energy, five cross sections
+            lcg_doubles6(jump6(jt, r0 + J[k], gseed), x);
+            const double e = x[0], x1 = x[1], x2 = x[2], x3 = x[3], x4 = x[4], x5 = x[5];
             double2 *d = reinterpret_cast<double2 *>(rec_i + 6 * (size_t)k);
             __stcs(d, make_double2(e, x1));  // evict-first, like the index rows
             __stcs(d + 1, make_double2(x2, x3));

@@ -52,6 +52,17 @@ __device__ __forceinline__ double lcg_double(uint64_t &s) {
   s = lcg_next(s);
   return __ull2double_rn(s) * 0x1p-63;
 }
+// the six draws after state s (a record's draws 6r+1..6r+6) as six
+// independent maps s -> A^k s + C_k (k = 1..6): the same states as six
+// lcg_double calls, without their k-step dependency chain
+__host__ __device__ constexpr uint64_t lcg_pow_a(int k) { uint64_t a = 1ULL; for (int i = 0; i < k; i++) a *= kLcgA; return a; }
+__host__ __device__ constexpr uint64_t lcg_pow_c(int k) { uint64_t c = 0ULL; for (int i = 0; i < k; i++) c = kLcgA * c + 1ULL; return c; }
+__device__ __forceinline__ void lcg_doubles6(uint64_t s, double (&x)[6]) {
+  constexpr uint64_t A[6] = {lcg_pow_a(1), lcg_pow_a(2), lcg_pow_a(3), lcg_pow_a(4), lcg_pow_a(5), lcg_pow_a(6)};
+  constexpr uint64_t C[6] = {lcg_pow_c(1), lcg_pow_c(2), lcg_pow_c(3), lcg_pow_c(4), lcg_pow_c(5), lcg_pow_c(6)};
+#pragma unroll
+  for (int k = 0; k < 6; k++) x[k] = __ull2double_rn((A[k] * s + C[k]) & kMask63) * 0x1p-63;
+}
 __device__ __forceinline__ uint64_t lcg_int(uint64_t &s) {
   s = lcg_next(s);
   return s;
