@@ -246,7 +246,7 @@ ENS_HD long long xs_uchunks(const XsParams &p) {
 // arena layout (byte offsets, 256-B aligned)
 struct XsLayout {
   uint64_t recs;      // [n_iso][n_gp] x 48 B records, sorted per nuclide
-  uint64_t keys;      // [n_u] (hash / nuclide: [cs][n_gp]) x 16 B {energy bits, record id}, bucket-sorted
+  uint64_t keys;      // unionized: [n_u] u32 record ids sorted by energy (block path) or [n_iso][n_gp] u64 sorted energies (warp path); hash / nuclide: [cs][n_gp] u64 sorted energies
   uint64_t bkt;       // [xs_buckets] u32 bucket counts -> offsets
   uint64_t uenergy;   // unionized: [n_u] sorted union energies (u64 bits)
   uint64_t ufind;     // unionized: [xs_ubins] u32 union search table (private accelerator)
@@ -304,7 +304,7 @@ ENS_HD XsLayout xs_layout(const XsParams &p, int cs = 1) {
   // unionized: one sort of all n_u records; otherwise one nuclide at a time
   const uint64_t n_s = p.grid == XS_UNIONIZED ? n_u : (uint64_t)p.n_gp * (uint64_t)cs;
   L.recs = o; o = align_up(o + n_u * 48, 256);
-  L.keys = o; o = align_up(o + n_s * 16, 256);
+  L.keys = o; o = align_up(o + n_s * 8, 256);  // u32 ids (unionized, block path) or u64 energies
   L.bkt = o;
   if (p.grid == XS_UNIONIZED) o = align_up(o + (uint64_t)xs_buckets(p) * 4, 256);
   if (p.grid == XS_UNIONIZED) {

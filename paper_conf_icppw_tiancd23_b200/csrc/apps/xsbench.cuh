@@ -6,9 +6,9 @@
 //
 // B200 design (results identical to the oracle):
 //  * init keeps shared memory small (material tables + bucket counters) so
-//    the L1 stays large for the lookup phase: only {energy, record id} keys
-//    are sorted (energies are uniform in [0,1): counts -> scan -> scatter ->
-//    insertion sort of ~1.4-element buckets); each record is then written
+//    the L1 stays large for the lookup phase: only record ids are sorted, by
+//    energy (uniform in [0,1): counts -> scan -> scatter -> sort of ~4-record
+//    buckets, energies re-drawn from the ids); each record is then written
 //    once, at its sorted position, its cross sections re-drawn from the LCG
 //    through jump tables (no generation-order copy);
 //  * the hash index grid is stored nuclide-major [n_iso][bins+1] (entry
@@ -130,11 +130,6 @@ __device__ __forceinline__ long long gs_u64(const uint64_t *A, double q, long lo
 #else
 #define XS_STOP(k) phase_mark_if(trc, c, (k))  // tracing (ENS_F_PHASES): end of init phase k
 #endif
-
-struct XsKey {
-  unsigned long long key;  // energy bit pattern (positive doubles order as integers)
-  unsigned int idx, pad;
-};
 
 // init-sort bucket of record r with energy e in [0, 1]: by energy alone
 // (unionized) or by (nuclide, energy); nb / nbn are powers of two, so
@@ -280,8 +275,12 @@ struct XsApp {
     if (r >> 24) s = jt[256 + ((r >> 24) & 63u)](s);
     return s;
   }
-  // sort keys[lo, hi) by (energy, record id): <= 8 in registers, else in place
-  __device__ static __forceinline__ void sort_bucket(XsKey *keys, long long lo, long long hi) {
+  // sort the record ids ids[lo, hi) by (energy, record id), each energy
+  // re-drawn once from its id (draw 6r+1): <= 8 in registers, <= 64 in a
+  // local array (~2 % of the buckets at ~4 records each), else in place with
+  // the energies re-drawn per comparison (never at these bucket sizes)
+  __device__ static __forceinline__ void sort_bucket(uint32_t *ids, long long lo, long long hi, const Affine *jt,
+                                                     uint64_t gseed) {
     const int cnt = (int)(hi - lo);
     if (cnt <= 1) return;
     if (cnt <= 8) {
@@ -290,9 +289,8 @@ struct XsApp {
 #pragma unroll
       for (int q = 0; q < 8; q++)
         if (q < cnt) {
-          const XsKey v = keys[lo + q];
-          kk[q] = v.key;
-          ii[q] = v.idx;
+          ii[q] = ids[lo + q];
+          kk[q] = dbits(rec_energy(jt, ii[q], gseed));
         }
 #pragma unroll
       for (int x = 1; x < 8; x++) {
@@ -310,23 +308,38 @@ struct XsApp {
       }
 #pragma unroll
       for (int q = 0; q < 8; q++)
-        if (q < cnt) {
-          XsKey v;
-          v.key = kk[q];
-          v.idx = ii[q];
-          v.pad = 0;
-          keys[lo + q] = v;
+        if (q < cnt) ids[lo + q] = ii[q];
+      return;
+    }
+    if (cnt <= 64) {
+      unsigned long long kk[64];
+      unsigned ii[64];
+      for (int x = 0; x < cnt; x++) {
+        const unsigned v = ids[lo + x];
+        const unsigned long long ve = dbits(rec_energy(jt, v, gseed));
+        int y = x - 1;
+        while (y >= 0 && (kk[y] > ve || (kk[y] == ve && ii[y] > v))) {
+          kk[y + 1] = kk[y];
+          ii[y + 1] = ii[y];
+          y--;
         }
+        kk[y + 1] = ve;
+        ii[y + 1] = v;
+      }
+      for (int x = 0; x < cnt; x++) ids[lo + x] = ii[x];
       return;
     }
     for (long long x = lo + 1; x < hi; x++) {
-      const XsKey v = keys[x];
+      const unsigned v = ids[x];
+      const unsigned long long ve = dbits(rec_energy(jt, v, gseed));
       long long y = x - 1;
-      while (y >= lo && (keys[y].key > v.key || (keys[y].key == v.key && keys[y].idx > v.idx))) {
-        keys[y + 1] = keys[y];
-        y--;
+      for (; y >= lo; y--) {
+        const unsigned w = ids[y];
+        const unsigned long long we = dbits(rec_energy(jt, w, gseed));
+        if (!(we > ve || (we == ve && w > v))) break;
+        ids[y + 1] = w;
       }
-      keys[y + 1] = v;
+      ids[y + 1] = v;
     }
   }
 
@@ -338,7 +351,7 @@ struct XsApp {
   // before its increment is the sorted position s of that record: the
   // record id goes to inv[s] (each owner's positions are written in order),
   // so that (R) writes the records in sorted order.
-  __device__ static __forceinline__ void sweep(const XsKey *keys, uint32_t *inv, const uint32_t *chist, int *ig,
+  __device__ static __forceinline__ void sweep(const uint32_t *ids, uint32_t *inv, const uint32_t *chist, int *ig,
                                                int *sw, long long n_u,
                                                int n_iso, int n_gp, long long nch, int crank, int csize) {
     const int tid = threadIdx.x, T = blockDim.x, lane = tid & 31, warp = tid >> 5, nw = T >> 5;
@@ -354,10 +367,10 @@ struct XsApp {
       }
       __syncwarp();
       // record ids of the next 32 rows are prefetched while this group is swept
-      unsigned id_next = e0 + lane < e1 ? keys[e0 + lane].idx : 0u;
+      unsigned id_next = e0 + lane < e1 ? ids[e0 + lane] : 0u;
       for (long long g = e0; g < e1; g += 32) {
         const int own_cur = (int)(id_next / (unsigned)n_gp);
-        id_next = g + 32 + lane < e1 ? keys[g + 32 + lane].idx : 0u;
+        id_next = g + 32 + lane < e1 ? ids[g + 32 + lane] : 0u;
         const int ng = (int)(e1 - g < 32 ? e1 - g : 32);
         int4 *row = reinterpret_cast<int4 *>(ig + (size_t)g * ip);
         for (int sl = 0; sl < ng; sl++, row += ng4) {
@@ -365,7 +378,7 @@ struct XsApp {
             const int c = cnt[own_cur];
             cnt[own_cur] = c + 1;
             val[own_cur] = clip(c + 1);
-            inv[(size_t)own_cur * n_gp + c] = keys[g + sl].idx;
+            inv[(size_t)own_cur * n_gp + c] = ids[g + sl];
           }
           __syncwarp();
           for (int q = lane; q < ng4; q += 32) __stcs(row + q, reinterpret_cast<const int4 *>(val)[q]);  // evict-first
@@ -661,8 +674,9 @@ struct XsApp {
   // ---- XS-3/4/5, unionized grid: one block-wide sort of all records ------
   // One bucket sort of all n_u records by energy replaces n_iso per-nuclide
   // sorts and the union merge: (G) count each record's energy bucket (energy
-  // = draw 6r+1, XS-3); (S) scan; (P) scatter {energy, record id}; (B)
-  // insertion-sort each ~2-element bucket.  The sorted keys ARE the union
+  // = draw 6r+1, XS-3); (S) scan; (P) scatter the record ids (4 B: the
+  // energies are re-drawn where needed); (B) sort each ~4-record bucket by
+  // (energy, id).  The sorted records ARE the union
   // (XS-5) and a nuclide's records in union order are its sorted records
   // (XS-4).  Ties are measure-zero (reading Q13) and broken by record id.
   // (U) union tables, (W) index sweep, (R) every record written once to its
@@ -684,7 +698,7 @@ struct XsApp {
     const int nbn = xs_nbn(n_gp);
     const Affine *jt = (const Affine *)(ens_smem(c) + S.jmp);
     double *recs = (double *)(c.arena + L.recs);
-    XsKey *keys = (XsKey *)(c.arena + L.keys);
+    uint32_t *ids = (uint32_t *)(c.arena + L.keys);  // record ids, sorted by (energy, id)
     const bool sm_bkt = xs_smem_nb(p) != 0;
     uint32_t *bkt = sm_bkt ? (uint32_t *)(ens_smem(c) + S.ubkt) : (uint32_t *)(c.arena + L.bkt);
     int *ig = (int *)(c.arena + L.index);
@@ -731,11 +745,7 @@ struct XsApp {
         for (int q = 0; q < kQ; q++) {
           const long long r = r0 + (long long)q * GS;
           if (r < n_u) {
-            XsKey k;
-            k.key = eb[q];
-            k.idx = (unsigned)r;
-            k.pad = 0;
-            keys[pos[q]] = k;
+            ids[pos[q]] = (uint32_t)r;
           }
         }
       }
@@ -743,11 +753,12 @@ struct XsApp {
     sync();
     XS_STOP(3);
     // (B) sort each bucket by (energy, record id); bkt[b] = end of bucket b
-    for (long long b = g0; b < NB; b += GS) sort_bucket(keys, b ? (long long)bkt[b - 1] : 0, (long long)bkt[b]);
+    for (long long b = g0; b < NB; b += GS)
+      sort_bucket(ids, b ? (long long)bkt[b - 1] : 0, (long long)bkt[b], jt, p.gseed);
     sync();
     XS_STOP(4);
 
-    // (U) keys[] is the union (XS-5); owner = record id / n_gp
+    // (U) ids[] in order is the union (XS-5); owner = record id / n_gp
     uint64_t *uA = (uint64_t *)(c.arena + L.uenergy);
     uint32_t *chist = sm_bkt ? bkt : (uint32_t *)(c.arena + L.chist);  // the sort's counters are dead
     const long long nch = (n_u + kXsSweepRows - 1) / kXsSweepRows;
@@ -764,11 +775,12 @@ struct XsApp {
       return bk < UB ? bk : UB;
     };
     for (long long e = g0; e < n_u; e += GS) {  // union energies, chunk owner counts, search table:
-      const XsKey k = keys[e];                   // ufind[b] = #{k >= 1 : u_k <= b / UB} = e on
-      uA[e] = k.key;                             // [b_e, b_e+1) (b_0 := 0, b_n_u := UB)
-      atomicAdd(&chist[(e / kXsSweepRows) * n_iso + k.idx / n_gp], 1u);
-      const long long lo = e == 0 ? 0 : bfirst(k.key);
-      const long long hi = e + 1 < n_u ? bfirst(keys[e + 1].key) : UB;
+      const uint32_t id = ids[e];                // ufind[b] = #{k >= 1 : u_k <= b / UB} = e on
+      const unsigned long long key = dbits(rec_energy(jt, id, p.gseed));  // [b_e, b_e+1) (b_0 := 0,
+      uA[e] = key;                                                         // b_n_u := UB)
+      atomicAdd(&chist[(e / kXsSweepRows) * n_iso + id / n_gp], 1u);
+      const long long lo = e == 0 ? 0 : bfirst(key);
+      const long long hi = e + 1 < n_u ? bfirst(dbits(rec_energy(jt, ids[e + 1], p.gseed))) : UB;
       for (long long b = lo; b < hi; b++) uf[b] = (uint32_t)e;
     }
     sync();
@@ -798,7 +810,7 @@ struct XsApp {
     // is clip(#{k>=1: E_i[k] <= u_e}, 0, n_gp-2) = clip(cnt_i(e) - 1, ...),
     // and the owner's new count is the sorted position of that record (XS-4).
     uint32_t *inv = (uint32_t *)(c.arena + L.inv);
-    sweep(keys, inv, chist, ig, (int *)(ens_smem(c) + S.nbkt), n_u, n_iso, n_gp, nch, team ? (int)c.crank : 0,
+    sweep(ids, inv, chist, ig, (int *)(ens_smem(c) + S.nbkt), n_u, n_iso, n_gp, nch, team ? (int)c.crank : 0,
           team ? (int)c.csize : 1);
     sync();
     XS_STOP(7);
