@@ -774,14 +774,28 @@ struct XsApp {
       if ((double)bk < x) bk++;
       return bk < UB ? bk : UB;
     };
-    for (long long e = g0; e < n_u; e += GS) {  // union energies, chunk owner counts, search table:
-      const uint32_t id = ids[e];                // ufind[b] = #{k >= 1 : u_k <= b / UB} = e on
-      const unsigned long long key = dbits(rec_energy(jt, id, p.gseed));  // [b_e, b_e+1) (b_0 := 0,
-      uA[e] = key;                                                         // b_n_u := UB)
-      atomicAdd(&chist[(e / kXsSweepRows) * n_iso + id / n_gp], 1u);
-      const long long lo = e == 0 ? 0 : bfirst(key);
-      const long long hi = e + 1 < n_u ? bfirst(dbits(rec_energy(jt, ids[e + 1], p.gseed))) : UB;
-      for (long long b = lo; b < hi; b++) uf[b] = (uint32_t)e;
+    // union energies, chunk owner counts, search table: ufind[b] = #{k >= 1 :
+    // u_k <= b / UB} = e on [b_e, b_e+1) (b_0 := 0, b_n_u := UB).  The warp's
+    // lanes hold consecutive e: u_{e+1} comes from the next lane (lane 31
+    // re-draws it)
+    const int lane = tid & 31;
+    for (long long w0 = g0 - lane; w0 < n_u; w0 += GS) {
+      const long long e = w0 + lane;
+      uint32_t id = 0;
+      unsigned long long key = 0;
+      if (e < n_u) {
+        id = ids[e];
+        key = dbits(rec_energy(jt, id, p.gseed));
+      }
+      unsigned long long knext = __shfl_down_sync(0xffffffffu, key, 1);
+      if (lane == 31 && e + 1 < n_u) knext = dbits(rec_energy(jt, ids[e + 1], p.gseed));
+      if (e < n_u) {
+        uA[e] = key;
+        atomicAdd(&chist[(e / kXsSweepRows) * n_iso + id / n_gp], 1u);
+        const long long lo = e == 0 ? 0 : bfirst(key);
+        const long long hi = e + 1 < n_u ? bfirst(knext) : UB;
+        for (long long b = lo; b < hi; b++) uf[b] = (uint32_t)e;
+      }
     }
     sync();
     for (long long i = g0; i < n_iso; i += GS) {  // exclusive scan over chunks per owner, kU loads in
