@@ -1702,8 +1702,9 @@ struct XsApp {
       ENS_CHECK(s0 <= s1 && s1 <= n);
       for (int f = lane; f < nf; f += 32) cnt[f] = 0u;
       __syncwarp();
-      // buckets of <= 32 * kR energies (~325 at C2's size) are loaded once,
-      // all loads in flight, and kept in registers; larger ones re-read
+      // buckets of <= 32 * kR energies (~325 on average at C2's size) are
+      // loaded once, all loads in flight, and kept in registers; larger ones
+      // (the frequent materials' buckets) are re-read in batches of 32 * kR
       constexpr int kR = 16;
       const bool inreg = s1 - s0 <= 32 * kR;
       double v[kR];
@@ -1717,7 +1718,17 @@ struct XsApp {
         for (int r = 0; r < kR; r++)
           if (s0 + lane + 32 * r < s1) atomicAdd(&cnt[fine(v[r])], 1u);
       } else {
-        for (long long i = s0 + lane; i < s1; i += 32) atomicAdd(&cnt[fine(__ldcg(tmp + i))], 1u);
+        for (long long b = s0; b < s1; b += 32 * kR) {
+          double w[kR];
+#pragma unroll
+          for (int r = 0; r < kR; r++) {
+            const long long i = b + lane + 32 * r;
+            w[r] = i < s1 ? __ldcg(tmp + i) : 0.0;
+          }
+#pragma unroll
+          for (int r = 0; r < kR; r++)
+            if (b + lane + 32 * r < s1) atomicAdd(&cnt[fine(w[r])], 1u);
+        }
       }
       __syncwarp();
       {  // exclusive scan of cnt[0, nf): lane l owns entries [l*per, (l+1)*per)
@@ -1752,9 +1763,16 @@ struct XsApp {
             lk_pe[pos] = v[r];
           }
       } else {
-        for (long long i = s0 + lane; i < s1; i += 32) {
-          const double pe = __ldcg(tmp + i);
-          lk_pe[s0 + atomicAdd(&cnt[fine(pe)], 1u)] = pe;
+        for (long long b = s0; b < s1; b += 32 * kR) {
+          double w[kR];
+#pragma unroll
+          for (int r = 0; r < kR; r++) {
+            const long long i = b + lane + 32 * r;
+            w[r] = i < s1 ? __ldcg(tmp + i) : 0.0;
+          }
+#pragma unroll
+          for (int r = 0; r < kR; r++)
+            if (b + lane + 32 * r < s1) lk_pe[s0 + atomicAdd(&cnt[fine(w[r])], 1u)] = w[r];
         }
       }
       __syncwarp();
