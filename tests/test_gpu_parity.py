@@ -146,6 +146,18 @@ def test_xs_union_paths(oracle, line, generic):
     assert_parity(g, o)
 
 
+@pytest.mark.parametrize("team", [1, 3, 5, 16])
+def test_xs_union_block_arena_team(oracle, team):
+    """The block-wide unionized init with its sort counters in the arena (n_u = 355 x 1100 >
+    4 x kXsSmemBkt): ~4-record buckets of record ids, their energies re-drawn; the union pass's
+    next energy from the neighbouring lane; the sweep's inverse map and the record pass in sorted
+    order — on 1..16-CTA teams (non-power-of-two striding), two instances."""
+    lines = ["xsbench -s large -g 1100 -l 3000 -G unionized -r 31",
+             "xsbench -s large -g 1050 -l 2000 -G unionized -r 32"]
+    g, o = run_both(oracle, lines, threads=256, team_ctas=team)
+    assert_parity(g, o)
+
+
 @pytest.mark.parametrize("threads", [32, 64, 128, 512])
 def test_xs_warp_union_threads(oracle, threads):
     """The warp path with 1..16 warps per team (T=32 runs every nuclide and chunk on one warp)."""
