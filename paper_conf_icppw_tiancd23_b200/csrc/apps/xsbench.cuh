@@ -532,6 +532,12 @@ struct XsApp {
       // otherwise the sorted energies go to `ekey` (arena scratch)
       auto bfirst = [&](double e) {  // first bin b with e <= b*du (bins if none; bins <= 10^7: int)
         int bb = (int)(e * p.bins);
+        // the usual answer is bb or bb+1: the three edge tests are independent
+        // (no compare-then-multiply chain); anything else takes the walk
+        const bool dn = bb > 0 && (double)(bb - 1) * du >= e;
+        const bool u0 = bb < p.bins && (double)bb * du < e;
+        const bool u1 = bb + 1 < p.bins && (double)(bb + 1) * du < e;
+        if (!dn && !u1) return bb + (u0 ? 1 : 0);
         while (bb > 0 && (double)(bb - 1) * du >= e) bb--;
         while (bb < p.bins && (double)bb * du < e) bb++;
         return bb;
